@@ -1,0 +1,223 @@
+"""Seeded synthetic inputs shared by the oracle tests, the GPU parity tests and bench.py.
+
+This module holds NONE of the method's arithmetic (no recursion, no schedule,
+no scoring). It only draws sequences and model parameters and writes down the
+fixed scoring tables the workloads name, so both sides of every parity check
+see byte-identical problem definitions (task ③: "only the seeded input
+generators serve both, from a module of their own").
+
+Workload recipe (SURVEY.md §8(d) D1–D5):
+  * master seed 20120611 + config index, numpy PCG64;
+  * RNA  : bases i.i.d. uniform over ACGU (codes 0..3);
+  * protein: residues i.i.d. uniform over the 20 standard amino acids (codes 0..19
+    in the BLOSUM62 order ARNDCQEGHILKMFPSTWYV; BZX* = 20..23 exist in the table);
+  * HMM  : S=64 states, DNA alphabet (ACGT), rows of A, E and pi ~ Dirichlet(1),
+    sequences sampled from the model itself;
+  * Viterbi log-scores: int32 milli-bits round(1000*log2 p), computed once here.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+MASTER_SEED = 20120611
+
+RNA = "ACGU"
+DNA = "ACGT"
+PROTEIN = "ARNDCQEGHILKMFPSTWYVBZX*"
+EN = "abcdefghijklmnopqrstuvwxyz"  # Fig.7's `en` alphabet, used by the edit-distance mode
+
+# NCBI BLOSUM62 in the order of PROTEIN (a published constant; scoring input of
+# the substitution-matrix extension, §5.1; matrix named by
+# the decisions register SURVEY.md App. B).
+_B62_ROWS = """
+ 4 -1 -2 -2  0 -1 -1  0 -2 -1 -1 -1 -1 -2 -1  1  0 -3 -2  0 -2 -1  0 -4
+-1  5  0 -2 -3  1  0 -2  0 -3 -2  2 -1 -3 -2 -1 -1 -3 -2 -3 -1  0 -1 -4
+-2  0  6  1 -3  0  0  0  1 -3 -3  0 -2 -3 -2  1  0 -4 -2 -3  3  0 -1 -4
+-2 -2  1  6 -3  0  2 -1 -1 -3 -4 -1 -3 -3 -1  0 -1 -4 -3 -3  4  1 -1 -4
+ 0 -3 -3 -3  9 -3 -4 -3 -3 -1 -1 -3 -1 -2 -3 -1 -1 -2 -2 -1 -3 -3 -2 -4
+-1  1  0  0 -3  5  2 -2  0 -3 -2  1  0 -3 -1  0 -1 -2 -1 -2  0  3 -1 -4
+-1  0  0  2 -4  2  5 -2  0 -3 -3  1 -2 -3 -1  0 -1 -3 -2 -2  1  4 -1 -4
+ 0 -2  0 -1 -3 -2 -2  6 -2 -4 -4 -2 -3 -3 -2  0 -2 -2 -3 -3 -1 -2 -1 -4
+-2  0  1 -1 -3  0  0 -2  8 -3 -3 -1 -2 -1 -2 -1 -2 -2  2 -3  0  0 -1 -4
+-1 -3 -3 -3 -1 -3 -3 -4 -3  4  2 -3  1  0 -3 -2 -1 -3 -1  3 -3 -3 -1 -4
+-1 -2 -3 -4 -1 -2 -3 -4 -3  2  4 -2  2  0 -3 -2 -1 -2 -1  1 -4 -3 -1 -4
+-1  2  0 -1 -3  1  1 -2 -1 -3 -2  5 -1 -3 -1  0 -1 -3 -2 -2  0  1 -1 -4
+-1 -1 -2 -3 -1  0 -2 -3 -2  1  2 -1  5  0 -2 -1 -1 -1 -1  1 -3 -1 -1 -4
+-2 -3 -3 -3 -2 -3 -3 -3 -1  0  0 -3  0  6 -4 -2 -2  1  3 -1 -3 -3 -1 -4
+-1 -2 -2 -1 -3 -1 -1 -2 -2 -3 -3 -1 -2 -4  7 -1 -1 -4 -3 -2 -2 -1 -2 -4
+ 1 -1  1  0 -1  0  0  0 -1 -2 -2  0 -1 -2 -1  4  1 -3 -2 -2  0  0  0 -4
+ 0 -1  0 -1 -1 -1 -1 -2 -2 -1 -1 -1 -1 -2 -1  1  5 -2 -2  0 -1 -1  0 -4
+-3 -3 -4 -4 -2 -2 -3 -2 -2 -3 -2 -3 -1  1 -4 -3 -2 11  2 -3 -4 -3 -2 -4
+-2 -2 -2 -3 -2 -1 -2 -3  2 -1 -1 -2 -1  3 -3 -2 -2  2  7 -1 -3 -2 -1 -4
+ 0 -3 -3 -3 -1 -2 -2 -3 -3  3  1 -2  1 -1 -2 -2  0 -3 -1  4 -3 -2 -1 -4
+-2 -1  3  4 -3  0  1 -1  0 -3 -4  0 -3 -3 -2  0 -1 -4 -3 -3  4  1 -1 -4
+-1  0  0  1 -3  3  4 -2  0 -3 -3  1 -1 -3 -1  0 -1 -3 -2 -2  1  4 -1 -4
+ 0 -1 -1 -1 -2 -1 -1 -1 -1 -1 -1 -1 -1 -1 -2  0  0 -2 -1 -1 -1 -1 -1 -4
+-4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4 -4  1
+"""
+
+SW_GAP = 4          # linear gap penalty g (BLOSUM62's '*' score)
+NUSS_HAIRPIN = 3    # minimum hairpin loop h
+HMM_STATES = 64
+MILLIBIT_FLOOR = -100000  # score used for p == 0 (2^-100); Dirichlet(1) draws never hit it in practice
+
+
+def rng(config_index: int, extra: int = 0) -> np.random.Generator:
+    """numpy PCG64 seeded with 20120611 + config index (+ extra sub-stream)."""
+    return np.random.Generator(np.random.PCG64(MASTER_SEED + config_index + 1000003 * extra))
+
+
+def blosum62() -> np.ndarray:
+    m = np.array([int(v) for v in _B62_ROWS.split()], dtype=np.int8).reshape(24, 24)
+    return m
+
+
+def edit_sigma(asz: int = 26) -> np.ndarray:
+    """Unit-cost table for the edit-distance mode, stated as a scoring input
+    (0 on the diagonal, -1 elsewhere). Only the GPU's max-plus alignment kernel
+    consumes it; the oracle evaluates Fig.7's comparison s[i-1]==t[j-1] itself."""
+    m = -np.ones((asz, asz), dtype=np.int8)
+    np.fill_diagonal(m, 0)
+    return m
+
+
+def rna_pair_mask(gu: bool = True) -> np.ndarray:
+    """4x4 uint8 mask over ACGU: 1 where the two bases may pair (WC + optional GU wobble)."""
+    m = np.zeros((4, 4), dtype=np.uint8)
+    for a, b in ("AU", "UA", "GC", "CG") + (("GU", "UG") if gu else ()):
+        m[RNA.index(a), RNA.index(b)] = 1
+    return m
+
+
+def encode(s: str, alphabet: str) -> np.ndarray:
+    return np.frombuffer(bytes(alphabet.index(c) for c in s), dtype=np.uint8).copy()
+
+
+def decode(codes, alphabet: str) -> str:
+    return "".join(alphabet[int(c)] for c in codes)
+
+
+def random_seq(g: np.random.Generator, n: int, k: int) -> np.ndarray:
+    return g.integers(0, k, size=n, dtype=np.uint8)
+
+
+def pack(seqs) -> tuple[np.ndarray, np.ndarray]:
+    """Concatenate uint8 sequences; returns (cat, offsets[n+1] int64)."""
+    lens = np.array([len(s) for s in seqs], dtype=np.int64)
+    off = np.zeros(len(seqs) + 1, dtype=np.int64)
+    np.cumsum(lens, out=off[1:])
+    cat = np.concatenate([np.asarray(s, dtype=np.uint8) for s in seqs]) if len(seqs) else np.zeros(0, np.uint8)
+    return cat, off
+
+
+def unpack(cat: np.ndarray, off: np.ndarray, i: int) -> np.ndarray:
+    return cat[off[i]:off[i + 1]]
+
+
+# ----------------------------------------------------------------------------- configs
+def config1_rna64() -> np.ndarray:
+    """D1: one 64-nt RNA, seed 20120611+1."""
+    return random_seq(rng(1), 64, 4)
+
+
+def config2_protein_pairs(n_pairs: int = 100_000, length: int = 256, first: int = 0):
+    """D2: n_pairs protein pairs of the given length, seed 20120611+2.
+
+    Returns (a_cat, a_off, b_cat, b_off). `first` skips that many pairs of the
+    same stream (so a bounded sample is a prefix-consistent slice)."""
+    g = rng(2)
+    total = first + n_pairs
+    a = g.integers(0, 20, size=(total, length), dtype=np.uint8)
+    b = g.integers(0, 20, size=(total, length), dtype=np.uint8)
+    a = a[first:]
+    b = b[first:]
+    off = np.arange(n_pairs + 1, dtype=np.int64) * length
+    return a.reshape(-1).copy(), off, b.reshape(-1).copy(), off.copy()
+
+
+def hmm_params(g: np.random.Generator, S: int = HMM_STATES, K: int = 4):
+    """Rows of pi (1xS), A (SxS), E (SxK) ~ Dirichlet(1), float64."""
+    pi = g.dirichlet(np.ones(S))
+    A = g.dirichlet(np.ones(S), size=S)
+    E = g.dirichlet(np.ones(K), size=S)
+    return pi, A, E
+
+
+def sample_hmm(g: np.random.Generator, pi, A, E, n: int, T: int) -> np.ndarray:
+    """n sequences of length T drawn from the HMM (states by pi then A, symbols by E)."""
+    S = len(pi)
+    cA = np.cumsum(A, axis=1)
+    cE = np.cumsum(E, axis=1)
+    cpi = np.cumsum(pi)
+    out = np.empty((n, T), dtype=np.uint8)
+    if T == 0 or n == 0:
+        return out
+    st = np.minimum(np.searchsorted(cpi, g.random(n), side="right"), S - 1)
+    for t in range(T):
+        u = g.random(n)
+        sym = (cE[st] <= u[:, None]).sum(axis=1)
+        out[:, t] = np.minimum(sym, E.shape[1] - 1)
+        u = g.random(n)
+        st = np.minimum((cA[st] <= u[:, None]).sum(axis=1), S - 1)
+    return out
+
+
+def millibits(p) -> np.ndarray:
+    """int32 round(1000*log2 p); p == 0 -> MILLIBIT_FLOOR. Computed once, here only."""
+    p = np.asarray(p, dtype=np.float64)
+    with np.errstate(divide="ignore"):
+        v = np.where(p > 0, np.rint(1000.0 * np.log2(np.where(p > 0, p, 1.0))), MILLIBIT_FLOOR)
+    return np.maximum(v, MILLIBIT_FLOOR).astype(np.int32)
+
+
+def config3_hmm(n_seqs: int = 10_000, T: int = 1000, S: int = HMM_STATES):
+    """D3: 64-state dense HMM over DNA, params seed +3, sequences seed +4.
+
+    Returns dict with fp32 probabilities (pi, A, E) — the values both sides use —
+    their int32 milli-bit scores (lpi, lA, lE), and sequences (n_seqs x T uint8)."""
+    pi, A, E = hmm_params(rng(3), S, 4)
+    pi32, A32, E32 = (x.astype(np.float32) for x in (pi, A, E))
+    seqs = sample_hmm(rng(4), pi, A, E, n_seqs, T)
+    return {
+        "pi": pi32, "A": A32, "E": E32,
+        "lpi": millibits(pi32), "lA": millibits(A32), "lE": millibits(E32),
+        "seqs": seqs, "S": S, "K": 4,
+    }
+
+
+def config4_rna8192(n: int = 8192) -> np.ndarray:
+    """D4: one RNA of length n (8192), seed 20120611+5."""
+    return random_seq(rng(5), n, 4)
+
+
+def config5_lengths(n_seqs: int = 1_000_000, lo: int = 128, hi: int = 512) -> np.ndarray:
+    return rng(6).integers(lo, hi + 1, size=n_seqs, dtype=np.int64)
+
+
+def config5_rna_batch(n_seqs: int = 1_000_000, lo: int = 128, hi: int = 512, ids=None):
+    """D5: RNAs with lengths i.i.d. uniform in [lo, hi], bases i.i.d. ACGU, seed +6.
+
+    Sequence i's bases come from its own sub-stream (seed +6, extra=i+1) so any
+    subset `ids` is generated without drawing the whole million."""
+    lens = config5_lengths(n_seqs, lo, hi)
+    if ids is None:
+        g = rng(6, extra=1)
+        cat = g.integers(0, 4, size=int(lens.sum()), dtype=np.uint8)
+        off = np.zeros(n_seqs + 1, dtype=np.int64)
+        np.cumsum(lens, out=off[1:])
+        return cat, off
+    seqs = []
+    full_off = np.zeros(n_seqs + 1, dtype=np.int64)
+    np.cumsum(lens, out=full_off[1:])
+    g = rng(6, extra=1)
+    # regenerate the full stream lazily in chunks only up to the largest id needed
+    need = int(full_off[max(ids) + 1])
+    cat = g.integers(0, 4, size=need, dtype=np.uint8)
+    for i in ids:
+        seqs.append(cat[full_off[i]:full_off[i + 1]])
+    return pack(seqs)
+
+
+def config5_sample_ids(n_seqs: int = 1_000_000, k: int = 10_000) -> np.ndarray:
+    """The fixed 1% subset (seed +7) used for the on-box oracle timing."""
+    return np.sort(rng(7).choice(n_seqs, size=k, replace=False))

@@ -1,0 +1,144 @@
+"""Pins for the oracle's edit distance (Fig.7) and Smith–Waterman (§6.1) functions.
+
+Brute force over every (local) alignment on tiny inputs, closed forms and
+textbook special cases."""
+import numpy as np
+import pytest
+
+import dpgen
+from tests import brute
+
+EN = dpgen.EN
+
+
+def enc(s):
+    return dpgen.encode(s, EN)
+
+
+def test_edit_textbook(orc):
+    # Levenshtein's textbook example (not in PAPER.md): kitten -> sitting = 3.
+    assert orc.edit(enc("kitten"), enc("sitting")) == 3
+    assert orc.edit(enc("flaw"), enc("lawn")) == 2
+
+
+def test_edit_closed_forms(orc):
+    g = np.random.default_rng(1)
+    for _ in range(50):
+        s = g.integers(0, 4, size=g.integers(0, 12)).astype(np.uint8)
+        t = g.integers(0, 4, size=g.integers(0, 12)).astype(np.uint8)
+        d = orc.edit(s, t)
+        assert orc.edit(s, np.zeros(0, np.uint8)) == len(s)        # d(s, eps) = |s|
+        assert orc.edit(np.zeros(0, np.uint8), t) == len(t)
+        assert orc.edit(s, s) == 0
+        assert d == orc.edit(t, s)                                 # symmetry
+        assert abs(len(s) - len(t)) <= d <= max(len(s), len(t))
+        u = g.integers(0, 4, size=g.integers(0, 8)).astype(np.uint8)
+        assert d <= orc.edit(s, u) + orc.edit(u, t)                # triangle inequality
+
+
+def test_edit_brute_force(orc):
+    g = np.random.default_rng(2)
+    for _ in range(60):
+        s = g.integers(0, 3, size=g.integers(0, 7)).astype(np.uint8)
+        t = g.integers(0, 3, size=g.integers(0, 7)).astype(np.uint8)
+        assert orc.edit(s, t) == brute.brute_edit(list(s), list(t))
+
+
+def test_edit_traceback_canonical(orc):
+    """Ops are an optimal alignment and the canonical one: the smallest reversed op
+    sequence under diag < up(D) < left(I) among all optimal alignments."""
+    g = np.random.default_rng(3)
+    rank = {"M": 0, "X": 0, "S": 0, "D": 1, "I": 2}
+    for _ in range(40):
+        s = list(g.integers(0, 3, size=g.integers(0, 6)))
+        t = list(g.integers(0, 3, size=g.integers(0, 6)))
+        ops = orc.edit_traceback(np.array(s, np.uint8), np.array(t, np.uint8))
+        d = orc.edit(np.array(s, np.uint8), np.array(t, np.uint8))
+        cost = brute.score_alignment(s, t, ops.replace("M", "S").replace("X", "S"),
+                                     lambda a, b: -int(a != b), 1)
+        assert -cost == d
+        i = j = 0
+        for o in ops:  # M/X labels agree with the residues
+            if o in "MX":
+                assert (o == "M") == (s[i] == t[j]); i += 1; j += 1
+            elif o == "D":
+                i += 1
+            else:
+                j += 1
+        best = None
+        for al in brute.all_global_alignments(len(s), len(t)):
+            if -brute.score_alignment(s, t, al, lambda a, b: -int(a != b), 1) == d:
+                key = tuple(rank[o] for o in reversed(al))
+                best = key if best is None or key < best else best
+        assert tuple(rank[o] for o in reversed(ops)) == best
+
+
+def test_sw_brute_force_cells_and_end(orc):
+    """Score and end cell equal the brute-force max over all local alignments."""
+    g = np.random.default_rng(4)
+    sig = dpgen.blosum62()
+    for _ in range(25):
+        s = list(g.integers(0, 24, size=g.integers(0, 5)))
+        t = list(g.integers(0, 24, size=g.integers(0, 5)))
+        gap = int(g.integers(1, 6))
+        _, best, (bi, bj) = brute.brute_local_cells(s, t, sig, gap)
+        sc, ei, ej = orc.sw(np.array(s, np.uint8), np.array(t, np.uint8), sig, gap)
+        assert sc == best
+        assert (ei, ej) == (bi, bj)
+
+
+def test_sw_traceback_canonical(orc):
+    g = np.random.default_rng(5)
+    sig = dpgen.blosum62()
+    rank = {"S": 0, "M": 0, "X": 0, "D": 1, "I": 2}
+    for _ in range(25):
+        s = list(g.integers(0, 6, size=g.integers(0, 5)))
+        t = list(g.integers(0, 6, size=g.integers(0, 5)))
+        gap = int(g.integers(1, 5))
+        sc, ei, ej = orc.sw(np.array(s, np.uint8), np.array(t, np.uint8), sig, gap)
+        ops, (si, sj, ei2, ej2) = orc.sw_traceback(np.array(s, np.uint8), np.array(t, np.uint8), sig, gap)
+        assert (ei2, ej2) == ((ei, ej) if sc > 0 else (0, 0))
+        sub = lambda a, b: int(sig[a][b])
+        if sc == 0:
+            assert ops == ""
+            continue
+        assert brute.score_alignment(s[si:ei], t[sj:ej], ops.replace("M", "S").replace("X", "S"), sub, gap) == sc
+        best = None
+        for i0 in range(ei + 1):
+            for j0 in range(ej + 1):
+                for al in brute.all_global_alignments(ei - i0, ej - j0):
+                    if brute.score_alignment(s[i0:ei], t[j0:ej], al, sub, gap) == sc:
+                        key = tuple(rank[o] for o in reversed(al))
+                        best = key if best is None or key < best else best
+        assert tuple(rank[o] for o in reversed(ops)) == best
+
+
+def test_sw_longest_common_substring(orc):
+    """match=+1, mismatch=-inf-like, gap=inf-like reduces SW to longest common substring."""
+    g = np.random.default_rng(6)
+    sig = np.full((4, 4), -100, dtype=np.int8)
+    np.fill_diagonal(sig, 1)
+    for _ in range(40):
+        s = g.integers(0, 4, size=g.integers(0, 14)).astype(np.uint8)
+        t = g.integers(0, 4, size=g.integers(0, 14)).astype(np.uint8)
+        lcs = 0
+        for i in range(len(s)):
+            for j in range(len(t)):
+                k = 0
+                while i + k < len(s) and j + k < len(t) and s[i + k] == t[j + k]:
+                    k += 1
+                lcs = max(lcs, k)
+        assert orc.sw(s, t, sig, 100)[0] == lcs
+
+
+def test_sw_bounds(orc):
+    g = np.random.default_rng(7)
+    sig = dpgen.blosum62()
+    for _ in range(30):
+        s = g.integers(0, 20, size=g.integers(1, 40)).astype(np.uint8)
+        t = g.integers(0, 20, size=g.integers(1, 40)).astype(np.uint8)
+        sc = orc.sw(s, t, sig, 4)[0]
+        assert sc >= max(0, max(int(sig[a][b]) for a in s for b in t))
+        assert sc <= 11 * min(len(s), len(t))
+        assert sc == orc.sw(t, s, sig.T.copy(), 4)[0]  # transposition symmetry
+        assert orc.sw(s, s, sig, 4)[0] == int(sum(int(sig[a][a]) for a in s))  # identity: diagonal is optimal
