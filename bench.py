@@ -1,0 +1,462 @@
+#!/usr/bin/env python
+"""Benchmark: DP cell-updates/s (GCUPS) on B200 with the roofline fraction of the
+dominant kernel (BASELINE.json metric).
+
+Default workload (N = 1): BASELINE config 2 — 100k synthetic protein pairs of
+length 256, Smith–Waterman (BLOSUM62, linear gap 4) on the anti-diagonal
+schedule. A step = one pass of the whole hot path over one batch: schedule
+(plan) already derived, solve with traceback retention, canonical traceback of
+every pair, and (N > 1) the NCCL gather of scores and tracebacks to rank 0.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--config sw|nuss1|hmm|nuss4|nuss5]
+
+Multi-GPU: one process per GPU (torchrun), each rank processes its own batch
+of the config's size from the same seeded stream (weak scaling), no data-path
+collective; ranks are timed with CUDA events and the max over ranks is used.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import dpgen  # noqa: E402
+
+MEASURED_UBENCH = {  # profiles/ubench_r01.jsonl, lane-ops per SM clock on B200 (this pool)
+    "viaddmnmx_s32": 64.0, "viaddmnmx_s16x2": 128.0, "ffma": 128.0, "lds_bytes": 128.0,
+}
+SMS = 148
+
+
+def peaks():
+    p = {"hbm_gbs": 6570.6, "sm_max_mhz": 1965.0, "source": "fallback"}
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            m = json.load(f)
+        p.update({"hbm_gbs": m["hbm_gbs"], "sm_max_mhz": m.get("sm_max_mhz", 1965.0), "source": "measured"})
+    except Exception:
+        pass
+    return p
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled during the timed region."""
+
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self.proc = None
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 6:
+                self.samples.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        reasons = sorted({names[k] for s in self.samples for k in range(4) if s[2 + k].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+# ----------------------------------------------------------------------------- workloads
+def workload(name, rank, world):
+    """Returns dict with host arrays, a plan factory, cells and algorithmic ops per step."""
+    if name == "sw":
+        n = 100_000
+        a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(n, 256, first=rank * n)
+        return {"kind": "sw", "n": n, "a_cat": a_cat, "a_off": a_off, "b_cat": b_cat, "b_off": b_off,
+                "max_la": 256, "max_lb": 256, "cells": n * 256 * 256, "ops_per_cell": 3, "tb_stride": 513,
+                "workload": "BASELINE config 2: 100k protein pairs x 256 (uniform 20 aa), Smith-Waterman, "
+                            "BLOSUM62, linear gap 4, with tracebacks"}
+    if name == "nuss1":
+        x = dpgen.config1_rna64()
+        cat, off = dpgen.pack([x])
+        n = 64
+        return {"kind": "nuss", "n": 1, "a_cat": cat, "a_off": off, "max_la": 64, "cells": n * (n - 1) // 2,
+                "inner": sum((64 - d) * (d - 1) for d in range(1, 64)), "tb_stride": 64,
+                "workload": "BASELINE config 1: one 64-nt RNA, Nussinov (h=3, WC+GU), with traceback"}
+    if name == "nuss4":
+        x = dpgen.config4_rna8192()
+        cat, off = dpgen.pack([x])
+        n = 8192
+        return {"kind": "nuss", "n": 1, "a_cat": cat, "a_off": off, "max_la": n, "cells": n * (n - 1) // 2,
+                "inner": sum((n - d) * (d - 1) for d in range(1, n)), "tb_stride": n,
+                "workload": "BASELINE config 4: one 8192-nt RNA, Nussinov grid-wide hyperplane sweep, with traceback"}
+    if name == "nuss5":
+        nseq = 1_000_000 // world if world > 1 else 1_000_000
+        nseq = int(os.environ.get("DP_NUSS5_N", nseq))
+        cat, off = dpgen.config5_rna_batch(nseq)
+        lens = np.diff(off)
+        return {"kind": "nuss", "n": nseq, "a_cat": cat, "a_off": off, "max_la": int(lens.max()),
+                "cells": int((lens * (lens - 1) // 2).sum()),
+                "inner": int((lens * (lens - 1) * (lens - 2) // 6).sum()), "tb_stride": 512,
+                "workload": "BASELINE config 5: RNAs of length U[128,512], Nussinov batch, with tracebacks"}
+    if name == "hmm":
+        n = 10_000
+        d = dpgen.config3_hmm(n_seqs=n)
+        seqs = d["seqs"]
+        off = np.arange(n + 1, dtype=np.int64) * seqs.shape[1]
+        return {"kind": "hmm", "n": n, "a_cat": seqs.reshape(-1).copy(), "a_off": off, "max_la": 1000, "hmm": d,
+                "cells": 2 * n * 64 * 1000, "inner": n * 64 * 64 * 999, "tb_stride": 1000,
+                "workload": "BASELINE config 3: 64-state dense HMM, 10k DNA sequences x 1000, forward + Viterbi "
+                            "with Viterbi tracebacks (cells = 2 tables x S x T x n)"}
+    raise SystemExit(f"unknown config {name}")
+
+
+# ----------------------------------------------------------------------------- our arm
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_pldi_carteylm12_b200 as dp
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    W = workload(args.config, rank, world)
+    stream = torch.cuda.Stream(device=dev)
+
+    def cu(x):
+        return torch.from_numpy(np.ascontiguousarray(x)).to(dev)
+
+    plans = []
+    if W["kind"] == "sw":
+        sig = dpgen.blosum62()
+        plans.append(dp.Plan(dp.SW_LINEAR, W["max_la"], W["max_lb"], sigma=sig, gap=dpgen.SW_GAP,
+                             want_traceback=True))
+        dev_in = (cu(W["a_cat"]), cu(W["a_off"]), cu(W["b_cat"]), cu(W["b_off"]))
+    elif W["kind"] == "nuss":
+        plans.append(dp.Plan(dp.NUSSINOV, W["max_la"], pair_mask=dpgen.rna_pair_mask(),
+                             min_hairpin=dpgen.NUSS_HAIRPIN, want_traceback=True))
+        dev_in = (cu(W["a_cat"]), cu(W["a_off"]), None, None)
+    else:
+        h = W["hmm"]
+        plans.append(dp.Plan(dp.HMM_FORWARD, W["max_la"], pi=h["pi"], A=h["A"], E=h["E"]))
+        plans.append(dp.Plan(dp.HMM_VITERBI, W["max_la"], lpi=h["lpi"], lA=h["lA"], lE=h["lE"],
+                             want_traceback=True))
+        dev_in = (cu(W["a_cat"]), cu(W["a_off"]), None, None)
+    n = W["n"]
+    scores = [torch.empty(n, dtype=torch.float32 if (W["kind"] == "hmm" and k == 0) else torch.int32, device=dev)
+              for k in range(len(plans))]
+    tb_plan = plans[-1]
+    stride = W["tb_stride"]
+    tb_out = torch.empty((n, stride), dtype=torch.uint8, device=dev)
+    tb_len = torch.empty(n, dtype=torch.int32, device=dev)
+    tb_co = torch.empty((n, 4), dtype=torch.int32, device=dev) if W["kind"] == "sw" else None
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    gathered = None
+    if world > 1:
+        gathered = torch.empty(world * n, dtype=torch.int32, device=dev)
+
+    ev_k = []  # (start, end) events around the dominant kernel launch
+
+    def step(timed):
+        with torch.cuda.stream(stream):
+            for k, p in enumerate(plans):
+                if timed and k == 0:
+                    e0 = torch.cuda.Event(enable_timing=True)
+                    e1 = torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
+                p.solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=W.get("max_lb", 0), out=scores[k],
+                              stream=stream)
+                if timed and k == 0:
+                    e1.record(stream)
+                    ev_k.append((e0, e1))
+            tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
+            if world > 1:
+                dist.all_gather_into_tensor(gathered, scores[-1] if W["kind"] != "hmm" else scores[1])
+                # tracebacks go to rank 0 only
+                if rank == 0:
+                    bufs = [torch.empty_like(tb_out) for _ in range(world)]
+                    dist.gather(tb_out, gather_list=bufs, dst=0)
+                else:
+                    dist.gather(tb_out, dst=0)
+
+    for _ in range(args.warmup):
+        step(False)
+    torch.cuda.synchronize(dev)
+    launches0 = sum(p.launches for p in plans)
+    step_ms = []
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    with ClockSampler(local_rank) as clk:
+        for _ in range(args.steps):
+            flush.zero_()  # L2 flush between steps, outside the step events
+            s0 = torch.cuda.Event(enable_timing=True)
+            s1 = torch.cuda.Event(enable_timing=True)
+            s0.record(stream)
+            step(True)
+            s1.record(stream)
+            step_ms.append((s0, s1))
+        torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    launches = sum(p.launches for p in plans) - launches0
+    ms = [a.elapsed_time(b) for a, b in step_ms]
+    kms = [a.elapsed_time(b) for a, b in ev_k]
+    ms_step = sum(ms) / len(ms)
+    k_ms = sum(kms) / len(kms)
+    if world > 1:
+        t = torch.tensor([ms_step, k_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_step, k_ms = float(t[0]), float(t[1])
+
+    # ---- end to end through the C ABI with host buffers (pinned), same work per step
+    e2e = e2e_host(args, W, plans, dev, stream, world)
+
+    # ---- roofline of the dominant kernel
+    pk = peaks()
+    roof = roofline(W, k_ms, pk)
+    res = {
+        "metric": "DP cell-updates/sec (GCUPS) at 1/2/4/8 B200 and fraction of roofline",
+        "value": round(W["cells"] * world / (ms_step * 1e-3) / 1e9, 3),
+        "unit": "GCUPS",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(ms_step, 4),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": {"sw": "int32", "nuss": "int16 table / int32 arithmetic", "hmm": "f32 (forward) + int32 (Viterbi)"}[W["kind"]],
+        "data": "synthetic (seeded, dpgen)",
+        "config": {"workload": W["workload"], "config": args.config, "problems_per_gpu": n,
+                   "cells_per_gpu": W["cells"], "l2": "flushed between steps (256 MiB write outside step events)",
+                   "parallelism": f"dp{world} (independent problems per rank)"},
+        "kernel_ms": round(k_ms, 4),
+        "roofline": roof,
+        "gpu_launches": int(launches),
+        "e2e": e2e,
+        "clocks": clk.summary(),
+    }
+    if rank == 0 and not args.no_cpu:
+        res["cpu_baseline"] = cpu_baseline(args.config, W)
+    for p in plans:
+        p.close()
+    return res
+
+
+def roofline(W, k_ms, pk):
+    clock_hz = pk["sm_max_mhz"] * 1e6
+    if W["kind"] == "sw":
+        ops = W["cells"] * W["ops_per_cell"]
+        peak = MEASURED_UBENCH["viaddmnmx_s16x2"] * SMS * clock_hz
+        peak32 = MEASURED_UBENCH["viaddmnmx_s32"] * SMS * clock_hz
+        ach = ops / (k_ms * 1e-3)
+        return {"bound": "alu", "kernel": "k_align<8,SW,TB>", "achieved": round(ach / 1e12, 3),
+                "peak": round(peak / 1e12, 3), "unit": "Tops/s", "frac": round(ach / peak, 4),
+                "frac_vs_int32_peak": round(ach / peak32, 4), "traffic": None,
+                "ops_per_cell": W["ops_per_cell"],
+                "peak_source": "ubench_r01 (VIADDMNMX.S16x2 128 lane-ops/clk/SM) x 148 SMs x sm_max_mhz"}
+    if W["kind"] == "nuss":
+        ops = W["inner"]  # one max-plus (VIADDMNMX) per split evaluation
+        peak = MEASURED_UBENCH["viaddmnmx_s16x2"] * SMS * clock_hz
+        ach = ops / (k_ms * 1e-3)
+        return {"bound": "alu", "kernel": "k_nuss", "achieved": round(ach / 1e12, 4), "peak": round(peak / 1e12, 3),
+                "unit": "Tops/s", "frac": round(ach / peak, 5), "traffic": None,
+                "peak_source": "ubench_r01 (VIADDMNMX.S16x2) x 148 SMs x sm_max_mhz"}
+    ops = 2 * W["inner"]  # forward: one FMA (2 flop) per (p, s) per step
+    peak = MEASURED_UBENCH["ffma"] * SMS * clock_hz * 2
+    ach = ops / (k_ms * 1e-3)
+    return {"bound": "alu", "kernel": "k_forward", "achieved": round(ach / 1e12, 3), "peak": round(peak / 1e12, 3),
+            "unit": "TFLOP/s (fp32 FFMA)", "frac": round(ach / peak, 4), "traffic": None,
+            "peak_source": "ubench_r01 (FFMA 128 lanes/clk/SM) x 148 SMs x sm_max_mhz x 2"}
+
+
+def e2e_host(args, W, plans, dev, stream, world):
+    """Same metric through dp_solve_batch_host: pinned host inputs, H2D, solve, traceback, D2H."""
+    import torch
+    import paper_conf_pldi_carteylm12_b200 as dp
+
+    def pin(x):
+        return torch.from_numpy(np.ascontiguousarray(x)).pin_memory().numpy()
+
+    a_cat, a_off = pin(W["a_cat"]), pin(W["a_off"])
+    b_cat = pin(W["b_cat"]) if "b_cat" in W else None
+    b_off = pin(W["b_off"]) if "b_off" in W else None
+    n, stride = W["n"], W["tb_stride"]
+    outs = []
+    for k, p in enumerate(plans):
+        sc = pin(np.empty(n, np.float32 if (W["kind"] == "hmm" and k == 0) else np.int32))
+        tb = pin(np.empty((n, stride), np.uint8)) if p.want_traceback else None
+        tl = pin(np.empty(n, np.int32)) if p.want_traceback else None
+        tc = pin(np.empty((n, 4), np.int32)) if (p.want_traceback and W["kind"] == "sw") else None
+        outs.append((sc, tb, tl, tc))
+    h2d = a_cat.nbytes + a_off.nbytes + (b_cat.nbytes + b_off.nbytes if b_cat is not None else 0)
+    h2d *= len(plans)
+    d2h = sum(o[0].nbytes + (o[1].nbytes + o[2].nbytes if o[1] is not None else 0) +
+              (o[3].nbytes if o[3] is not None else 0) for o in outs)
+
+    def one():
+        for p, (sc, tb, tl, tc) in zip(plans, outs):
+            p.solve_batch_host_into(a_cat, a_off, b_cat, b_off, sc, tb, stride, tl, tc, stream=stream)
+
+    one()
+    torch.cuda.synchronize(dev)
+    steps = max(1, min(args.steps, 5))
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        one()
+    e1.record(stream)
+    torch.cuda.synchronize(dev)
+    ms = e0.elapsed_time(e1) / steps
+    if world > 1:
+        import torch.distributed as dist
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t[0])
+    return {"value": round(W["cells"] * world / (ms * 1e-3) / 1e9, 3), "unit": "GCUPS", "ms_per_step": round(ms, 3),
+            "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+            "api": "dp_solve_batch_host (pinned host buffers; H2D + solve + traceback + D2H)"}
+
+
+# ----------------------------------------------------------------------------- oracle (CPU)
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def oracle_sample(config, W, budget_s):
+    """Times the oracle as it stands on a bounded sample; returns (cells/s, sample text, cores)."""
+    import oracle
+    cores = host_cores()
+    if config == "sw":
+        k = 4000
+        a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(k)
+        sig = dpgen.blosum62()
+        t = time.perf_counter()
+        oracle.sw_batch(a_cat, a_off, b_cat, b_off, sig, dpgen.SW_GAP, threads=cores)
+        oracle.sw_traceback_batch(a_cat, a_off, b_cat, b_off, sig, dpgen.SW_GAP, 513, threads=cores)
+        dt = time.perf_counter() - t
+        return k * 65536 / dt, f"first {k} pairs of config 2 (scores + canonical tracebacks)", cores
+    if config in ("nuss1",):
+        x = dpgen.config1_rna64()
+        reps = 200
+        t = time.perf_counter()
+        for _ in range(reps):
+            oracle.nussinov_traceback(x, dpgen.rna_pair_mask(), 3)
+        dt = time.perf_counter() - t
+        return reps * W["cells"] / dt, f"config 1 x{reps} repetitions (score + traceback), 1 core", 1
+    if config in ("nuss4", "nuss5"):
+        ids = dpgen.config5_sample_ids(k=2000 if config == "nuss5" else 200)
+        cat, off = dpgen.config5_rna_batch(ids=ids)
+        lens = np.diff(off)
+        t = time.perf_counter()
+        oracle.nussinov_batch(cat, off, dpgen.rna_pair_mask(), 3, threads=cores)
+        dt = time.perf_counter() - t
+        cells = int((lens * (lens - 1) // 2).sum())
+        return cells / dt, f"{len(ids)} sequences of the fixed config-5 subset (seed +7), scores only", cores
+    d = W["hmm"]
+    k = 200
+    seqs = d["seqs"][:k]
+    off = np.arange(k + 1, dtype=np.int64) * seqs.shape[1]
+    t = time.perf_counter()
+    oracle.forward_batch(seqs.reshape(-1), off, *(d[q].astype(np.float64) for q in ("pi", "A", "E")), threads=cores)
+    oracle.viterbi_batch(seqs.reshape(-1), off, d["lpi"], d["lA"], d["lE"], threads=cores)
+    dt = time.perf_counter() - t
+    return k * 64 * 1000 / dt, f"first {k} sequences of config 3 (forward + Viterbi)", cores
+
+
+def cpu_baseline(config, W):
+    v, sample, cores = oracle_sample(config, W, 20)
+    return {"value": round(v / 1e9, 6), "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": sample}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle as it stands on the host cores, bounded samples per step."""
+    if rank != 0:
+        return None
+    W = workload(args.config, 0, 1) if args.config != "nuss5" else {"cells": 0}
+    vals = []
+    sample = cores = None
+    for k in range(args.warmup + args.steps):
+        v, sample, cores = oracle_sample(args.config, W, 5)
+        if k >= args.warmup:
+            vals.append(v)
+    val = sum(vals) / len(vals)
+    return {
+        "impl": "reference",
+        "metric": "DP cell-updates/sec (GCUPS) at 1/2/4/8 B200 and fraction of roofline",
+        "value": round(val / 1e9, 6), "unit": "GCUPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "int64 (oracle)", "data": "synthetic (seeded, dpgen)",
+        "config": {"workload": workload(args.config, 0, 1)["workload"] if args.config != "nuss5" else "config 5",
+                   "config": args.config},
+        "cpu_baseline": {"value": round(val / 1e9, 6), "unit": "GCUPS", "cores": cores, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": round(val / 1e9, 6), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="sw", choices=["sw", "nuss1", "hmm", "nuss4", "nuss5"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    args = ap.parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        res = run_reference(args, rank, world)
+        if res is not None:
+            print(json.dumps(res), flush=True)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    res = run_ours(args, rank, world, local_rank)
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

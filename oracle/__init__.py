@@ -64,6 +64,8 @@ def lib():
         L.orc_viterbi.argtypes = [u8p, i64, ctypes.c_int, ctypes.c_int, i32p, i32p, i32p, u8p]
         L.orc_sw_batch.restype = None
         L.orc_sw_batch.argtypes = [i64, i64, u8p, i64p, u8p, i64p, i8p, ctypes.c_int, i64, i64p]
+        L.orc_sw_traceback_batch.restype = None
+        L.orc_sw_traceback_batch.argtypes = [i64, i64, u8p, i64p, u8p, i64p, i8p, ctypes.c_int, i64, u8p, i64, i64p]
         L.orc_nussinov_batch.restype = None
         L.orc_nussinov_batch.argtypes = [i64, i64, u8p, i64p, u8p, ctypes.c_int, i64p]
         L.orc_forward_batch.restype = None
@@ -168,6 +170,19 @@ def sw_batch(a_cat, a_off, b_cat, b_off, sigma, g, threads=1) -> np.ndarray:
     a_off, b_off = np.ascontiguousarray(a_off, np.int64), np.ascontiguousarray(b_off, np.int64)
     _parallel(n, lambda f, c: lib().orc_sw_batch(f, c, a_cat, a_off, b_cat, b_off, sig, sig.shape[0], int(g), out), threads)
     return out
+
+
+def sw_traceback_batch(a_cat, a_off, b_cat, b_off, sigma, g, stride, threads=1):
+    """Canonical tracebacks of a batch (ops, lengths); each problem's score is recomputed inside."""
+    n = len(a_off) - 1
+    ops = np.zeros((n, stride), dtype=np.uint8)
+    lens = np.zeros(n, dtype=np.int64)
+    sig = np.ascontiguousarray(sigma, dtype=np.int8)
+    a_cat, b_cat = _u8(a_cat), _u8(b_cat)
+    a_off, b_off = np.ascontiguousarray(a_off, np.int64), np.ascontiguousarray(b_off, np.int64)
+    _parallel(n, lambda f, c: lib().orc_sw_traceback_batch(f, c, a_cat, a_off, b_cat, b_off, sig, sig.shape[0],
+                                                           int(g), ops.reshape(-1), stride, lens), threads)
+    return ops, lens
 
 
 def nussinov_batch(x_cat, x_off, pair_mask, h, threads=1) -> np.ndarray:

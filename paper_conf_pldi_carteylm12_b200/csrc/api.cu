@@ -1,0 +1,470 @@
+// C ABI (include/dp.h): plan lifecycle, dispatch to the kernels, traceback,
+// host-buffer entry point. No exception crosses this boundary.
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <vector>
+#include <cuda_runtime.h>
+
+#include "dp.h"
+#include "dp_internal.h"
+
+namespace {
+
+struct DevBuf {
+  void* ptr = nullptr;
+  size_t bytes = 0;
+  cudaError_t ensure(size_t want) {
+    if (want <= bytes) return cudaSuccess;
+    if (ptr) cudaFree(ptr);
+    ptr = nullptr;
+    bytes = 0;
+    cudaError_t e = cudaMalloc(&ptr, want);
+    if (e == cudaSuccess) bytes = want;
+    return e;
+  }
+  void release() {
+    if (ptr) cudaFree(ptr);
+    ptr = nullptr;
+    bytes = 0;
+  }
+};
+
+}  // namespace
+
+struct dp_plan {
+  int kind = 0;
+  int device = 0;
+  int64_t max_la = 0, max_lb = 0;
+  int asz = 0, gap = 0, hairpin = 0, S = 0, K = 0;
+  bool want_tb = false;
+  int ndim = 2;
+  int32_t coeff[DP_MAX_DIM] = {0, 0, 0, 0};
+  int64_t p_lo = 0, p_hi = 0;
+  int64_t ext[2] = {1, 1};
+  int32_t window = -1;
+  // device parameters
+  int8_t* d_sigma = nullptr;
+  uint8_t* d_pair = nullptr;
+  float *d_pi = nullptr, *d_A = nullptr, *d_E = nullptr;
+  int32_t *d_lpi = nullptr, *d_lA = nullptr, *d_lE = nullptr;
+  // retained state of the most recent solve
+  DevBuf tb_state, tb_aux, tb_aux2, scratch;
+  int64_t last_n = -1;
+  int64_t last_max_la = 0, last_max_lb = 0;
+  const uint8_t *last_a = nullptr, *last_b = nullptr;
+  const int64_t *last_aoff = nullptr, *last_boff = nullptr;
+  int32_t* last_scores = nullptr;  // device (alignment traceback reads the score)
+  DevBuf own_scores;               // when the caller's scores are float/host we keep a copy
+  // host-API staging
+  DevBuf h_a, h_b, h_aoff, h_boff, h_scores, h_tb, h_tblen, h_coords;
+  int64_t launches = 0;
+};
+
+namespace {
+
+dp_status cuda_status(cudaError_t e) {
+  if (e == cudaSuccess) return DP_OK;
+  if (e == cudaErrorMemoryAllocation) return DP_E_NOMEM;
+  return DP_E_CUDA;
+}
+
+template <typename T>
+cudaError_t upload(T** dst, const T* src, size_t count) {
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(dst), count * sizeof(T));
+  if (e != cudaSuccess) return e;
+  return cudaMemcpy(*dst, src, count * sizeof(T), cudaMemcpyHostToDevice);
+}
+
+// Dependency families of each recurrence, in the index
+// order of its definition. Alignment: (i, j); Nussinov: (i, j); HMM: (s, i).
+int families(int kind, int64_t la, int64_t lb, int S, int64_t ext[2], int* triangular, dp_dep deps[8]) {
+  memset(deps, 0, sizeof(dp_dep) * 8);
+  for (int d = 0; d < 8; ++d) deps[d].ranged_axis = -1;
+  *triangular = 0;
+  switch (kind) {
+    case DP_EDIT:
+    case DP_SW_LINEAR:  // d(i-1,j), d(i,j-1), d(i-1,j-1)  (Fig.7; §6.1)
+      ext[0] = la + 1; ext[1] = lb + 1;
+      deps[0].offset[0] = -1;
+      deps[1].offset[1] = -1;
+      deps[2].offset[0] = -1; deps[2].offset[1] = -1;
+      return 3;
+    case DP_NUSSINOV: {  // gamma(i+1,j), gamma(i,j-1), gamma(i+1,j-1), gamma(i,k), gamma(k+1,j), i<k<j
+      const int64_t n = la > 1 ? la : 2;
+      ext[0] = n; ext[1] = n;
+      *triangular = 1;
+      deps[0].offset[0] = 1;
+      deps[1].offset[1] = -1;
+      deps[2].offset[0] = 1; deps[2].offset[1] = -1;
+      deps[3].ranged_axis = 1; deps[3].lo = -(n - 1); deps[3].hi = -1;  // (0, k - j)
+      deps[4].ranged_axis = 0; deps[4].lo = 1; deps[4].hi = n - 1;      // (k + 1 - i, 0)
+      return 5;
+    }
+    case DP_HMM_FORWARD:
+    case DP_HMM_VITERBI:  // F(t.start, i-1) for t in s.transitionsto: any state (§5.2)
+      ext[0] = S; ext[1] = la + 1;
+      deps[0].offset[1] = -1;
+      deps[0].ranged_axis = 0; deps[0].lo = -(S - 1); deps[0].hi = S - 1;
+      return 1;
+  }
+  return -1;
+}
+
+}  // namespace
+
+extern "C" {
+
+int dp_abi_version(void) { return DP_ABI_VERSION; }
+
+const char* dp_status_string(dp_status s) {
+  switch (s) {
+    case DP_OK: return "ok";
+    case DP_E_INVALID: return "invalid argument";
+    case DP_E_NO_SCHEDULE: return "no valid schedule (cyclic dependencies)";
+    case DP_E_UNSUPPORTED: return "unsupported";
+    case DP_E_TOO_LARGE: return "size exceeds plan maximum or device limit";
+    case DP_E_NOMEM: return "out of memory";
+    case DP_E_CUDA: return "CUDA error";
+    case DP_E_NO_TRACEBACK: return "no traceback retained";
+  }
+  return "unknown status";
+}
+
+void dp_plan_destroy(dp_plan_t p) {
+  if (!p) return;
+  int cur = 0;
+  cudaGetDevice(&cur);
+  cudaSetDevice(p->device);
+  cudaFree(p->d_sigma); cudaFree(p->d_pair);
+  cudaFree(p->d_pi); cudaFree(p->d_A); cudaFree(p->d_E);
+  cudaFree(p->d_lpi); cudaFree(p->d_lA); cudaFree(p->d_lE);
+  DevBuf* bufs[] = {&p->tb_state, &p->tb_aux, &p->tb_aux2, &p->scratch, &p->own_scores, &p->h_a, &p->h_b,
+                    &p->h_aoff, &p->h_boff, &p->h_scores, &p->h_tb, &p->h_tblen, &p->h_coords};
+  for (DevBuf* b : bufs) b->release();
+  cudaSetDevice(cur);
+  delete p;
+}
+
+dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
+  if (!d || !out) return DP_E_INVALID;
+  *out = nullptr;
+  if (d->struct_size != sizeof(dp_desc)) return DP_E_INVALID;
+  if (d->kind < DP_EDIT || d->kind > DP_HMM_VITERBI) return DP_E_INVALID;
+  if (d->max_len_a < 0 || d->max_len_b < 0) return DP_E_INVALID;
+  dp_plan* p = new (std::nothrow) dp_plan();
+  if (!p) return DP_E_NOMEM;
+  p->kind = d->kind;
+  p->max_la = d->max_len_a;
+  p->max_lb = d->max_len_b;
+  p->want_tb = d->want_traceback != 0;
+  cudaGetDevice(&p->device);
+  dp_status st = DP_OK;
+  cudaError_t e = cudaSuccess;
+  switch (d->kind) {
+    case DP_EDIT:
+      p->asz = d->alphabet_size > 0 ? d->alphabet_size : 32;
+      if (p->asz > 32) st = DP_E_UNSUPPORTED;
+      p->gap = 1;
+      if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) st = DP_E_TOO_LARGE;
+      break;
+    case DP_SW_LINEAR:
+      p->asz = d->alphabet_size;
+      if (!d->sigma || p->asz < 1 || d->gap <= 0) { st = DP_E_INVALID; break; }
+      if (p->asz > 32) { st = DP_E_UNSUPPORTED; break; }
+      p->gap = d->gap;
+      if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) { st = DP_E_TOO_LARGE; break; }
+      e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
+      break;
+    case DP_NUSSINOV:
+      if (!d->pair_mask || d->min_hairpin < 0) { st = DP_E_INVALID; break; }
+      if (d->max_len_a > 32767 * 2) { st = DP_E_TOO_LARGE; break; }
+      p->hairpin = d->min_hairpin;
+      e = upload(&p->d_pair, d->pair_mask, 16);
+      break;
+    case DP_HMM_FORWARD:
+    case DP_HMM_VITERBI:
+      p->S = d->n_states;
+      p->K = d->alphabet_size;
+      if (p->S < 1 || p->K < 1) { st = DP_E_INVALID; break; }
+      if (p->S > 64 || p->K > 16) { st = DP_E_UNSUPPORTED; break; }
+      if (d->kind == DP_HMM_FORWARD) {
+        if (!d->pi || !d->A || !d->E) { st = DP_E_INVALID; break; }
+        if (p->want_tb) { st = DP_E_UNSUPPORTED; break; }
+        e = upload(&p->d_pi, d->pi, p->S);
+        if (e == cudaSuccess) e = upload(&p->d_A, d->A, (size_t)p->S * p->S);
+        if (e == cudaSuccess) e = upload(&p->d_E, d->E, (size_t)p->S * p->K);
+      } else {
+        if (!d->lpi || !d->lA || !d->lE) { st = DP_E_INVALID; break; }
+        e = upload(&p->d_lpi, d->lpi, p->S);
+        if (e == cudaSuccess) e = upload(&p->d_lA, d->lA, (size_t)p->S * p->S);
+        if (e == cudaSuccess) e = upload(&p->d_lE, d->lE, (size_t)p->S * p->K);
+      }
+      break;
+  }
+  if (st == DP_OK && e != cudaSuccess) st = cuda_status(e);
+  if (st == DP_OK) {
+    // schedule (A1–A4): derive, or verify the user's
+    int tri = 0;
+    dp_dep deps[8];
+    int nd = families(d->kind, p->max_la, p->max_lb, p->S, p->ext, &tri, deps);
+    p->ndim = 2;
+    st = dp_schedule_derive(2, p->ext, tri, nd, deps, d->coeff_bound, d->user_coeff, p->coeff, &p->p_lo, &p->p_hi,
+                            &p->window);
+  }
+  if (st == DP_OK) {
+    // The kernels implement the derived schedule; a user schedule that is valid
+    // but differs would need another kernel (conditional schedules, §4.7: NEXT).
+    // Coefficients of a dimension of extent 1 do not change the partitions.
+    static const int32_t expect[5][2] = {{1, 1}, {1, 1}, {-1, 1}, {0, 1}, {0, 1}};
+    for (int i = 0; i < 2; ++i)
+      if (p->ext[i] > 1 && p->coeff[i] != expect[d->kind][i]) st = DP_E_UNSUPPORTED;
+  }
+  if (st != DP_OK) {
+    dp_plan_destroy(p);
+    return st;
+  }
+  *out = p;
+  return DP_OK;
+}
+
+dp_status dp_plan_get_schedule(dp_plan_t p, int32_t coeff[], int* ndim, int64_t* p_lo, int64_t* p_hi,
+                               int32_t* window) {
+  if (!p) return DP_E_INVALID;
+  if (coeff) for (int i = 0; i < p->ndim; ++i) coeff[i] = p->coeff[i];
+  if (ndim) *ndim = p->ndim;
+  if (p_lo) *p_lo = p->p_lo;
+  if (p_hi) *p_hi = p->p_hi;
+  if (window) *window = p->window;
+  return DP_OK;
+}
+
+int64_t dp_plan_launch_count(dp_plan_t p) { return p ? p->launches : -1; }
+
+dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int64_t* a_off, const uint8_t* b_cat,
+                         const int64_t* b_off, int64_t max_len_a, int64_t max_len_b, void* scores_out,
+                         void* stream) {
+  if (!p || n < 0) return DP_E_INVALID;
+  if (n > 0 && (!a_off || !scores_out)) return DP_E_INVALID;
+  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR;
+  if (align && n > 0 && !b_off) return DP_E_INVALID;
+  if (max_len_a < 0 || max_len_b < 0) return DP_E_INVALID;
+  if (max_len_a > p->max_la || (align && max_len_b > p->max_lb)) return DP_E_TOO_LARGE;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  int cur = 0;
+  cudaGetDevice(&cur);
+  if (cur != p->device) cudaSetDevice(p->device);
+  cudaError_t e = cudaSuccess;
+  p->last_n = n;
+  p->last_a = a_cat; p->last_b = b_cat; p->last_aoff = a_off; p->last_boff = b_off;
+  p->last_max_la = max_len_a; p->last_max_lb = max_len_b;
+  switch (p->kind) {
+    case DP_EDIT:
+    case DP_SW_LINEAR: {
+      dpk::AlignArgs A{};
+      A.n = n; A.a_cat = a_cat; A.b_cat = b_cat; A.a_off = a_off; A.b_off = b_off;
+      A.max_la = max_len_a > 0 ? max_len_a : 1; A.max_lb = max_len_b > 0 ? max_len_b : 1;
+      A.sigma = p->d_sigma; A.asz = p->asz; A.gap = p->gap; A.local = p->kind == DP_SW_LINEAR;
+      A.scores = static_cast<int32_t*>(scores_out);
+      if (p->want_tb) {
+        A.dir_stride = dpk::align_dir_words(A.max_la, A.max_lb);
+        e = p->tb_state.ensure((size_t)(n * A.dir_stride * 4 + 16));
+        if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 2 * 4 + 16));
+        if (e != cudaSuccess) break;
+        A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
+        A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
+        p->last_scores = A.scores;
+      }
+      e = dpk::align_solve(A, s, &p->launches);
+      break;
+    }
+    case DP_NUSSINOV: {
+      dpk::NussArgs A{};
+      A.n = n; A.x_cat = a_cat; A.x_off = a_off; A.max_len = max_len_a > 0 ? max_len_a : 1;
+      A.pair_mask = p->d_pair; A.hairpin = p->hairpin;
+      A.scores = static_cast<int32_t*>(scores_out);
+      if (p->want_tb) {
+        A.db_stride = A.max_len;
+        e = p->tb_state.ensure((size_t)(n * A.db_stride + 16));
+        if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 4 + 16));
+        if (e != cudaSuccess) break;
+        A.db = static_cast<uint8_t*>(p->tb_state.ptr);
+        A.db_len = static_cast<int32_t*>(p->tb_aux.ptr);
+      }
+      A.scratch_bytes = dpk::nuss_scratch_bytes(A.max_len, n, p->device);
+      e = p->scratch.ensure((size_t)A.scratch_bytes);
+      if (e != cudaSuccess) break;
+      A.scratch = p->scratch.ptr;
+      e = dpk::nuss_solve(A, s, &p->launches);
+      break;
+    }
+    case DP_HMM_FORWARD:
+    case DP_HMM_VITERBI: {
+      dpk::HmmArgs H{};
+      H.n = n; H.x_cat = a_cat; H.x_off = a_off; H.max_len = max_len_a; H.S = p->S; H.K = p->K;
+      if (p->kind == DP_HMM_FORWARD) {
+        H.pi = p->d_pi; H.A = p->d_A; H.E = p->d_E;
+        H.ll_out = static_cast<float*>(scores_out);
+        e = dpk::hmm_forward(H, s, &p->launches);
+      } else {
+        H.lpi = p->d_lpi; H.lA = p->d_lA; H.lE = p->d_lE;
+        H.vit_out = static_cast<int32_t*>(scores_out);
+        if (p->want_tb) {
+          e = p->tb_state.ensure((size_t)(n * (max_len_a > 0 ? max_len_a : 1) * 64 + 16));
+          if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 4 + 16));
+          if (e != cudaSuccess) break;
+          H.bp = static_cast<uint8_t*>(p->tb_state.ptr);
+          H.final_state = static_cast<int32_t*>(p->tb_aux.ptr);
+        }
+        e = dpk::hmm_viterbi(H, s, &p->launches);
+      }
+      break;
+    }
+  }
+  if (cur != p->device) cudaSetDevice(cur);
+  if (e != cudaSuccess) {
+    p->last_n = -1;
+    return cuda_status(e);
+  }
+  return DP_OK;
+}
+
+dp_status dp_solve(dp_plan_t p, const uint8_t* a, int64_t len_a, const uint8_t* b, int64_t len_b, void* score_out,
+                   void* stream) {
+  if (!p || len_a < 0 || len_b < 0) return DP_E_INVALID;
+  // offsets {0, len} live in plan workspace
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  cudaError_t e = p->tb_aux2.ensure(64);
+  if (e != cudaSuccess) return cuda_status(e);
+  int64_t off[4] = {0, len_a, 0, len_b};
+  e = cudaMemcpyAsync(p->tb_aux2.ptr, off, sizeof(off), cudaMemcpyHostToDevice, s);
+  if (e != cudaSuccess) return cuda_status(e);
+  const int64_t* d = static_cast<const int64_t*>(p->tb_aux2.ptr);
+  return dp_solve_batch(p, 1, a, d, b, d + 2, len_a, len_b, score_out, stream);
+}
+
+dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, int64_t stride, int32_t* out_len,
+                       int32_t* coords, void* stream) {
+  if (!p) return DP_E_INVALID;
+  if (p->kind == DP_HMM_FORWARD) return DP_E_UNSUPPORTED;
+  if (!p->want_tb || p->last_n < 0) return DP_E_NO_TRACEBACK;
+  if (first < 0 || count < 0 || first + count > p->last_n || stride < 0) return DP_E_INVALID;
+  if (count > 0 && (!out || !out_len)) return DP_E_INVALID;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaSuccess;
+  switch (p->kind) {
+    case DP_EDIT:
+    case DP_SW_LINEAR: {
+      if (stride < p->last_max_la + p->last_max_lb) return DP_E_TOO_LARGE;
+      dpk::AlignArgs A{};
+      A.n = p->last_n; A.a_cat = p->last_a; A.b_cat = p->last_b; A.a_off = p->last_aoff; A.b_off = p->last_boff;
+      A.max_la = p->last_max_la > 0 ? p->last_max_la : 1; A.max_lb = p->last_max_lb > 0 ? p->last_max_lb : 1;
+      A.sigma = p->d_sigma; A.asz = p->asz; A.gap = p->gap; A.local = p->kind == DP_SW_LINEAR;
+      A.scores = p->last_scores;
+      A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
+      A.dir_stride = dpk::align_dir_words(A.max_la, A.max_lb);
+      A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
+      e = dpk::align_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
+      break;
+    }
+    case DP_NUSSINOV: {
+      if (stride < p->last_max_la) return DP_E_TOO_LARGE;
+      const int64_t ds = p->last_max_la > 0 ? p->last_max_la : 1;
+      if (stride == ds) {
+        e = cudaMemcpyAsync(out, static_cast<uint8_t*>(p->tb_state.ptr) + first * ds, count * ds,
+                            cudaMemcpyDeviceToDevice, s);
+      } else {
+        e = cudaMemcpy2DAsync(out, stride, static_cast<uint8_t*>(p->tb_state.ptr) + first * ds, ds, ds, count,
+                              cudaMemcpyDeviceToDevice, s);
+      }
+      if (e == cudaSuccess)
+        e = cudaMemcpyAsync(out_len, static_cast<int32_t*>(p->tb_aux.ptr) + first, count * 4,
+                            cudaMemcpyDeviceToDevice, s);
+      break;
+    }
+    case DP_HMM_VITERBI: {
+      if (stride < p->last_max_la) return DP_E_TOO_LARGE;
+      dpk::HmmArgs H{};
+      H.n = p->last_n; H.x_cat = p->last_a; H.x_off = p->last_aoff; H.max_len = p->last_max_la; H.S = p->S;
+      H.K = p->K; H.bp = static_cast<uint8_t*>(p->tb_state.ptr); H.final_state = static_cast<int32_t*>(p->tb_aux.ptr);
+      e = dpk::hmm_viterbi_traceback(H, first, count, out, stride, out_len, s, &p->launches);
+      break;
+    }
+  }
+  return cuda_status(e);
+}
+
+dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int64_t* a_off,
+                              const uint8_t* b_cat, const int64_t* b_off, void* scores_out, uint8_t* tb_out,
+                              int64_t tb_stride, int32_t* tb_len, int32_t* tb_coords, void* stream) {
+  if (!p || n < 0 || (n > 0 && (!a_off || !a_cat || !scores_out))) return DP_E_INVALID;
+  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR;
+  if (align && n > 0 && (!b_off || !b_cat)) return DP_E_INVALID;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  int64_t max_la = 0, max_lb = 0;
+  for (int64_t q = 0; q < n; ++q) {
+    const int64_t la = a_off[q + 1] - a_off[q];
+    if (la < 0) return DP_E_INVALID;
+    if (la > max_la) max_la = la;
+    if (align) {
+      const int64_t lb = b_off[q + 1] - b_off[q];
+      if (lb < 0) return DP_E_INVALID;
+      if (lb > max_lb) max_lb = lb;
+    }
+  }
+  if (max_la > p->max_la || max_lb > p->max_lb) return DP_E_TOO_LARGE;
+  const int64_t abytes = n > 0 ? a_off[n] - a_off[0] : 0;
+  const int64_t bbytes = (align && n > 0) ? b_off[n] - b_off[0] : 0;
+  cudaError_t e = p->h_a.ensure((size_t)abytes + 16);
+  if (e == cudaSuccess) e = p->h_aoff.ensure((size_t)(n + 1) * 8);
+  if (e == cudaSuccess && align) e = p->h_b.ensure((size_t)bbytes + 16);
+  if (e == cudaSuccess && align) e = p->h_boff.ensure((size_t)(n + 1) * 8);
+  if (e == cudaSuccess) e = p->h_scores.ensure((size_t)n * 4 + 16);
+  if (e != cudaSuccess) return cuda_status(e);
+  // offsets are rebased to 0 when a_off[0] != 0
+  std::vector<int64_t> ao, bo;
+  const int64_t* aoff_h = a_off;
+  const int64_t* boff_h = b_off;
+  if (n > 0 && a_off[0] != 0) {
+    ao.resize(n + 1);
+    for (int64_t q = 0; q <= n; ++q) ao[q] = a_off[q] - a_off[0];
+    aoff_h = ao.data();
+  }
+  if (align && n > 0 && b_off[0] != 0) {
+    bo.resize(n + 1);
+    for (int64_t q = 0; q <= n; ++q) bo[q] = b_off[q] - b_off[0];
+    boff_h = bo.data();
+  }
+  if (n > 0) {
+    e = cudaMemcpyAsync(p->h_a.ptr, a_cat + a_off[0], abytes, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(p->h_aoff.ptr, aoff_h, (n + 1) * 8, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess && align) e = cudaMemcpyAsync(p->h_b.ptr, b_cat + b_off[0], bbytes, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess && align) e = cudaMemcpyAsync(p->h_boff.ptr, boff_h, (n + 1) * 8, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_status(e);
+  }
+  dp_status st = dp_solve_batch(p, n, static_cast<uint8_t*>(p->h_a.ptr), static_cast<int64_t*>(p->h_aoff.ptr),
+                                align ? static_cast<uint8_t*>(p->h_b.ptr) : nullptr,
+                                align ? static_cast<int64_t*>(p->h_boff.ptr) : nullptr, max_la, max_lb,
+                                p->h_scores.ptr, stream);
+  if (st != DP_OK) return st;
+  if (n > 0) e = cudaMemcpyAsync(scores_out, p->h_scores.ptr, n * 4, cudaMemcpyDeviceToHost, s);
+  if (e != cudaSuccess) return cuda_status(e);
+  if (p->want_tb && tb_out && tb_len && p->kind != DP_HMM_FORWARD && n > 0) {
+    e = p->h_tb.ensure((size_t)(n * tb_stride) + 16);
+    if (e == cudaSuccess) e = p->h_tblen.ensure((size_t)n * 4 + 16);
+    if (e == cudaSuccess && tb_coords) e = p->h_coords.ensure((size_t)n * 16 + 16);
+    if (e != cudaSuccess) return cuda_status(e);
+    st = dp_traceback(p, 0, n, static_cast<uint8_t*>(p->h_tb.ptr), tb_stride, static_cast<int32_t*>(p->h_tblen.ptr),
+                      tb_coords ? static_cast<int32_t*>(p->h_coords.ptr) : nullptr, stream);
+    if (st != DP_OK) return st;
+    e = cudaMemcpyAsync(tb_out, p->h_tb.ptr, n * tb_stride, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(tb_len, p->h_tblen.ptr, n * 4, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && tb_coords)
+      e = cudaMemcpyAsync(tb_coords, p->h_coords.ptr, n * 16, cudaMemcpyDeviceToHost, s);
+    if (e != cudaSuccess) return cuda_status(e);
+  }
+  return cuda_status(cudaStreamSynchronize(s));
+}
+
+}  // extern "C"

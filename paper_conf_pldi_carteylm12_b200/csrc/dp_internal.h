@@ -1,0 +1,69 @@
+// Internal launcher interface between the C-ABI layer (api.cu) and the
+// kernels (align.cu, nussinov.cu, hmm.cu). Not installed; not part of dp.h.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace dpk {
+
+constexpr int kWarps = 8;  // warps per CTA for the warp-per-problem kernels
+
+// ---------------------------------------------------------------- alignment
+struct AlignArgs {
+  int64_t n;
+  const uint8_t *a_cat, *b_cat;
+  const int64_t *a_off, *b_off;
+  int64_t max_la, max_lb;
+  const int8_t* sigma;   // device [asz x asz] (SW) or nullptr (edit)
+  int asz;
+  int gap;
+  bool local;            // SW (true) vs edit distance (false)
+  int32_t* scores;
+  // traceback retention (nullptr when not wanted)
+  uint32_t* dirs;        // direction codes, 2 bits per cell
+  int64_t dir_stride;    // words per problem
+  int32_t* ends;         // n x 2 (end_i, end_j)
+};
+int64_t align_dir_words(int64_t max_la, int64_t max_lb);  // words per problem for `dirs`
+cudaError_t align_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
+cudaError_t align_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
+                            int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
+
+// ---------------------------------------------------------------- Nussinov
+struct NussArgs {
+  int64_t n;
+  const uint8_t* x_cat;
+  const int64_t* x_off;
+  int64_t max_len;
+  const uint8_t* pair_mask;  // device [16]
+  int hairpin;
+  int32_t* scores;
+  uint8_t* db;               // dot-brackets (n x db_stride) or nullptr
+  int64_t db_stride;
+  int32_t* db_len;
+  void* scratch;             // global table scratch for large n
+  int64_t scratch_bytes;
+};
+int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device);
+cudaError_t nuss_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
+
+// ---------------------------------------------------------------- HMM
+struct HmmArgs {
+  int64_t n;
+  const uint8_t* x_cat;
+  const int64_t* x_off;
+  int64_t max_len;
+  int S, K;
+  const float *pi, *A, *E;          // device, forward
+  const int32_t *lpi, *lA, *lE;     // device, Viterbi
+  float* ll_out;                    // forward
+  int32_t* vit_out;                 // Viterbi
+  uint8_t* bp;                      // Viterbi back-pointers (n x max_len x 64) or nullptr
+  int32_t* final_state;             // n
+};
+cudaError_t hmm_forward(const HmmArgs& a, cudaStream_t s, int64_t* launches);
+cudaError_t hmm_viterbi(const HmmArgs& a, cudaStream_t s, int64_t* launches);
+cudaError_t hmm_viterbi_traceback(const HmmArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
+                                  int32_t* out_len, cudaStream_t s, int64_t* launches);
+
+}  // namespace dpk

@@ -1,0 +1,237 @@
+// Nussinov interval DP on the hyperplanes of the derived schedule
+// S(i,j) = -i + j (partition d = j - i):
+//   gamma(i,j) = max{ gamma(i+1,j), gamma(i,j-1), gamma(i+1,j-1) + 1 [pair, j-i-1 >= h],
+//                     max_{i<k<j} gamma(i,k) + gamma(k+1,j) }.
+// The recurrence is not in PAPER.md (RNA folding is Further Work, L585–L589);
+// the definition follows the paper's ref [3] (DESIGN.md R-NUSS).
+//
+// Table layout (int16, scores <= n/2): two triangular copies so that both
+// operand streams of a split term are contiguous in k:
+//   U[i][k] = gamma(i, k),   k = i .. n-1      (row i)
+//   L[j][k] = gamma(k+1, j), k = 0 .. j-1      (row j)
+// split(i,j) = max_k U[i][k] + L[j][k] over i < k < j.
+// Cells of one partition are independent (eq.2), so a partition is computed
+// by all threads of the CTA (or grid) and closed by one barrier (Fig.8).
+// Each cell is reduced by a power-of-two group of lanes (k strided over the
+// group, then __shfl_xor_sync), sized to the partition's cell count.
+#include <algorithm>
+#include <cstdint>
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+
+#include "dp_internal.h"
+
+namespace cg = cooperative_groups;
+
+namespace dpk {
+namespace {
+
+constexpr int kNussThreads = 512;
+constexpr int64_t kSmemMaxN = 340;  // 2 n^2 bytes of int16 table <= 227 KiB
+
+__host__ __device__ __forceinline__ int64_t ustart(int64_t i, int64_t n) { return i * n - (i * (i - 1)) / 2; }
+__host__ __device__ __forceinline__ int64_t lstart(int64_t j) { return (j * (j - 1)) / 2; }
+// n(n+1)/2 (U) + n(n-1)/2 (L), rounded to 8 elements so what follows stays 16-byte aligned
+__host__ __device__ __forceinline__ int64_t table_elems(int64_t n) { return (n * n + 7) & ~int64_t(7); }
+
+// Evaluate the cells of partition d assigned to this thread. `tid`/`nthr`
+// span the CTA (or the whole grid).
+__device__ __forceinline__ void nuss_partition(int16_t* U, int16_t* L, const uint8_t* x, int n, int d,
+                                               const uint8_t* pm, int h, int64_t tid, int64_t nthr) {
+  const int ncells = n - d;
+  // group size G: power of two <= 32, about nthr / ncells lanes per cell, no more than the split count
+  int G = 1;
+  while (G < 32 && (int64_t)G * 2 * ncells <= nthr && G * 2 <= max(1, d - 1)) G *= 2;
+  const int64_t ngroups = nthr / G;
+  const int q = (int)(tid % G);
+  const int64_t grp = tid / G;
+  // every group runs the same number of iterations so the shuffles stay converged
+  const int64_t iters = (ncells + ngroups - 1) / ngroups;
+  for (int64_t it = 0; it < iters; ++it) {
+    const int64_t cidx = grp + it * ngroups;
+    const bool live = cidx < ncells && grp < ngroups;
+    const int i = live ? (int)cidx : 0;
+    const int j = i + d;
+    int best = 0;
+    if (live) {
+      const int16_t* Ui = U + ustart(i, n);
+      const int16_t* Lj = L + lstart(j);
+      for (int k = i + 1 + q; k < j; k += G) best = max(best, (int)Ui[k - i] + (int)Lj[k]);
+    }
+    const unsigned mask = 0xffffffffu;
+    if (G > 1) {
+      for (int o = G / 2; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(mask, best, o, G));
+    }
+    if (live && q == 0) {
+      const int16_t* Ui = U + ustart(i, n);
+      const int16_t* Ui1 = U + ustart(i + 1, n);
+      int v = best;
+      v = max(v, (int)Ui1[j - (i + 1)]);               // gamma(i+1, j)
+      v = max(v, (int)Ui[j - 1 - i]);                  // gamma(i, j-1)
+      if (pm[x[i] * 4 + x[j]] && d - 1 >= h) {
+        const int inner = (d >= 2) ? (int)Ui1[j - 1 - (i + 1)] : 0;  // gamma(i+1, j-1), empty -> 0
+        v = max(v, inner + 1);
+      }
+      U[ustart(i, n) + d] = (int16_t)v;
+      if (i >= 1) L[lstart(j) + (i - 1)] = (int16_t)v;
+    }
+  }
+}
+
+__device__ void nuss_init(int16_t* U, int16_t* L, int n, int64_t tid, int64_t nthr) {
+  // diagonal d = 0: gamma(i,i) = 0 in U; L[j][j-1] = gamma(j,j) = 0
+  for (int64_t i = tid; i < n; i += nthr) {
+    U[ustart(i, n)] = 0;
+    if (i >= 1) L[lstart(i) + i - 1] = 0;
+  }
+}
+
+// Canonical traceback (DESIGN.md R-TB-NUSS): Durbin order, smallest split k.
+// One thread; explicit stack in global scratch.
+__device__ void nuss_traceback(const int16_t* U, const int16_t* L, const uint8_t* x, int n, const uint8_t* pm, int h,
+                               uint8_t* db, int* stack) {
+  for (int k = 0; k < n; ++k) db[k] = '.';
+  if (n <= 1) return;
+  auto gam = [&](int i, int j) -> int { return (j - i < 1) ? 0 : (int)U[ustart(i, n) + (j - i)]; };
+  int sp = 0;
+  stack[sp++] = 0; stack[sp++] = n - 1;
+  while (sp > 0) {
+    const int j = stack[--sp], i = stack[--sp];
+    if (j - i < 1) continue;
+    const int v = gam(i, j);
+    if (v == gam(i + 1, j)) { stack[sp++] = i + 1; stack[sp++] = j; continue; }
+    if (v == gam(i, j - 1)) { stack[sp++] = i; stack[sp++] = j - 1; continue; }
+    if (pm[x[i] * 4 + x[j]] && j - i - 1 >= h && v == gam(i + 1, j - 1) + 1) {
+      db[i] = '('; db[j] = ')';
+      stack[sp++] = i + 1; stack[sp++] = j - 1;
+      continue;
+    }
+    const int16_t* Ui = U + ustart(i, n);
+    const int16_t* Lj = L + lstart(j);
+    for (int k = i + 1; k < j; ++k)
+      if (v == (int)Ui[k - i] + (int)Lj[k]) {
+        stack[sp++] = k + 1; stack[sp++] = j;
+        stack[sp++] = i; stack[sp++] = k;
+        break;
+      }
+  }
+}
+
+// One CTA per problem (persistent over the batch). The table lives in shared
+// memory when it fits (SMEM=true) or in this CTA's slice of a global scratch
+// that stays L2-resident (SMEM=false).
+template <bool SMEM>
+__global__ void __launch_bounds__(kNussThreads) k_nuss_cta(NussArgs A, int64_t slice_elems) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  __shared__ uint8_t pm[16];
+  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
+  uint8_t* xs = smem;  // sequence bytes
+  int16_t* tab;
+  if (SMEM) tab = reinterpret_cast<int16_t*>(smem + ((A.max_len + 15) & ~15));
+  else tab = reinterpret_cast<int16_t*>(A.scratch) + (int64_t)blockIdx.x * slice_elems;
+  int* stack = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * (SMEM ? 0 : slice_elems)) +
+               (int64_t)blockIdx.x * (4 * A.max_len + 8);
+  for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
+    const uint8_t* xg = A.x_cat + A.x_off[p];
+    const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+    __syncthreads();
+    for (int q = threadIdx.x; q < n; q += blockDim.x) xs[q] = xg[q];
+    int16_t* U = tab;
+    int16_t* L = tab + (int64_t)n * (n + 1) / 2;
+    nuss_init(U, L, n, threadIdx.x, blockDim.x);
+    __syncthreads();
+    for (int d = 1; d < n; ++d) {
+      nuss_partition(U, L, xs, n, d, pm, A.hairpin, threadIdx.x, blockDim.x);
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+      A.scores[p] = n <= 1 ? 0 : (int)U[ustart(0, n) + n - 1];
+      if (A.db) {
+        nuss_traceback(U, L, xs, n, pm, A.hairpin, A.db + p * A.db_stride, stack);
+        A.db_len[p] = n;
+      }
+    }
+  }
+}
+
+// One problem over the whole grid: partitions separated by grid-wide barriers
+// (cooperative launch), the table in global memory (L2-resident).
+__global__ void __launch_bounds__(kNussThreads) k_nuss_grid(NussArgs A, int64_t p) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ uint8_t pm[16];
+  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
+  __syncthreads();
+  const uint8_t* x = A.x_cat + A.x_off[p];
+  const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+  int16_t* U = reinterpret_cast<int16_t*>(A.scratch);
+  int16_t* L = U + (int64_t)n * (n + 1) / 2;
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+  nuss_init(U, L, n, tid, nthr);
+  grid.sync();
+  for (int d = 1; d < n; ++d) {
+    nuss_partition(U, L, x, n, d, pm, A.hairpin, tid, nthr);
+    grid.sync();
+  }
+  if (tid == 0) {
+    A.scores[p] = n <= 1 ? 0 : (int)U[ustart(0, n) + n - 1];
+    if (A.db) {
+      int* stack = reinterpret_cast<int*>(U + table_elems(n));
+      nuss_traceback(U, L, x, n, pm, A.hairpin, A.db + p * A.db_stride, stack);
+      A.db_len[p] = n;
+    }
+  }
+}
+
+int num_sms(int device) {
+  int v = 0;
+  cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device);
+  return v > 0 ? v : 148;
+}
+
+}  // namespace
+
+int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device) {
+  const int64_t stack_bytes = (4 * max_len + 8) * 4;
+  if (max_len <= kSmemMaxN) {
+    const int64_t grid = std::min<int64_t>(n, (int64_t)num_sms(device) * 4);
+    return grid * stack_bytes + 256;
+  }
+  if (n == 1) return table_elems(max_len) * 2 + stack_bytes + 256;
+  const int64_t grid = std::min<int64_t>(n, (int64_t)num_sms(device) * 2);
+  return grid * (table_elems(max_len) * 2 + stack_bytes) + 256;
+}
+
+cudaError_t nuss_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
+  if (A.n == 0) return cudaSuccess;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const int sms = num_sms(dev);
+  if (A.max_len <= kSmemMaxN) {
+    const size_t smem = ((A.max_len + 15) & ~15) + (size_t)table_elems(A.max_len) * 2;
+    cudaError_t e = cudaFuncSetAttribute(k_nuss_cta<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const int64_t grid = std::min<int64_t>(A.n, (int64_t)sms * 4);
+    ++*launches;
+    k_nuss_cta<true><<<(unsigned)grid, kNussThreads, smem, s>>>(A, 0);
+    return cudaGetLastError();
+  }
+  if (A.n == 1) {
+    int per_sm = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_nuss_grid, kNussThreads, 0);
+    if (e != cudaSuccess) return e;
+    const int grid = sms * std::max(1, std::min(per_sm, 2));
+    int64_t p = 0;
+    NussArgs a2 = A;
+    void* args[2] = {&a2, &p};
+    ++*launches;
+    return cudaLaunchCooperativeKernel((void*)k_nuss_grid, grid, kNussThreads, args, 0, s);
+  }
+  const size_t smem = ((A.max_len + 15) & ~15);
+  const int64_t grid = std::min<int64_t>(A.n, (int64_t)sms * 2);
+  ++*launches;
+  k_nuss_cta<false><<<(unsigned)grid, kNussThreads, smem, s>>>(A, table_elems(A.max_len));
+  return cudaGetLastError();
+}
+
+}  // namespace dpk

@@ -1,0 +1,131 @@
+"""Host-side tests of the product (no GPU): the C-ABI library loads and exports
+every symbol include/dp.h declares, and its symbolic schedule front-end
+(dp_schedule_derive) agrees with the brute-force schedule oracle on explicit
+call graphs and with the paper's worked examples."""
+import json
+import os
+import re
+
+import pytest
+
+from oracle import schedule as sch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+GOLD = json.load(open(os.path.join(ROOT, "tests", "golden", "schedule_pins.json")))
+
+
+@pytest.fixture(scope="module")
+def dp():
+    from paper_conf_pldi_carteylm12_b200 import _build
+    _build.build()
+    import paper_conf_pldi_carteylm12_b200 as dp
+    dp.lib()
+    return dp
+
+
+def test_exports_match_header(dp):
+    hdr = open(os.path.join(ROOT, "include", "dp.h")).read()
+    declared = set(re.findall(r"\b(dp_[a-z_]+)\s*\(", hdr))
+    assert declared == set(dp.EXPORTS)
+    L = dp.lib()
+    for name in declared:
+        assert hasattr(L, name), name
+    assert L.dp_abi_version() == 1
+    for code in range(8):
+        assert L.dp_status_string(code)
+
+
+def U(*off):
+    return (off, None, 0, 0)
+
+
+def test_edit_and_sw_schedule(dp):
+    for n, m in [(2, 2), (256, 256), (5, 9)]:
+        r = dp.schedule_derive((n + 1, m + 1), [U(-1, 0), U(0, -1), U(-1, -1)])
+        assert list(r["a"]) == GOLD["edit_schedule"]["a"]
+        assert (r["p_lo"], r["p_hi"]) == (0, n + m)
+        assert r["window"] == 2
+        dom, calls, ext = sch.edit_instance(min(n, 5), min(m, 5))
+        o = sch.derive(dom, calls, ext)
+        assert o["a"] == r["a"]
+    assert dp.schedule_derive((3, 3), [U(-1, 0), U(0, -1), U(-1, -1)])["p_hi"] + 1 == 5   # Fig.3
+
+
+def test_user_schedule_verification(dp):
+    deps = [U(-1, 0), U(0, -1), U(-1, -1)]
+    r = dp.schedule_derive((5, 5), deps, user_coeff=(2, 1))          # valid, more partitions (L168-L170)
+    assert r["a"] == (2, 1) and r["p_hi"] == 12
+    with pytest.raises(dp.DPError) as e:
+        dp.schedule_derive((5, 5), deps, user_coeff=(1, -1))
+    assert e.value.code == 2
+
+
+@pytest.mark.parametrize("nx,ny", [(3, 5), (5, 3), (4, 4), (7, 2)])
+def test_diagonal_only_matches_oracle(dp, nx, ny):
+    r = dp.schedule_derive((nx, ny), [U(-1, -1)])
+    dom, calls, ext = sch.diagonal_instance(nx, ny)
+    assert r["a"] == sch.derive(dom, calls, ext)["a"]
+    want = GOLD["diagonal_only"]["nx_lt_ny"] if nx < ny else GOLD["diagonal_only"]["nx_gt_ny"]
+    assert list(r["a"]) == want
+
+
+@pytest.mark.parametrize("n", [3, 6, 64, 8192])
+def test_nussinov_schedule(dp, n):
+    deps = [U(1, 0), U(0, -1), U(1, -1), ((0, 0), 1, -(n - 1), -1), ((0, 0), 0, 1, n - 1)]
+    r = dp.schedule_derive((n, n), deps, triangular=True)
+    assert r["a"] == (-1, 1)
+    assert (r["p_lo"], r["p_hi"]) == (0, n - 1)     # n partitions over the triangle
+    assert r["window"] == -1                        # ranged descent: no sliding window (§4.8)
+    if n <= 6:
+        dom, calls, ext = sch.nussinov_instance(n)
+        o = sch.derive(dom, calls, ext)
+        assert o["a"] == r["a"] and (o["p_lo"], o["p_hi"]) == (r["p_lo"], r["p_hi"])
+
+
+@pytest.mark.parametrize("S,T", [(4, 5), (64, 1000)])
+def test_hmm_schedule(dp, S, T):
+    r = dp.schedule_derive((S, T + 1), [((0, -1), 0, -(S - 1), S - 1)])
+    assert list(r["a"]) == GOLD["hmm_forward"]["a"]
+    assert r["window"] == 1 and (r["p_lo"], r["p_hi"]) == (0, T)
+    if S * T < 40:
+        dom, calls, ext = sch.hmm_instance(S, T)
+        assert sch.derive(dom, calls, ext)["a"] == r["a"]
+
+
+def test_fibonacci_and_cyclic(dp):
+    r = dp.schedule_derive((9,), [U(-1), U(-2)])
+    assert r["a"] == (1,) and r["window"] == 2
+    with pytest.raises(dp.DPError) as e:
+        dp.schedule_derive((5,), [U(-1), U(1)])
+    assert e.value.code == 2
+
+
+def test_random_families_match_bruteforce(dp):
+    """Random uniform dependency sets in 2-D: symbolic criteria == explicit call graph."""
+    import random
+    rnd = random.Random(7)
+    for _ in range(40):
+        deps = set()
+        while len(deps) < rnd.randint(1, 3):
+            d = (rnd.randint(-2, 1), rnd.randint(-2, 1))
+            if d != (0, 0):
+                deps.add(d)
+        nx, ny = rnd.randint(2, 5), rnd.randint(2, 5)
+        dom = [(x, y) for x in range(nx) for y in range(ny)]
+        calls = lambda c, deps=tuple(deps): [(c[0] + a, c[1] + b) for a, b in deps]
+        o = sch.derive(dom, calls, (nx, ny))
+        # the call graph only contains in-domain edges; keep cases where every family has an edge
+        if any(not any((x + a, y + b) in set(dom) for x, y in dom) for a, b in deps):
+            continue
+        try:
+            r = dp.schedule_derive((nx, ny), [U(a, b) for a, b in deps])
+        except dp.DPError as e:
+            assert e.code == 2 and o is None
+            continue
+        assert o is not None and r["a"] == o["a"], (deps, nx, ny, r, o)
+
+
+def test_bad_arguments(dp):
+    with pytest.raises(dp.DPError) as e:
+        dp.schedule_derive((0, 3), [U(-1, 0)])
+    assert e.value.code == 1

@@ -1,0 +1,309 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by
+element on seeded inputs. Integer scores and tracebacks bit-exact; forward
+log-likelihoods within relative 1e-5 (north_star)."""
+import os
+
+import numpy as np
+import pytest
+
+import dpgen
+
+pytestmark = pytest.mark.gpu
+THREADS = os.cpu_count() or 4
+
+
+@pytest.fixture(scope="module")
+def dp():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_pldi_carteylm12_b200 import _build
+    _build.build()
+    import paper_conf_pldi_carteylm12_b200 as dp
+    return dp
+
+
+def cuda(x):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(x)).cuda()
+
+
+def host(t):
+    return t.cpu().numpy()
+
+
+def rand_batch(g, n, lo, hi, k):
+    seqs = [g.integers(0, k, size=int(g.integers(lo, hi + 1))).astype(np.uint8) for _ in range(n)]
+    return seqs, dpgen.pack(seqs)
+
+
+# ----------------------------------------------------------------------------- alignment
+def run_align(dp, kind, a_seqs, b_seqs, sigma=None, gap=0, asz=26, tb=True):
+    a_cat, a_off = dpgen.pack(a_seqs)
+    b_cat, b_off = dpgen.pack(b_seqs)
+    la = max((len(s) for s in a_seqs), default=0)
+    lb = max((len(s) for s in b_seqs), default=0)
+    plan = dp.Plan(kind, max(la, 1), max(lb, 1), sigma=sigma, gap=gap, alphabet_size=asz, want_traceback=tb)
+    A = (cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off))
+    sc = plan.solve_batch(*A, max_len_a=la, max_len_b=lb)
+    res = {"scores": host(sc)}
+    if tb:
+        out, ln, co = plan.traceback(0, len(a_seqs), la + lb + 1)
+        res["ops"] = [bytes(host(out[q, :int(l)])).decode() for q, l in enumerate(host(ln))]
+        res["coords"] = host(co)
+    plan.close()
+    return res
+
+
+def test_edit_random_ragged(dp, orc):
+    g = np.random.default_rng(100)
+    a, _ = rand_batch(g, 300, 0, 150, 26)
+    b, _ = rand_batch(g, 300, 0, 150, 26)
+    a += [np.zeros(0, np.uint8), dpgen.encode("kitten", dpgen.EN)]
+    b += [dpgen.encode("abc", dpgen.EN), dpgen.encode("sitting", dpgen.EN)]
+    r = run_align(dp, dp.EDIT, a, b)
+    for q in range(len(a)):
+        assert r["scores"][q] == orc.edit(a[q], b[q]), q
+        assert r["ops"][q] == orc.edit_traceback(a[q], b[q]), q
+
+
+@pytest.mark.parametrize("maxlen", [40, 300, 700])
+def test_sw_random_ragged(dp, orc, maxlen):
+    """Lengths span several lane tiles, strips (> 256 rows) and ragged tails."""
+    g = np.random.default_rng(101 + maxlen)
+    sig = dpgen.blosum62()
+    n = 200
+    a, _ = rand_batch(g, n, 0, maxlen, 24)
+    b, _ = rand_batch(g, n, 0, maxlen, 24)
+    r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24)
+    for q in range(n):
+        sc, ei, ej = orc.sw(a[q], b[q], sig, 4)
+        assert r["scores"][q] == sc, q
+        if q % 4 == 0:
+            ops, co = orc.sw_traceback(a[q], b[q], sig, 4)
+            assert r["ops"][q] == ops, q
+            assert tuple(r["coords"][q]) == co, q
+
+
+def test_sw_score_only_matches_traceback_mode(dp):
+    g = np.random.default_rng(102)
+    sig = dpgen.blosum62()
+    a, _ = rand_batch(g, 64, 1, 256, 20)
+    b, _ = rand_batch(g, 64, 1, 256, 20)
+    r1 = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24, tb=False)
+    r2 = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24, tb=True)
+    assert (r1["scores"] == r2["scores"]).all()
+
+
+def test_sw_config2_full_size_sampled(dp, orc):
+    """BASELINE config 2 at full size (100k x 256, the bench launch), sampled against the oracle."""
+    a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs()
+    sig = dpgen.blosum62()
+    plan = dp.Plan(dp.SW_LINEAR, 256, 256, sigma=sig, gap=dpgen.SW_GAP, want_traceback=True)
+    A = (cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off))
+    sc = host(plan.solve_batch(*A, max_len_a=256, max_len_b=256))
+    n = len(a_off) - 1
+    ids = np.random.default_rng(103).choice(n, size=150, replace=False)
+    ids = np.concatenate([ids, [0, n - 1]])
+    out, ln, co = plan.traceback(0, n, 513)
+    out, ln, co = host(out), host(ln), host(co)
+    for q in ids:
+        s, t = a_cat[a_off[q]:a_off[q + 1]], b_cat[b_off[q]:b_off[q + 1]]
+        assert sc[q] == orc.sw(s, t, sig, dpgen.SW_GAP)[0]
+        ops, c = orc.sw_traceback(s, t, sig, dpgen.SW_GAP)
+        assert bytes(out[q, :ln[q]]).decode() == ops
+        assert tuple(co[q]) == c
+    assert sc.min() >= 0 and sc.max() <= 11 * 256
+    plan.close()
+
+
+def test_align_degenerate(dp, orc):
+    sig = dpgen.blosum62()
+    e = np.zeros(0, np.uint8)
+    x = dpgen.encode("ARND", dpgen.PROTEIN)
+    r = run_align(dp, dp.SW_LINEAR, [e, x, e], [x, e, e], sigma=sig, gap=4, asz=24)
+    assert list(r["scores"]) == [0, 0, 0] and r["ops"] == ["", "", ""]
+    r = run_align(dp, dp.EDIT, [e, x, e], [x, e, e], asz=24)
+    assert list(r["scores"]) == [4, 4, 0]
+    assert r["ops"] == ["IIII", "DDDD", ""]
+
+
+# ----------------------------------------------------------------------------- Nussinov
+def run_nuss(dp, seqs, h=3, pm=None, tb=True):
+    pm = dpgen.rna_pair_mask() if pm is None else pm
+    cat, off = dpgen.pack(seqs)
+    ml = max((len(s) for s in seqs), default=1)
+    plan = dp.Plan(dp.NUSSINOV, max(ml, 1), pair_mask=pm, min_hairpin=h, want_traceback=tb)
+    sc = host(plan.solve_batch(cuda(cat), cuda(off), max_len_a=ml))
+    res = {"scores": sc}
+    if tb:
+        out, ln, _ = plan.traceback(0, len(seqs), max(ml, 1), coords=False)
+        res["db"] = [bytes(host(out[q, :int(l)])).decode() for q, l in enumerate(host(ln))]
+    plan.close()
+    return res
+
+
+def test_nussinov_config1(dp, orc):
+    x = dpgen.config1_rna64()
+    r = run_nuss(dp, [x])
+    assert r["scores"][0] == orc.nussinov(x, dpgen.rna_pair_mask(), 3)
+    assert r["db"][0] == orc.nussinov_traceback(x, dpgen.rna_pair_mask(), 3)[1]
+
+
+@pytest.mark.parametrize("h", [0, 3])
+def test_nussinov_random_smem(dp, orc, h):
+    g = np.random.default_rng(110 + h)
+    seqs, _ = rand_batch(g, 120, 0, 200, 4)
+    seqs += [dpgen.encode("GGGGAAAACCCC", dpgen.RNA), dpgen.encode("A" * 50, dpgen.RNA)]
+    pm = dpgen.rna_pair_mask(gu=(h == 3))
+    r = run_nuss(dp, seqs, h=h, pm=pm)
+    for q, x in enumerate(seqs):
+        sc, db = orc.nussinov_traceback(x, pm, h)
+        assert r["scores"][q] == sc, q
+        assert r["db"][q] == db, q
+
+
+def test_nussinov_global_scratch_path(dp, orc):
+    """Lengths above the shared-memory limit use the L2-resident table."""
+    g = np.random.default_rng(112)
+    seqs, _ = rand_batch(g, 6, 341, 512, 4)
+    r = run_nuss(dp, seqs)
+    pm = dpgen.rna_pair_mask()
+    for q, x in enumerate(seqs):
+        sc, db = orc.nussinov_traceback(x, pm, 3)
+        assert r["scores"][q] == sc and r["db"][q] == db, q
+
+
+def test_nussinov_grid_sweep(dp, orc):
+    """A single large table swept by the whole grid (config 4's path) at n = 1500."""
+    x = dpgen.random_seq(dpgen.rng(5, extra=9), 1500, 4)
+    r = run_nuss(dp, [x])
+    sc, db = orc.nussinov_traceback(x, dpgen.rna_pair_mask(), 3)
+    assert r["scores"][0] == sc and r["db"][0] == db
+
+
+def test_nussinov_config4_properties(dp):
+    """n = 8192 (oracle ~20+ min): the structure is valid and has score-many pairs."""
+    from tests import brute
+    x = dpgen.config4_rna8192()
+    r = run_nuss(dp, [x])
+    pairs = brute.dotbracket_pairs(r["db"][0])
+    pm = dpgen.rna_pair_mask()
+    assert len(pairs) == r["scores"][0]
+    assert all(pm[x[i]][x[j]] and j - i - 1 >= 3 for i, j in pairs)
+    assert 0.25 * 8192 < r["scores"][0] <= (8192 - 3) // 2
+
+
+def test_nussinov_config5_sampled(dp, orc):
+    ids = dpgen.config5_sample_ids(k=400)
+    cat, off = dpgen.config5_rna_batch(ids=ids)
+    seqs = [cat[off[q]:off[q + 1]] for q in range(len(ids))]
+    r = run_nuss(dp, seqs, tb=False)
+    want = orc.nussinov_batch(cat, off, dpgen.rna_pair_mask(), 3, threads=THREADS)
+    assert (r["scores"] == want).all()
+
+
+# ----------------------------------------------------------------------------- HMM
+def hmm_case(g, S, n, tlo, thi):
+    pi, A, E = dpgen.hmm_params(g, S, 4)
+    pi32, A32, E32 = (v.astype(np.float32) for v in (pi, A, E))
+    seqs = [dpgen.sample_hmm(g, pi, A, E, 1, int(g.integers(tlo, thi + 1)))[0] for _ in range(n)]
+    return pi32, A32, E32, seqs
+
+
+@pytest.mark.parametrize("S", [1, 5, 64])
+def test_forward_random(dp, orc, S):
+    g = np.random.default_rng(120 + S)
+    pi, A, E, seqs = hmm_case(g, S, 60, 0, 300)
+    cat, off = dpgen.pack(seqs)
+    plan = dp.Plan(dp.HMM_FORWARD, max(len(s) for s in seqs), pi=pi, A=A, E=E)
+    ll = host(plan.solve_batch(cuda(cat), cuda(off)))
+    want = orc.forward_batch(cat, off, pi.astype(np.float64), A.astype(np.float64), E.astype(np.float64),
+                             threads=THREADS)
+    for q in range(len(seqs)):
+        if len(seqs[q]) == 0:
+            assert ll[q] == 0.0
+        else:
+            assert abs(ll[q] - want[q]) <= 1e-5 * abs(want[q]), (q, ll[q], want[q])
+
+
+@pytest.mark.parametrize("S", [1, 7, 64])
+def test_viterbi_random(dp, orc, S):
+    g = np.random.default_rng(130 + S)
+    pi, A, E, seqs = hmm_case(g, S, 60, 0, 300)
+    lpi, lA, lE = dpgen.millibits(pi), dpgen.millibits(A), dpgen.millibits(E)
+    cat, off = dpgen.pack(seqs)
+    ml = max(len(s) for s in seqs)
+    plan = dp.Plan(dp.HMM_VITERBI, ml, lpi=lpi, lA=lA, lE=lE, want_traceback=True)
+    sc = host(plan.solve_batch(cuda(cat), cuda(off)))
+    out, ln, _ = plan.traceback(0, len(seqs), max(ml, 1), coords=False)
+    out, ln = host(out), host(ln)
+    for q, x in enumerate(seqs):
+        v, path = orc.viterbi(x, lpi, lA, lE)
+        assert sc[q] == v, q
+        assert ln[q] == len(x) and (out[q, :len(x)] == path).all(), q
+
+
+def test_hmm_config3_sampled(dp, orc):
+    """BASELINE config 3 at full size (10k x 1000, S = 64), sampled against the oracle."""
+    d = dpgen.config3_hmm()
+    seqs = d["seqs"]
+    n, T = seqs.shape
+    off = np.arange(n + 1, dtype=np.int64) * T
+    cat = seqs.reshape(-1)
+    pf = dp.Plan(dp.HMM_FORWARD, T, pi=d["pi"], A=d["A"], E=d["E"])
+    ll = host(pf.solve_batch(cuda(cat), cuda(off), max_len_a=T))
+    pv = dp.Plan(dp.HMM_VITERBI, T, lpi=d["lpi"], lA=d["lA"], lE=d["lE"], want_traceback=True)
+    vs = host(pv.solve_batch(cuda(cat), cuda(off), max_len_a=T))
+    out, ln, _ = pv.traceback(0, n, T, coords=False)
+    out = host(out)
+    ids = np.random.default_rng(140).choice(n, size=24, replace=False)
+    sub_off = np.arange(len(ids) + 1, dtype=np.int64) * T
+    sub = seqs[ids].reshape(-1)
+    want = orc.forward_batch(sub, sub_off, *(d[k].astype(np.float64) for k in ("pi", "A", "E")), threads=THREADS)
+    for k, q in enumerate(ids):
+        assert abs(ll[q] - want[k]) <= 1e-5 * abs(want[k])
+        v, path = orc.viterbi(seqs[q], d["lpi"], d["lA"], d["lE"])
+        assert vs[q] == v and (out[q] == path).all()
+
+
+# ----------------------------------------------------------------------------- boundary
+def test_errors_and_empty(dp):
+    import torch
+    sig = dpgen.blosum62()
+    plan = dp.Plan(dp.SW_LINEAR, 16, 16, sigma=sig, gap=4)
+    z = torch.zeros(1, dtype=torch.int64, device="cuda")
+    e = torch.zeros(0, dtype=torch.uint8, device="cuda")
+    out = plan.solve_batch(e, z, e, z, max_len_a=0, max_len_b=0)
+    assert out.numel() == 0
+    a = cuda(np.zeros(20, np.uint8))
+    off = cuda(np.array([0, 20], np.int64))
+    with pytest.raises(dp.DPError) as ex:
+        plan.solve_batch(a, off, a, off, max_len_a=20, max_len_b=20)
+    assert ex.value.code == 4   # DP_E_TOO_LARGE
+    with pytest.raises(dp.DPError) as ex:
+        plan.traceback(0, 1, 64)
+    assert ex.value.code == 7   # DP_E_NO_TRACEBACK
+    with pytest.raises(dp.DPError) as ex:
+        dp.Plan(dp.HMM_FORWARD, 10, pi=np.ones(2, np.float32), A=np.ones((2, 2), np.float32),
+                E=np.ones((2, 4), np.float32), want_traceback=True)
+    assert ex.value.code == 3   # forward has no traceback
+    with pytest.raises(dp.DPError) as ex:
+        dp.Plan(dp.SW_LINEAR, 16, 16, sigma=sig, gap=4, user_coeff=(1, -1))
+    assert ex.value.code == 2   # user schedule violates eq.(3)
+    plan.close()
+
+
+def test_host_entry_point(dp, orc):
+    """dp_solve_batch_host (H2D + solve + traceback + D2H) equals the device path."""
+    g = np.random.default_rng(150)
+    sig = dpgen.blosum62()
+    a, (a_cat, a_off) = rand_batch(g, 50, 1, 256, 20)
+    b, (b_cat, b_off) = rand_batch(g, 50, 1, 256, 20)
+    plan = dp.Plan(dp.SW_LINEAR, 256, 256, sigma=sig, gap=4, want_traceback=True)
+    sc, tb, tbl, tbc = plan.solve_batch_host(a_cat, a_off, b_cat, b_off, tb_stride=512)
+    for q in range(50):
+        s0, _, _ = orc.sw(a[q], b[q], sig, 4)
+        ops, co = orc.sw_traceback(a[q], b[q], sig, 4)
+        assert sc[q] == s0 and bytes(tb[q, :tbl[q]]).decode() == ops and tuple(tbc[q]) == co
+    plan.close()
