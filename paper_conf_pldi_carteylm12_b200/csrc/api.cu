@@ -46,6 +46,8 @@ struct dp_plan {
   int32_t window = -1;
   // device parameters
   int8_t* d_sigma = nullptr;
+  std::vector<int8_t> h_sigma;
+  bool packed16 = false;  // SW on the s16x2 two-problems-per-warp kernels
   uint8_t* d_pair = nullptr;
   float *d_pi = nullptr, *d_A = nullptr, *d_E = nullptr;
   int32_t *d_lpi = nullptr, *d_lA = nullptr, *d_lE = nullptr;
@@ -112,6 +114,28 @@ int families(int kind, int64_t la, int64_t lb, int S, int64_t ext[2], int* trian
   return -1;
 }
 
+// Packed-SW arguments; with traceback the checkpoint buffers live in the plan.
+cudaError_t sw16_args(dp_plan* p, int64_t n, const uint8_t* a_cat, const int64_t* a_off, const uint8_t* b_cat,
+                      const int64_t* b_off, int64_t max_la, int64_t max_lb, int32_t* scores, dpk::Sw16Args* A) {
+  A->n = n; A->a_cat = a_cat; A->b_cat = b_cat; A->a_off = a_off; A->b_off = b_off;
+  A->max_la = max_la > 0 ? max_la : 1; A->max_lb = max_lb > 0 ? max_lb : 1;
+  A->sigma = p->d_sigma; A->asz = p->asz; A->gap = p->gap;
+  A->smem_per_warp = dpk::sw16_smem_per_warp(p->asz, A->max_la, A->max_lb);
+  A->scores = scores;
+  if (!p->want_tb) return cudaSuccess;
+  int64_t strips, nslab, rw, cw, bw;
+  dpk::sw16_state_words(n, A->max_la, A->max_lb, &strips, &nslab, &rw, &cw, &bw);
+  cudaError_t e = p->tb_state.ensure((size_t)(rw + cw + bw) * 4 + 64);
+  if (e != cudaSuccess) return e;
+  A->rowck = static_cast<uint32_t*>(p->tb_state.ptr);
+  A->colck = A->rowck + rw;
+  A->slabbest = A->colck + cw;
+  A->strips_max = strips;
+  A->nslab_max = nslab > 0 ? nslab : 1;
+  p->last_scores = scores;
+  return cudaSuccess;
+}
+
 }  // namespace
 
 extern "C" {
@@ -176,6 +200,9 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       p->gap = d->gap;
       if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) { st = DP_E_TOO_LARGE; break; }
       e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
+      p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
+      p->packed16 = dpk::sw16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap) &&
+                    getenv("DP_FORCE_INT32") == nullptr;
       break;
     case DP_NUSSINOV:
       if (!d->pair_mask || d->min_hairpin < 0) { st = DP_E_INVALID; break; }
@@ -260,8 +287,15 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
   p->last_a = a_cat; p->last_b = b_cat; p->last_aoff = a_off; p->last_boff = b_off;
   p->last_max_la = max_len_a; p->last_max_lb = max_len_b;
   switch (p->kind) {
-    case DP_EDIT:
-    case DP_SW_LINEAR: {
+    case DP_SW_LINEAR:
+      if (p->packed16) {
+        dpk::Sw16Args A{};
+        e = sw16_args(p, n, a_cat, a_off, b_cat, b_off, max_len_a, max_len_b, static_cast<int32_t*>(scores_out), &A);
+        if (e == cudaSuccess) e = dpk::sw16_solve(A, p->want_tb, s, &p->launches);
+        break;
+      }
+      /* fall through */
+    case DP_EDIT: {
       dpk::AlignArgs A{};
       A.n = n; A.a_cat = a_cat; A.b_cat = b_cat; A.a_off = a_off; A.b_off = b_off;
       A.max_la = max_len_a > 0 ? max_len_a : 1; A.max_lb = max_len_b > 0 ? max_len_b : 1;
@@ -292,11 +326,16 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         A.db = static_cast<uint8_t*>(p->tb_state.ptr);
         A.db_len = static_cast<int32_t*>(p->tb_aux.ptr);
       }
-      A.scratch_bytes = dpk::nuss_scratch_bytes(A.max_len, n, p->device);
+      // cell-level CTA kernel (table in shared memory) for short sequences, tiled
+      // max-plus kernels above (SURVEY §8(a) A6b'); DP_NUSS_CELL=1 forces the cell level
+      const bool tiled = A.max_len > 128 && getenv("DP_NUSS_CELL") == nullptr &&
+                         (n == 1 || A.max_len <= 4096);
+      A.scratch_bytes = tiled ? dpk::nuss_tiled_scratch_bytes(A.max_len, n, p->device)
+                              : dpk::nuss_scratch_bytes(A.max_len, n, p->device);
       e = p->scratch.ensure((size_t)A.scratch_bytes);
       if (e != cudaSuccess) break;
       A.scratch = p->scratch.ptr;
-      e = dpk::nuss_solve(A, s, &p->launches);
+      e = tiled ? dpk::nuss_tiled_solve(A, s, &p->launches) : dpk::nuss_solve(A, s, &p->launches);
       break;
     }
     case DP_HMM_FORWARD:
@@ -354,8 +393,17 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   cudaError_t e = cudaSuccess;
   switch (p->kind) {
-    case DP_EDIT:
-    case DP_SW_LINEAR: {
+    case DP_SW_LINEAR:
+      if (p->packed16) {
+        if (stride < p->last_max_la + p->last_max_lb) return DP_E_TOO_LARGE;
+        dpk::Sw16Args A{};
+        e = sw16_args(p, p->last_n, p->last_a, p->last_aoff, p->last_b, p->last_boff, p->last_max_la,
+                      p->last_max_lb, p->last_scores, &A);
+        if (e == cudaSuccess) e = dpk::sw16_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
+        break;
+      }
+      /* fall through */
+    case DP_EDIT: {
       if (stride < p->last_max_la + p->last_max_lb) return DP_E_TOO_LARGE;
       dpk::AlignArgs A{};
       A.n = p->last_n; A.a_cat = p->last_a; A.b_cat = p->last_b; A.a_off = p->last_aoff; A.b_off = p->last_boff;

@@ -29,6 +29,30 @@ cudaError_t align_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t align_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                             int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
 
+// ---------------------------------------------------------------- packed SW (two problems per warp)
+struct Sw16Args {
+  int64_t n;
+  const uint8_t *a_cat, *b_cat;
+  const int64_t *a_off, *b_off;
+  int64_t max_la, max_lb;
+  const int8_t* sigma;   // device [asz x asz]
+  int asz, gap;
+  int smem_per_warp;
+  int32_t* scores;
+  // traceback checkpoints (nullptr in score-only mode)
+  uint32_t* rowck;       // [groups][strips][8 bands][max_lb]    G of each 32-row band's bottom row (packed pair)
+  uint32_t* colck;       // [groups][strips][nslab][256]         G of every 32nd column
+  uint32_t* slabbest;    // [groups][strips][nslab][32]           per-lane best G per 32-column slab
+  int64_t strips_max, nslab_max;
+};
+bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap);
+int sw16_smem_per_warp(int asz, int64_t max_la, int64_t max_lb);
+void sw16_state_words(int64_t n, int64_t max_la, int64_t max_lb, int64_t* strips, int64_t* nslab, int64_t* rowck,
+                      int64_t* colck, int64_t* slabbest);
+cudaError_t sw16_solve(const Sw16Args& a, bool tb, cudaStream_t s, int64_t* launches);
+cudaError_t sw16_traceback(const Sw16Args& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
+                           int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
+
 // ---------------------------------------------------------------- Nussinov
 struct NussArgs {
   int64_t n;
@@ -45,6 +69,9 @@ struct NussArgs {
   int64_t scratch_bytes;
 };
 int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device);
+bool nuss_tiled_supported(int64_t max_len);
+int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device);
+cudaError_t nuss_tiled_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t nuss_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
 
 // ---------------------------------------------------------------- HMM

@@ -1,0 +1,436 @@
+// Tiled Nussinov (SURVEY.md §8(a) A6b'): the schedule vector (-1,1) of the
+// cell-level analysis applied to 32x32 TILES. Tile (I,J) reads tiles (I,K) and
+// (K,J) for I < K < J, which are all strictly earlier tile-partitions, so a
+// tile-diagonal D = J - I is one hyperplane of independent tiles:
+//
+//   phase A  C(I,J) = max_{I<K<J} U(I,K) (x) L(K,J)     max-plus tile product,
+//            U(I,K)[r][k] = gamma(32I+r, 32K+k), L(K,J)[k][c] = gamma(32K+k+1, 32J+c)
+//   phase B  in-tile wavefront over the 63 local anti-diagonals: neighbours,
+//            the pair term and the split points k inside tiles I and J.
+//
+// Phase A is the bulk of the work (n^3/6 split evaluations) and runs as an
+// s16x2 max-plus micro-kernel: a warp owns a 32x32 C tile, lane (ty, tx)
+// holds rows 4ty..4ty+3 x column pairs 8tx..8tx+7 (16 packed accumulators);
+// per k it reads one 16-byte A word (4 rows, each value duplicated into both
+// halves) and one 16-byte B word (8 columns) from shared memory and issues 16
+// VIADDMNMX.S16x2 (32 split evaluations).
+//
+// Tables live in global memory (L2-resident), one 4 KB record per tile:
+// UT[c][r] = gamma(32I+r, 32J+c) (column-major int16; A operand and in-tile
+// reads) and L[k][c] (row-major int16; B operand).
+//
+// Two drivers share the tile routines:
+//   k_nuss_tiled_cta   one problem per CTA (batches), C tiles in shared memory,
+//                      __syncthreads between phases;
+//   k_nuss_tiled_grid  one large problem on the whole grid (cooperative launch):
+//                      phase A split-K over every warp of the grid with
+//                      atomicMax into global C, grid.sync between phases.
+// The canonical traceback (Durbin order, smallest k) runs right after the fill
+// with the split search spread over a warp.
+#include <algorithm>
+#include <cstdint>
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+
+#include "dp_internal.h"
+
+namespace cg = cooperative_groups;
+
+namespace dpk {
+namespace {
+
+constexpr int T = 32;
+constexpr int kTileWords = T * T;      // int16 per tile record half
+constexpr int kRec = 2 * kTileWords;   // int16 per tile record (UT + L)
+constexpr int kCtaWarps = 16;
+constexpr int kCS = T + 1;             // row stride of in-tile buffers
+constexpr int kGridMin = 1024;         // single problems longer than this use the whole grid
+
+__host__ __device__ __forceinline__ int64_t tile_id(int I, int J, int nt) {
+  return (int64_t)I * nt - (int64_t)I * (I - 1) / 2 + (J - I);
+}
+__host__ __device__ __forceinline__ int64_t tiles_of(int nt) { return (int64_t)nt * (nt + 1) / 2; }
+
+struct Tab {
+  int16_t* base;  // tile records
+  int nt;
+  __device__ __forceinline__ int16_t* UT(int I, int J) const { return base + tile_id(I, J, nt) * kRec; }
+  __device__ __forceinline__ int16_t* L(int I, int J) const { return base + tile_id(I, J, nt) * kRec + kTileWords; }
+  // gamma(i, j) for 0 <= i, j < 32 nt (0 when j - i < 1)
+  __device__ __forceinline__ int gamma(int i, int j) const {
+    if (j - i < 1) return 0;
+    return UT(i / T, j / T)[(j % T) * T + (i % T)];
+  }
+};
+
+__device__ __forceinline__ uint32_t dup16(uint32_t w, int hi) {
+  uint32_t r;
+  const uint32_t sel = hi ? 0x3232u : 0x1010u;
+  asm("prmt.b32 %0, %1, %1, %2;" : "=r"(r) : "r"(w), "r"(sel));
+  return r;
+}
+
+// Stage A = UT(I,K) (duplicated halves, [k][r]) and B = L(K,J) ([k][c]) in this warp's buffers.
+__device__ __forceinline__ void stage(const int16_t* ut, const int16_t* l, uint32_t* As, uint16_t* Bs, int lane) {
+#pragma unroll
+  for (int t = 0; t < 8; ++t) {
+    const int chunk = lane + 32 * t;  // 4-row chunk: k = chunk / 8, rows 4 (chunk % 8) ..
+    const uint2 w = *reinterpret_cast<const uint2*>(ut + chunk * 4);
+    *reinterpret_cast<uint4*>(As + chunk * 4) = make_uint4(dup16(w.x, 0), dup16(w.x, 1), dup16(w.y, 0), dup16(w.y, 1));
+  }
+#pragma unroll
+  for (int t = 0; t < 4; ++t) {
+    const int chunk = lane + 32 * t;  // 8 int16 per chunk
+    *reinterpret_cast<uint4*>(Bs + chunk * 8) = *reinterpret_cast<const uint4*>(l + chunk * 8);
+  }
+}
+
+// acc[4 rows][4 pairs] = max(acc, A (x) B) over the 32 k of one staged K tile.
+__device__ __forceinline__ void micro(const uint32_t* As, const uint16_t* Bs, uint32_t (&acc)[16], int lane) {
+  const int ty = lane >> 2, tx = lane & 3;
+#pragma unroll 8
+  for (int k = 0; k < T; ++k) {
+    const uint4 a = *reinterpret_cast<const uint4*>(As + k * T + 4 * ty);
+    const uint4 b = *reinterpret_cast<const uint4*>(Bs + k * T + 8 * tx);
+    const uint32_t av[4] = {a.x, a.y, a.z, a.w};
+    const uint32_t bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+    for (int r = 0; r < 4; ++r)
+#pragma unroll
+      for (int q = 0; q < 4; ++q) acc[r * 4 + q] = __viaddmax_s16x2(av[r], bv[q], acc[r * 4 + q]);
+  }
+}
+
+// Phase A for one (tile, K range) work unit; result max-merged into C (int32 [32][32]).
+template <bool SHARED_C>
+__device__ void product_unit(const Tab& tab, int I, int J, int K0, int K1, int* C, uint32_t* As, uint16_t* Bs,
+                             int lane) {
+  uint32_t acc[16];
+#pragma unroll
+  for (int q = 0; q < 16; ++q) acc[q] = 0;  // gamma >= 0, so 0 is a neutral start
+  for (int K = K0; K < K1; ++K) {
+    __syncwarp();
+    stage(tab.UT(I, K), tab.L(K, J), As, Bs, lane);
+    __syncwarp();
+    micro(As, Bs, acc, lane);
+  }
+  const int ty = lane >> 2, tx = lane & 3;
+#pragma unroll
+  for (int r = 0; r < 4; ++r)
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t v = acc[r * 4 + q];
+      int* c = C + (4 * ty + r) * T + 8 * tx + 2 * q;
+      const int lo = (int)(int16_t)(v & 0xffffu), hi = (int)(int16_t)(v >> 16);
+      if (SHARED_C) { atomicMax(c, lo); atomicMax(c + 1, hi); }
+      else { atomicMax(c, lo); atomicMax(c + 1, hi); }
+    }
+}
+
+struct InTileBuf {
+  int cur[T * kCS];        // CUR[r][c]
+  int16_t uii[T * kCS];    // U(I,I)[r][k]
+  int16_t ljj[T * kCS];    // L(J,J)[k][c]
+  int below[T];        // U(I+1,J)[0][c]
+  int left[T];         // U(I,J-1)[r][31]
+  int corner;          // gamma(32I+32, 32J-1)
+};
+
+__device__ __forceinline__ bool pairable(const uint8_t* x, const uint8_t* pm, int n, int i, int j, int h) {
+  return i < n && j < n && pm[x[i] * 4 + x[j]] && j - i - 1 >= h;
+}
+
+// Phase B: finalise tile (I,J) from C (max of the middle products), write UT/L records.
+__device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, InTileBuf& B, const uint8_t* x,
+                        const uint8_t* pm, int n, int h, int lane) {
+  const int i0 = I * T, j0 = J * T;
+  if (I == J) {
+    // diagonal tile: the cell-level recursion inside one 32x32 triangle
+    for (int q = lane; q < T * kCS; q += 32) B.cur[q] = 0;
+    __syncwarp();
+    for (int d = 1; d < T; ++d) {
+      const int r = lane, c = lane + d;
+      if (c < T) {
+        int v = max(B.cur[(r + 1) * kCS + c], B.cur[r * kCS + c - 1]);
+        if (pairable(x, pm, n, i0 + r, j0 + c, h)) v = max(v, (d >= 2 ? B.cur[(r + 1) * kCS + c - 1] : 0) + 1);
+        for (int k = r + 1; k < c; ++k) v = max(v, B.cur[r * kCS + k] + B.cur[(k + 1) * kCS + c]);
+        B.cur[r * kCS + c] = v;
+      }
+      __syncwarp();
+    }
+  } else {
+    const int16_t* utii = tab.UT(I, I);
+    const int16_t* ljj = tab.L(J, J);
+    const int16_t* utb = tab.UT(I + 1, J);
+    const int16_t* utl = tab.UT(I, J - 1);
+    for (int q = lane; q < T * T; q += 32) {
+      const int a = q / T, b = q % T;
+      B.uii[a * kCS + b] = utii[b * T + a];  // U(I,I)[a][b]
+      B.ljj[a * kCS + b] = ljj[q];           // L(J,J)[a][b]
+      B.cur[a * kCS + b] = has_c ? C[q] : 0;
+    }
+    B.below[lane] = utb[lane * T + 0];
+    B.left[lane] = utl[(T - 1) * T + lane];
+    if (lane == 0) B.corner = (I + 1 <= J - 1) ? tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
+    __syncwarp();
+    for (int dl = -(T - 1); dl <= T - 1; ++dl) {
+      const int r = lane, c = lane + dl;
+      if (c >= 0 && c < T) {
+        int v = B.cur[r * kCS + c];
+        const int bl = (r < T - 1) ? B.cur[(r + 1) * kCS + c] : B.below[c];
+        const int le = (c > 0) ? B.cur[r * kCS + c - 1] : B.left[r];
+        v = max(v, max(bl, le));
+        if (pairable(x, pm, n, i0 + r, j0 + c, h)) {
+          int inner;
+          if (r < T - 1 && c > 0) inner = B.cur[(r + 1) * kCS + c - 1];
+          else if (r == T - 1 && c > 0) inner = B.below[c - 1];
+          else if (r < T - 1 && c == 0) inner = B.left[r + 1];
+          else inner = B.corner;
+          v = max(v, inner + 1);
+        }
+        // split k inside tile I: gamma(i,k) + gamma(k+1,j), k = i0+r+1 .. i0+31
+        for (int k = r + 1; k < T; ++k)
+          v = max(v, (int)B.uii[r * kCS + k] + (k < T - 1 ? B.cur[(k + 1) * kCS + c] : B.below[c]));
+        // split k inside tile J: k = j0 .. j-1
+        for (int k = 0; k < c; ++k) v = max(v, B.cur[r * kCS + k] + (int)B.ljj[k * kCS + c]);
+        B.cur[r * kCS + c] = v;
+      }
+      __syncwarp();
+    }
+  }
+  // write the records: UT[c][r] and L[k][c] = gamma(i0+k+1, j0+c)
+  int16_t* ut = tab.UT(I, J);
+  int16_t* l = tab.L(I, J);
+  for (int r = 0; r < T; ++r) ut[lane * T + r] = (int16_t)B.cur[r * kCS + lane];
+  for (int k = 0; k < T - 1; ++k) l[k * T + lane] = (int16_t)B.cur[(k + 1) * kCS + lane];
+  l[(T - 1) * T + lane] = (I == J) ? 0 : (int16_t)B.below[lane];
+}
+
+// Canonical traceback (DESIGN.md R-TB-NUSS) by one warp: the split search is lane-parallel.
+__device__ void tiled_traceback(const Tab& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
+                                int* stack, int lane) {
+  for (int k = lane; k < n; k += 32) db[k] = '.';
+  __syncwarp();
+  if (n <= 1) return;
+  int sp = 0;
+  if (lane == 0) { stack[0] = 0; stack[1] = n - 1; }
+  sp = 2;
+  __syncwarp();
+  while (sp > 0) {
+    const int j = stack[sp - 1], i = stack[sp - 2];
+    sp -= 2;
+    __syncwarp();
+    if (j - i < 1) continue;
+    const int v = tab.gamma(i, j);
+    int action = 0, kk = -1;
+    if (v == tab.gamma(i + 1, j)) action = 1;
+    else if (v == tab.gamma(i, j - 1)) action = 2;
+    else if (pairable(x, pm, n, i, j, h) && v == tab.gamma(i + 1, j - 1) + 1) action = 3;
+    else {
+      for (int k0 = i + 1; k0 < j && kk < 0; k0 += 32) {
+        const int k = k0 + lane;
+        const bool hit = k < j && v == tab.gamma(i, k) + tab.gamma(k + 1, j);
+        const unsigned m = __ballot_sync(0xffffffffu, hit);
+        if (m) kk = k0 + __ffs(m) - 1;
+      }
+      action = 4;
+    }
+    if (lane == 0) {
+      if (action == 1) { stack[sp] = i + 1; stack[sp + 1] = j; }
+      else if (action == 2) { stack[sp] = i; stack[sp + 1] = j - 1; }
+      else if (action == 3) { db[i] = '('; db[j] = ')'; stack[sp] = i + 1; stack[sp + 1] = j - 1; }
+      else { stack[sp] = kk + 1; stack[sp + 1] = j; stack[sp + 2] = i; stack[sp + 3] = kk; }
+    }
+    sp += (action == 4) ? 4 : 2;
+    __syncwarp();
+  }
+}
+
+// ------------------------------------------------------------------ batch driver
+__global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  __shared__ uint8_t pm[16];
+  __shared__ uint8_t xs[4096];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
+  int* Cs = reinterpret_cast<int*>(smem);                                   // [kCtaWarps][1024]
+  uint8_t* wbuf = smem + sizeof(int) * kCtaWarps * T * T;                    // per-warp scratch
+  const size_t wbytes = sizeof(InTileBuf) > (T * T * 4 + T * T * 2) ? sizeof(InTileBuf) : (T * T * 4 + T * T * 2);
+  uint8_t* mine = wbuf + warp * ((wbytes + 15) & ~size_t(15));
+  uint32_t* As = reinterpret_cast<uint32_t*>(mine);
+  uint16_t* Bs = reinterpret_cast<uint16_t*>(mine + T * T * 4);
+  InTileBuf& IB = *reinterpret_cast<InTileBuf*>(mine);
+  Tab tab;
+  tab.base = reinterpret_cast<int16_t*>(A.scratch) + (int64_t)blockIdx.x * slot_elems;
+  int* stack = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * slot_elems) +
+               (int64_t)blockIdx.x * (4 * A.max_len + 8);
+  for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
+    const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+    __syncthreads();
+    for (int q = threadIdx.x; q < n; q += blockDim.x) xs[q] = A.x_cat[A.x_off[p] + q];
+    const int nt = (n + T - 1) / T;
+    tab.nt = nt;
+    __syncthreads();
+    for (int D = 0; D < nt; ++D) {
+      const int nT = nt - D;  // tiles on this diagonal (<= nt <= 128 for n <= 4096)
+      // phase A: work units (tile, K chunk); C per tile in shared memory (tiles > 16 processed in groups)
+      for (int g0 = 0; g0 < nT; g0 += kCtaWarps) {
+        const int gT = min(kCtaWarps, nT - g0);
+        if (D >= 2) {
+          for (int q = threadIdx.x; q < gT * T * T; q += blockDim.x) Cs[q] = 0;
+          __syncthreads();
+          const int ksteps = D - 1;
+          const int chunks = max(1, min(ksteps, kCtaWarps / gT));
+          const int units = gT * chunks;
+          for (int u = warp; u < units; u += kCtaWarps) {
+            const int t = u / chunks, ch = u % chunks;
+            const int I = g0 + t, J = I + D;
+            const int K0 = I + 1 + (ksteps * ch) / chunks, K1 = I + 1 + (ksteps * (ch + 1)) / chunks;
+            product_unit<true>(tab, I, J, K0, K1, Cs + t * T * T, As, Bs, lane);
+          }
+          __syncthreads();
+        }
+        // phase B: one warp per tile
+        if (warp < gT) {
+          const int I = g0 + warp, J = I + D;
+          in_tile(tab, I, J, Cs + warp * T * T, D >= 2, IB, xs, pm, n, A.hairpin, lane);
+        }
+        __syncthreads();
+      }
+    }
+    if (warp == 0) {
+      const int sc = n <= 1 ? 0 : tab.gamma(0, n - 1);
+      if (lane == 0) A.scores[p] = sc;
+      if (A.db) {
+        tiled_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, lane);
+        if (lane == 0) A.db_len[p] = n;
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ grid driver (one large problem)
+__global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_grid(NussArgs A, int64_t p) {
+  cg::grid_group grid = cg::this_grid();
+  extern __shared__ __align__(16) uint8_t smem[];
+  __shared__ uint8_t pm[16];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
+  __syncthreads();
+  const size_t wbytes = sizeof(InTileBuf) > (T * T * 4 + T * T * 2) ? sizeof(InTileBuf) : (T * T * 4 + T * T * 2);
+  uint8_t* mine = smem + warp * ((wbytes + 15) & ~size_t(15));
+  uint32_t* As = reinterpret_cast<uint32_t*>(mine);
+  uint16_t* Bs = reinterpret_cast<uint16_t*>(mine + T * T * 4);
+  InTileBuf& IB = *reinterpret_cast<InTileBuf*>(mine);
+  const uint8_t* x = A.x_cat + A.x_off[p];
+  const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+  const int nt = (n + T - 1) / T;
+  Tab tab;
+  tab.base = reinterpret_cast<int16_t*>(A.scratch);
+  tab.nt = nt;
+  int* Cg = reinterpret_cast<int*>(tab.base + tiles_of(nt) * kRec);  // 2 x nt x 1024 int32
+  int* stack = Cg + 2 * (int64_t)nt * T * T;
+  const int64_t gw = (int64_t)blockIdx.x * kCtaWarps + warp;
+  const int64_t nw = (int64_t)gridDim.x * kCtaWarps;
+  // C buffers start at zero
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T;
+       q += (int64_t)gridDim.x * blockDim.x)
+    Cg[q] = 0;
+  grid.sync();
+  for (int D = 0; D < nt; ++D) {
+    const int nT = nt - D;
+    int* C = Cg + (int64_t)(D & 1) * nt * T * T;
+    if (D >= 2) {
+      // phase A: split the (tile, K) pairs of this diagonal evenly over all warps
+      const int64_t total = (int64_t)nT * (D - 1);
+      const int64_t per = (total + nw - 1) / nw;
+      const int64_t b0 = gw * per, b1 = min(total, b0 + per);
+      int64_t it = b0;
+      while (it < b1) {
+        const int t = (int)(it / (D - 1));
+        const int kk = (int)(it % (D - 1));
+        const int64_t tile_end = (int64_t)(t + 1) * (D - 1);
+        const int64_t e = min(b1, tile_end);
+        const int I = t, J = t + D;
+        product_unit<false>(tab, I, J, I + 1 + kk, I + 1 + kk + (int)(e - it), C + (int64_t)t * T * T, As, Bs, lane);
+        it = e;
+      }
+      grid.sync();
+    }
+    // phase B: one warp per tile; the other buffer is cleared for diagonal D+1
+    int* Cn = Cg + (int64_t)((D + 1) & 1) * nt * T * T;
+    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < (int64_t)(nT - 1) * T * T;
+         q += (int64_t)gridDim.x * blockDim.x)
+      Cn[q] = 0;
+    for (int64_t t = gw; t < nT; t += nw) {
+      const int I = (int)t, J = I + D;
+      in_tile(tab, I, J, C + t * T * T, D >= 2, IB, x, pm, n, A.hairpin, lane);
+    }
+    grid.sync();
+  }
+  if (gw == 0) {
+    const int sc = n <= 1 ? 0 : tab.gamma(0, n - 1);
+    if (lane == 0) A.scores[p] = sc;
+    if (A.db) {
+      tiled_traceback(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, stack, lane);
+      if (lane == 0) A.db_len[p] = n;
+    }
+  }
+}
+
+size_t warp_bytes() {
+  const size_t w = sizeof(InTileBuf) > (T * T * 4 + T * T * 2) ? sizeof(InTileBuf) : (T * T * 4 + T * T * 2);
+  return (w + 15) & ~size_t(15);
+}
+
+int num_sms_t(int device) {
+  int v = 0;
+  cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device);
+  return v > 0 ? v : 148;
+}
+
+}  // namespace
+
+bool nuss_tiled_supported(int64_t max_len) { return max_len <= 65536; }
+
+int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
+  const int nt = (int)((max_len + T - 1) / T);
+  const int64_t stack_bytes = (4 * max_len + 8) * 4;
+  if (n == 1 && max_len > kGridMin) {
+    return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
+  }
+  const int64_t grid = std::min<int64_t>(n, num_sms_t(device));
+  return grid * (tiles_of(nt) * kRec * 2 + stack_bytes) + 256;
+}
+
+cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
+  if (A.n == 0) return cudaSuccess;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const int sms = num_sms_t(dev);
+  const int nt = (int)((A.max_len + T - 1) / T);
+  if (A.n == 1 && A.max_len > kGridMin) {
+    const size_t smem = kCtaWarps * warp_bytes();
+    cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_grid, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_nuss_tiled_grid, kCtaWarps * 32, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) return cudaErrorInvalidConfiguration;
+    NussArgs a2 = A;
+    int64_t p = 0;
+    void* args[2] = {&a2, &p};
+    ++*launches;
+    return cudaLaunchCooperativeKernel((void*)k_nuss_tiled_grid, sms, kCtaWarps * 32, args, smem, s);
+  }
+  if (A.max_len > 4096) return cudaErrorInvalidValue;  // batch path keeps the sequence in shared memory
+  const size_t smem = sizeof(int) * kCtaWarps * T * T + kCtaWarps * warp_bytes();
+  cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const int64_t grid = std::min<int64_t>(A.n, sms);
+  ++*launches;
+  k_nuss_tiled_cta<<<(unsigned)grid, kCtaWarps * 32, smem, s>>>(A, tiles_of(nt) * kRec);
+  return cudaGetLastError();
+}
+
+}  // namespace dpk

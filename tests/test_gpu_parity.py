@@ -85,6 +85,34 @@ def test_sw_random_ragged(dp, orc, maxlen):
             assert tuple(r["coords"][q]) == co, q
 
 
+def test_sw_int32_kernel_path(dp, orc, monkeypatch):
+    """The general int32 kernel (used when s16x2 could overflow) on the same cases."""
+    monkeypatch.setenv("DP_FORCE_INT32", "1")
+    g = np.random.default_rng(104)
+    sig = dpgen.blosum62()
+    a, _ = rand_batch(g, 60, 0, 300, 24)
+    b, _ = rand_batch(g, 60, 0, 300, 24)
+    r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24)
+    for q in range(60):
+        assert r["scores"][q] == orc.sw(a[q], b[q], sig, 4)[0], q
+        ops, co = orc.sw_traceback(a[q], b[q], sig, 4)
+        assert r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+
+
+def test_sw_packed_odd_batch_and_ties(dp, orc):
+    """Odd batch (last warp half empty), mismatched pair lengths in one warp, and
+    a low-entropy alphabet that makes ties frequent (end cell / traceback tie-breaks)."""
+    g = np.random.default_rng(105)
+    sig = dpgen.blosum62()
+    a, _ = rand_batch(g, 77, 1, 260, 3)
+    b, _ = rand_batch(g, 77, 1, 90, 3)
+    r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=2, asz=24)
+    for q in range(77):
+        sc, ei, ej = orc.sw(a[q], b[q], sig, 2)
+        ops, co = orc.sw_traceback(a[q], b[q], sig, 2)
+        assert r["scores"][q] == sc and r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+
+
 def test_sw_score_only_matches_traceback_mode(dp):
     g = np.random.default_rng(102)
     sig = dpgen.blosum62()
@@ -161,6 +189,30 @@ def test_nussinov_random_smem(dp, orc, h):
         sc, db = orc.nussinov_traceback(x, pm, h)
         assert r["scores"][q] == sc, q
         assert r["db"][q] == db, q
+
+
+def test_nussinov_cell_level_path(dp, orc, monkeypatch):
+    """The cell-level CTA kernels (shared-memory table; L2 table above 340) on the same cases."""
+    monkeypatch.setenv("DP_NUSS_CELL", "1")
+    g = np.random.default_rng(113)
+    seqs, _ = rand_batch(g, 40, 0, 420, 4)
+    r = run_nuss(dp, seqs)
+    pm = dpgen.rna_pair_mask()
+    for q, x in enumerate(seqs):
+        sc, db = orc.nussinov_traceback(x, pm, 3)
+        assert r["scores"][q] == sc and r["db"][q] == db, q
+
+
+def test_nussinov_tiled_ragged(dp, orc):
+    """Tiled batch kernel: lengths around tile multiples (31, 32, 33, 64, 65 ...)."""
+    g = np.random.default_rng(114)
+    lens = [129, 130, 159, 160, 161, 191, 192, 193, 255, 256, 257, 300, 2, 1, 0, 31, 32, 33]
+    seqs = [g.integers(0, 4, size=l).astype(np.uint8) for l in lens]
+    r = run_nuss(dp, seqs)
+    pm = dpgen.rna_pair_mask()
+    for q, x in enumerate(seqs):
+        sc, db = orc.nussinov_traceback(x, pm, 3)
+        assert r["scores"][q] == sc and r["db"][q] == db, (q, len(x))
 
 
 def test_nussinov_global_scratch_path(dp, orc):
