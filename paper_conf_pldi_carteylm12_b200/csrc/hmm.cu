@@ -2,21 +2,24 @@
 // L467–L472: "our schedule can only be S_forward(s,i) = i").
 // Partition i holds the S cells F(., i); the window is one partition (§4.8).
 //
-// B200 design (SIMT, round 1): one warp per sequence, lane l owns states l and
-// l + 32 (S <= 64). The column of the transition matrix for each owned state
-// (64 + 64 values) stays in registers for the whole sequence, the previous
-// partition's S values are broadcast from shared memory, so one step is
-// 128 FFMA (forward) or 128 VIADDMNMX (Viterbi) per lane with no global traffic.
+// B200 design (SIMT): one warp carries NS sequences, lane l owns states l and
+// l + 32 (S <= 64). The columns of the transition matrix for the two owned
+// states (64 + 64 values) stay in registers for the whole batch and are
+// reused by all NS sequences; the previous partition of each sequence is
+// broadcast from shared memory by LDS.128. One step is 128 x NS FFMA (forward)
+// or VIADDMNMX (Viterbi) per lane, with NS independent chains to hide the
+// per-step reduction latency. NS is picked so the batch fits in one wave.
 //
 // Forward (Fig.11a; DESIGN.md R-HMM-FWD): begin state with
 // transitions pi, tau == 1. Probabilities are kept in scaled linear space
 // (one of the representations §3.2 L222–L225 allows): alpha_i = a_i / c_i with
-// c_i = sum_s a_i(s), log P(x) = sum_i log c_i accumulated in fp64.
+// c_i = sum_s a_i(s); log P(x) = sum_i log c_i, the c_i multiplied in fp32 and
+// folded into an fp64 log sum whenever the product leaves [2^-60, 2^60].
 // Viterbi (max-variant, L463–L464; DESIGN.md R-VIT): int32 milli-bit scores,
 // exact integer arithmetic. The predecessor argmax with lowest-index ties uses
 // packed keys key(p) = V(p) * 64 + (63 - p), so one VIADDMNMX per (p, s) yields
-// both the max and the argmax; V is renormalised by its max every step
-// (integer offset kept in int64) so keys never overflow.
+// both the max and the argmax; V is renormalised by its max every 32 steps
+// (exact integer offset kept in int64) so keys never overflow.
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -27,6 +30,8 @@ namespace {
 
 constexpr int kMaxS = 64;
 constexpr int kMaxK = 16;
+constexpr int kHW = 1;      // warps per CTA (one: fine-grained occupancy for the register-heavy kernels)
+constexpr int kChunk = 32;  // sequence symbols staged per refill
 
 __device__ __forceinline__ float warp_sum(float v) {
 #pragma unroll
@@ -39,18 +44,33 @@ __device__ __forceinline__ int warp_max(int v) {
   return v;
 }
 
-__global__ void __launch_bounds__(kWarps * 32, 1) k_forward(HmmArgs H) {
-  __shared__ __align__(16) float alpha[kWarps][kMaxS];
-  __shared__ float Es[kMaxS * kMaxK];
+// Stage symbols [t0, t0 + kChunk) of the warp's sequences (0 past the end).
+template <int NS>
+__device__ __forceinline__ void stage_symbols(const HmmArgs& H, int64_t p0, const int* T, int t0, uint8_t (*xs)[kChunk],
+                                              int lane) {
+#pragma unroll
+  for (int q = 0; q < NS; ++q) {
+    const int64_t p = p0 + q;
+    const int t = t0 + lane;
+    xs[q][lane] = (p < H.n && t < T[q]) ? H.x_cat[H.x_off[p] + t] : 0;
+  }
+}
+
+template <int NS>
+__global__ void __launch_bounds__(kHW * 32) k_forward(HmmArgs H) {
+  __shared__ __align__(16) float alpha[kHW][NS][kMaxS];
+  __shared__ float Es[kMaxK][kMaxS];
+  __shared__ uint8_t xs_all[kHW][NS][kChunk];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = H.S, K = H.K;
   for (int q = threadIdx.x; q < kMaxS * kMaxK; q += blockDim.x) {
-    const int s = q / kMaxK, c = q % kMaxK;
-    Es[q] = (s < S && c < K) ? H.E[s * K + c] : 0.f;
+    const int c = q / kMaxS, s = q % kMaxS;
+    Es[c][s] = (s < S && c < K) ? H.E[s * K + c] : 0.f;
   }
   __syncthreads();
-  const int64_t p = (int64_t)blockIdx.x * kWarps + warp;
-  if (p >= H.n) return;
+  const int64_t p0 = ((int64_t)blockIdx.x * kHW + warp) * NS;
+  if (p0 >= H.n) return;
+  uint8_t (*xs)[kChunk] = xs_all[warp];
   const int s0 = lane, s1 = lane + 32;
   float a0[kMaxS], a1[kMaxS];
 #pragma unroll
@@ -58,68 +78,100 @@ __global__ void __launch_bounds__(kWarps * 32, 1) k_forward(HmmArgs H) {
     a0[q] = (q < S && s0 < S) ? H.A[q * S + s0] : 0.f;
     a1[q] = (q < S && s1 < S) ? H.A[q * S + s1] : 0.f;
   }
-  const uint8_t* x = H.x_cat + H.x_off[p];
-  const int T = (int)(H.x_off[p + 1] - H.x_off[p]);
-  if (T == 0) {
-    if (lane == 0) H.ll_out[p] = 0.f;
-    return;
-  }
-  double ll = 0.0;
-  // i = 1: a(s) = pi_s e_s(x_1)
-  int c = x[0];
-  float v0 = (s0 < S) ? H.pi[s0] * Es[s0 * kMaxK + c] : 0.f;
-  float v1 = (s1 < S) ? H.pi[s1] * Es[s1 * kMaxK + c] : 0.f;
-  float tot = warp_sum(v0 + v1);
-  ll += log((double)tot);
-  float inv = 1.f / tot;
-  alpha[warp][s0] = v0 * inv;
-  alpha[warp][s1] = v1 * inv;
-  __syncwarp();
-  int cn = (T > 1) ? x[1] : 0;
-  for (int i = 2; i <= T; ++i) {
-    c = cn;
-    if (i < T) cn = x[i];  // prefetch the next symbol
-    float acc0[4] = {0.f, 0.f, 0.f, 0.f}, acc1[4] = {0.f, 0.f, 0.f, 0.f};
-    const float4* al = reinterpret_cast<const float4*>(alpha[warp]);
+  int T[NS];
+  int Tmax = 0;
 #pragma unroll
-    for (int q4 = 0; q4 < kMaxS / 4; ++q4) {
-      const float4 v = al[q4];
-      acc0[0] = fmaf(v.x, a0[4 * q4 + 0], acc0[0]);
-      acc0[1] = fmaf(v.y, a0[4 * q4 + 1], acc0[1]);
-      acc0[2] = fmaf(v.z, a0[4 * q4 + 2], acc0[2]);
-      acc0[3] = fmaf(v.w, a0[4 * q4 + 3], acc0[3]);
-      acc1[0] = fmaf(v.x, a1[4 * q4 + 0], acc1[0]);
-      acc1[1] = fmaf(v.y, a1[4 * q4 + 1], acc1[1]);
-      acc1[2] = fmaf(v.z, a1[4 * q4 + 2], acc1[2]);
-      acc1[3] = fmaf(v.w, a1[4 * q4 + 3], acc1[3]);
+  for (int q = 0; q < NS; ++q) {
+    T[q] = (p0 + q < H.n) ? (int)(H.x_off[p0 + q + 1] - H.x_off[p0 + q]) : 0;
+    Tmax = max(Tmax, T[q]);
+  }
+  double ll[NS];
+  float prod[NS];
+  stage_symbols<NS>(H, p0, T, 0, xs, lane);
+  __syncwarp();
+  // i = 1: a(s) = pi_s e_s(x_1)
+#pragma unroll
+  for (int q = 0; q < NS; ++q) {
+    ll[q] = 0.0;
+    prod[q] = 1.f;
+    const int c = xs[q][0];
+    const float v0 = (s0 < S) ? H.pi[s0] * Es[c][s0] : 0.f;
+    const float v1 = (s1 < S) ? H.pi[s1] * Es[c][s1] : 0.f;
+    const float tot = warp_sum(v0 + v1);
+    const float inv = 1.f / tot;
+    prod[q] = tot;
+    alpha[warp][q][s0] = v0 * inv;
+    alpha[warp][q][s1] = v1 * inv;
+  }
+  __syncwarp();
+  for (int i = 2; i <= Tmax; ++i) {
+    if (((i - 1) & (kChunk - 1)) == 0) {
+      __syncwarp();
+      stage_symbols<NS>(H, p0, T, i - 1, xs, lane);
+      __syncwarp();
     }
-    v0 = ((acc0[0] + acc0[1]) + (acc0[2] + acc0[3])) * Es[s0 * kMaxK + c];
-    v1 = ((acc1[0] + acc1[1]) + (acc1[2] + acc1[3])) * Es[s1 * kMaxK + c];
-    tot = warp_sum(v0 + v1);
-    ll += log((double)tot);
-    inv = 1.f / tot;
+    float v0[NS], v1[NS];
+#pragma unroll
+    for (int q = 0; q < NS; ++q) {
+      float acc0a = 0.f, acc0b = 0.f, acc1a = 0.f, acc1b = 0.f;
+      const float4* al = reinterpret_cast<const float4*>(alpha[warp][q]);
+#pragma unroll
+      for (int q4 = 0; q4 < kMaxS / 4; ++q4) {
+        const float4 v = al[q4];
+        acc0a = fmaf(v.x, a0[4 * q4 + 0], acc0a);
+        acc0b = fmaf(v.y, a0[4 * q4 + 1], acc0b);
+        acc0a = fmaf(v.z, a0[4 * q4 + 2], acc0a);
+        acc0b = fmaf(v.w, a0[4 * q4 + 3], acc0b);
+        acc1a = fmaf(v.x, a1[4 * q4 + 0], acc1a);
+        acc1b = fmaf(v.y, a1[4 * q4 + 1], acc1b);
+        acc1a = fmaf(v.z, a1[4 * q4 + 2], acc1a);
+        acc1b = fmaf(v.w, a1[4 * q4 + 3], acc1b);
+      }
+      const int c = xs[q][(i - 1) & (kChunk - 1)];
+      v0[q] = (acc0a + acc0b) * Es[c][s0];
+      v1[q] = (acc1a + acc1b) * Es[c][s1];
+    }
     __syncwarp();
-    alpha[warp][s0] = v0 * inv;
-    alpha[warp][s1] = v1 * inv;
+#pragma unroll
+    for (int q = 0; q < NS; ++q) {
+      if (i > T[q]) continue;  // warp-uniform
+      const float tot = warp_sum(v0[q] + v1[q]);
+      const float inv = 1.f / tot;
+      alpha[warp][q][s0] = v0[q] * inv;
+      alpha[warp][q][s1] = v1[q] * inv;
+      prod[q] *= tot;
+      if (!(prod[q] > 8.6736e-19f && prod[q] < 1.1529215e18f)) {  // outside [2^-60, 2^60]
+        ll[q] += log((double)prod[q]);
+        prod[q] = 1.f;
+      }
+    }
     __syncwarp();
   }
-  if (lane == 0) H.ll_out[p] = (float)ll;
+  if (lane == 0) {
+#pragma unroll
+    for (int q = 0; q < NS; ++q)
+      if (p0 + q < H.n) H.ll_out[p0 + q] = T[q] == 0 ? 0.f : (float)(ll[q] + log((double)prod[q]));
+  }
 }
 
 constexpr int kNegKey = -(1 << 30);
+constexpr int kRenorm = 32;
 
-__global__ void __launch_bounds__(kWarps * 32, 1) k_viterbi(HmmArgs H) {
-  __shared__ __align__(16) int key[kWarps][kMaxS];
-  __shared__ int Es[kMaxS * kMaxK];
+template <int NS>
+__global__ void __launch_bounds__(kHW * 32) k_viterbi(HmmArgs H) {
+  __shared__ __align__(16) int key[kHW][NS][kMaxS];
+  __shared__ int Es[kMaxK][kMaxS];
+  __shared__ uint8_t xs_all[kHW][NS][kChunk];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = H.S, K = H.K;
   for (int q = threadIdx.x; q < kMaxS * kMaxK; q += blockDim.x) {
-    const int s = q / kMaxK, c = q % kMaxK;
-    Es[q] = (s < S && c < K) ? H.lE[s * K + c] : 0;
+    const int c = q / kMaxS, s = q % kMaxS;
+    Es[c][s] = (s < S && c < K) ? H.lE[s * K + c] : 0;
   }
   __syncthreads();
-  const int64_t p = (int64_t)blockIdx.x * kWarps + warp;
-  if (p >= H.n) return;
+  const int64_t p0 = ((int64_t)blockIdx.x * kHW + warp) * NS;
+  if (p0 >= H.n) return;
+  uint8_t (*xs)[kChunk] = xs_all[warp];
   const int s0 = lane, s1 = lane + 32;
   const bool ok0 = s0 < S, ok1 = s1 < S;
   int la0[kMaxS], la1[kMaxS];  // transition scores x 64 (key units)
@@ -128,63 +180,91 @@ __global__ void __launch_bounds__(kWarps * 32, 1) k_viterbi(HmmArgs H) {
     la0[q] = (q < S && ok0) ? H.lA[q * S + s0] * 64 : 0;
     la1[q] = (q < S && ok1) ? H.lA[q * S + s1] * 64 : 0;
   }
-  const uint8_t* x = H.x_cat + H.x_off[p];
-  const int T = (int)(H.x_off[p + 1] - H.x_off[p]);
-  if (T == 0) {
-    if (lane == 0) { H.vit_out[p] = 0; if (H.final_state) H.final_state[p] = -1; }
-    return;
-  }
-  uint8_t* bp = H.bp ? H.bp + (p * H.max_len) * kMaxS : nullptr;
-  // i = 1: V(s) = lpi_s + lE[s, x_1]
-  int c = x[0];
-  int V0 = ok0 ? H.lpi[s0] + Es[s0 * kMaxK + c] : kNegKey;
-  int V1 = ok1 ? H.lpi[s1] + Es[s1 * kMaxK + c] : kNegKey;
-  int m = warp_max(max(V0, V1));
-  int64_t off = m;
-  V0 -= m; V1 -= m;
-  key[warp][s0] = ok0 ? V0 * 64 + (63 - s0) : kNegKey;
-  key[warp][s1] = ok1 ? V1 * 64 + (63 - s1) : kNegKey;
-  __syncwarp();
-  int cn = (T > 1) ? x[1] : 0;
-  for (int i = 2; i <= T; ++i) {
-    c = cn;
-    if (i < T) cn = x[i];
-    int b0[4] = {INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN}, b1[4] = {INT32_MIN, INT32_MIN, INT32_MIN, INT32_MIN};
-    const int4* kv = reinterpret_cast<const int4*>(key[warp]);
+  int T[NS];
+  int Tmax = 0;
 #pragma unroll
-    for (int q4 = 0; q4 < kMaxS / 4; ++q4) {
-      const int4 v = kv[q4];
-      b0[0] = __viaddmax_s32(v.x, la0[4 * q4 + 0], b0[0]);
-      b0[1] = __viaddmax_s32(v.y, la0[4 * q4 + 1], b0[1]);
-      b0[2] = __viaddmax_s32(v.z, la0[4 * q4 + 2], b0[2]);
-      b0[3] = __viaddmax_s32(v.w, la0[4 * q4 + 3], b0[3]);
-      b1[0] = __viaddmax_s32(v.x, la1[4 * q4 + 0], b1[0]);
-      b1[1] = __viaddmax_s32(v.y, la1[4 * q4 + 1], b1[1]);
-      b1[2] = __viaddmax_s32(v.z, la1[4 * q4 + 2], b1[2]);
-      b1[3] = __viaddmax_s32(v.w, la1[4 * q4 + 3], b1[3]);
+  for (int q = 0; q < NS; ++q) {
+    T[q] = (p0 + q < H.n) ? (int)(H.x_off[p0 + q + 1] - H.x_off[p0 + q]) : 0;
+    Tmax = max(Tmax, T[q]);
+  }
+  stage_symbols<NS>(H, p0, T, 0, xs, lane);
+  __syncwarp();
+  int V0[NS], V1[NS];
+  int64_t off[NS];
+#pragma unroll
+  for (int q = 0; q < NS; ++q) {
+    const int c = xs[q][0];
+    V0[q] = ok0 ? H.lpi[s0] + Es[c][s0] : kNegKey;
+    V1[q] = ok1 ? H.lpi[s1] + Es[c][s1] : kNegKey;
+    const int m = warp_max(max(V0[q], V1[q]));
+    off[q] = m;
+    V0[q] -= m; V1[q] -= m;
+    key[warp][q][s0] = ok0 ? V0[q] * 64 + (63 - s0) : kNegKey;
+    key[warp][q][s1] = ok1 ? V1[q] * 64 + (63 - s1) : kNegKey;
+  }
+  __syncwarp();
+  for (int i = 2; i <= Tmax; ++i) {
+    if (((i - 1) & (kChunk - 1)) == 0) {
+      __syncwarp();
+      stage_symbols<NS>(H, p0, T, i - 1, xs, lane);
+      __syncwarp();
     }
-    const int k0 = max(max(b0[0], b0[1]), max(b0[2], b0[3]));
-    const int k1 = max(max(b1[0], b1[1]), max(b1[2], b1[3]));
-    // key = V(p)*64 + (63-p) + lA*64  ->  floor(key / 64) = V(p) + lA, low 6 bits = 63 - argmax
-    V0 = ok0 ? (k0 >> 6) + Es[s0 * kMaxK + c] : kNegKey;
-    V1 = ok1 ? (k1 >> 6) + Es[s1 * kMaxK + c] : kNegKey;
-    if (bp) {
-      if (ok0) bp[(int64_t)(i - 1) * kMaxS + s0] = (uint8_t)(63 - (k0 & 63));
-      if (ok1) bp[(int64_t)(i - 1) * kMaxS + s1] = (uint8_t)(63 - (k1 & 63));
+    int k0[NS], k1[NS];
+#pragma unroll
+    for (int q = 0; q < NS; ++q) {
+      int b0a = INT32_MIN, b0b = INT32_MIN, b1a = INT32_MIN, b1b = INT32_MIN;
+      const int4* kv = reinterpret_cast<const int4*>(key[warp][q]);
+#pragma unroll
+      for (int q4 = 0; q4 < kMaxS / 4; ++q4) {
+        const int4 v = kv[q4];
+        b0a = __viaddmax_s32(v.x, la0[4 * q4 + 0], b0a);
+        b0b = __viaddmax_s32(v.y, la0[4 * q4 + 1], b0b);
+        b0a = __viaddmax_s32(v.z, la0[4 * q4 + 2], b0a);
+        b0b = __viaddmax_s32(v.w, la0[4 * q4 + 3], b0b);
+        b1a = __viaddmax_s32(v.x, la1[4 * q4 + 0], b1a);
+        b1b = __viaddmax_s32(v.y, la1[4 * q4 + 1], b1b);
+        b1a = __viaddmax_s32(v.z, la1[4 * q4 + 2], b1a);
+        b1b = __viaddmax_s32(v.w, la1[4 * q4 + 3], b1b);
+      }
+      k0[q] = max(b0a, b0b);
+      k1[q] = max(b1a, b1b);
     }
-    m = warp_max(max(V0, V1));
-    off += m;
-    V0 -= m; V1 -= m;
     __syncwarp();
-    key[warp][s0] = ok0 ? V0 * 64 + (63 - s0) : kNegKey;
-    key[warp][s1] = ok1 ? V1 * 64 + (63 - s1) : kNegKey;
+#pragma unroll
+    for (int q = 0; q < NS; ++q) {
+      if (i > T[q]) continue;  // warp-uniform
+      const int c = xs[q][(i - 1) & (kChunk - 1)];
+      // key = V(p)*64 + (63-p) + lA*64  ->  floor(key / 64) = V(p) + lA, low 6 bits = 63 - argmax
+      V0[q] = ok0 ? (k0[q] >> 6) + Es[c][s0] : kNegKey;
+      V1[q] = ok1 ? (k1[q] >> 6) + Es[c][s1] : kNegKey;
+      if (H.bp) {
+        uint8_t* bp = H.bp + ((p0 + q) * H.max_len + (i - 1)) * kMaxS;
+        if (ok0) bp[s0] = (uint8_t)(63 - (k0[q] & 63));
+        if (ok1) bp[s1] = (uint8_t)(63 - (k1[q] & 63));
+      }
+      if ((i & (kRenorm - 1)) == 0) {
+        const int m = warp_max(max(V0[q], V1[q]));
+        off[q] += m;
+        V0[q] -= m; V1[q] -= m;
+      }
+      key[warp][q][s0] = ok0 ? V0[q] * 64 + (63 - s0) : kNegKey;
+      key[warp][q][s1] = ok1 ? V1[q] * 64 + (63 - s1) : kNegKey;
+    }
     __syncwarp();
   }
   // best final state: max V, lowest index on ties -> max of V*64 + (63 - s)
-  const int fk = warp_max(max(key[warp][s0], key[warp][s1]));
-  if (lane == 0) {
-    H.vit_out[p] = (int32_t)(off + (fk >> 6));
-    if (H.final_state) H.final_state[p] = 63 - (fk & 63);
+#pragma unroll
+  for (int q = 0; q < NS; ++q) {
+    const int fk = warp_max(max(key[warp][q][s0], key[warp][q][s1]));
+    if (lane == 0 && p0 + q < H.n) {
+      if (T[q] == 0) {
+        H.vit_out[p0 + q] = 0;
+        if (H.final_state) H.final_state[p0 + q] = -1;
+      } else {
+        H.vit_out[p0 + q] = (int32_t)(off[q] + (fk >> 6));
+        if (H.final_state) H.final_state[p0 + q] = 63 - (fk & 63);
+      }
+    }
   }
 }
 
@@ -205,20 +285,59 @@ __global__ void k_viterbi_tb(HmmArgs H, int64_t first, int64_t count, uint8_t* o
   out_len[q] = T;
 }
 
+int sms_of_current() {
+  int dev = 0, v = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+  return v > 0 ? v : 148;
+}
+
+template <int NS>
+void* fwd_ptr(bool viterbi) { return viterbi ? (void*)k_viterbi<NS> : (void*)k_forward<NS>; }
+
+// Sequences per warp: minimise (waves of resident warps) x NS, the per-warp time
+// being proportional to NS; ties go to the smaller NS (more warps in flight).
+int pick_ns(int64_t n, bool viterbi, void** kern) {
+  void* ks[8] = {fwd_ptr<1>(viterbi), fwd_ptr<2>(viterbi), fwd_ptr<3>(viterbi), fwd_ptr<4>(viterbi),
+                 fwd_ptr<5>(viterbi), fwd_ptr<6>(viterbi), fwd_ptr<7>(viterbi), fwd_ptr<8>(viterbi)};
+  const int sms = sms_of_current();
+  int best = 1;
+  int64_t best_cost = INT64_MAX;
+  for (int ns = 1; ns <= 8; ++ns) {
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ks[ns - 1], kHW * 32, 0) != cudaSuccess || per_sm < 1)
+      continue;
+    const int64_t warps = (n + ns - 1) / ns;
+    const int64_t wave = (int64_t)sms * per_sm * kHW;
+    const int64_t cost = ((warps + wave - 1) / wave) * ns;
+    if (cost < best_cost) { best_cost = cost; best = ns; }
+  }
+  *kern = ks[best - 1];
+  return best;
+}
+
 }  // namespace
 
 cudaError_t hmm_forward(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
   if (H.n == 0) return cudaSuccess;
+  void* kern = nullptr;
+  const int ns = pick_ns(H.n, false, &kern);
+  const int64_t warps = (H.n + ns - 1) / ns;
+  HmmArgs h2 = H;
+  void* args[1] = {&h2};
   ++*launches;
-  k_forward<<<(unsigned)((H.n + kWarps - 1) / kWarps), kWarps * 32, 0, s>>>(H);
-  return cudaGetLastError();
+  return cudaLaunchKernel(kern, dim3((unsigned)((warps + kHW - 1) / kHW)), dim3(kHW * 32), args, 0, s);
 }
 
 cudaError_t hmm_viterbi(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
   if (H.n == 0) return cudaSuccess;
+  void* kern = nullptr;
+  const int ns = pick_ns(H.n, true, &kern);
+  const int64_t warps = (H.n + ns - 1) / ns;
+  HmmArgs h2 = H;
+  void* args[1] = {&h2};
   ++*launches;
-  k_viterbi<<<(unsigned)((H.n + kWarps - 1) / kWarps), kWarps * 32, 0, s>>>(H);
-  return cudaGetLastError();
+  return cudaLaunchKernel(kern, dim3((unsigned)((warps + kHW - 1) / kHW)), dim3(kHW * 32), args, 0, s);
 }
 
 cudaError_t hmm_viterbi_traceback(const HmmArgs& H, int64_t first, int64_t count, uint8_t* out, int64_t stride,

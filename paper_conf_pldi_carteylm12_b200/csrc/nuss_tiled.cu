@@ -216,7 +216,8 @@ __device__ void tiled_traceback(const Tab& tab, const uint8_t* x, const uint8_t*
   if (lane == 0) { stack[0] = 0; stack[1] = n - 1; }
   sp = 2;
   __syncwarp();
-  while (sp > 0) {
+  int guard = 4 * n + 8;  // every pop consumes a pair or an end of an interval: bounded by 4n
+  while (sp > 0 && --guard > 0) {
     const int j = stack[sp - 1], i = stack[sp - 2];
     sp -= 2;
     __syncwarp();
@@ -233,15 +234,15 @@ __device__ void tiled_traceback(const Tab& tab, const uint8_t* x, const uint8_t*
         const unsigned m = __ballot_sync(0xffffffffu, hit);
         if (m) kk = k0 + __ffs(m) - 1;
       }
-      action = 4;
+      action = kk >= 0 ? 4 : 0;  // 0: inconsistent table (cannot happen); stop expanding
     }
     if (lane == 0) {
       if (action == 1) { stack[sp] = i + 1; stack[sp + 1] = j; }
       else if (action == 2) { stack[sp] = i; stack[sp + 1] = j - 1; }
       else if (action == 3) { db[i] = '('; db[j] = ')'; stack[sp] = i + 1; stack[sp + 1] = j - 1; }
-      else { stack[sp] = kk + 1; stack[sp + 1] = j; stack[sp + 2] = i; stack[sp + 3] = kk; }
+      else if (action == 4) { stack[sp] = kk + 1; stack[sp + 1] = j; stack[sp + 2] = i; stack[sp + 3] = kk; }
     }
-    sp += (action == 4) ? 4 : 2;
+    sp += (action == 4) ? 4 : (action == 0 ? 0 : 2);
     __syncwarp();
   }
 }

@@ -95,7 +95,8 @@ __device__ void nuss_traceback(const int16_t* U, const int16_t* L, const uint8_t
   auto gam = [&](int i, int j) -> int { return (j - i < 1) ? 0 : (int)U[ustart(i, n) + (j - i)]; };
   int sp = 0;
   stack[sp++] = 0; stack[sp++] = n - 1;
-  while (sp > 0) {
+  int guard = 4 * n + 8;
+  while (sp > 0 && --guard > 0) {
     const int j = stack[--sp], i = stack[--sp];
     if (j - i < 1) continue;
     const int v = gam(i, j);
