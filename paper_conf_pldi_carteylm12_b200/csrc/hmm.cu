@@ -295,8 +295,9 @@ int sms_of_current() {
 template <int NS>
 void* fwd_ptr(bool viterbi) { return viterbi ? (void*)k_viterbi<NS> : (void*)k_forward<NS>; }
 
-// Sequences per warp: minimise (waves of resident warps) x NS, the per-warp time
-// being proportional to NS; ties go to the smaller NS (more warps in flight).
+// Sequences per warp: minimise (waves of resident warps) x (NS + 2): the per-warp
+// time grows with NS plus a latency term (the per-step reduction and the
+// broadcast) that NS independent sequences share; ties go to the smaller NS.
 int pick_ns(int64_t n, bool viterbi, void** kern) {
   void* ks[8] = {fwd_ptr<1>(viterbi), fwd_ptr<2>(viterbi), fwd_ptr<3>(viterbi), fwd_ptr<4>(viterbi),
                  fwd_ptr<5>(viterbi), fwd_ptr<6>(viterbi), fwd_ptr<7>(viterbi), fwd_ptr<8>(viterbi)};
@@ -309,7 +310,7 @@ int pick_ns(int64_t n, bool viterbi, void** kern) {
       continue;
     const int64_t warps = (n + ns - 1) / ns;
     const int64_t wave = (int64_t)sms * per_sm * kHW;
-    const int64_t cost = ((warps + wave - 1) / wave) * ns;
+    const int64_t cost = ((warps + wave - 1) / wave) * (ns + 2);
     if (cost < best_cost) { best_cost = cost; best = ns; }
   }
   *kern = ks[best - 1];

@@ -42,7 +42,8 @@ namespace {
 constexpr int T = 32;
 constexpr int kTileWords = T * T;      // int16 per tile record half
 constexpr int kRec = 2 * kTileWords;   // int16 per tile record (UT + L)
-constexpr int kCtaWarps = 16;
+constexpr int kCtaWarps = 8;   // batch driver: two CTAs (two sequences) per SM
+constexpr int kGridWarps = 16; // grid driver
 constexpr int kCS = T + 1;             // row stride of in-tile buffers
 constexpr int kGridMin = 1024;         // single problems longer than this use the whole grid
 
@@ -127,13 +128,21 @@ __device__ void product_unit(const Tab& tab, int I, int J, int K0, int K1, int* 
     }
 }
 
+constexpr int kVS = 40;                  // int16 row stride of the in-tile operand copies (80 B)
+constexpr int16_t kNeg = -16000;         // masks split points outside a cell's range
+
 struct InTileBuf {
-  int cur[T * kCS];        // CUR[r][c]
-  int16_t uii[T * kCS];    // U(I,I)[r][k]
-  int16_t ljj[T * kCS];    // L(J,J)[k][c]
-  int below[T];        // U(I+1,J)[0][c]
-  int left[T];         // U(I,J-1)[r][31]
-  int corner;          // gamma(32I+32, 32J-1)
+  union {
+    struct {
+      int16_t uiis[T * kVS];  // UIIs[r][m] = U(I,I)[r][m-1] for m >= r+2, kNeg below (m = 0..32)
+      int16_t ct[T * kVS];    // CT[c][m]  = CUR[m][c] (m < 32), CT[c][32] = U(I+1,J)[0][c]
+      int16_t cr[T * kVS];    // CR[r][k]  = CUR[r][k]
+      int16_t lt[T * kVS];    // LT[c][k]  = L(J,J)[k][c] for k < c, kNeg otherwise
+    };
+    int cur[T * kCS];         // diagonal tiles only: CUR[r][c]
+  };
+  int left[T];                // U(I,J-1)[r][31]
+  int corner;                 // gamma(32I+32, 32J-1)
 };
 
 __device__ __forceinline__ bool pairable(const uint8_t* x, const uint8_t* pm, int n, int i, int j, int h) {
@@ -141,9 +150,14 @@ __device__ __forceinline__ bool pairable(const uint8_t* x, const uint8_t* pm, in
 }
 
 // Phase B: finalise tile (I,J) from C (max of the middle products), write UT/L records.
+// Off-diagonal tiles run the 63 local anti-diagonals with one cell per lane; each cell's
+// split points inside tiles I and J are reduced 8 at a time with VIADDMNMX.S16x2 over
+// masked operand copies (warp-uniform chunk ranges, no divergence).
 __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, InTileBuf& B, const uint8_t* x,
                         const uint8_t* pm, int n, int h, int lane) {
   const int i0 = I * T, j0 = J * T;
+  int16_t* ut = tab.UT(I, J);
+  int16_t* l = tab.L(I, J);
   if (I == J) {
     // diagonal tile: the cell-level recursion inside one 32x32 triangle
     for (int q = lane; q < T * kCS; q += 32) B.cur[q] = 0;
@@ -158,104 +172,178 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
       }
       __syncwarp();
     }
-  } else {
-    const int16_t* utii = tab.UT(I, I);
-    const int16_t* ljj = tab.L(J, J);
-    const int16_t* utb = tab.UT(I + 1, J);
-    const int16_t* utl = tab.UT(I, J - 1);
-    for (int q = lane; q < T * T; q += 32) {
-      const int a = q / T, b = q % T;
-      B.uii[a * kCS + b] = utii[b * T + a];  // U(I,I)[a][b]
-      B.ljj[a * kCS + b] = ljj[q];           // L(J,J)[a][b]
-      B.cur[a * kCS + b] = has_c ? C[q] : 0;
-    }
-    B.below[lane] = utb[lane * T + 0];
-    B.left[lane] = utl[(T - 1) * T + lane];
-    if (lane == 0) B.corner = (I + 1 <= J - 1) ? tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
-    __syncwarp();
-    for (int dl = -(T - 1); dl <= T - 1; ++dl) {
-      const int r = lane, c = lane + dl;
-      if (c >= 0 && c < T) {
-        int v = B.cur[r * kCS + c];
-        const int bl = (r < T - 1) ? B.cur[(r + 1) * kCS + c] : B.below[c];
-        const int le = (c > 0) ? B.cur[r * kCS + c - 1] : B.left[r];
-        v = max(v, max(bl, le));
-        if (pairable(x, pm, n, i0 + r, j0 + c, h)) {
-          int inner;
-          if (r < T - 1 && c > 0) inner = B.cur[(r + 1) * kCS + c - 1];
-          else if (r == T - 1 && c > 0) inner = B.below[c - 1];
-          else if (r < T - 1 && c == 0) inner = B.left[r + 1];
-          else inner = B.corner;
-          v = max(v, inner + 1);
-        }
-        // split k inside tile I: gamma(i,k) + gamma(k+1,j), k = i0+r+1 .. i0+31
-        for (int k = r + 1; k < T; ++k)
-          v = max(v, (int)B.uii[r * kCS + k] + (k < T - 1 ? B.cur[(k + 1) * kCS + c] : B.below[c]));
-        // split k inside tile J: k = j0 .. j-1
-        for (int k = 0; k < c; ++k) v = max(v, B.cur[r * kCS + k] + (int)B.ljj[k * kCS + c]);
-        B.cur[r * kCS + c] = v;
+    for (int r = 0; r < T; ++r) ut[lane * T + r] = (int16_t)B.cur[r * kCS + lane];
+    for (int k = 0; k < T - 1; ++k) l[k * T + lane] = (int16_t)B.cur[(k + 1) * kCS + lane];
+    l[(T - 1) * T + lane] = 0;
+    return;
+  }
+  const int16_t* utii = tab.UT(I, I);
+  const int16_t* ljj = tab.L(J, J);
+  const int16_t* utb = tab.UT(I + 1, J);
+  const int16_t* utl = tab.UT(I, J - 1);
+  for (int q = lane; q < T * kVS; q += 32) {
+    const int a = q / kVS, b = q % kVS;  // row a, column b of each copy
+    // UIIs[a][b] = U(I,I)[a][b-1] = UT(I,I)[b-1][a]
+    B.uiis[q] = (b >= a + 2 && b <= T) ? utii[(b - 1) * T + a] : kNeg;
+    // CT[a][b] = CUR[b][a] (initially C), CT[a][32] = below
+    B.ct[q] = (b < T) ? (int16_t)(has_c ? __ldcg(C + b * T + a) : 0) : (b == T ? utb[a * T + 0] : (int16_t)0);
+    B.cr[q] = (b < T) ? (int16_t)(has_c ? __ldcg(C + a * T + b) : 0) : (int16_t)0;
+    B.lt[q] = (b < a) ? ljj[b * T + a] : kNeg;
+  }
+  B.left[lane] = utl[(T - 1) * T + lane];
+  if (lane == 0) B.corner = (I + 1 <= J - 1) ? tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
+  __syncwarp();
+  const int r = lane;
+  const uint4* urow = reinterpret_cast<const uint4*>(B.uiis + r * kVS);
+  const uint4* crow = reinterpret_cast<const uint4*>(B.cr + r * kVS);
+  for (int dl = -(T - 1); dl <= T - 1; ++dl) {
+    const int c = r + dl;
+    const int rmin = max(0, -dl), cmax = min(T - 1, T - 1 + dl);
+    const int q0 = (rmin + 2) / 8;       // first K=I chunk any lane needs
+    const int q1 = (cmax + 7) / 8;       // K=J chunks 0 .. q1-1
+    if (c >= 0 && c < T) {
+      const uint4* ccol = reinterpret_cast<const uint4*>(B.ct + c * kVS);
+      const uint4* lcol = reinterpret_cast<const uint4*>(B.lt + c * kVS);
+      uint32_t acc = 0;
+      for (int q = q0; q <= 4; ++q) {  // k + 1 = m in [r+2, 32]
+        const uint4 a = urow[q], b = ccol[q];
+        acc = __viaddmax_s16x2(a.x, b.x, acc);
+        acc = __viaddmax_s16x2(a.y, b.y, acc);
+        acc = __viaddmax_s16x2(a.z, b.z, acc);
+        acc = __viaddmax_s16x2(a.w, b.w, acc);
       }
-      __syncwarp();
+      for (int q = 0; q < q1; ++q) {   // k in [0, c)
+        const uint4 a = crow[q], b = lcol[q];
+        acc = __viaddmax_s16x2(a.x, b.x, acc);
+        acc = __viaddmax_s16x2(a.y, b.y, acc);
+        acc = __viaddmax_s16x2(a.z, b.z, acc);
+        acc = __viaddmax_s16x2(a.w, b.w, acc);
+      }
+      int v = max((int)(int16_t)(acc & 0xffffu), (int)(int16_t)(acc >> 16));
+      v = max(v, (int)B.cr[r * kVS + c]);                              // C (middle products)
+      v = max(v, (int)B.ct[c * kVS + r + 1]);                          // gamma(i+1, j) (row 32 = below)
+      v = max(v, c > 0 ? (int)B.cr[r * kVS + c - 1] : B.left[r]);     // gamma(i, j-1)
+      if (pairable(x, pm, n, i0 + r, j0 + c, h)) {
+        const int inner = c > 0 ? (int)B.ct[(c - 1) * kVS + r + 1] : (r < T - 1 ? B.left[r + 1] : B.corner);
+        v = max(v, inner + 1);
+      }
+      B.cr[r * kVS + c] = (int16_t)v;
+      B.ct[c * kVS + r] = (int16_t)v;
     }
+    __syncwarp();
   }
   // write the records: UT[c][r] and L[k][c] = gamma(i0+k+1, j0+c)
-  int16_t* ut = tab.UT(I, J);
-  int16_t* l = tab.L(I, J);
-  for (int r = 0; r < T; ++r) ut[lane * T + r] = (int16_t)B.cur[r * kCS + lane];
-  for (int k = 0; k < T - 1; ++k) l[k * T + lane] = (int16_t)B.cur[(k + 1) * kCS + lane];
-  l[(T - 1) * T + lane] = (I == J) ? 0 : (int16_t)B.below[lane];
+  const uint32_t* ctw = reinterpret_cast<const uint32_t*>(B.ct + lane * kVS);
+  uint32_t* utw = reinterpret_cast<uint32_t*>(ut + lane * T);
+#pragma unroll
+  for (int q = 0; q < T / 2; ++q) utw[q] = ctw[q];
+  for (int k = 0; k < T - 1; ++k) l[k * T + lane] = B.ct[lane * kVS + k + 1];
+  l[(T - 1) * T + lane] = B.ct[lane * kVS + T];
 }
 
-// Canonical traceback (DESIGN.md R-TB-NUSS) by one warp: the split search is lane-parallel.
-__device__ void tiled_traceback(const Tab& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
-                                int* stack, int lane) {
-  for (int k = lane; k < n; k += 32) db[k] = '.';
-  __syncwarp();
+__device__ __forceinline__ void tb_lock(int* l) {
+  while (atomicCAS(l, 0, 1) != 0) __nanosleep(32);
+  __threadfence_block();
+}
+__device__ __forceinline__ void tb_unlock(int* l) {
+  __threadfence_block();
+  atomicExch(l, 0);
+}
+
+// Canonical traceback (DESIGN.md R-TB-NUSS: Durbin order, smallest split k) by ALL warps
+// of the CTA. Intervals live on a shared worklist (`stk` in global memory, counters `ctl`
+// in shared memory); a warp follows one interval through its unpaired / pair steps and
+// pushes the right part of every split, so independent branches of the structure are
+// traced concurrently (the set of pairs does not depend on the order). One step costs
+// one round trip: lanes 0-3 load gamma(i,j), gamma(i+1,j), gamma(i,j-1), gamma(i+1,j-1)
+// while all lanes load the first 32 split candidates.
+__device__ void cta_traceback(const Tab& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
+                              int2* stk, int cap, int* ctl, int lane) {
+  for (int k = threadIdx.x; k < n; k += blockDim.x) db[k] = '.';
+  if (threadIdx.x == 0) {
+    ctl[0] = 0;  // stack top
+    ctl[1] = 0;  // warps holding an interval
+    ctl[2] = 0;  // lock
+    if (n > 1) { stk[0] = make_int2(0, n - 1); ctl[0] = 1; }
+  }
+  __threadfence_block();
+  __syncthreads();
   if (n <= 1) return;
-  int sp = 0;
-  if (lane == 0) { stack[0] = 0; stack[1] = n - 1; }
-  sp = 2;
-  __syncwarp();
-  int guard = 4 * n + 8;  // every pop consumes a pair or an end of an interval: bounded by 4n
-  while (sp > 0 && --guard > 0) {
-    const int j = stack[sp - 1], i = stack[sp - 2];
-    sp -= 2;
-    __syncwarp();
-    if (j - i < 1) continue;
-    const int v = tab.gamma(i, j);
-    int action = 0, kk = -1;
-    if (v == tab.gamma(i + 1, j)) action = 1;
-    else if (v == tab.gamma(i, j - 1)) action = 2;
-    else if (pairable(x, pm, n, i, j, h) && v == tab.gamma(i + 1, j - 1) + 1) action = 3;
-    else {
-      for (int k0 = i + 1; k0 < j && kk < 0; k0 += 32) {
-        const int k = k0 + lane;
-        const bool hit = k < j && v == tab.gamma(i, k) + tab.gamma(k + 1, j);
-        const unsigned m = __ballot_sync(0xffffffffu, hit);
+  const unsigned full = 0xffffffffu;
+  for (;;) {
+    int i = 0, j = -1, done = 0;
+    if (lane == 0) {
+      for (;;) {
+        tb_lock(&ctl[2]);
+        const int t = ctl[0];
+        if (t > 0) {
+          const int2 iv = stk[t - 1];
+          ctl[0] = t - 1;
+          ctl[1] += 1;
+          i = iv.x; j = iv.y;
+        }
+        const int busy = ctl[1];
+        tb_unlock(&ctl[2]);
+        if (t > 0) break;
+        if (busy == 0) { done = 1; break; }
+        __nanosleep(100);
+      }
+    }
+    done = __shfl_sync(full, done, 0);
+    if (done) break;
+    i = __shfl_sync(full, i, 0);
+    j = __shfl_sync(full, j, 0);
+    int guard = 4 * n + 8;
+    while (j - i >= 1 && --guard > 0) {
+      int a = 0;
+      if (lane == 0) a = tab.gamma(i, j);
+      else if (lane == 1) a = tab.gamma(i + 1, j);
+      else if (lane == 2) a = tab.gamma(i, j - 1);
+      else if (lane == 3) a = tab.gamma(i + 1, j - 1);
+      const int k = i + 1 + lane;
+      const int sk = (k < j) ? tab.gamma(i, k) + tab.gamma(k + 1, j) : -1;
+      const int v = __shfl_sync(full, a, 0), g1 = __shfl_sync(full, a, 1);
+      const int g2 = __shfl_sync(full, a, 2), g3 = __shfl_sync(full, a, 3);
+      if (v == g1) { i += 1; continue; }
+      if (v == g2) { j -= 1; continue; }
+      if (pairable(x, pm, n, i, j, h) && v == g3 + 1) {
+        if (lane == 0) { db[i] = '('; db[j] = ')'; }
+        i += 1; j -= 1;
+        continue;
+      }
+      int kk = -1;
+      unsigned m = __ballot_sync(full, sk == v);
+      if (m) kk = i + __ffs(m);
+      for (int k0 = i + 33; kk < 0 && k0 < j; k0 += 32) {
+        const int kq = k0 + lane;
+        m = __ballot_sync(full, kq < j && v == tab.gamma(i, kq) + tab.gamma(kq + 1, j));
         if (m) kk = k0 + __ffs(m) - 1;
       }
-      action = kk >= 0 ? 4 : 0;  // 0: inconsistent table (cannot happen); stop expanding
+      if (kk < 0) break;  // inconsistent table: cannot happen
+      if (lane == 0) {    // right part to the worklist, keep following the left part
+        tb_lock(&ctl[2]);
+        if (ctl[0] < cap) { stk[ctl[0]] = make_int2(kk + 1, j); ctl[0] += 1; }
+        tb_unlock(&ctl[2]);
+      }
+      j = kk;
     }
     if (lane == 0) {
-      if (action == 1) { stack[sp] = i + 1; stack[sp + 1] = j; }
-      else if (action == 2) { stack[sp] = i; stack[sp + 1] = j - 1; }
-      else if (action == 3) { db[i] = '('; db[j] = ')'; stack[sp] = i + 1; stack[sp + 1] = j - 1; }
-      else if (action == 4) { stack[sp] = kk + 1; stack[sp + 1] = j; stack[sp + 2] = i; stack[sp + 3] = kk; }
+      tb_lock(&ctl[2]);
+      ctl[1] -= 1;
+      tb_unlock(&ctl[2]);
     }
-    sp += (action == 4) ? 4 : (action == 0 ? 0 : 2);
-    __syncwarp();
   }
 }
 
 // ------------------------------------------------------------------ batch driver
-__global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
+__global__ void __launch_bounds__(kCtaWarps * 32, 2) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint8_t pm[16];
   __shared__ uint8_t xs[4096];
+  __shared__ int tbctl[4];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
-  int* Cs = reinterpret_cast<int*>(smem);                                   // [kCtaWarps][1024]
-  uint8_t* wbuf = smem + sizeof(int) * kCtaWarps * T * T;                    // per-warp scratch
+  uint8_t* wbuf = smem;                                                      // per-warp scratch
   const size_t wbytes = sizeof(InTileBuf) > (T * T * 4 + T * T * 2) ? sizeof(InTileBuf) : (T * T * 4 + T * T * 2);
   uint8_t* mine = wbuf + warp * ((wbytes + 15) & ~size_t(15));
   uint32_t* As = reinterpret_cast<uint32_t*>(mine);
@@ -263,8 +351,11 @@ __global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_cta(NussArgs A
   InTileBuf& IB = *reinterpret_cast<InTileBuf*>(mine);
   Tab tab;
   tab.base = reinterpret_cast<int16_t*>(A.scratch) + (int64_t)blockIdx.x * slot_elems;
+  // per-slot C tiles (global, L2 atomics) after the tables, then the traceback stacks
+  int* Cs = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * slot_elems) +
+            (int64_t)blockIdx.x * kCtaWarps * T * T;
   int* stack = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * slot_elems) +
-               (int64_t)blockIdx.x * (4 * A.max_len + 8);
+               (int64_t)gridDim.x * kCtaWarps * T * T + (int64_t)blockIdx.x * (4 * A.max_len + 8);
   for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
     const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
     __syncthreads();
@@ -287,7 +378,7 @@ __global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_cta(NussArgs A
             const int t = u / chunks, ch = u % chunks;
             const int I = g0 + t, J = I + D;
             const int K0 = I + 1 + (ksteps * ch) / chunks, K1 = I + 1 + (ksteps * (ch + 1)) / chunks;
-            product_unit<true>(tab, I, J, K0, K1, Cs + t * T * T, As, Bs, lane);
+            product_unit<false>(tab, I, J, K0, K1, Cs + t * T * T, As, Bs, lane);
           }
           __syncthreads();
         }
@@ -299,19 +390,18 @@ __global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_cta(NussArgs A
         __syncthreads();
       }
     }
-    if (warp == 0) {
-      const int sc = n <= 1 ? 0 : tab.gamma(0, n - 1);
-      if (lane == 0) A.scores[p] = sc;
-      if (A.db) {
-        tiled_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, lane);
-        if (lane == 0) A.db_len[p] = n;
-      }
+    if (threadIdx.x == 0) {
+      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
+      if (A.db) A.db_len[p] = n;
     }
+    if (A.db)
+      cta_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack),
+                    2 * (int)A.max_len + 4, tbctl, lane);
   }
 }
 
 // ------------------------------------------------------------------ grid driver (one large problem)
-__global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_grid(NussArgs A, int64_t p) {
+__global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_tiled_grid(NussArgs A, int64_t p) {
   cg::grid_group grid = cg::this_grid();
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint8_t pm[16];
@@ -331,8 +421,8 @@ __global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_grid(NussArgs 
   tab.nt = nt;
   int* Cg = reinterpret_cast<int*>(tab.base + tiles_of(nt) * kRec);  // 2 x nt x 1024 int32
   int* stack = Cg + 2 * (int64_t)nt * T * T;
-  const int64_t gw = (int64_t)blockIdx.x * kCtaWarps + warp;
-  const int64_t nw = (int64_t)gridDim.x * kCtaWarps;
+  const int64_t gw = (int64_t)blockIdx.x * kGridWarps + warp;
+  const int64_t nw = (int64_t)gridDim.x * kGridWarps;
   // C buffers start at zero
   for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T;
        q += (int64_t)gridDim.x * blockDim.x)
@@ -369,13 +459,15 @@ __global__ void __launch_bounds__(kCtaWarps * 32, 1) k_nuss_tiled_grid(NussArgs 
     }
     grid.sync();
   }
-  if (gw == 0) {
-    const int sc = n <= 1 ? 0 : tab.gamma(0, n - 1);
-    if (lane == 0) A.scores[p] = sc;
-    if (A.db) {
-      tiled_traceback(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, stack, lane);
-      if (lane == 0) A.db_len[p] = n;
+  if (blockIdx.x == 0) {
+    __shared__ int tbctl[4];
+    if (threadIdx.x == 0) {
+      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
+      if (A.db) A.db_len[p] = n;
     }
+    if (A.db)
+      cta_traceback(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack),
+                    2 * n + 4, tbctl, lane);
   }
 }
 
@@ -400,8 +492,8 @@ int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
   if (n == 1 && max_len > kGridMin) {
     return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
   }
-  const int64_t grid = std::min<int64_t>(n, num_sms_t(device));
-  return grid * (tiles_of(nt) * kRec * 2 + stack_bytes) + 256;
+  const int64_t grid = std::min<int64_t>(n, 2 * (int64_t)num_sms_t(device));
+  return grid * (tiles_of(nt) * kRec * 2 + (int64_t)kCtaWarps * T * T * 4 + stack_bytes) + 256;
 }
 
 cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
@@ -411,24 +503,24 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
   const int sms = num_sms_t(dev);
   const int nt = (int)((A.max_len + T - 1) / T);
   if (A.n == 1 && A.max_len > kGridMin) {
-    const size_t smem = kCtaWarps * warp_bytes();
+    const size_t smem = kGridWarps * warp_bytes();
     cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_grid, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int per_sm = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_nuss_tiled_grid, kCtaWarps * 32, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_nuss_tiled_grid, kGridWarps * 32, smem);
     if (e != cudaSuccess) return e;
     if (per_sm < 1) return cudaErrorInvalidConfiguration;
     NussArgs a2 = A;
     int64_t p = 0;
     void* args[2] = {&a2, &p};
     ++*launches;
-    return cudaLaunchCooperativeKernel((void*)k_nuss_tiled_grid, sms, kCtaWarps * 32, args, smem, s);
+    return cudaLaunchCooperativeKernel((void*)k_nuss_tiled_grid, sms, kGridWarps * 32, args, smem, s);
   }
   if (A.max_len > 4096) return cudaErrorInvalidValue;  // batch path keeps the sequence in shared memory
-  const size_t smem = sizeof(int) * kCtaWarps * T * T + kCtaWarps * warp_bytes();
+  const size_t smem = kCtaWarps * warp_bytes();
   cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  const int64_t grid = std::min<int64_t>(A.n, sms);
+  const int64_t grid = std::min<int64_t>(A.n, 2 * (int64_t)sms);
   ++*launches;
   k_nuss_tiled_cta<<<(unsigned)grid, kCtaWarps * 32, smem, s>>>(A, tiles_of(nt) * kRec);
   return cudaGetLastError();

@@ -15,11 +15,11 @@
 // state (all lanes inside the table) carries no bounds checks.
 //
 // Traceback retention without per-cell direction codes: the forward pass
-// stores checkpoints of G — the bottom row of every 32-row band (every 4th
-// lane, every column) and every 32nd column (all rows) — plus each lane's
-// best per 32-column slab (0.19 B/cell, coalesced). k_sw16_tb then recomputes
-// only the 32x32 blocks the canonical traceback needs (warp-parallel
-// wavefront, one row per lane) and walks them with the oracle's tie-break
+// stores checkpoints of G — the bottom row of every 16-row band (odd lanes,
+// every column) and every 32nd column (all rows) — plus each lane's best per
+// 32-column slab (0.25 B/cell, coalesced). k_sw16_tb then recomputes only the
+// 32x32 blocks the canonical traceback needs (one row per lane, the two
+// 16-row halves in parallel) and walks them with the oracle's tie-break
 // (diag > up > left, stop at H = 0; end cell = first maximum in row-major order).
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -31,9 +31,10 @@ namespace {
 
 constexpr int kRows = 8;              // rows per lane
 constexpr int kStrip = 32 * kRows;    // rows per strip
-constexpr int kBand = 32;             // checkpoint band height (four lanes)
+constexpr int kBand = 16;             // checkpoint band height (two lanes)
 constexpr int kLanesPerBand = kBand / kRows;
 constexpr int kBandsPerStrip = kStrip / kBand;
+constexpr int kBlk = 32;              // traceback recompute block height (two independent bands)
 constexpr int kSlab = 32;             // checkpoint column spacing
 constexpr int kHS = kSlab + 2;        // row stride of the recomputed block (conflict-free anti-diagonals)
 constexpr int kDead = -100;           // profile value for rows/columns outside a problem
@@ -97,7 +98,7 @@ __device__ __forceinline__ void sw_step(FwdState& S, int j, int lbm, int lane, u
   S.bbest = __vimax3_s16x2(S.bbest, S.G[6], S.G[7]);
   S.last = g;
   if (TB) {
-    if ((lane & (kLanesPerBand - 1)) == kLanesPerBand - 1) rowck_p[j - 1] = g;  // bottom row of a 32-row band
+    if ((lane & (kLanesPerBand - 1)) == kLanesPerBand - 1) rowck_p[j - 1] = g;  // bottom row of a 16-row band
     if ((j & (kSlab - 1)) == 0 || j == lbm) {
       const int sl = (j - 1) / kSlab;
       if ((j & (kSlab - 1)) == 0) {
@@ -206,6 +207,7 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
       }
       __syncwarp();
     }
+#pragma unroll 2
     for (; k < k_steady1; ++k) {
       const int j = k - lane + 1;
       sw_step<TB, false>(S, j, lbm, lane, NEG_G2, bnd, from_bnd, offA, offB, pA8, pB8, rowck_p, colck_p, slab_p);
@@ -255,35 +257,47 @@ struct TbView {
   }
 };
 
-// Recompute block (band, slab) into Hb[(r+1)*kHS + c] (row 0 / column 0 = boundaries); one row per lane.
-__device__ void recompute_block(const TbView& V, const uint8_t* a, const uint8_t* b, int band, int slab, int* Hb,
-                                const int8_t* sig_s, int asz, int g) {
+// Recompute the 32-row block `blk` x slab into Hb[(r+1)*kHS + c] (row 0 / column 0 =
+// boundaries); one row per lane. The two 16-row halves are independent given the
+// checkpoint row between them, so lanes 0-15 and 16-31 run concurrently (47 steps).
+__device__ void recompute_block(const TbView& V, const uint8_t* a, const uint8_t* b, int blk, int slab, int* Hb,
+                                int* mid, const int8_t* sig_s, int asz, int g) {
   const int lane = threadIdx.x & 31;
-  const int R0 = band * kBand, C0 = slab * kSlab;
-  for (int c = lane; c <= kSlab; c += 32) Hb[c] = (C0 + c <= V.lb) ? V.top_h(band, C0 + c) : 0;
+  const int R0 = blk * kBlk, C0 = slab * kSlab;
+  const int band0 = R0 / kBand;
+  for (int c = lane; c <= kSlab; c += 32) {
+    Hb[c] = (C0 + c <= V.lb) ? V.top_h(band0, C0 + c) : 0;
+    mid[c] = (C0 + c <= V.lb) ? V.top_h(band0 + 1, C0 + c) : 0;
+  }
   const int i = R0 + lane + 1;
   const bool row_ok = i <= V.la;
   int left = row_ok ? V.left_h(i, slab) : 0;
   Hb[(lane + 1) * kHS] = left;
   __syncwarp();
+  const int hl = lane & (kBand - 1);  // row within the half
+  const int* top = (lane < kBand) ? Hb : mid;
   const int ai = row_ok ? a[i - 1] : 0;
   const int8_t* srow = sig_s + ai * asz;
+  const uint8_t* bb = b + C0 - 1;      // bb[c] = b[C0 + c - 1]
+  const int cmax = min(kSlab, V.lb - C0);  // live columns of this slab
+  int* hrow = Hb + (lane + 1) * kHS;
   int diag = __shfl_up_sync(0xffffffffu, left, 1);
-  if (lane == 0) diag = Hb[0];
+  if (hl == 0) diag = top[0];
   int last = 0;
-  for (int s = 0; s < kSlab + 31; ++s) {
-    const int c = s - lane + 1;
+  // branch-free wavefront: every lane evaluates every step, out-of-range steps are masked
+#pragma unroll 4
+  for (int s = 0; s < kSlab + kBand - 1; ++s) {
+    const int c = s - hl + 1;
     const int from = __shfl_up_sync(0xffffffffu, last, 1);
-    if (c >= 1 && c <= kSlab) {
-      const int up = (lane == 0) ? Hb[c] : from;
-      const int j = C0 + c;
-      int h = 0;
-      if (row_ok && j <= V.lb) h = max(max(diag + srow[b[j - 1]], 0), max(up, left) - g);
-      Hb[(lane + 1) * kHS + c] = h;
-      diag = up;
-      left = h;
-      last = h;
-    }
+    const bool in = (unsigned)(c - 1) < (unsigned)kSlab;
+    const int cc = in ? c : 1;
+    const int up = (hl == 0) ? top[cc] : from;
+    int h = max(max(diag + srow[bb[cc]], 0), max(up, left) - g);
+    h = (row_ok && cc <= cmax) ? h : 0;
+    if (in) hrow[cc] = h;
+    diag = in ? up : diag;
+    left = in ? h : left;
+    last = in ? h : last;
   }
   __syncwarp();
 }
@@ -302,9 +316,10 @@ __global__ void __launch_bounds__(128) k_sw16_tb(Sw16Args A, int64_t first, int6
   V.A = &A;
   V.grp = p >> 1;
   V.half = (int)(p & 1);
-  uint8_t* wsm = tsm + (size_t)warp * (seq_bytes + (kBand + 1) * kHS * 4);
+  uint8_t* wsm = tsm + (size_t)warp * (seq_bytes + ((kBlk + 1) * kHS + kHS) * 4);
   int* Hb = reinterpret_cast<int*>(wsm);
-  uint8_t* a = wsm + (kBand + 1) * kHS * 4;
+  int* mid = Hb + (kBlk + 1) * kHS;
+  uint8_t* a = wsm + ((kBlk + 1) * kHS + kHS) * 4;
   V.la = (int)(A.a_off[p + 1] - A.a_off[p]);
   V.lb = (int)(A.b_off[p + 1] - A.b_off[p]);
   const int la = V.la, lb = V.lb, asz = A.asz, g = A.gap;
@@ -337,14 +352,14 @@ __global__ void __launch_bounds__(128) k_sw16_tb(Sw16Args A, int64_t first, int6
   }
   const int lane8 = band8 % 32, st8 = band8 / 32;
   // 2) first cell with H == best: recompute only the slabs of band8 holding the best,
-  //    within the 32-row checkpoint band that contains band8's rows
-  const int band = (st8 * kStrip + lane8 * kRows) / kBand;
+  //    within the 32-row block that contains band8's rows
+  const int band = (st8 * kStrip + lane8 * kRows) / kBlk;
   int myc = 1 << 30;
   for (int sl = 0; sl < nsl; ++sl) {
     const uint32_t v = A.slabbest[((V.grp * A.strips_max + st8) * A.nslab_max + sl) * 32 + lane8];
     if (half16(v, V.half) + g != best) continue;
-    recompute_block(V, a, b, band, sl, Hb, sig_s, asz, g);
-    const int i = band * kBand + lane + 1;
+    recompute_block(V, a, b, band, sl, Hb, mid, sig_s, asz, g);
+    const int i = band * kBlk + lane + 1;
     if (myc == (1 << 30) && i <= la)
       for (int c = 1; c <= kSlab; ++c) {
         const int j = sl * kSlab + c;
@@ -355,16 +370,16 @@ __global__ void __launch_bounds__(128) k_sw16_tb(Sw16Args A, int64_t first, int6
   const unsigned hm = __ballot_sync(0xffffffffu, myc != (1 << 30));
   const int rowl = __ffs(hm) - 1;
   const int ej = __shfl_sync(0xffffffffu, myc, rowl < 0 ? 0 : rowl);
-  const int ei = band * kBand + rowl + 1;
+  const int ei = band * kBlk + rowl + 1;
   // 3) walk back block by block
   int i = ei, j = ej, h = best;
   int64_t n = 0;
   bool overflow = false;
   while (h > 0) {
-    const int bg = (i - 1) / kBand, sl = (j - 1) / kSlab;
-    recompute_block(V, a, b, bg, sl, Hb, sig_s, asz, g);
+    const int bg = (i - 1) / kBlk, sl = (j - 1) / kSlab;
+    recompute_block(V, a, b, bg, sl, Hb, mid, sig_s, asz, g);
     if (lane == 0) {
-      const int R0 = bg * kBand, C0 = sl * kSlab;
+      const int R0 = bg * kBlk, C0 = sl * kSlab;
       while (h > 0 && i > R0 && j > C0) {
         const int ri = i - R0, cj = j - C0;
         const int sub = sig_s[a[i - 1] * asz + b[j - 1]];
@@ -437,7 +452,7 @@ cudaError_t sw16_traceback(const Sw16Args& A, int64_t first, int64_t count, uint
                            int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches) {
   if (count == 0) return cudaSuccess;
   const int seq_bytes = (int)(((A.max_la + 15) & ~15) + ((A.max_lb + 15) & ~15));
-  const size_t smem = 4 * ((size_t)seq_bytes + (kBand + 1) * kHS * 4);
+  const size_t smem = 4 * ((size_t)seq_bytes + ((kBlk + 1) * kHS + kHS) * 4);
   cudaError_t e = cudaFuncSetAttribute(k_sw16_tb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   ++*launches;
