@@ -345,7 +345,9 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       if (p->kind == DP_HMM_FORWARD) {
         H.pi = p->d_pi; H.A = p->d_A; H.E = p->d_E;
         H.ll_out = static_cast<float*>(scores_out);
-        e = dpk::hmm_forward(H, s, &p->launches);
+        // the [batch x S] x [S x S] step on tcgen05 (SIMT fallback kernel via DP_HMM_SIMT=1)
+        e = dpk::hmm_forward_tc_supported(p->S) ? dpk::hmm_forward_tc(H, s, &p->launches)
+                                                 : dpk::hmm_forward(H, s, &p->launches);
       } else {
         H.lpi = p->d_lpi; H.lA = p->d_lA; H.lE = p->d_lE;
         H.vit_out = static_cast<int32_t*>(scores_out);

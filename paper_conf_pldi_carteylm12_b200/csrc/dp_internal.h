@@ -89,6 +89,8 @@ struct HmmArgs {
   int32_t* final_state;             // n
 };
 cudaError_t hmm_forward(const HmmArgs& a, cudaStream_t s, int64_t* launches);
+bool hmm_forward_tc_supported(int S);
+cudaError_t hmm_forward_tc(const HmmArgs& a, cudaStream_t s, int64_t* launches);  // tcgen05 path
 cudaError_t hmm_viterbi(const HmmArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t hmm_viterbi_traceback(const HmmArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                                   int32_t* out_len, cudaStream_t s, int64_t* launches);

@@ -181,17 +181,46 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
   const int16_t* ljj = tab.L(J, J);
   const int16_t* utb = tab.UT(I + 1, J);
   const int16_t* utl = tab.UT(I, J - 1);
-  for (int q = lane; q < T * kVS; q += 32) {
-    const int a = q / kVS, b = q % kVS;  // row a, column b of each copy
-    // UIIs[a][b] = U(I,I)[a][b-1] = UT(I,I)[b-1][a]
-    B.uiis[q] = (b >= a + 2 && b <= T) ? utii[(b - 1) * T + a] : kNeg;
-    // CT[a][b] = CUR[b][a] (initially C), CT[a][32] = below
-    B.ct[q] = (b < T) ? (int16_t)(has_c ? __ldcg(C + b * T + a) : 0) : (b == T ? utb[a * T + 0] : (int16_t)0);
-    B.cr[q] = (b < T) ? (int16_t)(has_c ? __ldcg(C + a * T + b) : 0) : (int16_t)0;
-    B.lt[q] = (b < a) ? ljj[b * T + a] : kNeg;
+  // Operand copies, built with coalesced global reads (lane = row/column of the copy)
+  // and 16-byte shared-memory stores of whole rows.
+  {
+    const int t = lane;
+    int16_t v[T];
+    auto store_row = [&](int16_t* dst, auto&& value) {
+      uint4* d = reinterpret_cast<uint4*>(dst + t * kVS);
+#pragma unroll
+      for (int w = 0; w < kVS / 8; ++w) {
+        uint32_t q[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int m0 = 8 * w + 2 * e;
+          q[e] = (uint32_t)(uint16_t)value(m0) | ((uint32_t)(uint16_t)value(m0 + 1) << 16);
+        }
+        d[w] = make_uint4(q[0], q[1], q[2], q[3]);
+      }
+    };
+    // UIIs[t][m] = U(I,I)[t][m-1] = UT(I,I)[m-1][t]  for t+2 <= m <= 32
+#pragma unroll
+    for (int k = 0; k < T; ++k) v[k] = utii[k * T + t];
+    store_row(B.uiis, [&](int m) -> int16_t { return (m >= t + 2 && m <= T) ? v[m - 1] : kNeg; });
+    // CT[t][m] = C[m][t] (m < 32), CT[t][32] = U(I+1,J)[0][t]
+#pragma unroll
+    for (int m = 0; m < T; ++m) v[m] = has_c ? (int16_t)__ldcg(C + m * T + t) : (int16_t)0;
+    const int16_t bel = utb[t * T + 0];
+    store_row(B.ct, [&](int m) -> int16_t { return m < T ? v[m] : (m == T ? bel : (int16_t)0); });
+    // LT[t][k] = L(J,J)[k][t] for k < t
+#pragma unroll
+    for (int k = 0; k < T; ++k) v[k] = ljj[k * T + t];
+    store_row(B.lt, [&](int k) -> int16_t { return (k < t && k < T) ? v[k] : kNeg; });
+    B.left[t] = utl[(T - 1) * T + t];
+    if (lane == 0) B.corner = (I + 1 <= J - 1) ? tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
+    __syncwarp();
+    // CR[t][k] = C[t][k] = CT[k][t] (transpose through shared memory)
+#pragma unroll
+    for (int k = 0; k < T; ++k) v[k] = B.ct[k * kVS + t];
+    __syncwarp();
+    store_row(B.cr, [&](int k) -> int16_t { return k < T ? v[k] : (int16_t)0; });
   }
-  B.left[lane] = utl[(T - 1) * T + lane];
-  if (lane == 0) B.corner = (I + 1 <= J - 1) ? tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
   __syncwarp();
   const int r = lane;
   const uint4* urow = reinterpret_cast<const uint4*>(B.uiis + r * kVS);
@@ -241,59 +270,26 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
   l[(T - 1) * T + lane] = B.ct[lane * kVS + T];
 }
 
-__device__ __forceinline__ void tb_lock(int* l) {
-  while (atomicCAS(l, 0, 1) != 0) __nanosleep(32);
-  __threadfence_block();
-}
-__device__ __forceinline__ void tb_unlock(int* l) {
-  __threadfence_block();
-  atomicExch(l, 0);
-}
-
-// Canonical traceback (DESIGN.md R-TB-NUSS: Durbin order, smallest split k) by ALL warps
-// of the CTA. Intervals live on a shared worklist (`stk` in global memory, counters `ctl`
-// in shared memory); a warp follows one interval through its unpaired / pair steps and
-// pushes the right part of every split, so independent branches of the structure are
-// traced concurrently (the set of pairs does not depend on the order). One step costs
-// one round trip: lanes 0-3 load gamma(i,j), gamma(i+1,j), gamma(i,j-1), gamma(i+1,j-1)
-// while all lanes load the first 32 split candidates.
-__device__ void cta_traceback(const Tab& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
-                              int2* stk, int cap, int* ctl, int lane) {
-  for (int k = threadIdx.x; k < n; k += blockDim.x) db[k] = '.';
-  if (threadIdx.x == 0) {
-    ctl[0] = 0;  // stack top
-    ctl[1] = 0;  // warps holding an interval
-    ctl[2] = 0;  // lock
-    if (n > 1) { stk[0] = make_int2(0, n - 1); ctl[0] = 1; }
-  }
-  __threadfence_block();
-  __syncthreads();
+// Canonical traceback (DESIGN.md R-TB-NUSS: Durbin order, smallest split k) by one
+// warp, right after the fill while the table is L2-resident. A warp follows an
+// interval through its unpaired / pair steps and pushes the right part of every
+// split on a stack in global memory. One step costs one round trip: lanes 0-3 load
+// gamma(i,j), gamma(i+1,j), gamma(i,j-1), gamma(i+1,j-1) while all lanes load the
+// first 32 split candidates.
+__device__ void warp_traceback(const Tab& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
+                               int2* stk, int lane) {
+  for (int k = lane; k < n; k += 32) db[k] = '.';
   if (n <= 1) return;
   const unsigned full = 0xffffffffu;
-  for (;;) {
-    int i = 0, j = -1, done = 0;
-    if (lane == 0) {
-      for (;;) {
-        tb_lock(&ctl[2]);
-        const int t = ctl[0];
-        if (t > 0) {
-          const int2 iv = stk[t - 1];
-          ctl[0] = t - 1;
-          ctl[1] += 1;
-          i = iv.x; j = iv.y;
-        }
-        const int busy = ctl[1];
-        tb_unlock(&ctl[2]);
-        if (t > 0) break;
-        if (busy == 0) { done = 1; break; }
-        __nanosleep(100);
-      }
-    }
-    done = __shfl_sync(full, done, 0);
-    if (done) break;
-    i = __shfl_sync(full, i, 0);
-    j = __shfl_sync(full, j, 0);
-    int guard = 4 * n + 8;
+  int sp = 1;
+  if (lane == 0) stk[0] = make_int2(0, n - 1);
+  __syncwarp();
+  int guard = 4 * n + 8;
+  while (sp > 0 && --guard > 0) {
+    const int2 iv = stk[sp - 1];
+    --sp;
+    int i = iv.x, j = iv.y;
+    __syncwarp();
     while (j - i >= 1 && --guard > 0) {
       int a = 0;
       if (lane == 0) a = tab.gamma(i, j);
@@ -320,17 +316,10 @@ __device__ void cta_traceback(const Tab& tab, const uint8_t* x, const uint8_t* p
         if (m) kk = k0 + __ffs(m) - 1;
       }
       if (kk < 0) break;  // inconsistent table: cannot happen
-      if (lane == 0) {    // right part to the worklist, keep following the left part
-        tb_lock(&ctl[2]);
-        if (ctl[0] < cap) { stk[ctl[0]] = make_int2(kk + 1, j); ctl[0] += 1; }
-        tb_unlock(&ctl[2]);
-      }
+      if (lane == 0) stk[sp] = make_int2(kk + 1, j);  // right part later, left part now
+      ++sp;
+      __syncwarp();
       j = kk;
-    }
-    if (lane == 0) {
-      tb_lock(&ctl[2]);
-      ctl[1] -= 1;
-      tb_unlock(&ctl[2]);
     }
   }
 }
@@ -340,7 +329,6 @@ __global__ void __launch_bounds__(kCtaWarps * 32, 2) k_nuss_tiled_cta(NussArgs A
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint8_t pm[16];
   __shared__ uint8_t xs[4096];
-  __shared__ int tbctl[4];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
   uint8_t* wbuf = smem;                                                      // per-warp scratch
@@ -394,9 +382,10 @@ __global__ void __launch_bounds__(kCtaWarps * 32, 2) k_nuss_tiled_cta(NussArgs A
       A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
       if (A.db) A.db_len[p] = n;
     }
-    if (A.db)
-      cta_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack),
-                    2 * (int)A.max_len + 4, tbctl, lane);
+    // warp 0 traces back while the other warps move on to the next problem's staging
+    // barrier (the second CTA on the SM keeps the SM busy meanwhile)
+    if (A.db && warp == 0)
+      warp_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack), lane);
   }
 }
 
@@ -459,15 +448,12 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_tiled_grid(NussArgs
     }
     grid.sync();
   }
-  if (blockIdx.x == 0) {
-    __shared__ int tbctl[4];
-    if (threadIdx.x == 0) {
+  if (gw == 0) {
+    if (lane == 0) {
       A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
       if (A.db) A.db_len[p] = n;
     }
-    if (A.db)
-      cta_traceback(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack),
-                    2 * n + 4, tbctl, lane);
+    if (A.db) warp_traceback(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack), lane);
   }
 }
 

@@ -37,6 +37,11 @@ constexpr int kBandsPerStrip = kStrip / kBand;
 constexpr int kBlk = 32;              // traceback recompute block height (two independent bands)
 constexpr int kSlab = 32;             // checkpoint column spacing
 constexpr int kHS = kSlab + 2;        // row stride of the recomputed block (conflict-free anti-diagonals)
+// word index of H(row, col) in a recomputed block: rows 17..32 (the lower 16-row half)
+// are shifted by 16 words so the two halves, which run the same anti-diagonal
+// concurrently, hit disjoint banks
+__device__ __forceinline__ int hbi(int row, int col) { return row * kHS + col + (row > kBand ? 16 : 0); }
+constexpr int kHbWords = (kBlk + 1) * kHS + 16;
 constexpr int kDead = -100;           // profile value for rows/columns outside a problem
 constexpr int kPad = 32;              // dead columns on each side of the residue array
 
@@ -272,7 +277,7 @@ __device__ void recompute_block(const TbView& V, const uint8_t* a, const uint8_t
   const int i = R0 + lane + 1;
   const bool row_ok = i <= V.la;
   int left = row_ok ? V.left_h(i, slab) : 0;
-  Hb[(lane + 1) * kHS] = left;
+  Hb[hbi(lane + 1, 0)] = left;
   __syncwarp();
   const int hl = lane & (kBand - 1);  // row within the half
   const int* top = (lane < kBand) ? Hb : mid;
@@ -280,7 +285,7 @@ __device__ void recompute_block(const TbView& V, const uint8_t* a, const uint8_t
   const int8_t* srow = sig_s + ai * asz;
   const uint8_t* bb = b + C0 - 1;      // bb[c] = b[C0 + c - 1]
   const int cmax = min(kSlab, V.lb - C0);  // live columns of this slab
-  int* hrow = Hb + (lane + 1) * kHS;
+  int* hrow = Hb + hbi(lane + 1, 0);
   int diag = __shfl_up_sync(0xffffffffu, left, 1);
   if (hl == 0) diag = top[0];
   int last = 0;
@@ -316,10 +321,10 @@ __global__ void __launch_bounds__(128) k_sw16_tb(Sw16Args A, int64_t first, int6
   V.A = &A;
   V.grp = p >> 1;
   V.half = (int)(p & 1);
-  uint8_t* wsm = tsm + (size_t)warp * (seq_bytes + ((kBlk + 1) * kHS + kHS) * 4);
+  uint8_t* wsm = tsm + (size_t)warp * (seq_bytes + (kHbWords + kHS) * 4);
   int* Hb = reinterpret_cast<int*>(wsm);
-  int* mid = Hb + (kBlk + 1) * kHS;
-  uint8_t* a = wsm + ((kBlk + 1) * kHS + kHS) * 4;
+  int* mid = Hb + kHbWords;
+  uint8_t* a = wsm + (kHbWords + kHS) * 4;
   V.la = (int)(A.a_off[p + 1] - A.a_off[p]);
   V.lb = (int)(A.b_off[p + 1] - A.b_off[p]);
   const int la = V.la, lb = V.lb, asz = A.asz, g = A.gap;
@@ -363,7 +368,7 @@ __global__ void __launch_bounds__(128) k_sw16_tb(Sw16Args A, int64_t first, int6
     if (myc == (1 << 30) && i <= la)
       for (int c = 1; c <= kSlab; ++c) {
         const int j = sl * kSlab + c;
-        if (j <= lb && Hb[(lane + 1) * kHS + c] == best) { myc = j; break; }
+        if (j <= lb && Hb[hbi(lane + 1, c)] == best) { myc = j; break; }
       }
     __syncwarp();
   }
@@ -384,15 +389,15 @@ __global__ void __launch_bounds__(128) k_sw16_tb(Sw16Args A, int64_t first, int6
         const int ri = i - R0, cj = j - C0;
         const int sub = sig_s[a[i - 1] * asz + b[j - 1]];
         uint8_t op;
-        if (h == Hb[(ri - 1) * kHS + cj - 1] + sub) {
+        if (h == Hb[hbi(ri - 1, cj - 1)] + sub) {
           op = (a[i - 1] == b[j - 1]) ? 'M' : 'X';
           --i; --j;
-        } else if (h == Hb[(ri - 1) * kHS + cj] - g) {
+        } else if (h == Hb[hbi(ri - 1, cj)] - g) {
           op = 'D'; --i;
         } else {
           op = 'I'; --j;
         }
-        h = Hb[(i - R0) * kHS + (j - C0)];
+        h = Hb[hbi(i - R0, j - C0)];
         if (n < stride) o[n] = op; else overflow = true;
         ++n;
       }
@@ -452,7 +457,7 @@ cudaError_t sw16_traceback(const Sw16Args& A, int64_t first, int64_t count, uint
                            int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches) {
   if (count == 0) return cudaSuccess;
   const int seq_bytes = (int)(((A.max_la + 15) & ~15) + ((A.max_lb + 15) & ~15));
-  const size_t smem = 4 * ((size_t)seq_bytes + ((kBlk + 1) * kHS + kHS) * 4);
+  const size_t smem = 4 * ((size_t)seq_bytes + (kHbWords + kHS) * 4);
   cudaError_t e = cudaFuncSetAttribute(k_sw16_tb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   ++*launches;

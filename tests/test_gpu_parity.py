@@ -279,6 +279,21 @@ def test_forward_random(dp, orc, S):
             assert abs(ll[q] - want[q]) <= 1e-5 * abs(want[q]), (q, ll[q], want[q])
 
 
+@pytest.mark.parametrize("S", [5, 64])
+def test_forward_simt_path(dp, orc, S, monkeypatch):
+    """The SIMT forward kernel (used when the tensor-core path is disabled)."""
+    monkeypatch.setenv("DP_HMM_SIMT", "1")
+    g = np.random.default_rng(125 + S)
+    pi, A, E, seqs = hmm_case(g, S, 40, 0, 300)
+    cat, off = dpgen.pack(seqs)
+    plan = dp.Plan(dp.HMM_FORWARD, max(len(s) for s in seqs), pi=pi, A=A, E=E)
+    ll = host(plan.solve_batch(cuda(cat), cuda(off)))
+    want = orc.forward_batch(cat, off, pi.astype(np.float64), A.astype(np.float64), E.astype(np.float64),
+                             threads=THREADS)
+    for q in range(len(seqs)):
+        assert abs(ll[q] - want[q]) <= 1e-5 * max(abs(want[q]), 1e-30), (q, ll[q], want[q])
+
+
 @pytest.mark.parametrize("S", [1, 7, 64])
 def test_viterbi_random(dp, orc, S):
     g = np.random.default_rng(130 + S)
