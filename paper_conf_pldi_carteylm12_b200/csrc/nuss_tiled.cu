@@ -42,7 +42,8 @@ namespace {
 constexpr int T = 32;
 constexpr int kTileWords = T * T;      // int16 per tile record half
 constexpr int kRec = 2 * kTileWords;   // int16 per tile record (UT + L)
-constexpr int kCtaWarps = 8;   // batch driver: two CTAs (two sequences) per SM
+constexpr int kCtaWarps = 2;   // batch driver: eight CTAs (eight sequences) per SM
+constexpr int kCtaPerSm = 8;
 constexpr int kGridWarps = 16; // grid driver
 constexpr int kCS = T + 1;             // row stride of in-tile buffers
 constexpr int kGridMin = 1024;         // single problems longer than this use the whole grid
@@ -167,8 +168,14 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
       if (c < T) {
         int v = max(B.cur[(r + 1) * kCS + c], B.cur[r * kCS + c - 1]);
         if (pairable(x, pm, n, i0 + r, j0 + c, h)) v = max(v, (d >= 2 ? B.cur[(r + 1) * kCS + c - 1] : 0) + 1);
-        for (int k = r + 1; k < c; ++k) v = max(v, B.cur[r * kCS + k] + B.cur[(k + 1) * kCS + c]);
-        B.cur[r * kCS + c] = v;
+        int v2 = v;  // two independent max chains
+        int k = r + 1;
+        for (; k + 1 < c; k += 2) {
+          v = __viaddmax_s32(B.cur[r * kCS + k], B.cur[(k + 1) * kCS + c], v);
+          v2 = __viaddmax_s32(B.cur[r * kCS + k + 1], B.cur[(k + 2) * kCS + c], v2);
+        }
+        if (k < c) v = __viaddmax_s32(B.cur[r * kCS + k], B.cur[(k + 1) * kCS + c], v);
+        B.cur[r * kCS + c] = max(v, v2);
       }
       __syncwarp();
     }
@@ -225,34 +232,53 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
   const int r = lane;
   const uint4* urow = reinterpret_cast<const uint4*>(B.uiis + r * kVS);
   const uint4* crow = reinterpret_cast<const uint4*>(B.cr + r * kVS);
+  // pair bits of my row: bit c set when (i0 + r, j0 + c) may pair (hairpin included)
+  uint32_t pairbits = 0;
+  for (int c = 0; c < T; ++c) pairbits |= (uint32_t)pairable(x, pm, n, i0 + r, j0 + c, h) << c;
+  // per-lane chunk ranges: K=I chunks [q0, 5) then K=J chunks [0, q1), merged into one loop
   for (int dl = -(T - 1); dl <= T - 1; ++dl) {
     const int c = r + dl;
+    const bool live = c >= 0 && c < T;
+    const int cc = live ? c : 0;
     const int rmin = max(0, -dl), cmax = min(T - 1, T - 1 + dl);
-    const int q0 = (rmin + 2) / 8;       // first K=I chunk any lane needs
+    const int q0 = (rmin + 2) / 8;       // first K=I chunk any lane needs (warp-uniform)
     const int q1 = (cmax + 7) / 8;       // K=J chunks 0 .. q1-1
-    if (c >= 0 && c < T) {
-      const uint4* ccol = reinterpret_cast<const uint4*>(B.ct + c * kVS);
-      const uint4* lcol = reinterpret_cast<const uint4*>(B.lt + c * kVS);
-      uint32_t acc = 0;
-      for (int q = q0; q <= 4; ++q) {  // k + 1 = m in [r+2, 32]
-        const uint4 a = urow[q], b = ccol[q];
-        acc = __viaddmax_s16x2(a.x, b.x, acc);
-        acc = __viaddmax_s16x2(a.y, b.y, acc);
-        acc = __viaddmax_s16x2(a.z, b.z, acc);
-        acc = __viaddmax_s16x2(a.w, b.w, acc);
-      }
-      for (int q = 0; q < q1; ++q) {   // k in [0, c)
-        const uint4 a = crow[q], b = lcol[q];
-        acc = __viaddmax_s16x2(a.x, b.x, acc);
-        acc = __viaddmax_s16x2(a.y, b.y, acc);
-        acc = __viaddmax_s16x2(a.z, b.z, acc);
-        acc = __viaddmax_s16x2(a.w, b.w, acc);
-      }
+    const uint4* ccol = reinterpret_cast<const uint4*>(B.ct + cc * kVS);
+    const uint4* lcol = reinterpret_cast<const uint4*>(B.lt + cc * kVS);
+    // all operand loads of the step are issued together (predicated full unroll), then reduced
+    uint4 ua[5], ub[5], ja[4], jb[4];
+#pragma unroll
+    for (int q = 0; q < 5; ++q) {
+      if (q >= q0) { ua[q] = urow[q]; ub[q] = ccol[q]; }
+      else { ua[q] = make_uint4(0, 0, 0, 0); ub[q] = make_uint4(0, 0, 0, 0); }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (q < q1) { ja[q] = crow[q]; jb[q] = lcol[q]; }
+      else { ja[q] = make_uint4(0, 0, 0, 0); jb[q] = make_uint4(0, 0, 0, 0); }
+    }
+    uint32_t a0 = 0, a1 = 0, a2 = 0, a3 = 0;  // four independent max chains (0 is neutral: gamma >= 0)
+#pragma unroll
+    for (int q = 0; q < 5; ++q) {             // k + 1 = m in [r+2, 32]
+      a0 = __viaddmax_s16x2(ua[q].x, ub[q].x, a0);
+      a1 = __viaddmax_s16x2(ua[q].y, ub[q].y, a1);
+      a2 = __viaddmax_s16x2(ua[q].z, ub[q].z, a2);
+      a3 = __viaddmax_s16x2(ua[q].w, ub[q].w, a3);
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {             // k in [0, c)
+      a0 = __viaddmax_s16x2(ja[q].x, jb[q].x, a0);
+      a1 = __viaddmax_s16x2(ja[q].y, jb[q].y, a1);
+      a2 = __viaddmax_s16x2(ja[q].z, jb[q].z, a2);
+      a3 = __viaddmax_s16x2(ja[q].w, jb[q].w, a3);
+    }
+    if (live) {
+      const uint32_t acc = __vmaxs2(__vmaxs2(a0, a1), __vmaxs2(a2, a3));
       int v = max((int)(int16_t)(acc & 0xffffu), (int)(int16_t)(acc >> 16));
       v = max(v, (int)B.cr[r * kVS + c]);                              // C (middle products)
       v = max(v, (int)B.ct[c * kVS + r + 1]);                          // gamma(i+1, j) (row 32 = below)
       v = max(v, c > 0 ? (int)B.cr[r * kVS + c - 1] : B.left[r]);     // gamma(i, j-1)
-      if (pairable(x, pm, n, i0 + r, j0 + c, h)) {
+      if ((pairbits >> c) & 1u) {
         const int inner = c > 0 ? (int)B.ct[(c - 1) * kVS + r + 1] : (r < T - 1 ? B.left[r + 1] : B.corner);
         v = max(v, inner + 1);
       }
@@ -325,7 +351,7 @@ __device__ void warp_traceback(const Tab& tab, const uint8_t* x, const uint8_t* 
 }
 
 // ------------------------------------------------------------------ batch driver
-__global__ void __launch_bounds__(kCtaWarps * 32, 2) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
+__global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint8_t pm[16];
   __shared__ uint8_t xs[4096];
@@ -417,34 +443,44 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_tiled_grid(NussArgs
        q += (int64_t)gridDim.x * blockDim.x)
     Cg[q] = 0;
   grid.sync();
+  // Round D: phase B of tile-diagonal D (the warp of tile t first adds the two boundary
+  // K-steps K = I+1 and K = J-1, whose operands lie on diagonal D-1) overlapped with the
+  // interior K-steps I+2 <= K <= J-2 of diagonal D+1 (operands on diagonals <= D-1) on
+  // the other warps: one grid-wide barrier per tile-diagonal instead of two.
   for (int D = 0; D < nt; ++D) {
     const int nT = nt - D;
-    int* C = Cg + (int64_t)(D & 1) * nt * T * T;
-    if (D >= 2) {
-      // phase A: split the (tile, K) pairs of this diagonal evenly over all warps
-      const int64_t total = (int64_t)nT * (D - 1);
-      const int64_t per = (total + nw - 1) / nw;
-      const int64_t b0 = gw * per, b1 = min(total, b0 + per);
+    int* C = Cg + (int64_t)(D & 1) * nt * T * T;        // diagonal D (interior products already in)
+    int* Cn = Cg + (int64_t)((D + 1) & 1) * nt * T * T; // diagonal D+1
+    const int64_t nB = min((int64_t)nT, nw / 2);  // warps on phase B (the rest on phase A)
+    if (gw < nB) {
+     for (int64_t tt = gw; tt < nT; tt += nB) {
+      const int t = (int)tt, I = t, J = t + D;
+      int* Ct = C + (int64_t)t * T * T;
+      if (D >= 2) {
+        product_unit<false>(tab, I, J, I + 1, I + 2, Ct, As, Bs, lane);
+        if (D >= 3) product_unit<false>(tab, I, J, J - 1, J, Ct, As, Bs, lane);
+        __threadfence();
+        __syncwarp();
+      }
+      in_tile(tab, I, J, Ct, D >= 2, IB, x, pm, n, A.hairpin, lane);
+      // this C slot is reused by diagonal D+2: clear it (in_tile has read it)
+      for (int q = lane; q < T * T; q += 32) Ct[q] = 0;
+     }
+    } else if (D + 1 < nt && D >= 3) {
+      // interior K-steps of diagonal D+1: tiles t' (I = t', J = t' + D + 1), K in [I+2, J-2]
+      const int nT1 = nt - (D + 1), ks = D - 2;
+      const int64_t total = (int64_t)nT1 * ks;
+      const int64_t nwA = nw - nB, wA = gw - nB;
+      const int64_t per = (total + nwA - 1) / nwA;
+      const int64_t b0 = wA * per, b1 = min(total, b0 + per);
       int64_t it = b0;
       while (it < b1) {
-        const int t = (int)(it / (D - 1));
-        const int kk = (int)(it % (D - 1));
-        const int64_t tile_end = (int64_t)(t + 1) * (D - 1);
-        const int64_t e = min(b1, tile_end);
-        const int I = t, J = t + D;
-        product_unit<false>(tab, I, J, I + 1 + kk, I + 1 + kk + (int)(e - it), C + (int64_t)t * T * T, As, Bs, lane);
+        const int t = (int)(it / ks), kk = (int)(it % ks);
+        const int64_t e = min(b1, (int64_t)(t + 1) * ks);
+        const int I = t, J = t + D + 1;
+        product_unit<false>(tab, I, J, I + 2 + kk, I + 2 + kk + (int)(e - it), Cn + (int64_t)t * T * T, As, Bs, lane);
         it = e;
       }
-      grid.sync();
-    }
-    // phase B: one warp per tile; the other buffer is cleared for diagonal D+1
-    int* Cn = Cg + (int64_t)((D + 1) & 1) * nt * T * T;
-    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < (int64_t)(nT - 1) * T * T;
-         q += (int64_t)gridDim.x * blockDim.x)
-      Cn[q] = 0;
-    for (int64_t t = gw; t < nT; t += nw) {
-      const int I = (int)t, J = I + D;
-      in_tile(tab, I, J, C + t * T * T, D >= 2, IB, x, pm, n, A.hairpin, lane);
     }
     grid.sync();
   }
@@ -478,7 +514,7 @@ int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
   if (n == 1 && max_len > kGridMin) {
     return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
   }
-  const int64_t grid = std::min<int64_t>(n, 2 * (int64_t)num_sms_t(device));
+  const int64_t grid = std::min<int64_t>(n, kCtaPerSm * (int64_t)num_sms_t(device));
   return grid * (tiles_of(nt) * kRec * 2 + (int64_t)kCtaWarps * T * T * 4 + stack_bytes) + 256;
 }
 
@@ -506,7 +542,7 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
   const size_t smem = kCtaWarps * warp_bytes();
   cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  const int64_t grid = std::min<int64_t>(A.n, 2 * (int64_t)sms);
+  const int64_t grid = std::min<int64_t>(A.n, kCtaPerSm * (int64_t)sms);
   ++*launches;
   k_nuss_tiled_cta<<<(unsigned)grid, kCtaWarps * 32, smem, s>>>(A, tiles_of(nt) * kRec);
   return cudaGetLastError();

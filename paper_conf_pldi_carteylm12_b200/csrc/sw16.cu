@@ -22,6 +22,7 @@
 // 16-row halves in parallel) and walks them with the oracle's tie-break
 // (diag > up > left, stop at H = 0; end cell = first maximum in row-major order).
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "dp_internal.h"
@@ -297,7 +298,7 @@ __device__ void recompute_block(const TbView& V, const uint8_t* a, const uint8_t
     const bool in = (unsigned)(c - 1) < (unsigned)kSlab;
     const int cc = in ? c : 1;
     const int up = (hl == 0) ? top[cc] : from;
-    int h = max(max(diag + srow[bb[cc]], 0), max(up, left) - g);
+    int h = max(max(diag + srow[cc <= cmax ? bb[cc] : 0], 0), max(up, left) - g);
     h = (row_ok && cc <= cmax) ? h : 0;
     if (in) hrow[cc] = h;
     diag = in ? up : diag;
@@ -414,6 +415,203 @@ __global__ void __launch_bounds__(128) k_sw16_tb(Sw16Args A, int64_t first, int6
   }
 }
 
+// ---------------------------------------------------------------- packed traceback
+// Two problems per warp (the pair group of the forward pass): lanes 0-15 serve
+// problem 2g, lanes 16-31 problem 2g+1. A 32-row block is recomputed by 16 lanes,
+// lane hl holding rows hl+1 (low half) and hl+17 (high half) in one s16x2
+// register — the two 16-row halves are independent given the checkpoint row
+// between them — so one VIADDMNMX.S16x2 chain step evaluates two cells.
+// Hp[t][c] packs (H(R0+t, C0+c), H(R0+16+t, C0+c)), t = 0..16: row 0 holds the
+// checkpoint rows (top, middle), column 0 the checkpoint column.
+constexpr int kPS = kSlab + 2;        // packed row stride (words)
+constexpr int kPW = 17 * kPS + 14;    // words per packed block (592 = 16 mod 32: the halves hit disjoint banks)
+
+struct PackedView {
+  const Sw16Args* A;
+  int64_t grp;
+  int half, la, lb;
+  __device__ __forceinline__ int top_h(int band, int j) const {  // H at row 16*band, column j
+    if (band == 0 || j == 0) return 0;
+    const int b = band - 1;
+    const int st = b / kBandsPerStrip, bi = b % kBandsPerStrip;
+    const uint32_t v = A->rowck[((grp * A->strips_max + st) * kBandsPerStrip + bi) * A->max_lb + (j - 1)];
+    return half16(v, half) + A->gap;
+  }
+  __device__ __forceinline__ int left_h(int i, int slab) const {  // H at row i, column 32*slab
+    if (slab == 0) return 0;
+    const int st = (i - 1) / kStrip, ri = (i - 1) % kStrip;
+    const uint32_t v = A->colck[((grp * A->strips_max + st) * A->nslab_max + (slab - 1)) * kStrip + ri];
+    return half16(v, half) + A->gap;
+  }
+};
+
+__device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(uint16_t)lo | ((uint32_t)(uint16_t)hi << 16); }
+__device__ __forceinline__ int hp_get(const uint32_t* Hp, int row, int col) {  // H(R0 + row, C0 + col), row 0..32
+  return row <= 16 ? lo16(Hp[row * kPS + col]) : hi16(Hp[(row - 16) * kPS + col]);
+}
+
+// Recompute this half's block (blk, slab) into Hp; `on` = this half has a block to do.
+__device__ void packed_block(const PackedView& V, const uint8_t* a, const uint8_t* b, int blk, int slab, bool on,
+                             uint32_t* Hp, const int8_t* sig_s, int asz, int g, int hl) {
+  const int R0 = blk * kBlk, C0 = slab * kSlab;
+  const int band0 = R0 / kBand;
+  if (on) {
+    for (int c = hl; c <= kSlab; c += 16)
+      Hp[c] = (C0 + c <= V.lb) ? pk(V.top_h(band0, C0 + c), V.top_h(band0 + 1, C0 + c)) : 0u;
+  }
+  const int iL = R0 + hl + 1, iH = R0 + hl + 17;
+  const bool okL = on && iL <= V.la, okH = on && iH <= V.la;
+  uint32_t left = pk(okL ? V.left_h(iL, slab) : 0, okH ? V.left_h(iH, slab) : 0);
+  if (on) Hp[(hl + 1) * kPS] = left;
+  __syncwarp();
+  const int8_t* sL = sig_s + (okL ? a[iL - 1] : 0) * asz;
+  const int8_t* sH = sig_s + (okH ? a[iH - 1] : 0) * asz;
+  const uint32_t rowmask = (okL ? 0xffffu : 0u) | (okH ? 0xffff0000u : 0u);
+  const uint8_t* bb = b + C0 - 1;
+  const int cmax = on ? min(kSlab, V.lb - C0) : 0;
+  const uint32_t NEG_G2 = (uint32_t)(uint16_t)(-g) * 0x10001u;
+  uint32_t* hrow = Hp + (hl + 1) * kPS;
+  uint32_t diag = __shfl_up_sync(0xffffffffu, left, 1, 16);
+  if (hl == 0) diag = on ? Hp[0] : 0u;
+  uint32_t last = 0;
+#pragma unroll 4
+  for (int s = 0; s < kSlab + 15; ++s) {
+    const int c = s - hl + 1;
+    const uint32_t from = __shfl_up_sync(0xffffffffu, last, 1, 16);
+    const bool in = (unsigned)(c - 1) < (unsigned)kSlab;
+    const int cc = in ? c : 1;
+    const uint32_t up = (hl == 0) ? Hp[cc] : from;
+    const int bj = (cc <= cmax) ? bb[cc] : 0;  // never read past the staged sequence
+    const uint32_t sg = prmt((uint32_t)(uint8_t)sL[bj], (uint32_t)(uint8_t)sH[bj], 0xC480u);
+    uint32_t h = __viaddmax_s16x2_relu(diag, sg, __vadd2(__vmaxs2(up, left), NEG_G2));
+    h = (cc <= cmax) ? (h & rowmask) : 0u;
+    if (in) hrow[cc] = h;
+    diag = in ? up : diag;
+    left = in ? h : left;
+    last = in ? h : last;
+  }
+  __syncwarp();
+}
+
+__global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int64_t count, uint8_t* out,
+                                                   int64_t stride, int32_t* out_len, int32_t* coords, int seq_bytes) {
+  extern __shared__ __align__(16) uint8_t tsm[];
+  __shared__ int8_t sig_s[32 * 32];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int q = threadIdx.x; q < A.asz * A.asz; q += blockDim.x) sig_s[q] = A.sigma[q];
+  __syncthreads();
+  const int half = lane >> 4, hl = lane & 15;
+  const int64_t g0 = first >> 1;
+  const int64_t grp = g0 + (int64_t)blockIdx.x * 4 + warp;
+  const int64_t p = 2 * grp + half;
+  const bool mine = p >= first && p < first + count;  // this half's problem is requested
+  if (2 * grp >= first + count) return;                  // warp-uniform
+  const int64_t qidx = p - first;
+  PackedView V;
+  V.A = &A; V.grp = grp; V.half = half;
+  V.la = mine ? (int)(A.a_off[p + 1] - A.a_off[p]) : 0;
+  V.lb = mine ? (int)(A.b_off[p + 1] - A.b_off[p]) : 0;
+  const int la = V.la, lb = V.lb, asz = A.asz, g = A.gap;
+  uint8_t* wsm = tsm + (size_t)warp * (2 * (kPW * 4 + seq_bytes));
+  uint32_t* Hp = reinterpret_cast<uint32_t*>(wsm) + half * kPW;  // the halves start 16 words apart mod 32
+  uint8_t* a = wsm + 2 * kPW * 4 + half * seq_bytes;
+  uint8_t* b = a + ((la + 15) & ~15);
+  for (int q = hl; q < la; q += 16) a[q] = A.a_cat[A.a_off[p] + q];
+  for (int q = hl; q < lb; q += 16) b[q] = A.b_cat[A.b_off[p] + q];
+  __syncwarp();
+  const int best = mine ? A.scores[p] : 0;
+  bool active = mine && best > 0 && la > 0 && lb > 0;
+  uint8_t* o = out + (mine ? qidx : 0) * stride;
+  // 1) first lane band (row-major) whose slab maxima reach the best value (per half)
+  int band8 = -1;
+  const int strips = (max(la, 1) + kStrip - 1) / kStrip;
+  const int nsl = (max(lb, 1) + kSlab - 1) / kSlab;
+  const int strips_w = max(__shfl_sync(0xffffffffu, strips, 0), __shfl_sync(0xffffffffu, strips, 16));
+  for (int st = 0; st < strips_w; ++st) {
+    for (int l2 = 0; l2 < 2; ++l2) {  // the half's 16 lanes cover the 32 lane bands in two rounds
+      const int ln = hl + 16 * l2;
+      bool hit = false;
+      if (active && band8 < 0 && st < strips)
+        for (int sl = 0; sl < nsl; ++sl)
+          hit |= half16(A.slabbest[((grp * A.strips_max + st) * A.nslab_max + sl) * 32 + ln], half) + g == best;
+      const unsigned m = __ballot_sync(0xffffffffu, hit) >> (16 * half) & 0xffffu;
+      if (band8 < 0 && m) band8 = st * 32 + 16 * l2 + __ffs(m) - 1;
+    }
+  }
+  // 2) first cell with H == best among the slabs of band8 holding the best (both halves together)
+  const int lane8 = band8 >= 0 ? band8 % 32 : 0, st8 = band8 >= 0 ? band8 / 32 : 0;
+  const int blk = (st8 * kStrip + lane8 * kRows) / kBlk;
+  int myr = 1 << 30, myc = 1 << 30;  // my best (row, col) candidate inside the block, row-major
+  const int nsl_w = max(__shfl_sync(0xffffffffu, nsl, 0), __shfl_sync(0xffffffffu, nsl, 16));
+  for (int sl = 0; sl < nsl_w; ++sl) {
+    const bool cand = active && sl < nsl &&
+        half16(A.slabbest[((grp * A.strips_max + st8) * A.nslab_max + sl) * 32 + lane8], half) + g == best;
+    if (!__any_sync(0xffffffffu, cand)) continue;
+    packed_block(V, a, b, blk, sl, cand, Hp, sig_s, asz, g, hl);
+    if (cand) {
+      for (int rr = 0; rr < 2; ++rr) {  // rows hl+1 and hl+17
+        const int row = hl + 1 + 16 * rr, i = blk * kBlk + row;
+        if (i > la || row > myr) continue;
+        for (int c = 1; c <= kSlab; ++c) {
+          const int j = sl * kSlab + c;
+          if (j <= lb && hp_get(Hp, row, c) == best) {
+            if (row < myr || (row == myr && j < myc)) { myr = row; myc = j; }
+            break;
+          }
+        }
+      }
+    }
+    __syncwarp();
+  }
+  // smallest (row, col) over the half's lanes
+  for (int o2 = 8; o2 > 0; o2 >>= 1) {
+    const int orr = __shfl_xor_sync(0xffffffffu, myr, o2, 16), occ = __shfl_xor_sync(0xffffffffu, myc, o2, 16);
+    if (orr < myr || (orr == myr && occ < myc)) { myr = orr; myc = occ; }
+  }
+  if (myr == (1 << 30)) active = false;  // cannot happen: the slab maxima name a cell holding the best
+  const int ei = active ? blk * kBlk + myr : 0, ej = active ? myc : 0;
+  // 3) walk back block by block; the two halves walk concurrently (leaders hl == 0)
+  int i = ei, j = ej, h = active ? best : 0;
+  int64_t n = 0;
+  bool overflow = false;
+  while (__any_sync(0xffffffffu, h > 0)) {
+    const bool on = h > 0;
+    const int bg = on ? (i - 1) / kBlk : 0, sl = on ? (j - 1) / kSlab : 0;
+    packed_block(V, a, b, bg, sl, on, Hp, sig_s, asz, g, hl);
+    if (hl == 0 && on) {
+      const int R0 = bg * kBlk, C0 = sl * kSlab;
+      while (h > 0 && i > R0 && j > C0) {
+        const int ri = i - R0, cj = j - C0;
+        const int sub = sig_s[a[i - 1] * asz + b[j - 1]];
+        uint8_t op;
+        if (h == hp_get(Hp, ri - 1, cj - 1) + sub) {
+          op = (a[i - 1] == b[j - 1]) ? 'M' : 'X';
+          --i; --j;
+        } else if (h == hp_get(Hp, ri - 1, cj) - g) {
+          op = 'D'; --i;
+        } else {
+          op = 'I'; --j;
+        }
+        h = hp_get(Hp, i - R0, j - C0);
+        if (n < stride) o[n] = op; else overflow = true;
+        ++n;
+      }
+    }
+    i = __shfl_sync(0xffffffffu, i, 16 * half);
+    j = __shfl_sync(0xffffffffu, j, 16 * half);
+    h = __shfl_sync(0xffffffffu, h, 16 * half);
+  }
+  if (hl == 0 && mine) {
+    if (!overflow)
+      for (int64_t u = 0, v = n - 1; u < v; ++u, --v) { const uint8_t t = o[u]; o[u] = o[v]; o[v] = t; }
+    out_len[qidx] = overflow ? -1 : (int32_t)n;
+    if (coords) {
+      coords[4 * qidx] = active ? i : 0; coords[4 * qidx + 1] = active ? j : 0;
+      coords[4 * qidx + 2] = ei; coords[4 * qidx + 3] = ej;
+    }
+  }
+}
+
 }  // namespace
 
 bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap) {
@@ -457,10 +655,19 @@ cudaError_t sw16_traceback(const Sw16Args& A, int64_t first, int64_t count, uint
                            int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches) {
   if (count == 0) return cudaSuccess;
   const int seq_bytes = (int)(((A.max_la + 15) & ~15) + ((A.max_lb + 15) & ~15));
+  ++*launches;
+  if (getenv("DP_SW_TB_UNPACKED") == nullptr) {  // packed: two problems per warp
+    const size_t smem = 4 * (2 * ((size_t)kPW * 4 + seq_bytes));
+    cudaError_t e = cudaFuncSetAttribute(k_sw16_tb2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const int64_t groups = ((first + count - 1) >> 1) - (first >> 1) + 1;
+    k_sw16_tb2<<<(unsigned)((groups + 3) / 4), 128, smem, s>>>(A, first, count, out, stride, out_len, coords,
+                                                               seq_bytes);
+    return cudaGetLastError();
+  }
   const size_t smem = 4 * ((size_t)seq_bytes + (kHbWords + kHS) * 4);
   cudaError_t e = cudaFuncSetAttribute(k_sw16_tb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  ++*launches;
   k_sw16_tb<<<(unsigned)((count + 3) / 4), 128, smem, s>>>(A, first, count, out, stride, out_len, coords, seq_bytes);
   return cudaGetLastError();
 }
