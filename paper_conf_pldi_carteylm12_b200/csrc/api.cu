@@ -1,6 +1,7 @@
 // C ABI (include/dp.h): plan lifecycle, dispatch to the kernels, traceback,
 // host-buffer entry point. No exception crosses this boundary.
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <new>
@@ -335,7 +336,17 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       e = p->scratch.ensure((size_t)A.scratch_bytes);
       if (e != cudaSuccess) break;
       A.scratch = p->scratch.ptr;
+      unsigned long long* rounds = nullptr;
+      if (getenv("DP_NUSS_ROUNDS") && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), A.round_ns = rounds;
       e = tiled ? dpk::nuss_tiled_solve(A, s, &p->launches) : dpk::nuss_solve(A, s, &p->launches);
+      if (rounds) {  // diagnostic: per tile-diagonal round durations of the grid sweep (stderr)
+        static unsigned long long h[8192];
+        cudaStreamSynchronize(s);
+        cudaMemcpy(h, rounds, sizeof(h), cudaMemcpyDeviceToHost);
+        const int nt = (int)((A.max_len + 31) / 32);
+        for (int d = 0; d + 1 < nt; ++d) fprintf(stderr, "round %d %.1f us\n", d, (h[d + 1] - h[d]) * 1e-3);
+        cudaFree(rounds);
+      }
       break;
     }
     case DP_HMM_FORWARD:

@@ -67,6 +67,7 @@ struct NussArgs {
   int32_t* db_len;
   void* scratch;             // global table scratch for large n
   int64_t scratch_bytes;
+  unsigned long long* round_ns;  // optional: %globaltimer at each tile-diagonal round (grid sweep)
 };
 int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device);
 bool nuss_tiled_supported(int64_t max_len);

@@ -73,18 +73,24 @@ __device__ __forceinline__ uint32_t dup16(uint32_t w, int hi) {
 }
 
 // Stage A = UT(I,K) (duplicated halves, [k][r]) and B = L(K,J) ([k][c]) in this warp's buffers.
-__device__ __forceinline__ void stage(const int16_t* ut, const int16_t* l, uint32_t* As, uint16_t* Bs, int lane) {
+// All global loads are issued before any shared-memory store (generic pointers could
+// alias, so interleaving them would serialise twelve L2 round trips).
+__device__ __forceinline__ void stage(const int16_t* __restrict__ ut, const int16_t* __restrict__ l,
+                                      uint32_t* __restrict__ As, uint16_t* __restrict__ Bs, int lane) {
+  uint2 wa[8];
+  uint4 wb[4];
+#pragma unroll
+  for (int t = 0; t < 8; ++t) wa[t] = __ldcg(reinterpret_cast<const uint2*>(ut + (lane + 32 * t) * 4));
+#pragma unroll
+  for (int t = 0; t < 4; ++t) wb[t] = __ldcg(reinterpret_cast<const uint4*>(l + (lane + 32 * t) * 8));
 #pragma unroll
   for (int t = 0; t < 8; ++t) {
     const int chunk = lane + 32 * t;  // 4-row chunk: k = chunk / 8, rows 4 (chunk % 8) ..
-    const uint2 w = *reinterpret_cast<const uint2*>(ut + chunk * 4);
-    *reinterpret_cast<uint4*>(As + chunk * 4) = make_uint4(dup16(w.x, 0), dup16(w.x, 1), dup16(w.y, 0), dup16(w.y, 1));
+    *reinterpret_cast<uint4*>(As + chunk * 4) =
+        make_uint4(dup16(wa[t].x, 0), dup16(wa[t].x, 1), dup16(wa[t].y, 0), dup16(wa[t].y, 1));
   }
 #pragma unroll
-  for (int t = 0; t < 4; ++t) {
-    const int chunk = lane + 32 * t;  // 8 int16 per chunk
-    *reinterpret_cast<uint4*>(Bs + chunk * 8) = *reinterpret_cast<const uint4*>(l + chunk * 8);
-  }
+  for (int t = 0; t < 4; ++t) *reinterpret_cast<uint4*>(Bs + (lane + 32 * t) * 8) = wb[t];
 }
 
 // acc[4 rows][4 pairs] = max(acc, A (x) B) over the 32 k of one staged K tile.
@@ -150,6 +156,23 @@ __device__ __forceinline__ bool pairable(const uint8_t* x, const uint8_t* pm, in
   return i < n && j < n && pm[x[i] * 4 + x[j]] && j - i - 1 >= h;
 }
 
+// Bit c of lane r: (i0 + r, j0 + c) may pair (pair set and hairpin). One coalesced load
+// per lane; the column bases are shuffled across the warp.
+__device__ __forceinline__ uint32_t pair_bits(const uint8_t* x, const uint8_t* pm, int n, int i0, int j0, int h,
+                                              int lane) {
+  const int i = i0 + lane;
+  const int xi = i < n ? x[i] : 0;
+  const int xjl = (j0 + lane < n) ? x[j0 + lane] : 0;
+  uint32_t bits = 0;
+#pragma unroll
+  for (int c = 0; c < T; ++c) {
+    const int xj = __shfl_sync(0xffffffffu, xjl, c);
+    const int j = j0 + c;
+    bits |= (uint32_t)(i < n && j < n && j - i - 1 >= h && pm[xi * 4 + xj]) << c;
+  }
+  return bits;
+}
+
 // Phase B: finalise tile (I,J) from C (max of the middle products), write UT/L records.
 // Off-diagonal tiles run the 63 local anti-diagonals with one cell per lane; each cell's
 // split points inside tiles I and J are reduced 8 at a time with VIADDMNMX.S16x2 over
@@ -162,12 +185,13 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
   if (I == J) {
     // diagonal tile: the cell-level recursion inside one 32x32 triangle
     for (int q = lane; q < T * kCS; q += 32) B.cur[q] = 0;
+    const uint32_t pbits = pair_bits(x, pm, n, i0, j0, h, lane);
     __syncwarp();
     for (int d = 1; d < T; ++d) {
       const int r = lane, c = lane + d;
       if (c < T) {
         int v = max(B.cur[(r + 1) * kCS + c], B.cur[r * kCS + c - 1]);
-        if (pairable(x, pm, n, i0 + r, j0 + c, h)) v = max(v, (d >= 2 ? B.cur[(r + 1) * kCS + c - 1] : 0) + 1);
+        if ((pbits >> c) & 1u) v = max(v, (d >= 2 ? B.cur[(r + 1) * kCS + c - 1] : 0) + 1);
         int v2 = v;  // two independent max chains
         int k = r + 1;
         for (; k + 1 < c; k += 2) {
@@ -230,47 +254,41 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
   }
   __syncwarp();
   const int r = lane;
-  const uint4* urow = reinterpret_cast<const uint4*>(B.uiis + r * kVS);
   const uint4* crow = reinterpret_cast<const uint4*>(B.cr + r * kVS);
-  // pair bits of my row: bit c set when (i0 + r, j0 + c) may pair (hairpin included)
-  uint32_t pairbits = 0;
-  for (int c = 0; c < T; ++c) pairbits |= (uint32_t)pairable(x, pm, n, i0 + r, j0 + c, h) << c;
-  // per-lane chunk ranges: K=I chunks [q0, 5) then K=J chunks [0, q1), merged into one loop
+  // my row of UIIs is constant for the whole tile: keep it in registers. It is already
+  // masked (kNeg for m < r + 2), so all five chunks are reduced unconditionally.
+  uint4 ur[5];
+#pragma unroll
+  for (int q = 0; q < 5; ++q) ur[q] = reinterpret_cast<const uint4*>(B.uiis + r * kVS)[q];
+  uint32_t pairbits = pair_bits(x, pm, n, i0, j0, h, lane);
   for (int dl = -(T - 1); dl <= T - 1; ++dl) {
     const int c = r + dl;
     const bool live = c >= 0 && c < T;
     const int cc = live ? c : 0;
-    const int rmin = max(0, -dl), cmax = min(T - 1, T - 1 + dl);
-    const int q0 = (rmin + 2) / 8;       // first K=I chunk any lane needs (warp-uniform)
-    const int q1 = (cmax + 7) / 8;       // K=J chunks 0 .. q1-1
+    const int cmax = min(T - 1, T - 1 + dl);
+    const int q1 = (cmax + 7) / 8;       // K=J chunks 0 .. q1-1 (warp-uniform)
     const uint4* ccol = reinterpret_cast<const uint4*>(B.ct + cc * kVS);
     const uint4* lcol = reinterpret_cast<const uint4*>(B.lt + cc * kVS);
-    // all operand loads of the step are issued together (predicated full unroll), then reduced
-    uint4 ua[5], ub[5], ja[4], jb[4];
+    uint4 ub[5];
 #pragma unroll
-    for (int q = 0; q < 5; ++q) {
-      if (q >= q0) { ua[q] = urow[q]; ub[q] = ccol[q]; }
-      else { ua[q] = make_uint4(0, 0, 0, 0); ub[q] = make_uint4(0, 0, 0, 0); }
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      if (q < q1) { ja[q] = crow[q]; jb[q] = lcol[q]; }
-      else { ja[q] = make_uint4(0, 0, 0, 0); jb[q] = make_uint4(0, 0, 0, 0); }
-    }
+    for (int q = 0; q < 5; ++q) ub[q] = ccol[q];
     uint32_t a0 = 0, a1 = 0, a2 = 0, a3 = 0;  // four independent max chains (0 is neutral: gamma >= 0)
 #pragma unroll
-    for (int q = 0; q < 5; ++q) {             // k + 1 = m in [r+2, 32]
-      a0 = __viaddmax_s16x2(ua[q].x, ub[q].x, a0);
-      a1 = __viaddmax_s16x2(ua[q].y, ub[q].y, a1);
-      a2 = __viaddmax_s16x2(ua[q].z, ub[q].z, a2);
-      a3 = __viaddmax_s16x2(ua[q].w, ub[q].w, a3);
+    for (int q = 0; q < 5; ++q) {             // K=I: k + 1 = m in [r+2, 32]
+      a0 = __viaddmax_s16x2(ur[q].x, ub[q].x, a0);
+      a1 = __viaddmax_s16x2(ur[q].y, ub[q].y, a1);
+      a2 = __viaddmax_s16x2(ur[q].z, ub[q].z, a2);
+      a3 = __viaddmax_s16x2(ur[q].w, ub[q].w, a3);
     }
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {             // k in [0, c)
-      a0 = __viaddmax_s16x2(ja[q].x, jb[q].x, a0);
-      a1 = __viaddmax_s16x2(ja[q].y, jb[q].y, a1);
-      a2 = __viaddmax_s16x2(ja[q].z, jb[q].z, a2);
-      a3 = __viaddmax_s16x2(ja[q].w, jb[q].w, a3);
+    for (int q = 0; q < 4; ++q) {             // K=J: k in [0, c)
+      if (q < q1) {
+        const uint4 ja = crow[q], jb = lcol[q];
+        a0 = __viaddmax_s16x2(ja.x, jb.x, a0);
+        a1 = __viaddmax_s16x2(ja.y, jb.y, a1);
+        a2 = __viaddmax_s16x2(ja.z, jb.z, a2);
+        a3 = __viaddmax_s16x2(ja.w, jb.w, a3);
+      }
     }
     if (live) {
       const uint32_t acc = __vmaxs2(__vmaxs2(a0, a1), __vmaxs2(a2, a3));
@@ -437,7 +455,6 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_tiled_grid(NussArgs
   int* Cg = reinterpret_cast<int*>(tab.base + tiles_of(nt) * kRec);  // 2 x nt x 1024 int32
   int* stack = Cg + 2 * (int64_t)nt * T * T;
   const int64_t gw = (int64_t)blockIdx.x * kGridWarps + warp;
-  const int64_t nw = (int64_t)gridDim.x * kGridWarps;
   // C buffers start at zero
   for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T;
        q += (int64_t)gridDim.x * blockDim.x)
@@ -448,29 +465,38 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_tiled_grid(NussArgs
   // interior K-steps I+2 <= K <= J-2 of diagonal D+1 (operands on diagonals <= D-1) on
   // the other warps: one grid-wide barrier per tile-diagonal instead of two.
   for (int D = 0; D < nt; ++D) {
+    if (A.round_ns && gw == 0 && lane == 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      A.round_ns[D] = t;
+    }
     const int nT = nt - D;
     int* C = Cg + (int64_t)(D & 1) * nt * T * T;        // diagonal D (interior products already in)
     int* Cn = Cg + (int64_t)((D + 1) & 1) * nt * T * T; // diagonal D+1
-    const int64_t nB = min((int64_t)nT, nw / 2);  // warps on phase B (the rest on phase A)
-    if (gw < nB) {
-     for (int64_t tt = gw; tt < nT; tt += nB) {
-      const int t = (int)tt, I = t, J = t + D;
-      int* Ct = C + (int64_t)t * T * T;
-      if (D >= 2) {
-        product_unit<false>(tab, I, J, I + 1, I + 2, Ct, As, Bs, lane);
-        if (D >= 3) product_unit<false>(tab, I, J, J - 1, J, Ct, As, Bs, lane);
-        __threadfence();
-        __syncwarp();
+    // Phase B runs on the first warp of each SM sub-partition group (warp % 4 == 0, i.e.
+    // SMSP 0), tiles spread over the SMs, so a latency-bound in-tile wavefront never
+    // shares its issue slots with another phase-B warp or with the phase-A warps, which
+    // run on the other three sub-partitions.
+    if ((warp & 3) == 0) {
+      for (int64_t tt = blockIdx.x + (int64_t)gridDim.x * (warp >> 2); tt < nT; tt += (int64_t)gridDim.x * (kGridWarps / 4)) {
+        const int t = (int)tt, I = t, J = t + D;
+        int* Ct = C + (int64_t)t * T * T;
+        if (D >= 2) {
+          product_unit<false>(tab, I, J, I + 1, I + 2, Ct, As, Bs, lane);
+          if (D >= 3) product_unit<false>(tab, I, J, J - 1, J, Ct, As, Bs, lane);
+          __threadfence();
+          __syncwarp();
+        }
+        in_tile(tab, I, J, Ct, D >= 2, IB, x, pm, n, A.hairpin, lane);
+        // this C slot is reused by diagonal D+2: clear it (in_tile has read it)
+        for (int q = lane; q < T * T; q += 32) Ct[q] = 0;
       }
-      in_tile(tab, I, J, Ct, D >= 2, IB, x, pm, n, A.hairpin, lane);
-      // this C slot is reused by diagonal D+2: clear it (in_tile has read it)
-      for (int q = lane; q < T * T; q += 32) Ct[q] = 0;
-     }
     } else if (D + 1 < nt && D >= 3) {
       // interior K-steps of diagonal D+1: tiles t' (I = t', J = t' + D + 1), K in [I+2, J-2]
       const int nT1 = nt - (D + 1), ks = D - 2;
       const int64_t total = (int64_t)nT1 * ks;
-      const int64_t nwA = nw - nB, wA = gw - nB;
+      const int64_t nwA = (int64_t)gridDim.x * (kGridWarps - kGridWarps / 4);
+      const int64_t wA = (int64_t)blockIdx.x * (kGridWarps - kGridWarps / 4) + (warp - (warp >> 2) - 1);
       const int64_t per = (total + nwA - 1) / nwA;
       const int64_t b0 = wA * per, b1 = min(total, b0 + per);
       int64_t it = b0;
