@@ -512,9 +512,10 @@ __global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int
   V.la = mine ? (int)(A.a_off[p + 1] - A.a_off[p]) : 0;
   V.lb = mine ? (int)(A.b_off[p + 1] - A.b_off[p]) : 0;
   const int la = V.la, lb = V.lb, asz = A.asz, g = A.gap;
-  uint8_t* wsm = tsm + (size_t)warp * (2 * (kPW * 4 + seq_bytes));
+  uint8_t* wsm = tsm + (size_t)warp * (2 * (kPW * 4 + 2 * seq_bytes));
   uint32_t* Hp = reinterpret_cast<uint32_t*>(wsm) + half * kPW;  // the halves start 16 words apart mod 32
-  uint8_t* a = wsm + 2 * kPW * 4 + half * seq_bytes;
+  uint8_t* a = wsm + 2 * kPW * 4 + half * 2 * seq_bytes;
+  uint8_t* ops = a + seq_bytes;  // the path, end -> start, staged in shared memory
   uint8_t* b = a + ((la + 15) & ~15);
   for (int q = hl; q < la; q += 16) a[q] = A.a_cat[A.a_off[p] + q];
   for (int q = hl; q < lb; q += 16) b[q] = A.b_cat[A.b_off[p] + q];
@@ -522,6 +523,7 @@ __global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int
   const int best = mine ? A.scores[p] : 0;
   bool active = mine && best > 0 && la > 0 && lb > 0;
   uint8_t* o = out + (mine ? qidx : 0) * stride;
+  const int ops_cap = seq_bytes;
   // 1) first lane band (row-major) whose slab maxima reach the best value (per half)
   int band8 = -1;
   const int strips = (max(la, 1) + kStrip - 1) / kStrip;
@@ -531,9 +533,16 @@ __global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int
     for (int l2 = 0; l2 < 2; ++l2) {  // the half's 16 lanes cover the 32 lane bands in two rounds
       const int ln = hl + 16 * l2;
       bool hit = false;
-      if (active && band8 < 0 && st < strips)
-        for (int sl = 0; sl < nsl; ++sl)
-          hit |= half16(A.slabbest[((grp * A.strips_max + st) * A.nslab_max + sl) * 32 + ln], half) + g == best;
+      if (active && band8 < 0 && st < strips) {
+        const uint32_t* sb = A.slabbest + ((grp * A.strips_max + st) * A.nslab_max) * 32 + ln;
+        for (int s0 = 0; s0 < nsl; s0 += 8) {  // eight independent loads in flight
+          uint32_t v[8];
+#pragma unroll
+          for (int q = 0; q < 8; ++q) v[q] = (s0 + q < nsl) ? __ldg(sb + (s0 + q) * 32) : 0u;
+#pragma unroll
+          for (int q = 0; q < 8; ++q) hit |= (s0 + q < nsl) && half16(v[q], half) + g == best;
+        }
+      }
       const unsigned m = __ballot_sync(0xffffffffu, hit) >> (16 * half) & 0xffffu;
       if (band8 < 0 && m) band8 = st * 32 + 16 * l2 + __ffs(m) - 1;
     }
@@ -593,7 +602,7 @@ __global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int
           op = 'I'; --j;
         }
         h = hp_get(Hp, i - R0, j - C0);
-        if (n < stride) o[n] = op; else overflow = true;
+        if (n < ops_cap) ops[n] = op;
         ++n;
       }
     }
@@ -601,9 +610,13 @@ __global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int
     j = __shfl_sync(0xffffffffu, j, 16 * half);
     h = __shfl_sync(0xffffffffu, h, 16 * half);
   }
+  // path start -> end, written by the half's 16 lanes
+  n = __shfl_sync(0xffffffffu, n, 16 * half);
+  overflow = n > stride || n > ops_cap;
+  __syncwarp();
+  if (mine && !overflow)
+    for (int64_t u = hl; u < n; u += 16) o[u] = ops[n - 1 - u];
   if (hl == 0 && mine) {
-    if (!overflow)
-      for (int64_t u = 0, v = n - 1; u < v; ++u, --v) { const uint8_t t = o[u]; o[u] = o[v]; o[v] = t; }
     out_len[qidx] = overflow ? -1 : (int32_t)n;
     if (coords) {
       coords[4 * qidx] = active ? i : 0; coords[4 * qidx + 1] = active ? j : 0;
@@ -657,7 +670,7 @@ cudaError_t sw16_traceback(const Sw16Args& A, int64_t first, int64_t count, uint
   const int seq_bytes = (int)(((A.max_la + 15) & ~15) + ((A.max_lb + 15) & ~15));
   ++*launches;
   if (getenv("DP_SW_TB_UNPACKED") == nullptr) {  // packed: two problems per warp
-    const size_t smem = 4 * (2 * ((size_t)kPW * 4 + seq_bytes));
+    const size_t smem = 4 * (2 * ((size_t)kPW * 4 + 2 * (size_t)seq_bytes));
     cudaError_t e = cudaFuncSetAttribute(k_sw16_tb2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     const int64_t groups = ((first + count - 1) >> 1) - (first >> 1) + 1;
