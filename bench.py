@@ -65,18 +65,25 @@ class ClockSampler:
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "20"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.started = threading.Event()
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
+            self.started.wait(timeout=5.0)  # first sample (pre-region) is discarded
         except Exception:
             self.proc = None
         return self
 
     def _read(self):
+        first = True
         for line in self.proc.stdout:
             parts = [x.strip() for x in line.split(",")]
             if len(parts) >= 6:
+                if first:
+                    first = False
+                    self.started.set()
+                    continue
                 self.samples.append(parts)
 
     def __exit__(self, *a):

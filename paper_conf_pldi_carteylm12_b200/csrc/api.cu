@@ -131,6 +131,7 @@ cudaError_t sw16_args(dp_plan* p, int64_t n, const uint8_t* a_cat, const int64_t
   A->rowck = static_cast<uint32_t*>(p->tb_state.ptr);
   A->colck = A->rowck + rw;
   A->slabbest = A->colck + cw;
+  A->corner = A->slabbest + bw / 2;
   A->strips_max = strips;
   A->nslab_max = nslab > 0 ? nslab : 1;
   p->last_scores = scores;
@@ -432,16 +433,8 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
     case DP_NUSSINOV: {
       if (stride < p->last_max_la) return DP_E_TOO_LARGE;
       const int64_t ds = p->last_max_la > 0 ? p->last_max_la : 1;
-      if (stride == ds) {
-        e = cudaMemcpyAsync(out, static_cast<uint8_t*>(p->tb_state.ptr) + first * ds, count * ds,
-                            cudaMemcpyDeviceToDevice, s);
-      } else {
-        e = cudaMemcpy2DAsync(out, stride, static_cast<uint8_t*>(p->tb_state.ptr) + first * ds, ds, ds, count,
-                              cudaMemcpyDeviceToDevice, s);
-      }
-      if (e == cudaSuccess)
-        e = cudaMemcpyAsync(out_len, static_cast<int32_t*>(p->tb_aux.ptr) + first, count * 4,
-                            cudaMemcpyDeviceToDevice, s);
+      e = dpk::nuss_copy_db(static_cast<uint8_t*>(p->tb_state.ptr), ds, static_cast<int32_t*>(p->tb_aux.ptr), first,
+                            count, out, stride, out_len, s, &p->launches);
       break;
     }
     case DP_HMM_VITERBI: {

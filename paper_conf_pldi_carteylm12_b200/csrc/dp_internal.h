@@ -41,8 +41,9 @@ struct Sw16Args {
   int32_t* scores;
   // traceback checkpoints (nullptr in score-only mode)
   uint32_t* rowck;       // [groups][strips][8 bands][max_lb]    G of each 32-row band's bottom row (packed pair)
-  uint32_t* colck;       // [groups][strips][nslab][256]         G of every 32nd column
-  uint32_t* slabbest;    // [groups][strips][nslab][32]           per-lane best G per 32-column slab
+  uint32_t* colck;       // [groups][strips][nslab][256]         G at each lane's checkpoint column 32 s - lane
+  uint32_t* slabbest;    // [groups][strips][nslab][32]           per-lane best G per slab (32 sweep steps)
+  uint32_t* corner;      // [groups][strips][nslab][32]           G of the row above the lane at its checkpoint column
   int64_t strips_max, nslab_max;
 };
 bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap);
@@ -74,6 +75,9 @@ bool nuss_tiled_supported(int64_t max_len);
 int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device);
 cudaError_t nuss_tiled_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t nuss_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
+// copy rows [first, first+count) of the dot-bracket scratch (row stride ds) and their lengths
+cudaError_t nuss_copy_db(const uint8_t* db, int64_t ds, const int32_t* lens, int64_t first, int64_t count,
+                         uint8_t* out, int64_t stride, int32_t* out_len, cudaStream_t s, int64_t* launches);
 
 // ---------------------------------------------------------------- HMM
 struct HmmArgs {

@@ -87,34 +87,57 @@ __device__ void nuss_init(int16_t* U, int16_t* L, int n, int64_t tid, int64_t nt
 }
 
 // Canonical traceback (DESIGN.md R-TB-NUSS): Durbin order, smallest split k.
-// One thread; explicit stack in global scratch.
-__device__ void nuss_traceback(const int16_t* U, const int16_t* L, const uint8_t* x, int n, const uint8_t* pm, int h,
-                               uint8_t* db, int* stack) {
-  for (int k = 0; k < n; ++k) db[k] = '.';
+// One warp: lane 0 owns the explicit stack (global scratch, L1/L2-resident);
+// the split search is spread over the 32 lanes and the smallest matching k is
+// taken with a ballot, so a step costs ceil((j-i-1)/32) table reads per lane
+// instead of j-i-1 serial ones.
+__device__ void nuss_traceback_warp(const int16_t* U, const int16_t* L, const uint8_t* x, int n, const uint8_t* pm,
+                                    int h, uint8_t* db, int* stack) {
+  const int lane = threadIdx.x & 31;
+  for (int k = lane; k < n; k += 32) db[k] = '.';
   if (n <= 1) return;
+  __syncwarp();
   auto gam = [&](int i, int j) -> int { return (j - i < 1) ? 0 : (int)U[ustart(i, n) + (j - i)]; };
-  int sp = 0;
-  stack[sp++] = 0; stack[sp++] = n - 1;
+  int sp = 0;  // identical in every lane
+  if (lane == 0) { stack[0] = 0; stack[1] = n - 1; }
+  sp = 2;
   int guard = 4 * n + 8;
   while (sp > 0 && --guard > 0) {
-    const int j = stack[--sp], i = stack[--sp];
+    __syncwarp();
+    const int j = stack[sp - 1], i = stack[sp - 2];
+    sp -= 2;
     if (j - i < 1) continue;
     const int v = gam(i, j);
-    if (v == gam(i + 1, j)) { stack[sp++] = i + 1; stack[sp++] = j; continue; }
-    if (v == gam(i, j - 1)) { stack[sp++] = i; stack[sp++] = j - 1; continue; }
-    if (pm[x[i] * 4 + x[j]] && j - i - 1 >= h && v == gam(i + 1, j - 1) + 1) {
-      db[i] = '('; db[j] = ')';
-      stack[sp++] = i + 1; stack[sp++] = j - 1;
-      continue;
-    }
-    const int16_t* Ui = U + ustart(i, n);
-    const int16_t* Lj = L + lstart(j);
-    for (int k = i + 1; k < j; ++k)
-      if (v == (int)Ui[k - i] + (int)Lj[k]) {
-        stack[sp++] = k + 1; stack[sp++] = j;
-        stack[sp++] = i; stack[sp++] = k;
-        break;
+    int ni0 = -1, nj0 = 0, ni1 = -1, nj1 = 0;  // up to two intervals to push (second on top)
+    if (v == gam(i + 1, j)) {
+      ni0 = i + 1; nj0 = j;
+    } else if (v == gam(i, j - 1)) {
+      ni0 = i; nj0 = j - 1;
+    } else if (pm[x[i] * 4 + x[j]] && j - i - 1 >= h && v == gam(i + 1, j - 1) + 1) {
+      if (lane == 0) { db[i] = '('; db[j] = ')'; }
+      ni0 = i + 1; nj0 = j - 1;
+    } else {
+      const int16_t* Ui = U + ustart(i, n);
+      const int16_t* Lj = L + lstart(j);
+      for (int k0 = i + 1; k0 < j; k0 += 32) {
+        const int k = k0 + lane;
+        const unsigned hit = __ballot_sync(0xffffffffu, k < j && v == (int)Ui[k - i] + (int)Lj[k]);
+        if (hit) {
+          const int kk = k0 + __ffs(hit) - 1;
+          ni0 = kk + 1; nj0 = j; ni1 = i; nj1 = kk;
+          break;
+        }
       }
+    }
+    __syncwarp();
+    if (ni0 >= 0) {
+      if (lane == 0) { stack[sp] = ni0; stack[sp + 1] = nj0; }
+      sp += 2;
+    }
+    if (ni1 >= 0) {
+      if (lane == 0) { stack[sp] = ni1; stack[sp + 1] = nj1; }
+      sp += 2;
+    }
   }
 }
 
@@ -145,12 +168,10 @@ __global__ void __launch_bounds__(kNussThreads) k_nuss_cta(NussArgs A, int64_t s
       nuss_partition(U, L, xs, n, d, pm, A.hairpin, threadIdx.x, blockDim.x);
       __syncthreads();
     }
-    if (threadIdx.x == 0) {
-      A.scores[p] = n <= 1 ? 0 : (int)U[ustart(0, n) + n - 1];
-      if (A.db) {
-        nuss_traceback(U, L, xs, n, pm, A.hairpin, A.db + p * A.db_stride, stack);
-        A.db_len[p] = n;
-      }
+    if (threadIdx.x == 0) A.scores[p] = n <= 1 ? 0 : (int)U[ustart(0, n) + n - 1];
+    if (A.db && threadIdx.x < 32) {
+      nuss_traceback_warp(U, L, xs, n, pm, A.hairpin, A.db + p * A.db_stride, stack);
+      if (threadIdx.x == 0) A.db_len[p] = n;
     }
   }
 }
@@ -174,13 +195,23 @@ __global__ void __launch_bounds__(kNussThreads) k_nuss_grid(NussArgs A, int64_t 
     nuss_partition(U, L, x, n, d, pm, A.hairpin, tid, nthr);
     grid.sync();
   }
-  if (tid == 0) {
-    A.scores[p] = n <= 1 ? 0 : (int)U[ustart(0, n) + n - 1];
-    if (A.db) {
-      int* stack = reinterpret_cast<int*>(U + table_elems(n));
-      nuss_traceback(U, L, x, n, pm, A.hairpin, A.db + p * A.db_stride, stack);
-      A.db_len[p] = n;
-    }
+  if (tid == 0) A.scores[p] = n <= 1 ? 0 : (int)U[ustart(0, n) + n - 1];
+  if (A.db && tid < 32) {
+    int* stack = reinterpret_cast<int*>(U + table_elems(n));
+    nuss_traceback_warp(U, L, x, n, pm, A.hairpin, A.db + p * A.db_stride, stack);
+    if (tid == 0) A.db_len[p] = n;
+  }
+}
+
+// One CTA per row: bytes of the row, then its length.
+__global__ void k_copy_db(const uint8_t* db, int64_t ds, const int32_t* lens, int64_t first, int64_t count,
+                          uint8_t* out, int64_t stride, int32_t* out_len) {
+  for (int64_t r = blockIdx.x; r < count; r += gridDim.x) {
+    const uint8_t* src = db + (first + r) * ds;
+    uint8_t* dst = out + r * stride;
+    const int len = lens[first + r];
+    for (int k = threadIdx.x; k < len; k += blockDim.x) dst[k] = src[k];
+    if (threadIdx.x == 0) out_len[r] = len;
   }
 }
 
@@ -191,6 +222,15 @@ int num_sms(int device) {
 }
 
 }  // namespace
+
+cudaError_t nuss_copy_db(const uint8_t* db, int64_t ds, const int32_t* lens, int64_t first, int64_t count,
+                         uint8_t* out, int64_t stride, int32_t* out_len, cudaStream_t s, int64_t* launches) {
+  if (count <= 0) return cudaSuccess;
+  const int64_t grid = std::min<int64_t>(count, 148 * 16);
+  ++*launches;
+  k_copy_db<<<(unsigned)grid, 128, 0, s>>>(db, ds, lens, first, count, out, stride, out_len);
+  return cudaGetLastError();
+}
 
 int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device) {
   const int64_t stack_bytes = (4 * max_len + 8) * 4;
