@@ -1,5 +1,6 @@
 // C ABI (include/dp.h): plan lifecycle, dispatch to the kernels, traceback,
 // host-buffer entry point. No exception crosses this boundary.
+#include <algorithm>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
@@ -60,8 +61,12 @@ struct dp_plan {
   const int64_t *last_aoff = nullptr, *last_boff = nullptr;
   int32_t* last_scores = nullptr;  // device (alignment traceback reads the score)
   DevBuf own_scores;               // when the caller's scores are float/host we keep a copy
-  // host-API staging
+  // host-API staging (dp_solve_batch_host): copies run on their own streams,
+  // chunk by chunk, overlapped with the solve of the neighbouring chunks
   DevBuf h_a, h_b, h_aoff, h_boff, h_scores, h_tb, h_tblen, h_coords;
+  cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+  static constexpr int kMaxChunks = 8;
+  cudaEvent_t ev_start = nullptr, ev_in[kMaxChunks] = {}, ev_out[kMaxChunks] = {};
   int64_t launches = 0;
 };
 
@@ -169,6 +174,13 @@ void dp_plan_destroy(dp_plan_t p) {
   DevBuf* bufs[] = {&p->tb_state, &p->tb_aux, &p->tb_aux2, &p->scratch, &p->own_scores, &p->h_a, &p->h_b,
                     &p->h_aoff, &p->h_boff, &p->h_scores, &p->h_tb, &p->h_tblen, &p->h_coords};
   for (DevBuf* b : bufs) b->release();
+  if (p->s_h2d) cudaStreamDestroy(p->s_h2d);
+  if (p->s_d2h) cudaStreamDestroy(p->s_d2h);
+  if (p->ev_start) cudaEventDestroy(p->ev_start);
+  for (int k = 0; k < dp_plan::kMaxChunks; ++k) {
+    if (p->ev_in[k]) cudaEventDestroy(p->ev_in[k]);
+    if (p->ev_out[k]) cudaEventDestroy(p->ev_out[k]);
+  }
   cudaSetDevice(cur);
   delete p;
 }
@@ -470,55 +482,78 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   if (max_la > p->max_la || max_lb > p->max_lb) return DP_E_TOO_LARGE;
   const int64_t abytes = n > 0 ? a_off[n] - a_off[0] : 0;
   const int64_t bbytes = (align && n > 0) ? b_off[n] - b_off[0] : 0;
+  const bool tb = p->want_tb && tb_out && tb_len && p->kind != DP_HMM_FORWARD && n > 0;
   cudaError_t e = p->h_a.ensure((size_t)abytes + 16);
   if (e == cudaSuccess) e = p->h_aoff.ensure((size_t)(n + 1) * 8);
   if (e == cudaSuccess && align) e = p->h_b.ensure((size_t)bbytes + 16);
   if (e == cudaSuccess && align) e = p->h_boff.ensure((size_t)(n + 1) * 8);
   if (e == cudaSuccess) e = p->h_scores.ensure((size_t)n * 4 + 16);
+  if (e == cudaSuccess && tb) e = p->h_tb.ensure((size_t)(n * tb_stride) + 16);
+  if (e == cudaSuccess && tb) e = p->h_tblen.ensure((size_t)n * 4 + 16);
+  if (e == cudaSuccess && tb && tb_coords) e = p->h_coords.ensure((size_t)n * 16 + 16);
+  if (e == cudaSuccess && !p->s_h2d) e = cudaStreamCreateWithFlags(&p->s_h2d, cudaStreamNonBlocking);
+  if (e == cudaSuccess && !p->s_d2h) e = cudaStreamCreateWithFlags(&p->s_d2h, cudaStreamNonBlocking);
+  if (e == cudaSuccess && !p->ev_start) e = cudaEventCreateWithFlags(&p->ev_start, cudaEventDisableTiming);
+  for (int k = 0; e == cudaSuccess && k < dp_plan::kMaxChunks; ++k) {
+    if (!p->ev_in[k]) e = cudaEventCreateWithFlags(&p->ev_in[k], cudaEventDisableTiming);
+    if (e == cudaSuccess && !p->ev_out[k]) e = cudaEventCreateWithFlags(&p->ev_out[k], cudaEventDisableTiming);
+  }
   if (e != cudaSuccess) return cuda_status(e);
-  // offsets are rebased to 0 when a_off[0] != 0
-  std::vector<int64_t> ao, bo;
-  const int64_t* aoff_h = a_off;
-  const int64_t* boff_h = b_off;
-  if (n > 0 && a_off[0] != 0) {
-    ao.resize(n + 1);
-    for (int64_t q = 0; q <= n; ++q) ao[q] = a_off[q] - a_off[0];
-    aoff_h = ao.data();
-  }
-  if (align && n > 0 && b_off[0] != 0) {
-    bo.resize(n + 1);
-    for (int64_t q = 0; q <= n; ++q) bo[q] = b_off[q] - b_off[0];
-    boff_h = bo.data();
-  }
-  if (n > 0) {
-    e = cudaMemcpyAsync(p->h_a.ptr, a_cat + a_off[0], abytes, cudaMemcpyHostToDevice, s);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(p->h_aoff.ptr, aoff_h, (n + 1) * 8, cudaMemcpyHostToDevice, s);
-    if (e == cudaSuccess && align) e = cudaMemcpyAsync(p->h_b.ptr, b_cat + b_off[0], bbytes, cudaMemcpyHostToDevice, s);
-    if (e == cudaSuccess && align) e = cudaMemcpyAsync(p->h_boff.ptr, boff_h, (n + 1) * 8, cudaMemcpyHostToDevice, s);
-    if (e != cudaSuccess) return cuda_status(e);
-  }
-  dp_status st = dp_solve_batch(p, n, static_cast<uint8_t*>(p->h_a.ptr), static_cast<int64_t*>(p->h_aoff.ptr),
-                                align ? static_cast<uint8_t*>(p->h_b.ptr) : nullptr,
-                                align ? static_cast<int64_t*>(p->h_boff.ptr) : nullptr, max_la, max_lb,
-                                p->h_scores.ptr, stream);
-  if (st != DP_OK) return st;
-  if (n > 0) e = cudaMemcpyAsync(scores_out, p->h_scores.ptr, n * 4, cudaMemcpyDeviceToHost, s);
+  if (n == 0) return dp_solve_batch(p, 0, nullptr, nullptr, nullptr, nullptr, 0, 0, p->h_scores.ptr, stream);
+  // Chunks of the batch: chunk c is copied in on s_h2d, solved (and traced) on
+  // the caller's stream, copied out on s_d2h, so the transfers of one chunk
+  // overlap the solve of its neighbours. Device copies keep the host layout:
+  // byte q of a_cat lives at h_a + (q - a_off[0]), so the kernels take the
+  // caller's (absolute) offsets with a rebased base pointer.
+  // a chunk must still fill the GPU: ~3 waves of the sweep kernels
+  const int64_t min_chunk = align ? 16384 : (p->kind == DP_NUSSINOV ? 65536 : 32768);
+  int nch = (int)std::min<int64_t>(dp_plan::kMaxChunks / 2, (n + min_chunk - 1) / min_chunk);
+  if (nch < 1) nch = 1;
+  const int64_t per = (n + nch - 1) / nch;
+  uint8_t* da = static_cast<uint8_t*>(p->h_a.ptr);
+  uint8_t* db = align ? static_cast<uint8_t*>(p->h_b.ptr) : nullptr;
+  int64_t* dao = static_cast<int64_t*>(p->h_aoff.ptr);
+  int64_t* dbo = align ? static_cast<int64_t*>(p->h_boff.ptr) : nullptr;
+  e = cudaEventRecord(p->ev_start, s);  // buffers are free once earlier work on the caller's stream is done
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(p->s_h2d, p->ev_start, 0);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(dao, a_off, (n + 1) * 8, cudaMemcpyHostToDevice, p->s_h2d);
+  if (e == cudaSuccess && align) e = cudaMemcpyAsync(dbo, b_off, (n + 1) * 8, cudaMemcpyHostToDevice, p->s_h2d);
   if (e != cudaSuccess) return cuda_status(e);
-  if (p->want_tb && tb_out && tb_len && p->kind != DP_HMM_FORWARD && n > 0) {
-    e = p->h_tb.ensure((size_t)(n * tb_stride) + 16);
-    if (e == cudaSuccess) e = p->h_tblen.ensure((size_t)n * 4 + 16);
-    if (e == cudaSuccess && tb_coords) e = p->h_coords.ensure((size_t)n * 16 + 16);
+  for (int c = 0; c < nch; ++c) {
+    const int64_t k0 = c * per, k1 = std::min(n, k0 + per), nk = k1 - k0;
+    if (nk <= 0) break;
+    e = cudaMemcpyAsync(da + (a_off[k0] - a_off[0]), a_cat + a_off[k0], a_off[k1] - a_off[k0],
+                        cudaMemcpyHostToDevice, p->s_h2d);
+    if (e == cudaSuccess && align)
+      e = cudaMemcpyAsync(db + (b_off[k0] - b_off[0]), b_cat + b_off[k0], b_off[k1] - b_off[k0],
+                          cudaMemcpyHostToDevice, p->s_h2d);
+    if (e == cudaSuccess) e = cudaEventRecord(p->ev_in[c], p->s_h2d);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(s, p->ev_in[c], 0);
     if (e != cudaSuccess) return cuda_status(e);
-    st = dp_traceback(p, 0, n, static_cast<uint8_t*>(p->h_tb.ptr), tb_stride, static_cast<int32_t*>(p->h_tblen.ptr),
-                      tb_coords ? static_cast<int32_t*>(p->h_coords.ptr) : nullptr, stream);
+    int32_t* dsc = static_cast<int32_t*>(p->h_scores.ptr) + k0;
+    dp_status st = dp_solve_batch(p, nk, da - a_off[0], dao + k0, align ? db - b_off[0] : nullptr,
+                                  align ? dbo + k0 : nullptr, max_la, max_lb, dsc, stream);
     if (st != DP_OK) return st;
-    e = cudaMemcpyAsync(tb_out, p->h_tb.ptr, n * tb_stride, cudaMemcpyDeviceToHost, s);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(tb_len, p->h_tblen.ptr, n * 4, cudaMemcpyDeviceToHost, s);
-    if (e == cudaSuccess && tb_coords)
-      e = cudaMemcpyAsync(tb_coords, p->h_coords.ptr, n * 16, cudaMemcpyDeviceToHost, s);
+    uint8_t* dtb = tb ? static_cast<uint8_t*>(p->h_tb.ptr) + k0 * tb_stride : nullptr;
+    int32_t* dtl = tb ? static_cast<int32_t*>(p->h_tblen.ptr) + k0 : nullptr;
+    int32_t* dco = (tb && tb_coords) ? static_cast<int32_t*>(p->h_coords.ptr) + 4 * k0 : nullptr;
+    if (tb) {
+      st = dp_traceback(p, 0, nk, dtb, tb_stride, dtl, dco, stream);
+      if (st != DP_OK) return st;
+    }
+    e = cudaEventRecord(p->ev_out[c], s);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(p->s_d2h, p->ev_out[c], 0);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(static_cast<uint8_t*>(scores_out) + 4 * k0, dsc, nk * 4, cudaMemcpyDeviceToHost, p->s_d2h);
+    if (e == cudaSuccess && tb) e = cudaMemcpyAsync(tb_out + k0 * tb_stride, dtb, nk * tb_stride,
+                                                    cudaMemcpyDeviceToHost, p->s_d2h);
+    if (e == cudaSuccess && tb) e = cudaMemcpyAsync(tb_len + k0, dtl, nk * 4, cudaMemcpyDeviceToHost, p->s_d2h);
+    if (e == cudaSuccess && dco) e = cudaMemcpyAsync(tb_coords + 4 * k0, dco, nk * 16, cudaMemcpyDeviceToHost, p->s_d2h);
     if (e != cudaSuccess) return cuda_status(e);
   }
-  return cuda_status(cudaStreamSynchronize(s));
+  e = cudaStreamSynchronize(p->s_d2h);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  return cuda_status(e);
 }
 
 }  // extern "C"

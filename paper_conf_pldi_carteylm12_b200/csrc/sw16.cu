@@ -495,7 +495,7 @@ __global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int
   const int ei = active ? blk * kBlk + myr : 0, ej = active ? myc : 0;
   // 3) walk back block by block; the two halves walk concurrently (leaders hl == 0)
   int i = ei, j = ej, h = active ? best : 0;
-  int64_t n = 0;
+  int n = 0;
   bool overflow = false;
   while (__any_sync(0xffffffffu, h > 0)) {
     const bool on = h > 0;
@@ -507,25 +507,32 @@ __global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int
     }
     packed_block(V, a, b, bg, sl, on, Hp, sig32, g, hl);
     if (hl == 0 && on) {
+      // walk in the block's sheared coordinates: packed row t (1..16) of half hf, column c
       const int R0 = bg * kBlk, D = sl * kSlab - (R0 % kStrip) / kRows;
-      while (h > 0 && i > R0) {
-        const int ri = i - R0, hf = ri > 16 ? 1 : 0, t = ri - 16 * hf;
-        const int c = j - D + ((ri - 1) >> 3);  // sheared column of (i, j)
-        if (c < 1) break;                       // left of this block
-        const int cu = j - D + shear_of(hf, t - 1);  // (i-1, j) in the row above's shear
-        const int sub = sig_s[a[i - 1] * 32 + b[j - 1]];
-        const int dV = hp_at(Hp, hf, t - 1, cu - 1), uV = hp_at(Hp, hf, t - 1, cu);
-        uint8_t op;
-        if (h == dV + sub) {
-          op = (a[i - 1] == b[j - 1]) ? 'M' : 'X';
-          --i; --j; h = dV;
-        } else if (h == uV - g) {
-          op = 'D'; --i; h = uV;
-        } else {
-          op = 'I'; --j; h = hp_at(Hp, hf, t, c - 1);
-        }
+      const int ri = i - R0;
+      int hf = ri > 16 ? 1 : 0, t = ri - 16 * hf;
+      int c = j - D + ((ri - 1) >> 3);
+      int sh = 16 * hf;
+      while (h > 0 && t >= 1 && c >= 1) {
+        // branch-free step: all three neighbours are read, the move is selected
+        const int tm = t - 1, cu = c - (t == 9 ? 1 : 0);  // row above: one column left at a forward-lane start
+        const uint32_t* up_row = Hp + tm * kPS;
+        const int dV = (int)(int16_t)(up_row[cu] >> sh), uV = (int)(int16_t)(up_row[cu + 1] >> sh);
+        const int lV = (int)(int16_t)(Hp[t * kPS + c] >> sh);
+        const int ra = a[i - 1], rb = b[j - 1];
+        const int sub = sig_s[ra * 32 + rb];
+        const bool isD = h == dV + sub;
+        const bool isU = !isD && h == uV - g;
+        const bool mvI = isD || isU;  // the row index moves
+        const uint8_t op = isD ? (ra == rb ? 'M' : 'X') : (isU ? 'D' : 'I');
+        h = isD ? dV : (isU ? uV : lV);
+        i -= mvI ? 1 : 0;
+        j -= isU ? 0 : 1;
+        c = isD ? cu - 1 : (isU ? cu : c - 1);
+        t = mvI ? tm : t;
         if (n < ops_cap) ops[n] = op;
         ++n;
+        if (t == 0 && hf == 1) { hf = 0; sh = 0; t = 16; --c; }  // row 16: continue in the low half (shear 1)
       }
     }
     i = __shfl_sync(0xffffffffu, i, 16 * half);
