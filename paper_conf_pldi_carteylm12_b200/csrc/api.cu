@@ -370,8 +370,26 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         H.pi = p->d_pi; H.A = p->d_A; H.E = p->d_E;
         H.ll_out = static_cast<float*>(scores_out);
         // the [batch x S] x [S x S] step on tcgen05 (SIMT fallback kernel via DP_HMM_SIMT=1)
+        unsigned long long* dbg = nullptr;
+        if (getenv("DP_HMM_TIMING")) cudaMalloc(&dbg, 8 * 4 * 66), cudaMemset(dbg, 0, 8 * 4 * 66), H.dbg = dbg;
         e = dpk::hmm_forward_tc_supported(p->S) ? dpk::hmm_forward_tc(H, s, &p->launches)
                                                  : dpk::hmm_forward(H, s, &p->launches);
+        if (dbg) {  // diagnostic: CTA 0 step phases (ns): MMA issue, wait for MMA, epilogue, barrier
+          unsigned long long h[4 * 66];
+          cudaStreamSynchronize(s);
+          cudaMemcpy(h, dbg, sizeof(h), cudaMemcpyDeviceToHost);
+          double acc[4] = {0, 0, 0, 0};
+          int cnt = 0;
+          for (int i = 10; i < 65; ++i) {
+            if (!h[4 * i] || !h[4 * (i + 1)]) continue;
+            acc[0] += h[4 * i + 1] - h[4 * i]; acc[1] += h[4 * i + 2] - h[4 * i + 1];
+            acc[2] += h[4 * i + 3] - h[4 * i + 2]; acc[3] += h[4 * (i + 1)] - h[4 * i + 3];
+            ++cnt;
+          }
+          if (cnt) fprintf(stderr, "forward step ns: issue %.0f wait %.0f epilogue %.0f barrier %.0f\n", acc[0] / cnt,
+                           acc[1] / cnt, acc[2] / cnt, acc[3] / cnt);
+          cudaFree(dbg);
+        }
       } else {
         H.lpi = p->d_lpi; H.lA = p->d_lA; H.lE = p->d_lE;
         H.vit_out = static_cast<int32_t*>(scores_out);

@@ -92,6 +92,7 @@ struct HmmArgs {
   int32_t* vit_out;                 // Viterbi
   uint8_t* bp;                      // Viterbi back-pointers (n x max_len x 64) or nullptr
   int32_t* final_state;             // n
+  unsigned long long* dbg = nullptr;  // diagnostic step timestamps (DP_HMM_TIMING), else nullptr
 };
 cudaError_t hmm_forward(const HmmArgs& a, cudaStream_t s, int64_t* launches);
 bool hmm_forward_tc_supported(int S);

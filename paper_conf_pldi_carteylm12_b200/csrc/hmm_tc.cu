@@ -5,19 +5,23 @@
 //     D[b][s] = sum_p alpha_{i-1}[b][p] * t_{p,s}
 // followed by the emission / normalisation epilogue of Fig.11a (L472–L474).
 //
-// One CTA = 128 sequences (the MMA's M), 4 warps. Thread b owns sequence b and
-// TMEM lane b. Per step:
-//   * thread 0 issues 12 tcgen05.mma.kind::f16 (M=128, N=64, K=16) into the
-//     fp32 TMEM accumulator: alpha_hi*A_hi + alpha_hi*A_lo + alpha_lo*A_hi,
-//     where x = x_hi + x_lo is a two-term bf16 split (product error ~2^-16 of
-//     a 2^-8 term: ~1e-7 relative per step);
-//   * tcgen05.commit arrives on an mbarrier; all threads wait on it, read
-//     their 64 columns with tcgen05.ld, multiply by e_s(x_i), normalise by the
-//     row sum c_i (log P = sum_i log c_i, fp64), split into bf16 hi/lo and
-//     store them in shared memory in the canonical K-major no-swizzle UMMA
-//     layout (8x16-byte core matrices) for the next step.
-// Operands live in shared memory (alpha hi/lo 2 x 16 KB, transitions hi/lo
-// 2 x 8 KB); the accumulator lives in TMEM (64 columns).
+// One CTA = 128 sequences (the MMA's M), 16 warps: warp w reads TMEM lane
+// quarter w % 4 (sequences 32 (w % 4) ..) and handles states 16 (w / 4) .. + 15.
+// Per step:
+//   * thread 0 issues 8 tcgen05.mma.kind::f16 (M=128, K=16) into the fp32 TMEM
+//     accumulator: alpha_hi x [A_hi | A_lo] (N=128) and alpha_lo x A_hi (N=64),
+//     where x = x_hi + x_lo is a two-term bf16 split (the dropped lo x lo term is
+//     ~2^-16 of a 2^-8 term: ~1e-7 relative per step);
+//     columns 64..127 hold alpha_hi A_lo and are added in the epilogue;
+//   * tcgen05.commit arrives on an mbarrier; every thread reads its 16 (+16)
+//     columns with tcgen05.ld, multiplies by e_s(x_i), scales by 1/R_{i-1} (the
+//     previous step's row sum: lagged scaling keeps the row reduction off the
+//     critical path, log P = sum_i log R_i), splits into bf16 hi/lo and stores
+//     the next A operand in the canonical K-major no-swizzle UMMA layout
+//     (8x16-byte core matrices).
+// Operands live in shared memory (alpha hi/lo 2 x 16 KB, transitions 16 KB);
+// the accumulator lives in TMEM (128 columns). DP_HMM_TIMING=1 prints per-phase
+// step times of CTA 0 (diagnostic).
 #include <cstdint>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -30,7 +34,8 @@ namespace {
 constexpr int kM = 128;       // sequences per CTA (UMMA M)
 constexpr int kS = 64;        // states (UMMA N and K)
 constexpr int kCore = 128;    // bytes per 8x(16 B) core matrix
-constexpr int kTmemCols = 64;
+constexpr int kN2 = 2 * kS;    // N of the alpha_hi x [A_hi | A_lo] product
+constexpr int kTmemCols = kN2;
 
 // K-major no-swizzle operand: core matrix (row group rg, k chunk kc) at
 // (kc * row_groups + rg) * 128 bytes, rows of a core matrix 16 bytes apart.
@@ -48,16 +53,18 @@ __device__ __forceinline__ uint64_t make_desc(uint32_t saddr, uint32_t lbo, uint
   return d;
 }
 
-// kind::f16 instruction descriptor: D f32, A/B bf16, both K-major, N = 64, M = 128
-constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(kS >> 3) << 17) | ((uint32_t)(kM >> 4) << 24);
+// kind::f16 instruction descriptors: D f32, A/B bf16, both K-major, M = 128, N = 64 / 128
+template <int N>
+__host__ __device__ constexpr uint32_t idesc() { return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(kM >> 4) << 24); }
 
+template <int N>
 __device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
   asm volatile(
       "{\n\t.reg .pred p;\n\t"
       "setp.ne.b32 p, %4, 0;\n\t"
       "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n"
       :
-      : "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(kIdesc), "r"(accumulate));
+      : "r"(tmem_d), "l"(adesc), "l"(bdesc), "n"(idesc<N>()), "r"(accumulate));
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -84,41 +91,52 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]) \
       : "r"(taddr))
 
+constexpr int kThreads = 512;  // 16 warps: warp w serves TMEM lane quarter w % 4 and states 16 (w / 4) ..
+
 struct TcSmem {
   alignas(128) uint8_t a_hi[kM * kS * 2];   // alpha (A operand), K-major core matrices
   alignas(128) uint8_t a_lo[kM * kS * 2];
-  alignas(128) uint8_t b_hi[kS * kS * 2];   // transitions (B operand): row = s (N), k = p
-  alignas(128) uint8_t b_lo[kS * kS * 2];
+  alignas(128) uint8_t b_cat[kN2 * kS * 2];  // transitions (B operand): row n = s (A_hi) or 64 + s (A_lo), k = p
   alignas(16) float E[16][kS + 4];          // emission rows, padded against bank conflicts
+  float psum[2][4][kM];                     // per-step partial row sums (double-buffered by step parity)
   uint64_t bar;
   uint32_t tmem_base;
 };
 
-// bf16 pair split: v = hi + lo with hi = bf16(v), lo = bf16(v - hi)
-__device__ __forceinline__ void split_bf16(float v, __nv_bfloat16& hi, __nv_bfloat16& lo) {
-  hi = __float2bfloat16_rn(v);
-  lo = __float2bfloat16_rn(v - __bfloat162float(hi));
+// Two bf16x2 words (hi, lo) with a + b = (hi.x + lo.x, hi.y + lo.y) to ~2^-16.
+__device__ __forceinline__ void split2(float a, float b, uint32_t& hi, uint32_t& lo) {
+  const __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  const float2 hf = __bfloat1622float2(h);
+  const __nv_bfloat162 l = __floats2bfloat162_rn(a - hf.x, b - hf.y);
+  hi = *reinterpret_cast<const uint32_t*>(&h);
+  lo = *reinterpret_cast<const uint32_t*>(&l);
 }
 
-__global__ void __launch_bounds__(kM, 1) k_forward_tc(HmmArgs H) {
+// Per step, with lagged scaling: alpha^_i = ((alpha^_{i-1} A) o e(x_i)) / R_{i-1},
+// R_i = sum_s alpha^_i(s); then P(x) = prod_{i<=T} R_i and log P = sum log R_i. Dividing by the
+// previous step's sum (known before the MMA finishes) keeps R_i within the emission range
+// because A is row-stochastic, and takes the row reduction off the critical path.
+__global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
   extern __shared__ __align__(1024) uint8_t tc_raw[];
   TcSmem& sm = *reinterpret_cast<TcSmem*>(tc_raw);
-  const int tid = threadIdx.x, warp = tid >> 5;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int lq = warp & 3, cg = warp >> 2;  // TMEM lane quarter, state group
+  const int b = 32 * lq + lane;             // this thread's sequence (row) in the CTA
+  const int s0 = 16 * cg;                   // this thread's 16 states
   const int S = H.S, K = H.K;
-  const int64_t p = (int64_t)blockIdx.x * kM + tid;
+  const int64_t p = (int64_t)blockIdx.x * kM + b;
   const bool live = p < H.n;
 
   // transitions: B[s][p] = t_{p,s} (K = p contiguous), split into bf16 hi/lo
-  for (int q = tid; q < kS * kS; q += kM) {
+  for (int q = tid; q < kS * kS; q += kThreads) {
     const int s = q / kS, pp = q % kS;
     const float v = (s < S && pp < S) ? H.A[pp * S + s] : 0.f;
-    __nv_bfloat16 hi, lo;
-    split_bf16(v, hi, lo);
-    const uint32_t off = op_offset(s, pp, kS / 8);
-    *reinterpret_cast<__nv_bfloat16*>(sm.b_hi + off) = hi;
-    *reinterpret_cast<__nv_bfloat16*>(sm.b_lo + off) = lo;
+    const __nv_bfloat16 hi = __float2bfloat16_rn(v);
+    const __nv_bfloat16 lo = __float2bfloat16_rn(v - __bfloat162float(hi));
+    *reinterpret_cast<__nv_bfloat16*>(sm.b_cat + op_offset(s, pp, kN2 / 8)) = hi;
+    *reinterpret_cast<__nv_bfloat16*>(sm.b_cat + op_offset(kS + s, pp, kN2 / 8)) = lo;
   }
-  for (int q = tid; q < 16 * (kS + 4); q += kM) {
+  for (int q = tid; q < 16 * (kS + 4); q += kThreads) {
     const int c = q / (kS + 4), s = q % (kS + 4);
     sm.E[c][s] = (c < K && s < S) ? H.E[s * K + c] : 0.f;
   }
@@ -131,91 +149,92 @@ __global__ void __launch_bounds__(kM, 1) k_forward_tc(HmmArgs H) {
                  "n"(kTmemCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
+  const uint8_t* x = live ? H.x_cat + H.x_off[p] : nullptr;
+  const int T = live ? (int)(H.x_off[p + 1] - H.x_off[p]) : 0;
+  __shared__ int tmax_s;
+  if (tid == 0) tmax_s = 0;
   asm volatile("fence.proxy.async.shared::cta;");
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = sm.tmem_base;
+  if (cg == 0) atomicMax(&tmax_s, T);
 
-  const uint8_t* x = live ? H.x_cat + H.x_off[p] : nullptr;
-  const int T = live ? (int)(H.x_off[p + 1] - H.x_off[p]) : 0;
-  int Tmax = T;
-  // the CTA runs to its longest sequence
-  {
-    __shared__ int tmax_s;
-    if (tid == 0) tmax_s = 0;
-    __syncthreads();
-    atomicMax(&tmax_s, T);
-    __syncthreads();
-    Tmax = tmax_s;
-  }
-  float alpha[kS];
-  double ll = 0.0;
-  // i = 1: a(s) = pi_s e_s(x_1)
+  const uint32_t a_hi = smem_u32(sm.a_hi), a_lo = smem_u32(sm.a_lo);
+  // descriptors: K chunk pairs 32 bytes... (2 core matrices of 8 k) apart by 2 x LBO
+  const uint64_t dA_hi = make_desc(a_hi, (kM / 8) * kCore, kCore), dA_lo = make_desc(a_lo, (kM / 8) * kCore, kCore);
+  const uint64_t dB = make_desc(smem_u32(sm.b_cat), (kN2 / 8) * kCore, kCore);
+  const uint32_t taddr = tmem + ((uint32_t)(lq * 32) << 16) + (uint32_t)s0;
+  // store 16 values of alpha^ as the A operand (k = s0 .. s0 + 15: two k chunks of 8)
+  auto store_operand = [&](const float* v) {
+    uint32_t hw[8], lw[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) split2(v[2 * q], v[2 * q + 1], hw[q], lw[q]);
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const uint32_t off = op_offset(b, s0 + 8 * h, kM / 8);
+      *reinterpret_cast<uint4*>(sm.a_hi + off) = make_uint4(hw[4 * h], hw[4 * h + 1], hw[4 * h + 2], hw[4 * h + 3]);
+      *reinterpret_cast<uint4*>(sm.a_lo + off) = make_uint4(lw[4 * h], lw[4 * h + 1], lw[4 * h + 2], lw[4 * h + 3]);
+    }
+  };
+  // i = 1: alpha^_1(s) = pi_s e_s(x_1) (no scaling)
   {
     const int c = T > 0 ? x[0] : 0;
-    float tot = 0.f;
+    float v[16], tot = 0.f;
 #pragma unroll
-    for (int s = 0; s < kS; ++s) {
-      alpha[s] = (s < S && T > 0) ? H.pi[s] * sm.E[c][s] : 0.f;
-      tot += alpha[s];
+    for (int q = 0; q < 16; ++q) {
+      const int s = s0 + q;
+      v[q] = (s < S && T > 0) ? H.pi[s] * sm.E[c][s] : 0.f;
+      tot += v[q];
     }
-    const float inv = tot > 0.f ? 1.f / tot : 0.f;
-    if (T > 0) ll = log((double)tot);
-#pragma unroll
-    for (int s = 0; s < kS; ++s) alpha[s] *= inv;
+    store_operand(v);
+    sm.psum[1][cg][b] = tot;
   }
-  const uint32_t a_hi = smem_u32(sm.a_hi), a_lo = smem_u32(sm.a_lo);
-  const uint32_t b_hi = smem_u32(sm.b_hi), b_lo = smem_u32(sm.b_lo);
-  const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16);  // this warp's 32 TMEM lanes
+  asm volatile("fence.proxy.async.shared::cta;");
+  asm volatile("tcgen05.fence::before_thread_sync;");
+  __syncthreads();
+  const int Tmax = tmax_s;
+  double prod = 1.0;  // prod of R_i, renormalised: P = prod * 2^pexp
+  int pexp = 0;
   uint32_t parity = 0;
   uint4 xs = make_uint4(0, 0, 0, 0);
-  for (int i = 2; i <= Tmax; ++i) {
-    // alpha_{i-1} -> shared memory (bf16 hi/lo, K-major core matrices)
-#pragma unroll
-    for (int kc = 0; kc < kS / 8; ++kc) {
-      uint32_t hw[4], lw[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        __nv_bfloat16 h0, l0, h1, l1;
-        split_bf16(alpha[kc * 8 + 2 * q], h0, l0);
-        split_bf16(alpha[kc * 8 + 2 * q + 1], h1, l1);
-        hw[q] = (uint32_t)__bfloat16_as_ushort(h0) | ((uint32_t)__bfloat16_as_ushort(h1) << 16);
-        lw[q] = (uint32_t)__bfloat16_as_ushort(l0) | ((uint32_t)__bfloat16_as_ushort(l1) << 16);
-      }
-      const uint32_t off = op_offset(tid, kc * 8, kM / 8);
-      *reinterpret_cast<uint4*>(sm.a_hi + off) = make_uint4(hw[0], hw[1], hw[2], hw[3]);
-      *reinterpret_cast<uint4*>(sm.a_lo + off) = make_uint4(lw[0], lw[1], lw[2], lw[3]);
+  auto stamp = [&](int i, int k) {
+    if (H.dbg && blockIdx.x == 0 && tid == 0 && i < 66) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      H.dbg[4 * i + k] = t;
     }
-    asm volatile("fence.proxy.async.shared::cta;");
-    asm volatile("tcgen05.fence::before_thread_sync;");
-    __syncthreads();
+  };
+  for (int i = 2; i <= Tmax; ++i) {
+    stamp(i, 0);
     if (tid == 0) {
       asm volatile("tcgen05.fence::after_thread_sync;");
-      // D = a_hi*b_hi + a_hi*b_lo + a_lo*b_hi, K = 64 in 4 steps of 16
+      // D[:, 0:64] = a_hi*A_hi + a_lo*A_hi, D[:, 64:128] = a_hi*A_lo; K = 64 in 4 steps of 16.
+      // Descriptor address fields count 16-byte units: a K step of 16 is two core matrices.
 #pragma unroll
-      for (int kk = 0; kk < kS / 16; ++kk) {
-        const uint32_t ka = (uint32_t)(2 * kk) * (kM / 8) * kCore;  // two k chunks per MMA
-        const uint32_t kb = (uint32_t)(2 * kk) * (kS / 8) * kCore;
-        mma_bf16(tmem, make_desc(a_hi + ka, (kM / 8) * kCore, kCore), make_desc(b_hi + kb, (kS / 8) * kCore, kCore),
-                 kk > 0);
-      }
+      for (int kk = 0; kk < kS / 16; ++kk)
+        mma_bf16<kN2>(tmem, dA_hi + (uint64_t)(2 * kk * (kM / 8) * kCore >> 4),
+                      dB + (uint64_t)(2 * kk * (kN2 / 8) * kCore >> 4), kk > 0);
 #pragma unroll
-      for (int kk = 0; kk < kS / 16; ++kk) {
-        const uint32_t ka = (uint32_t)(2 * kk) * (kM / 8) * kCore;
-        const uint32_t kb = (uint32_t)(2 * kk) * (kS / 8) * kCore;
-        mma_bf16(tmem, make_desc(a_hi + ka, (kM / 8) * kCore, kCore), make_desc(b_lo + kb, (kS / 8) * kCore, kCore), 1);
-      }
-#pragma unroll
-      for (int kk = 0; kk < kS / 16; ++kk) {
-        const uint32_t ka = (uint32_t)(2 * kk) * (kM / 8) * kCore;
-        const uint32_t kb = (uint32_t)(2 * kk) * (kS / 8) * kCore;
-        mma_bf16(tmem, make_desc(a_lo + ka, (kM / 8) * kCore, kCore), make_desc(b_hi + kb, (kS / 8) * kCore, kCore), 1);
-      }
+      for (int kk = 0; kk < kS / 16; ++kk)
+        mma_bf16<kS>(tmem, dA_lo + (uint64_t)(2 * kk * (kM / 8) * kCore >> 4),
+                     dB + (uint64_t)(2 * kk * (kN2 / 8) * kCore >> 4), 1);
       asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
           smem_u32(&sm.bar)));
     }
-    // next symbol (prefetched 16 at a time) while the MMAs run
+    stamp(i, 1);
+    // while the MMAs run: R_{i-1}, the scale, the symbol and its emission row
+    const float* ps = &sm.psum[(i - 1) & 1][0][0];
+    const float R = (ps[b] + ps[kM + b]) + (ps[2 * kM + b] + ps[3 * kM + b]);
+    const float inv = R > 0.f ? 1.f / R : 0.f;
+    if (i - 1 <= T) {
+      prod *= (double)R;
+      if ((i & 15) == 0) {  // keep the product normal: P = prod * 2^pexp
+        int e2;
+        prod = frexp(prod, &e2);
+        pexp += e2;
+      }
+    }
     if (((i - 2) & 15) == 0 && i - 1 < T) {
       uint8_t tmp[16];
 #pragma unroll
@@ -225,32 +244,37 @@ __global__ void __launch_bounds__(kM, 1) k_forward_tc(HmmArgs H) {
     const int sh = (i - 2) & 15;
     const uint32_t word = sh < 4 ? xs.x : sh < 8 ? xs.y : sh < 12 ? xs.z : xs.w;
     const int c = (word >> (8 * (sh & 3))) & 0xff;
+    const float4* er = reinterpret_cast<const float4*>(&sm.E[c][s0]);
+    const float4 e0 = er[0], e1 = er[1], e2 = er[2], e3 = er[3];
     mbar_wait(&sm.bar, parity);
+    stamp(i, 2);
     parity ^= 1;
     asm volatile("tcgen05.fence::after_thread_sync;");
-    uint32_t r[kS];
-    TMEM_LD16(taddr + 0, (&r[0]));
-    TMEM_LD16(taddr + 16, (&r[16]));
-    TMEM_LD16(taddr + 32, (&r[32]));
-    TMEM_LD16(taddr + 48, (&r[48]));
+    uint32_t r[16], r2[16];
+    TMEM_LD16(taddr, r);
+    TMEM_LD16(taddr + kS, r2);
     asm volatile("tcgen05.wait::ld.sync.aligned;");
     if (i <= T) {
-      const float4* er = reinterpret_cast<const float4*>(sm.E[c]);
-      float tot = 0.f;
+      const float ev[16] = {e0.x, e0.y, e0.z, e0.w, e1.x, e1.y, e1.z, e1.w,
+                            e2.x, e2.y, e2.z, e2.w, e3.x, e3.y, e3.z, e3.w};
+      float v[16], tot = 0.f;
 #pragma unroll
-      for (int q4 = 0; q4 < kS / 4; ++q4) {
-        const float4 e = er[q4];
-        alpha[4 * q4 + 0] = __uint_as_float(r[4 * q4 + 0]) * e.x;
-        alpha[4 * q4 + 1] = __uint_as_float(r[4 * q4 + 1]) * e.y;
-        alpha[4 * q4 + 2] = __uint_as_float(r[4 * q4 + 2]) * e.z;
-        alpha[4 * q4 + 3] = __uint_as_float(r[4 * q4 + 3]) * e.w;
-        tot += (alpha[4 * q4 + 0] + alpha[4 * q4 + 1]) + (alpha[4 * q4 + 2] + alpha[4 * q4 + 3]);
+      for (int q = 0; q < 16; ++q) {
+        v[q] = (__uint_as_float(r[q]) + __uint_as_float(r2[q])) * ev[q] * inv;
+        tot += v[q];
       }
-      const float inv = tot > 0.f ? 1.f / tot : 0.f;
-      ll += log((double)tot);
-#pragma unroll
-      for (int s = 0; s < kS; ++s) alpha[s] *= inv;
+      store_operand(v);
+      sm.psum[i & 1][cg][b] = tot;
     }
+    stamp(i, 3);
+    asm volatile("fence.proxy.async.shared::cta;");
+    asm volatile("tcgen05.fence::before_thread_sync;");
+    __syncthreads();
+  }
+  if (cg == 0 && Tmax >= 1 && Tmax <= T) {  // R_T of the sequences that run to the end
+    const float* ps = &sm.psum[Tmax & 1][0][0];
+    const float R = (ps[b] + ps[kM + b]) + (ps[2 * kM + b] + ps[3 * kM + b]);
+    prod *= (double)R;
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
@@ -258,7 +282,7 @@ __global__ void __launch_bounds__(kM, 1) k_forward_tc(HmmArgs H) {
     asm volatile("tcgen05.fence::after_thread_sync;");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kTmemCols));
   }
-  if (live) H.ll_out[p] = T == 0 ? 0.f : (float)ll;
+  if (live && cg == 0) H.ll_out[p] = T == 0 ? 0.f : (float)(log(prod) + (double)pexp * 0.69314718055994530942);
 }
 
 }  // namespace
@@ -271,7 +295,7 @@ cudaError_t hmm_forward_tc(const HmmArgs& H, cudaStream_t s, int64_t* launches) 
   cudaError_t e = cudaFuncSetAttribute(k_forward_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   ++*launches;
-  k_forward_tc<<<(unsigned)((H.n + kM - 1) / kM), kM, smem, s>>>(H);
+  k_forward_tc<<<(unsigned)((H.n + kM - 1) / kM), kThreads, smem, s>>>(H);
   return cudaGetLastError();
 }
 
