@@ -54,6 +54,16 @@ def lib():
         L.orc_sw.argtypes = [u8p, i64, u8p, i64, i8p, ctypes.c_int, i64, ctypes.POINTER(i64), ctypes.POINTER(i64)]
         L.orc_sw_traceback.restype = i64
         L.orc_sw_traceback.argtypes = [u8p, i64, u8p, i64, i8p, ctypes.c_int, i64, u8p, i64p]
+        L.orc_sw_affine.restype = i64
+        L.orc_sw_affine.argtypes = [u8p, i64, u8p, i64, i8p, ctypes.c_int, i64, i64, ctypes.POINTER(i64),
+                                    ctypes.POINTER(i64)]
+        L.orc_sw_affine_traceback.restype = i64
+        L.orc_sw_affine_traceback.argtypes = [u8p, i64, u8p, i64, i8p, ctypes.c_int, i64, i64, u8p, i64p]
+        L.orc_sw_affine_batch.restype = None
+        L.orc_sw_affine_batch.argtypes = [i64, i64, u8p, i64p, u8p, i64p, i8p, ctypes.c_int, i64, i64, i64p]
+        L.orc_sw_affine_traceback_batch.restype = None
+        L.orc_sw_affine_traceback_batch.argtypes = [i64, i64, u8p, i64p, u8p, i64p, i8p, ctypes.c_int, i64, i64,
+                                                    u8p, i64, i64p]
         L.orc_nussinov.restype = i64
         L.orc_nussinov.argtypes = [u8p, i64, u8p, ctypes.c_int]
         L.orc_nussinov_traceback.restype = i64
@@ -111,6 +121,49 @@ def sw_traceback(s, t, sigma, g) -> tuple[str, tuple[int, int, int, int]]:
     co = np.zeros(4, dtype=np.int64)
     n = lib().orc_sw_traceback(s, len(s), t, len(t), sig, sig.shape[0], int(g), buf, co)
     return bytes(buf[:n]).decode(), tuple(int(v) for v in co)
+
+
+def sw_affine(s, t, sigma, go, ge) -> tuple[int, int, int]:
+    """Affine-gap SW (gap of length k costs go + k*ge): (score, end_i, end_j)."""
+    s, t = _u8(s), _u8(t)
+    sig = np.ascontiguousarray(sigma, dtype=np.int8)
+    ei, ej = i64(0), i64(0)
+    sc = lib().orc_sw_affine(s, len(s), t, len(t), sig, sig.shape[0], int(go), int(ge), ctypes.byref(ei),
+                             ctypes.byref(ej))
+    return int(sc), int(ei.value), int(ej.value)
+
+
+def sw_affine_traceback(s, t, sigma, go, ge) -> tuple[str, tuple[int, int, int, int]]:
+    s, t = _u8(s), _u8(t)
+    sig = np.ascontiguousarray(sigma, dtype=np.int8)
+    buf = np.zeros(len(s) + len(t) + 1, dtype=np.uint8)
+    co = np.zeros(4, dtype=np.int64)
+    n = lib().orc_sw_affine_traceback(s, len(s), t, len(t), sig, sig.shape[0], int(go), int(ge), buf, co)
+    return bytes(buf[:n]).decode(), tuple(int(v) for v in co)
+
+
+def sw_affine_batch(a_cat, a_off, b_cat, b_off, sigma, go, ge, threads=1) -> np.ndarray:
+    n = len(a_off) - 1
+    out = np.zeros(n, dtype=np.int64)
+    sig = np.ascontiguousarray(sigma, dtype=np.int8)
+    a_cat, b_cat = _u8(a_cat), _u8(b_cat)
+    a_off, b_off = np.ascontiguousarray(a_off, np.int64), np.ascontiguousarray(b_off, np.int64)
+    _parallel(n, lambda f, c: lib().orc_sw_affine_batch(f, c, a_cat, a_off, b_cat, b_off, sig, sig.shape[0],
+                                                        int(go), int(ge), out), threads)
+    return out
+
+
+def sw_affine_traceback_batch(a_cat, a_off, b_cat, b_off, sigma, go, ge, stride, threads=1):
+    n = len(a_off) - 1
+    ops = np.zeros((n, stride), dtype=np.uint8)
+    lens = np.zeros(n, dtype=np.int64)
+    sig = np.ascontiguousarray(sigma, dtype=np.int8)
+    a_cat, b_cat = _u8(a_cat), _u8(b_cat)
+    a_off, b_off = np.ascontiguousarray(a_off, np.int64), np.ascontiguousarray(b_off, np.int64)
+    _parallel(n, lambda f, c: lib().orc_sw_affine_traceback_batch(f, c, a_cat, a_off, b_cat, b_off, sig,
+                                                                  sig.shape[0], int(go), int(ge), ops.reshape(-1),
+                                                                  stride, lens), threads)
+    return ops, lens
 
 
 def nussinov(x, pair_mask, h) -> int:

@@ -90,6 +90,47 @@ def brute_local_cells(s, t, sigma, gap):
     return H, best, (bi, bj)
 
 
+def score_alignment_affine(s, t, ops, sub, go, ge):
+    """Affine gap cost: every maximal run of k 'D' (or k 'I') ops costs go + k*ge; a
+    D-run directly followed by an I-run is two gaps."""
+    i = j = 0
+    tot = 0
+    prev = None
+    for o in ops:
+        if o in "SMX":
+            tot += sub(s[i], t[j]); i += 1; j += 1
+        else:
+            if o != prev:
+                tot -= go
+            tot -= ge
+            if o == "D":
+                i += 1
+            else:
+                j += 1
+        prev = o
+    assert i == len(s) and j == len(t)
+    return tot
+
+
+def brute_local_affine(s, t, sigma, go, ge):
+    """max over every local alignment (every pair of substrings, every global alignment
+    of them) of the affine score; the empty alignment scores 0."""
+    n, m = len(s), len(t)
+    sub = lambda a, b: int(sigma[a][b])
+    aligns = {}
+    best = 0
+    for i0 in range(n + 1):
+        for i in range(i0, n + 1):
+            for j0 in range(m + 1):
+                for j in range(j0, m + 1):
+                    key = (i - i0, j - j0)
+                    if key not in aligns:
+                        aligns[key] = all_global_alignments(*key)
+                    for ops in aligns[key]:
+                        best = max(best, score_alignment_affine(s[i0:i], t[j0:j], ops, sub, go, ge))
+    return best
+
+
 # ----------------------------------------------------------------------------- secondary structures
 def all_structures(n, can_pair, h):
     """Every secondary structure (set of non-crossing pairs (i,j), i<j, j-i-1>=h,
