@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define DP_ABI_VERSION 1
+#define DP_ABI_VERSION 2
 #define DP_MAX_DIM 4
 
 typedef enum dp_status {
@@ -53,7 +53,9 @@ typedef enum dp_kind {
   DP_SW_LINEAR = 1,   /* §6.1 L502–L507 + §5.1: local alignment, linear gap, int32 score */
   DP_NUSSINOV = 2,    /* interval DP with max over split k (ref [3], L598), int32 #pairs */
   DP_HMM_FORWARD = 3, /* Fig.11a, natural-log likelihood, float32 */
-  DP_HMM_VITERBI = 4  /* max-variant of Fig.11a (L463–L464), int32 milli-bit score */
+  DP_HMM_VITERBI = 4, /* max-variant of Fig.11a (L463–L464), int32 milli-bit score */
+  DP_SW_AFFINE = 5    /* SURVEY §8(f) NEXT 1 (Gotoh, L509–L520; mutual recursion = Further Work L585–L589):
+                         local alignment, gap of length k costs gap_open + k * gap_extend, int32 score */
 } dp_kind;
 
 /*
@@ -115,6 +117,9 @@ typedef struct dp_desc {
   int32_t coeff_bound;       /* 0 -> 10 */
   const int32_t* user_coeff; /* optional user schedule to verify (length = recurrence ndim) */
   int32_t want_traceback;    /* retain state for dp_traceback */
+  /* affine gaps (DP_SW_AFFINE; ABI 2): gap of length k costs gap_open + k * gap_extend */
+  int32_t gap_open;          /* >= 0 */
+  int32_t gap_extend;        /* >= 1 */
 } dp_desc;
 
 typedef struct dp_plan* dp_plan_t;

@@ -15,9 +15,9 @@ import numpy as np
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libdp.so")
 
-EDIT, SW_LINEAR, NUSSINOV, HMM_FORWARD, HMM_VITERBI = range(5)
+EDIT, SW_LINEAR, NUSSINOV, HMM_FORWARD, HMM_VITERBI, SW_AFFINE = range(6)
 KIND_NAMES = {EDIT: "edit", SW_LINEAR: "sw_linear", NUSSINOV: "nussinov", HMM_FORWARD: "hmm_forward",
-              HMM_VITERBI: "hmm_viterbi"}
+              HMM_VITERBI: "hmm_viterbi", SW_AFFINE: "sw_affine"}
 STATUS = {0: "DP_OK", 1: "DP_E_INVALID", 2: "DP_E_NO_SCHEDULE", 3: "DP_E_UNSUPPORTED", 4: "DP_E_TOO_LARGE",
           5: "DP_E_NOMEM", 6: "DP_E_CUDA", 7: "DP_E_NO_TRACEBACK"}
 MAX_DIM = 4
@@ -44,6 +44,7 @@ class Desc(ctypes.Structure):
         ("n_states", ctypes.c_int32), ("pi", ctypes.c_void_p), ("A", ctypes.c_void_p), ("E", ctypes.c_void_p),
         ("lpi", ctypes.c_void_p), ("lA", ctypes.c_void_p), ("lE", ctypes.c_void_p),
         ("coeff_bound", ctypes.c_int32), ("user_coeff", ctypes.c_void_p), ("want_traceback", ctypes.c_int32),
+        ("gap_open", ctypes.c_int32), ("gap_extend", ctypes.c_int32),
     ]
 
 
@@ -137,7 +138,7 @@ class Plan:
 
     def __init__(self, kind, max_len_a, max_len_b=0, *, sigma=None, gap=0, alphabet_size=0, pair_mask=None,
                  min_hairpin=0, pi=None, A=None, E=None, lpi=None, lA=None, lE=None, want_traceback=False,
-                 coeff_bound=0, user_coeff=None):
+                 coeff_bound=0, user_coeff=None, gap_open=0, gap_extend=0):
         self.kind = kind
         self._keep = []
         d = Desc()
@@ -146,6 +147,7 @@ class Plan:
         d.max_len_a, d.max_len_b = int(max_len_a), int(max_len_b)
         d.alphabet_size = int(alphabet_size)
         d.gap = int(gap)
+        d.gap_open, d.gap_extend = int(gap_open), int(gap_extend)
         d.min_hairpin = int(min_hairpin)
         d.want_traceback = int(bool(want_traceback))
         d.coeff_bound = int(coeff_bound)
@@ -259,7 +261,7 @@ class Plan:
         if self.want_traceback and tb_stride:
             tb = np.empty((n, tb_stride), dtype=np.uint8)
             tbl = np.empty(n, dtype=np.int32)
-            if self.kind in (EDIT, SW_LINEAR):
+            if self.kind in (EDIT, SW_LINEAR, SW_AFFINE):
                 tbc = np.empty((n, 4), dtype=np.int32)
         _check(lib().dp_solve_batch_host(self._h, n, _ptr(a_cat), _ptr(a_off), _ptr(b_cat), _ptr(b_off),
                                          _ptr(scores), _ptr(tb), int(tb_stride), _ptr(tbl), _ptr(tbc),

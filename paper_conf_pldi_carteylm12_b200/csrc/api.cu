@@ -40,6 +40,7 @@ struct dp_plan {
   int device = 0;
   int64_t max_la = 0, max_lb = 0;
   int asz = 0, gap = 0, hairpin = 0, S = 0, K = 0;
+  int gap_open = 0, gap_ext = 0;  // DP_SW_AFFINE
   bool want_tb = false;
   int ndim = 2;
   int32_t coeff[DP_MAX_DIM] = {0, 0, 0, 0};
@@ -94,6 +95,7 @@ int families(int kind, int64_t la, int64_t lb, int S, int64_t ext[2], int* trian
   switch (kind) {
     case DP_EDIT:
     case DP_SW_LINEAR:  // d(i-1,j), d(i,j-1), d(i-1,j-1)  (Fig.7; §6.1)
+    case DP_SW_AFFINE:  // E <- (0,-1), F <- (-1,0), H <- (-1,-1); same-cell H <- E, F orders a cell's tables
       ext[0] = la + 1; ext[1] = lb + 1;
       deps[0].offset[0] = -1;
       deps[1].offset[1] = -1;
@@ -189,7 +191,7 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
   if (!d || !out) return DP_E_INVALID;
   *out = nullptr;
   if (d->struct_size != sizeof(dp_desc)) return DP_E_INVALID;
-  if (d->kind < DP_EDIT || d->kind > DP_HMM_VITERBI) return DP_E_INVALID;
+  if (d->kind < DP_EDIT || d->kind > DP_SW_AFFINE) return DP_E_INVALID;
   if (d->max_len_a < 0 || d->max_len_b < 0) return DP_E_INVALID;
   dp_plan* p = new (std::nothrow) dp_plan();
   if (!p) return DP_E_NOMEM;
@@ -217,6 +219,15 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
       p->packed16 = dpk::sw16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap) &&
                     getenv("DP_FORCE_INT32") == nullptr;
+      break;
+    case DP_SW_AFFINE:
+      p->asz = d->alphabet_size;
+      if (!d->sigma || p->asz < 1 || d->gap_open < 0 || d->gap_extend < 1) { st = DP_E_INVALID; break; }
+      if (p->asz > 32) { st = DP_E_UNSUPPORTED; break; }
+      p->gap_open = d->gap_open; p->gap_ext = d->gap_extend;
+      if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) { st = DP_E_TOO_LARGE; break; }
+      e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
+      p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
       break;
     case DP_NUSSINOV:
       if (!d->pair_mask || d->min_hairpin < 0) { st = DP_E_INVALID; break; }
@@ -258,7 +269,7 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
     // The kernels implement the derived schedule; a user schedule that is valid
     // but differs would need another kernel (conditional schedules, §4.7: NEXT).
     // Coefficients of a dimension of extent 1 do not change the partitions.
-    static const int32_t expect[5][2] = {{1, 1}, {1, 1}, {-1, 1}, {0, 1}, {0, 1}};
+    static const int32_t expect[6][2] = {{1, 1}, {1, 1}, {-1, 1}, {0, 1}, {0, 1}, {1, 1}};
     for (int i = 0; i < 2; ++i)
       if (p->ext[i] > 1 && p->coeff[i] != expect[d->kind][i]) st = DP_E_UNSUPPORTED;
   }
@@ -288,7 +299,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
                          void* stream) {
   if (!p || n < 0) return DP_E_INVALID;
   if (n > 0 && (!a_off || !scores_out)) return DP_E_INVALID;
-  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR;
+  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE;
   if (align && n > 0 && !b_off) return DP_E_INVALID;
   if (max_len_a < 0 || max_len_b < 0) return DP_E_INVALID;
   if (max_len_a > p->max_la || (align && max_len_b > p->max_lb)) return DP_E_TOO_LARGE;
@@ -325,6 +336,25 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         p->last_scores = A.scores;
       }
       e = dpk::align_solve(A, s, &p->launches);
+      break;
+    }
+    case DP_SW_AFFINE: {
+      dpk::AlignArgs A{};
+      A.n = n; A.a_cat = a_cat; A.b_cat = b_cat; A.a_off = a_off; A.b_off = b_off;
+      A.max_la = max_len_a > 0 ? max_len_a : 1; A.max_lb = max_len_b > 0 ? max_len_b : 1;
+      A.sigma = p->d_sigma; A.asz = p->asz; A.local = true;
+      A.gap_open = p->gap_open; A.gap_ext = p->gap_ext;
+      A.scores = static_cast<int32_t*>(scores_out);
+      if (p->want_tb) {
+        A.dir_stride = dpk::align_affine_dir_words(A.max_la, A.max_lb);
+        e = p->tb_state.ensure((size_t)(n * A.dir_stride * 4 + 16));
+        if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 2 * 4 + 16));
+        if (e != cudaSuccess) break;
+        A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
+        A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
+        p->last_scores = A.scores;
+      }
+      e = dpk::align_affine_solve(A, s, &p->launches);
       break;
     }
     case DP_NUSSINOV: {
@@ -460,6 +490,20 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
       e = dpk::align_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
       break;
     }
+    case DP_SW_AFFINE: {
+      if (stride < p->last_max_la + p->last_max_lb) return DP_E_TOO_LARGE;
+      dpk::AlignArgs A{};
+      A.n = p->last_n; A.a_cat = p->last_a; A.b_cat = p->last_b; A.a_off = p->last_aoff; A.b_off = p->last_boff;
+      A.max_la = p->last_max_la > 0 ? p->last_max_la : 1; A.max_lb = p->last_max_lb > 0 ? p->last_max_lb : 1;
+      A.sigma = p->d_sigma; A.asz = p->asz; A.local = true;
+      A.gap_open = p->gap_open; A.gap_ext = p->gap_ext;
+      A.scores = p->last_scores;
+      A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
+      A.dir_stride = dpk::align_affine_dir_words(A.max_la, A.max_lb);
+      A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
+      e = dpk::align_affine_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
+      break;
+    }
     case DP_NUSSINOV: {
       if (stride < p->last_max_la) return DP_E_TOO_LARGE;
       const int64_t ds = p->last_max_la > 0 ? p->last_max_la : 1;
@@ -483,7 +527,7 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
                               const uint8_t* b_cat, const int64_t* b_off, void* scores_out, uint8_t* tb_out,
                               int64_t tb_stride, int32_t* tb_len, int32_t* tb_coords, void* stream) {
   if (!p || n < 0 || (n > 0 && (!a_off || !a_cat || !scores_out))) return DP_E_INVALID;
-  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR;
+  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE;
   if (align && n > 0 && (!b_off || !b_cat)) return DP_E_INVALID;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   int64_t max_la = 0, max_lb = 0;

@@ -18,6 +18,7 @@ struct AlignArgs {
   int asz;
   int gap;
   bool local;            // SW (true) vs edit distance (false)
+  int gap_open, gap_ext; // affine SW (align_affine.cu)
   int32_t* scores;
   // traceback retention (nullptr when not wanted)
   uint32_t* dirs;        // direction codes, 2 bits per cell
@@ -25,6 +26,10 @@ struct AlignArgs {
   int32_t* ends;         // n x 2 (end_i, end_j)
 };
 int64_t align_dir_words(int64_t max_la, int64_t max_lb);  // words per problem for `dirs`
+int64_t align_affine_dir_words(int64_t max_la, int64_t max_lb);  // affine: 4 bits per cell
+cudaError_t align_affine_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
+cudaError_t align_affine_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
+                                   int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
 cudaError_t align_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t align_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                             int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);

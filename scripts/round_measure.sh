@@ -14,7 +14,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file
 ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_nuss4.csv python bench.py --config nuss4 --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
 ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_nuss5.csv env DP_NUSS5_N=50000 python bench.py --config nuss5 --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_sw16" -c 2 -o gpurun_out/ncu_sw python bench.py --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_forward_tc|k_viterbi<" -c 2 -o gpurun_out/ncu_hmm python bench.py --config hmm --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:"k_forward_tc|k_viterbi" -c 3 -o gpurun_out/ncu_hmm python bench.py --config hmm --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_nuss" -c 1 -o gpurun_out/ncu_nuss4 python bench.py --config nuss4 --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_nuss" -c 1 -o gpurun_out/ncu_nuss5 env DP_NUSS5_N=5000 python bench.py --config nuss5 --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
 ls -la gpurun_out

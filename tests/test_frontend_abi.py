@@ -30,7 +30,7 @@ def test_exports_match_header(dp):
     L = dp.lib()
     for name in declared:
         assert hasattr(L, name), name
-    assert L.dp_abi_version() == 1
+    assert L.dp_abi_version() == 2
     for code in range(8):
         assert L.dp_status_string(code)
 

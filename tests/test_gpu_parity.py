@@ -38,12 +38,13 @@ def rand_batch(g, n, lo, hi, k):
 
 
 # ----------------------------------------------------------------------------- alignment
-def run_align(dp, kind, a_seqs, b_seqs, sigma=None, gap=0, asz=26, tb=True):
+def run_align(dp, kind, a_seqs, b_seqs, sigma=None, gap=0, asz=26, tb=True, go=0, ge=0):
     a_cat, a_off = dpgen.pack(a_seqs)
     b_cat, b_off = dpgen.pack(b_seqs)
     la = max((len(s) for s in a_seqs), default=0)
     lb = max((len(s) for s in b_seqs), default=0)
-    plan = dp.Plan(kind, max(la, 1), max(lb, 1), sigma=sigma, gap=gap, alphabet_size=asz, want_traceback=tb)
+    plan = dp.Plan(kind, max(la, 1), max(lb, 1), sigma=sigma, gap=gap, alphabet_size=asz, want_traceback=tb,
+                   gap_open=go, gap_extend=ge)
     A = (cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off))
     sc = plan.solve_batch(*A, max_len_a=la, max_len_b=lb)
     res = {"scores": host(sc)}
@@ -111,6 +112,48 @@ def test_sw_packed_odd_batch_and_ties(dp, orc):
         sc, ei, ej = orc.sw(a[q], b[q], sig, 2)
         ops, co = orc.sw_traceback(a[q], b[q], sig, 2)
         assert r["scores"][q] == sc and r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+
+
+@pytest.mark.parametrize("maxlen,go,ge", [(40, 11, 1), (300, 11, 1), (300, 3, 2), (600, 0, 4)])
+def test_sw_affine_random_ragged(dp, orc, maxlen, go, ge):
+    """Affine gaps (NEXT rank 1): ragged lengths across lane tiles and strips; scores
+    and canonical three-table tracebacks bit-exact."""
+    g = np.random.default_rng(110 + maxlen + go)
+    sig = dpgen.blosum62()
+    n = 120
+    a, _ = rand_batch(g, n, 0, maxlen, 24)
+    b, _ = rand_batch(g, n, 0, maxlen, 24)
+    a += [np.arange(20, dtype=np.uint8)]
+    b += [np.concatenate([np.arange(10), [5, 5, 5], np.arange(10, 20)]).astype(np.uint8)]  # one long gap
+    r = run_align(dp, dp.SW_AFFINE, a, b, sigma=sig, asz=24, go=go, ge=ge)
+    for q in range(len(a)):
+        sc, _, _ = orc.sw_affine(a[q], b[q], sig, go, ge)
+        assert r["scores"][q] == sc, q
+        if q % 3 == 0 or q == len(a) - 1:
+            ops, co = orc.sw_affine_traceback(a[q], b[q], sig, go, ge)
+            assert r["ops"][q] == ops, q
+            assert tuple(r["coords"][q]) == co, q
+
+
+def test_sw_affine_config2_sampled(dp, orc):
+    """BASELINE config 2's pairs with affine gaps (open 11, extend 1) at full size,
+    in the bench's launch configuration; sampled pairs against the oracle."""
+    n = 100_000
+    a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(n, 256, first=0)
+    sig = dpgen.blosum62()
+    plan = dp.Plan(dp.SW_AFFINE, 256, 256, sigma=sig, alphabet_size=24, want_traceback=True, gap_open=11,
+                   gap_extend=1)
+    sc = host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=256, max_len_b=256))
+    out, ln, co = plan.traceback(0, n, 513)
+    idx = np.random.default_rng(111).choice(n, 40, replace=False)
+    out, ln, co = host(out), host(ln), host(co)
+    for q in idx:
+        a = a_cat[a_off[q]:a_off[q + 1]]
+        b = b_cat[b_off[q]:b_off[q + 1]]
+        ops, c = orc.sw_affine_traceback(a, b, sig, 11, 1)
+        assert sc[q] == orc.sw_affine(a, b, sig, 11, 1)[0], q
+        assert bytes(out[q, :ln[q]]).decode() == ops and tuple(co[q]) == c, q
+    plan.close()
 
 
 def test_sw_score_only_matches_traceback_mode(dp):
