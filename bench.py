@@ -115,6 +115,13 @@ def workload(name, rank, world):
                 "max_la": 256, "max_lb": 256, "cells": n * 256 * 256, "ops_per_cell": 3, "tb_stride": 513,
                 "workload": "BASELINE config 2: 100k protein pairs x 256 (uniform 20 aa), Smith-Waterman, "
                             "BLOSUM62, linear gap 4, with tracebacks"}
+    if name == "swa":
+        n = 100_000
+        a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(n, 256, first=rank * n)
+        return {"kind": "swa", "n": n, "a_cat": a_cat, "a_off": a_off, "b_cat": b_cat, "b_off": b_off,
+                "max_la": 256, "max_lb": 256, "cells": n * 256 * 256, "ops_per_cell": 6, "tb_stride": 513,
+                "workload": "config 2 pairs with affine gaps (SURVEY 8(f) NEXT 1): 100k protein pairs x 256, "
+                            "BLOSUM62, gap open 11 / extend 1, with tracebacks"}
     if name == "nuss1":
         x = dpgen.config1_rna64()
         cat, off = dpgen.pack([x])
@@ -170,6 +177,10 @@ def run_ours(args, rank, world, local_rank):
         plans.append(dp.Plan(dp.SW_LINEAR, W["max_la"], W["max_lb"], sigma=sig, gap=dpgen.SW_GAP,
                              want_traceback=True))
         dev_in = (cu(W["a_cat"]), cu(W["a_off"]), cu(W["b_cat"]), cu(W["b_off"]))
+    elif W["kind"] == "swa":
+        plans.append(dp.Plan(dp.SW_AFFINE, W["max_la"], W["max_lb"], sigma=dpgen.blosum62(),
+                             gap_open=dpgen.SW_GAP_OPEN, gap_extend=dpgen.SW_GAP_EXTEND, want_traceback=True))
+        dev_in = (cu(W["a_cat"]), cu(W["a_off"]), cu(W["b_cat"]), cu(W["b_off"]))
     elif W["kind"] == "nuss":
         plans.append(dp.Plan(dp.NUSSINOV, W["max_la"], pair_mask=dpgen.rna_pair_mask(),
                              min_hairpin=dpgen.NUSS_HAIRPIN, want_traceback=True))
@@ -187,7 +198,7 @@ def run_ours(args, rank, world, local_rank):
     stride = W["tb_stride"]
     tb_out = torch.empty((n, stride), dtype=torch.uint8, device=dev)
     tb_len = torch.empty(n, dtype=torch.int32, device=dev)
-    tb_co = torch.empty((n, 4), dtype=torch.int32, device=dev) if W["kind"] == "sw" else None
+    tb_co = torch.empty((n, 4), dtype=torch.int32, device=dev) if W["kind"] in ("sw", "swa") else None
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     gathered = None
     if world > 1:
@@ -195,11 +206,12 @@ def run_ours(args, rank, world, local_rank):
 
     # CUDA events (on the launching stream) around each phase of the step: every solve
     # launch and the traceback launch; the dominant one carries the roofline
-    phase_names = ([{"sw": "k_sw16 (partition sweep)", "nuss": "k_nuss (fill + in-kernel traceback)",
+    phase_names = ([{"sw": "k_sw16 (partition sweep)", "swa": "k_align_affine (partition sweep)",
+                     "nuss": "k_nuss (fill + in-kernel traceback)",
                      "hmm": "k_forward_tc (tcgen05 forward)"}[W["kind"]]] +
                    (["k_viterbi (max-plus)"] if W["kind"] == "hmm" else []) +
-                   [{"sw": "k_sw16_tb (traceback)", "nuss": "dp_traceback (copy)",
-                     "hmm": "k_viterbi_tb (traceback)"}[W["kind"]]])
+                   [{"sw": "k_sw16_tb (traceback)", "swa": "k_align_affine_tb (traceback)",
+                     "nuss": "dp_traceback (copy)", "hmm": "k_viterbi_tb (traceback)"}[W["kind"]]])
     ev_phase = [[] for _ in phase_names]
 
     def ev():
@@ -275,7 +287,7 @@ def run_ours(args, rank, world, local_rank):
         "higher_is_better": True,
         "scaling": "weak",
         "vs_baseline": None,
-        "dtype": {"sw": "int32", "nuss": "int16 table / int32 arithmetic", "hmm": "f32 (forward) + int32 (Viterbi)"}[W["kind"]],
+        "dtype": {"sw": "int32", "swa": "int32", "nuss": "int16 table / int32 arithmetic", "hmm": "f32 (forward) + int32 (Viterbi)"}[W["kind"]],
         "data": "synthetic (seeded, dpgen)",
         "config": {"workload": W["workload"], "config": args.config, "problems_per_gpu": n,
                    "cells_per_gpu": W["cells"], "l2": "flushed between steps (256 MiB write outside step events)",
@@ -322,6 +334,11 @@ def roofline(W, phase_ms, pk):
             tb["sweep"] = sweep
             return tb
         return sweep
+    if W["kind"] == "swa":
+        # E, F: add + fused add-max each; H: fused add-max + max; int32 (scores of affine SW are not
+        # bounded to 16 bits by the plan check) -> the s32 peak
+        return alu("k_align_affine", W["cells"] * W["ops_per_cell"], phase_ms[0], peak32,
+                   "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz")
     if W["kind"] == "nuss":
         return alu("k_nuss_tiled (fill + traceback)", W["inner"], phase_ms[0], peak16,
                    "ubench_r01 VIADDMNMX.S16x2 x 148 SMs x sm_max_mhz (one split evaluation = one max-plus)")
@@ -359,7 +376,7 @@ def e2e_host(args, W, plans, dev, stream, world):
         sc = pin(np.empty(n, np.float32 if (W["kind"] == "hmm" and k == 0) else np.int32))
         tb = pin(np.empty((n, stride), np.uint8)) if p.want_traceback else None
         tl = pin(np.empty(n, np.int32)) if p.want_traceback else None
-        tc = pin(np.empty((n, 4), np.int32)) if (p.want_traceback and W["kind"] == "sw") else None
+        tc = pin(np.empty((n, 4), np.int32)) if (p.want_traceback and W["kind"] in ("sw", "swa")) else None
         outs.append((sc, tb, tl, tc))
     h2d = a_cat.nbytes + a_off.nbytes + (b_cat.nbytes + b_off.nbytes if b_cat is not None else 0)
     h2d *= len(plans)
@@ -412,6 +429,16 @@ def oracle_sample(config, W, budget_s):
         oracle.sw_traceback_batch(a_cat, a_off, b_cat, b_off, sig, dpgen.SW_GAP, 513, threads=cores)
         dt = time.perf_counter() - t
         return k * 65536 / dt, f"first {k} pairs of config 2 (scores + canonical tracebacks)", cores
+    if config == "swa":
+        k = 1500
+        a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(k)
+        sig = dpgen.blosum62()
+        go, ge = dpgen.SW_GAP_OPEN, dpgen.SW_GAP_EXTEND
+        t = time.perf_counter()
+        oracle.sw_affine_batch(a_cat, a_off, b_cat, b_off, sig, go, ge, threads=cores)
+        oracle.sw_affine_traceback_batch(a_cat, a_off, b_cat, b_off, sig, go, ge, 513, threads=cores)
+        dt = time.perf_counter() - t
+        return k * 65536 / dt, f"first {k} pairs of config 2, affine gaps (scores + canonical tracebacks)", cores
     if config in ("nuss1",):
         x = dpgen.config1_rna64()
         reps = 200
@@ -477,7 +504,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="sw", choices=["sw", "nuss1", "hmm", "nuss4", "nuss5"])
+    ap.add_argument("--config", default="sw", choices=["sw", "swa", "nuss1", "hmm", "nuss4", "nuss5"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))

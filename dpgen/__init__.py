@@ -57,6 +57,7 @@ _B62_ROWS = """
 """
 
 SW_GAP = 4          # linear gap penalty g (BLOSUM62's '*' score)
+SW_GAP_OPEN, SW_GAP_EXTEND = 11, 1  # affine SW (NEXT rank 1): gap of length k costs 11 + k (NCBI BLOSUM62 default)
 NUSS_HAIRPIN = 3    # minimum hairpin loop h
 HMM_STATES = 64
 MILLIBIT_FLOOR = -100000  # score used for p == 0 (2^-100); Dirichlet(1) draws never hit it in practice
