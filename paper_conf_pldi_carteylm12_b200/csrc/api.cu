@@ -138,7 +138,9 @@ cudaError_t sw16_args(dp_plan* p, int64_t n, const uint8_t* a_cat, const int64_t
   A->rowck = static_cast<uint32_t*>(p->tb_state.ptr);
   A->colck = A->rowck + rw;
   A->slabbest = A->colck + cw;
-  A->corner = A->slabbest + bw / 2;
+  const int64_t slab_words = ((n + 1) / 2) * strips * (nslab > 0 ? nslab : 1) * 32;
+  A->corner = A->slabbest + slab_words;
+  A->lanebest = A->corner + slab_words;
   A->strips_max = strips;
   A->nslab_max = nslab > 0 ? nslab : 1;
   p->last_scores = scores;
@@ -381,7 +383,19 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       A.scratch = p->scratch.ptr;
       unsigned long long* rounds = nullptr;
       if (getenv("DP_NUSS_ROUNDS") && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), A.round_ns = rounds;
+      unsigned long long* dbg = nullptr;
+      if (getenv("DP_NUSS_TIMING") && tiled) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
       e = tiled ? dpk::nuss_tiled_solve(A, s, &p->launches) : dpk::nuss_solve(A, s, &p->launches);
+      if (dbg) {  // diagnostic: batch-kernel phase cycles summed over warps (stderr)
+        unsigned long long h[8];
+        cudaStreamSynchronize(s);
+        cudaMemcpy(h, dbg, sizeof(h), cudaMemcpyDeviceToHost);
+        const char* nm[8] = {"stage", "clearC", "phaseA", "waitA", "phaseB", "waitB", "traceback", "-"};
+        double tot = 0;
+        for (int q = 0; q < 7; ++q) tot += (double)h[q];
+        for (int q = 0; q < 7; ++q) fprintf(stderr, "nuss %-9s %16llu %5.1f%%\n", nm[q], h[q], 100.0 * h[q] / (tot > 0 ? tot : 1));
+        cudaFree(dbg);
+      }
       if (rounds) {  // diagnostic: per tile-diagonal round durations of the grid sweep (stderr)
         static unsigned long long h[8192];
         cudaStreamSynchronize(s);
@@ -473,7 +487,19 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
         dpk::Sw16Args A{};
         e = sw16_args(p, p->last_n, p->last_a, p->last_aoff, p->last_b, p->last_boff, p->last_max_la,
                       p->last_max_lb, p->last_scores, &A);
+        unsigned long long* dbg = nullptr;
+        if (getenv("DP_SW_TIMING")) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
         if (e == cudaSuccess) e = dpk::sw16_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
+        if (dbg) {  // diagnostic: traceback phase cycles summed over warps
+          unsigned long long h[8];
+          cudaStreamSynchronize(s);
+          cudaMemcpy(h, dbg, sizeof(h), cudaMemcpyDeviceToHost);
+          const char* nm[8] = {"prologue", "probe", "setup", "recompute", "search", "walk", "output", "rounds"};
+          double tot = 0;
+          for (int q = 0; q < 7; ++q) tot += (double)h[q];
+          for (int q = 0; q < 8; ++q) fprintf(stderr, "tb %-9s %14llu %5.1f%%\n", nm[q], h[q], q < 7 ? 100.0 * h[q] / tot : 0.0);
+          cudaFree(dbg);
+        }
         break;
       }
       /* fall through */

@@ -6,6 +6,19 @@
 
 namespace dpk {
 
+// Diagnostic phase clock (DP_*_TIMING): per-phase SM cycles of lane 0 of every warp,
+// summed into 8 device counters at the end of the kernel. Off (dbg == nullptr) it costs
+// one predicated branch per lap.
+struct PhaseClock {
+  unsigned long long* dbg;
+  long long t, acc[8];
+  __device__ __forceinline__ void start() { if (dbg) { t = clock64(); for (int q = 0; q < 8; ++q) acc[q] = 0; } }
+  __device__ __forceinline__ void lap(int q) { if (dbg) { const long long u = clock64(); acc[q] += u - t; t = u; } }
+  __device__ __forceinline__ void flush(int lane) {
+    if (dbg && lane == 0) for (int q = 0; q < 8; ++q) atomicAdd(dbg + q, (unsigned long long)acc[q]);
+  }
+};
+
 constexpr int kWarps = 8;  // warps per CTA for the warp-per-problem kernels
 
 // ---------------------------------------------------------------- alignment
@@ -49,7 +62,9 @@ struct Sw16Args {
   uint32_t* colck;       // [groups][strips][nslab][256]         G at each lane's checkpoint column 32 s - lane
   uint32_t* slabbest;    // [groups][strips][nslab][32]           per-lane best G per slab (32 sweep steps)
   uint32_t* corner;      // [groups][strips][nslab][32]           G of the row above the lane at its checkpoint column
+  uint32_t* lanebest;    // [groups][strips][32]                  per-lane best G over the strip
   int64_t strips_max, nslab_max;
+  unsigned long long* dbg = nullptr;  // DP_SW_TIMING: traceback phase cycles (8 counters), else nullptr
 };
 bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap);
 int sw16_smem_per_warp(int asz, int64_t max_la, int64_t max_lb);
@@ -74,6 +89,7 @@ struct NussArgs {
   void* scratch;             // global table scratch for large n
   int64_t scratch_bytes;
   unsigned long long* round_ns;  // optional: %globaltimer at each tile-diagonal round (grid sweep)
+  unsigned long long* dbg = nullptr;  // DP_NUSS_TIMING: batch-kernel phase cycles (8 counters)
 };
 int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device);
 bool nuss_tiled_supported(int64_t max_len);

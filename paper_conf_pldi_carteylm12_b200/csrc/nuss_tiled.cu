@@ -45,7 +45,6 @@ constexpr int kRec = 2 * kTileWords;   // int16 per tile record (UT + L)
 constexpr int kCtaWarps = 2;   // batch driver: eight CTAs (eight sequences) per SM
 constexpr int kCtaPerSm = 8;
 constexpr int kGridWarps = 16; // grid driver
-constexpr int kCS = T + 1;             // row stride of in-tile buffers
 constexpr int kGridMin = 1024;         // single problems longer than this use the whole grid
 
 __host__ __device__ __forceinline__ int64_t tile_id(int I, int J, int nt) {
@@ -135,21 +134,23 @@ __device__ void product_unit(const Tab& tab, int I, int J, int K0, int K1, int* 
     }
 }
 
-constexpr int kVS = 40;                  // int16 row stride of the in-tile operand copies (80 B)
+constexpr int kAS = 72;                  // int16 row stride of the in-tile operand rows (64 entries + 8 pad)
+constexpr int kCC = 34;                  // int16 row stride of the staged middle products
 constexpr int16_t kNeg = -16000;         // masks split points outside a cell's range
 
+// Phase-B buffers. The split terms of cell (r, c) that lie inside tiles I and J form ONE
+// reduction over p' in [r+1, 32+c) (off-diagonal tiles) of AS[r][p'] + BC[c][p'], with
+//   AS[r][p'] = U(I,I)[r][p']  (p' < 32; kNeg for p' <= r)  |  X[r][p'-32]  (p' >= 32; kNeg until computed)
+//   BC[c][p'] = X[p'+1][c]     (p' < 32; p' = 31: the row below the tile)  |  L(J,J)[p'-32][c]  (p' >= 32)
+// (X = this tile). The K = I terms pair gamma(i, 32I+p') with gamma(32I+p'+1, j), the K = J
+// terms gamma(i, 32J+k) with gamma(32J+k+1, j). Every live cell of local anti-diagonal dl
+// has exactly 31 + dl such terms, so chunks of 8 run warp-uniformly with no mask waste
+// beyond the chunk edges; entries outside a cell's range are killed by kNeg on the A side.
+// Diagonal tiles: AS[r][p' < 32] = kNeg, BC[c][32+k] = X[k+1][c] (filled as computed).
 struct InTileBuf {
-  union {
-    struct {
-      int16_t uiis[T * kVS];  // UIIs[r][m] = U(I,I)[r][m-1] for m >= r+2, kNeg below (m = 0..32)
-      int16_t ct[T * kVS];    // CT[c][m]  = CUR[m][c] (m < 32), CT[c][32] = U(I+1,J)[0][c]
-      int16_t cr[T * kVS];    // CR[r][k]  = CUR[r][k]
-      int16_t lt[T * kVS];    // LT[c][k]  = L(J,J)[k][c] for k < c, kNeg otherwise
-    };
-    int cur[T * kCS];         // diagonal tiles only: CUR[r][c]
-  };
-  int left[T];                // U(I,J-1)[r][31]
-  int corner;                 // gamma(32I+32, 32J-1)
+  int16_t as[T * kAS];
+  int16_t bc[T * kAS];
+  int16_t cc[T * kCC];        // C[r][c], the max over the middle tiles (phase A)
 };
 
 __device__ __forceinline__ bool pairable(const uint8_t* x, const uint8_t* pm, int n, int i, int j, int h) {
@@ -173,145 +174,139 @@ __device__ __forceinline__ uint32_t pair_bits(const uint8_t* x, const uint8_t* p
   return bits;
 }
 
-// Phase B: finalise tile (I,J) from C (max of the middle products), write UT/L records.
-// Off-diagonal tiles run the 63 local anti-diagonals with one cell per lane; each cell's
-// split points inside tiles I and J are reduced 8 at a time with VIADDMNMX.S16x2 over
-// masked operand copies (warp-uniform chunk ranges, no divergence).
+__device__ __forceinline__ uint32_t pk16(int lo, int hi) { return (uint32_t)(uint16_t)lo | ((uint32_t)(uint16_t)hi << 16); }
+
+// Phase B: finalise tile (I,J) from C (max of the middle products), write its UT/L records.
+// One cell per lane (lane = row r) per local anti-diagonal; the neighbours come from the
+// lane's own previous cell (left) and lane r+1's (below, and the pair's inner cell one step
+// later); the in-tile split points are the uniform-length AS x BC reduction above.
 __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, InTileBuf& B, const uint8_t* x,
                         const uint8_t* pm, int n, int h, int lane) {
-  const int i0 = I * T, j0 = J * T;
+  const unsigned full = 0xffffffffu;
+  const bool diag = I == J;
+  const int i0 = I * T, j0 = J * T, r = lane;
   int16_t* ut = tab.UT(I, J);
   int16_t* l = tab.L(I, J);
-  if (I == J) {
-    // diagonal tile: the cell-level recursion inside one 32x32 triangle
-    for (int q = lane; q < T * kCS; q += 32) B.cur[q] = 0;
-    const uint32_t pbits = pair_bits(x, pm, n, i0, j0, h, lane);
-    __syncwarp();
-    for (int d = 1; d < T; ++d) {
-      const int r = lane, c = lane + d;
-      if (c < T) {
-        int v = max(B.cur[(r + 1) * kCS + c], B.cur[r * kCS + c - 1]);
-        if ((pbits >> c) & 1u) v = max(v, (d >= 2 ? B.cur[(r + 1) * kCS + c - 1] : 0) + 1);
-        int v2 = v;  // two independent max chains
-        int k = r + 1;
-        for (; k + 1 < c; k += 2) {
-          v = __viaddmax_s32(B.cur[r * kCS + k], B.cur[(k + 1) * kCS + c], v);
-          v2 = __viaddmax_s32(B.cur[r * kCS + k + 1], B.cur[(k + 2) * kCS + c], v2);
-        }
-        if (k < c) v = __viaddmax_s32(B.cur[r * kCS + k], B.cur[(k + 1) * kCS + c], v);
-        B.cur[r * kCS + c] = max(v, v2);
-      }
-      __syncwarp();
-    }
-    for (int r = 0; r < T; ++r) ut[lane * T + r] = (int16_t)B.cur[r * kCS + lane];
-    for (int k = 0; k < T - 1; ++k) l[k * T + lane] = (int16_t)B.cur[(k + 1) * kCS + lane];
-    l[(T - 1) * T + lane] = 0;
-    return;
-  }
-  const int16_t* utii = tab.UT(I, I);
-  const int16_t* ljj = tab.L(J, J);
-  const int16_t* utb = tab.UT(I + 1, J);
-  const int16_t* utl = tab.UT(I, J - 1);
-  // Operand copies, built with coalesced global reads (lane = row/column of the copy)
-  // and 16-byte shared-memory stores of whole rows.
+  // ---- staging (all global loads before the shared stores of each part)
   {
-    const int t = lane;
     int16_t v[T];
-    auto store_row = [&](int16_t* dst, auto&& value) {
-      uint4* d = reinterpret_cast<uint4*>(dst + t * kVS);
+    if (!diag) {
+      const int16_t* utii = tab.UT(I, I);
 #pragma unroll
-      for (int w = 0; w < kVS / 8; ++w) {
-        uint32_t q[4];
+      for (int p = 0; p < T; ++p) v[p] = utii[p * T + r];  // U(I,I)[r][p] = gamma(i0+r, i0+p)
+    }
+    uint4* row = reinterpret_cast<uint4*>(B.as + r * kAS);
 #pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const int m0 = 8 * w + 2 * e;
-          q[e] = (uint32_t)(uint16_t)value(m0) | ((uint32_t)(uint16_t)value(m0 + 1) << 16);
-        }
-        d[w] = make_uint4(q[0], q[1], q[2], q[3]);
+    for (int w = 0; w < kAS / 8; ++w) {
+      uint32_t q[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const int p0 = 8 * w + 2 * e;
+        const int lo = (!diag && p0 < T && p0 > r) ? v[p0 < T ? p0 : 0] : kNeg;
+        const int hi = (!diag && p0 + 1 < T && p0 + 1 > r) ? v[p0 + 1 < T ? p0 + 1 : 0] : kNeg;
+        q[e] = pk16(lo, hi);
       }
-    };
-    // UIIs[t][m] = U(I,I)[t][m-1] = UT(I,I)[m-1][t]  for t+2 <= m <= 32
-#pragma unroll
-    for (int k = 0; k < T; ++k) v[k] = utii[k * T + t];
-    store_row(B.uiis, [&](int m) -> int16_t { return (m >= t + 2 && m <= T) ? v[m - 1] : kNeg; });
-    // CT[t][m] = C[m][t] (m < 32), CT[t][32] = U(I+1,J)[0][t]
-#pragma unroll
-    for (int m = 0; m < T; ++m) v[m] = has_c ? (int16_t)__ldcg(C + m * T + t) : (int16_t)0;
-    const int16_t bel = utb[t * T + 0];
-    store_row(B.ct, [&](int m) -> int16_t { return m < T ? v[m] : (m == T ? bel : (int16_t)0); });
-    // LT[t][k] = L(J,J)[k][t] for k < t
-#pragma unroll
-    for (int k = 0; k < T; ++k) v[k] = ljj[k * T + t];
-    store_row(B.lt, [&](int k) -> int16_t { return (k < t && k < T) ? v[k] : kNeg; });
-    B.left[t] = utl[(T - 1) * T + t];
-    if (lane == 0) B.corner = (I + 1 <= J - 1) ? tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
-    __syncwarp();
-    // CR[t][k] = C[t][k] = CT[k][t] (transpose through shared memory)
-#pragma unroll
-    for (int k = 0; k < T; ++k) v[k] = B.ct[k * kVS + t];
-    __syncwarp();
-    store_row(B.cr, [&](int k) -> int16_t { return k < T ? v[k] : (int16_t)0; });
+      row[w] = make_uint4(q[0], q[1], q[2], q[3]);
+    }
   }
-  __syncwarp();
-  const int r = lane;
-  const uint4* crow = reinterpret_cast<const uint4*>(B.cr + r * kVS);
-  // my row of UIIs is constant for the whole tile: keep it in registers. It is already
-  // masked (kNeg for m < r + 2), so all five chunks are reduced unconditionally.
-  uint4 ur[5];
+  {
+    const int c = lane;
+    int16_t v[T];
+    if (!diag) {
+      const int16_t* ljj = tab.L(J, J);
 #pragma unroll
-  for (int q = 0; q < 5; ++q) ur[q] = reinterpret_cast<const uint4*>(B.uiis + r * kVS)[q];
-  uint32_t pairbits = pair_bits(x, pm, n, i0, j0, h, lane);
-  for (int dl = -(T - 1); dl <= T - 1; ++dl) {
+      for (int k = 0; k < T; ++k) v[k] = ljj[k * T + c];  // L(J,J)[k][c] = gamma(j0+k+1, j0+c)
+    }
+    const int below = diag ? 0 : (int)tab.UT(I + 1, J)[c * T + 0];  // X[32][c] = gamma(i0+32, j0+c)
+    uint4* col = reinterpret_cast<uint4*>(B.bc + c * kAS);
+#pragma unroll
+    for (int w = 0; w < kAS / 8; ++w) {
+      uint32_t q[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const int p0 = 8 * w + 2 * e;
+        auto val = [&](int p) -> int {
+          if (p == T - 1) return below;
+          if (p >= T && p < 2 * T) return diag ? 0 : (int)v[p - T < T && p >= T ? p - T : 0];
+          return 0;
+        };
+        q[e] = pk16(val(p0), val(p0 + 1));
+      }
+      col[w] = make_uint4(q[0], q[1], q[2], q[3]);
+    }
+    int cv[T];
+#pragma unroll
+    for (int rr = 0; rr < T; ++rr) cv[rr] = has_c ? __ldcg(C + rr * T + c) : 0;
+#pragma unroll
+    for (int rr = 0; rr < T; ++rr) B.cc[rr * kCC + c] = (int16_t)cv[rr];
+  }
+  const int left = diag ? 0 : (int)tab.UT(I, J - 1)[(T - 1) * T + r];  // gamma(i0+r, j0-1)
+  const int corner = (!diag && I + 1 <= J - 1) ? (int)tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
+  const uint32_t pairbits = pair_bits(x, pm, n, i0, j0, h, lane);
+  __syncwarp();
+  int v = left;                                                    // X[r][c-1]
+  int below_prev = __shfl_down_sync(full, left, 1);                // X[r+1][c-1]
+  if (r == T - 1) below_prev = corner;
+  if (diag) below_prev = 0;
+  const uint4* arow = reinterpret_cast<const uint4*>(B.as + r * kAS);
+  const int lo = diag ? T + 1 + r : r + 1;
+  const int qlo = lo >> 3;
+  for (int dl = diag ? 1 : -(T - 1); dl <= T - 1; ++dl) {
     const int c = r + dl;
     const bool live = c >= 0 && c < T;
     const int cc = live ? c : 0;
-    const int cmax = min(T - 1, T - 1 + dl);
-    const int q1 = (cmax + 7) / 8;       // K=J chunks 0 .. q1-1 (warp-uniform)
-    const uint4* ccol = reinterpret_cast<const uint4*>(B.ct + cc * kVS);
-    const uint4* lcol = reinterpret_cast<const uint4*>(B.lt + cc * kVS);
-    uint4 ub[5];
-#pragma unroll
-    for (int q = 0; q < 5; ++q) ub[q] = ccol[q];
+    int below = __shfl_down_sync(full, v, 1);
+    if (r == T - 1) below = diag ? 0 : (int)B.bc[cc * kAS + (T - 1)];
+    if (diag && dl == 1) below = 0;
+    const uint4* bcol = reinterpret_cast<const uint4*>(B.bc + cc * kAS);
+    const int nq = diag ? ((dl + 5) >> 3) + 1 : ((37 + dl) >> 3) + 1;  // covers [qlo, q_hi] of every live lane
     uint32_t a0 = 0, a1 = 0, a2 = 0, a3 = 0;  // four independent max chains (0 is neutral: gamma >= 0)
-#pragma unroll
-    for (int q = 0; q < 5; ++q) {             // K=I: k + 1 = m in [r+2, 32]
-      a0 = __viaddmax_s16x2(ur[q].x, ub[q].x, a0);
-      a1 = __viaddmax_s16x2(ur[q].y, ub[q].y, a1);
-      a2 = __viaddmax_s16x2(ur[q].z, ub[q].z, a2);
-      a3 = __viaddmax_s16x2(ur[q].w, ub[q].w, a3);
+    for (int t = 0; t < nq; ++t) {
+      const uint4 av = arow[qlo + t], bv = bcol[qlo + t];
+      a0 = __viaddmax_s16x2(av.x, bv.x, a0);
+      a1 = __viaddmax_s16x2(av.y, bv.y, a1);
+      a2 = __viaddmax_s16x2(av.z, bv.z, a2);
+      a3 = __viaddmax_s16x2(av.w, bv.w, a3);
     }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {             // K=J: k in [0, c)
-      if (q < q1) {
-        const uint4 ja = crow[q], jb = lcol[q];
-        a0 = __viaddmax_s16x2(ja.x, jb.x, a0);
-        a1 = __viaddmax_s16x2(ja.y, jb.y, a1);
-        a2 = __viaddmax_s16x2(ja.z, jb.z, a2);
-        a3 = __viaddmax_s16x2(ja.w, jb.w, a3);
-      }
-    }
+    const uint32_t acc = __vmaxs2(__vmaxs2(a0, a1), __vmaxs2(a2, a3));
+    int val = max((int)(int16_t)(acc & 0xffffu), (int)(int16_t)(acc >> 16));
+    val = max(val, (int)B.cc[r * kCC + cc]);
+    val = max(val, max(below, v));
+    if ((pairbits >> cc) & 1u) val = max(val, below_prev + 1);
     if (live) {
-      const uint32_t acc = __vmaxs2(__vmaxs2(a0, a1), __vmaxs2(a2, a3));
-      int v = max((int)(int16_t)(acc & 0xffffu), (int)(int16_t)(acc >> 16));
-      v = max(v, (int)B.cr[r * kVS + c]);                              // C (middle products)
-      v = max(v, (int)B.ct[c * kVS + r + 1]);                          // gamma(i+1, j) (row 32 = below)
-      v = max(v, c > 0 ? (int)B.cr[r * kVS + c - 1] : B.left[r]);     // gamma(i, j-1)
-      if ((pairbits >> c) & 1u) {
-        const int inner = c > 0 ? (int)B.ct[(c - 1) * kVS + r + 1] : (r < T - 1 ? B.left[r + 1] : B.corner);
-        v = max(v, inner + 1);
-      }
-      B.cr[r * kVS + c] = (int16_t)v;
-      B.ct[c * kVS + r] = (int16_t)v;
+      B.as[r * kAS + T + c] = (int16_t)val;
+      if (r >= 1) B.bc[c * kAS + (diag ? T + r - 1 : r - 1)] = (int16_t)val;
+      v = val;
+      below_prev = below;
     }
     __syncwarp();
   }
-  // write the records: UT[c][r] and L[k][c] = gamma(i0+k+1, j0+c)
-  const uint32_t* ctw = reinterpret_cast<const uint32_t*>(B.ct + lane * kVS);
-  uint32_t* utw = reinterpret_cast<uint32_t*>(ut + lane * T);
+  // ---- records: UT[c][r] = X[r][c], L[k][c] = X[k+1][c] (k < 31), L[31][c] = X[32][c]
+  {
+    const uint4* xr = reinterpret_cast<const uint4*>(B.as + r * kAS + T);
+    uint4 w[4];
 #pragma unroll
-  for (int q = 0; q < T / 2; ++q) utw[q] = ctw[q];
-  for (int k = 0; k < T - 1; ++k) l[k * T + lane] = B.ct[lane * kVS + k + 1];
-  l[(T - 1) * T + lane] = B.ct[lane * kVS + T];
+    for (int q = 0; q < 4; ++q) {
+      w[q] = xr[q];
+      if (diag) {  // entries with c <= r are gamma(i, j <= i) = 0 (held as kNeg)
+        w[q].x = __vmaxs2(w[q].x, 0u); w[q].y = __vmaxs2(w[q].y, 0u);
+        w[q].z = __vmaxs2(w[q].z, 0u); w[q].w = __vmaxs2(w[q].w, 0u);
+      }
+    }
+    const uint32_t ww[16] = {w[0].x, w[0].y, w[0].z, w[0].w, w[1].x, w[1].y, w[1].z, w[1].w,
+                             w[2].x, w[2].y, w[2].z, w[2].w, w[3].x, w[3].y, w[3].z, w[3].w};
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      ut[(2 * q) * T + r] = (int16_t)(ww[q] & 0xffffu);
+      ut[(2 * q + 1) * T + r] = (int16_t)(ww[q] >> 16);
+    }
+    if (r >= 1) {
+      uint4* lr = reinterpret_cast<uint4*>(l + (r - 1) * T);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) lr[q] = w[q];
+    }
+    l[(T - 1) * T + lane] = B.bc[lane * kAS + (T - 1)];
+  }
 }
 
 // Canonical traceback (DESIGN.md R-TB-NUSS: Durbin order, smallest split k) by one
@@ -388,6 +383,9 @@ __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(Nu
             (int64_t)blockIdx.x * kCtaWarps * T * T;
   int* stack = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * slot_elems) +
                (int64_t)gridDim.x * kCtaWarps * T * T + (int64_t)blockIdx.x * (4 * A.max_len + 8);
+  PhaseClock clk;
+  clk.dbg = A.dbg;
+  clk.start();
   for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
     const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
     __syncthreads();
@@ -395,6 +393,7 @@ __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(Nu
     const int nt = (n + T - 1) / T;
     tab.nt = nt;
     __syncthreads();
+    clk.lap(0);
     for (int D = 0; D < nt; ++D) {
       const int nT = nt - D;  // tiles on this diagonal (<= nt <= 128 for n <= 4096)
       // phase A: work units (tile, K chunk); C per tile in shared memory (tiles > 16 processed in groups)
@@ -403,6 +402,7 @@ __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(Nu
         if (D >= 2) {
           for (int q = threadIdx.x; q < gT * T * T; q += blockDim.x) Cs[q] = 0;
           __syncthreads();
+          clk.lap(1);
           const int ksteps = D - 1;
           const int chunks = max(1, min(ksteps, kCtaWarps / gT));
           const int units = gT * chunks;
@@ -412,14 +412,18 @@ __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(Nu
             const int K0 = I + 1 + (ksteps * ch) / chunks, K1 = I + 1 + (ksteps * (ch + 1)) / chunks;
             product_unit<false>(tab, I, J, K0, K1, Cs + t * T * T, As, Bs, lane);
           }
+          clk.lap(2);
           __syncthreads();
+          clk.lap(3);
         }
         // phase B: one warp per tile
         if (warp < gT) {
           const int I = g0 + warp, J = I + D;
           in_tile(tab, I, J, Cs + warp * T * T, D >= 2, IB, xs, pm, n, A.hairpin, lane);
         }
+        clk.lap(4);
         __syncthreads();
+        clk.lap(5);
       }
     }
     if (threadIdx.x == 0) {
@@ -430,7 +434,9 @@ __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(Nu
     // barrier (the second CTA on the SM keeps the SM busy meanwhile)
     if (A.db && warp == 0)
       warp_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack), lane);
+    clk.lap(6);
   }
+  clk.flush(lane);
 }
 
 // ------------------------------------------------------------------ grid driver (one large problem)

@@ -20,9 +20,10 @@
 // every column) and, after every block of 32 steps, every lane's 8 rows at the
 // column it is on (a staircase, column 32 s - lane: warp-uniform, coalesced,
 // no per-step branch), the G above it there and its best G over the block
-// (0.25 B/cell). k_sw16_tb2 recomputes only the 32x32 (sheared) blocks the
-// canonical traceback needs and walks them with the oracle's tie-break
-// (diag > up > left, stop at H = 0; end cell = first maximum in row-major order).
+// (0.25 B/cell), plus every lane's maximum over the strip. k_sw16_tb3 recomputes
+// only the 32x32 (sheared) blocks the canonical traceback needs and walks them
+// with the oracle's tie-break (diag > up > left, stop at H = 0; end cell = first
+// maximum in row-major order).
 #include <cstdint>
 #include <cstdlib>
 #include <cuda_runtime.h>
@@ -217,6 +218,7 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
     const bool from_bnd = st > 0;
     const bool spill31 = (st + 1 < strips) && lane == 31;
     uint32_t *rowck = nullptr, *colck = nullptr, *slab = nullptr, *corner = nullptr;
+    uint32_t sbest = NEG_G2;  // this lane's maximum over the strip (TB)
     if (TB) {
       rowck = A.rowck + ((grp * A.strips_max + st) * kBandsPerStrip + lane / kLanesPerBand) * A.max_lb;
       colck = A.colck + ((grp * A.strips_max + st) * A.nslab_max) * kStrip + lane * kRows;
@@ -262,11 +264,13 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
         col[1] = make_uint4(S.G[4], S.G[5], S.G[6], S.G[7]);
         slab[sl * 32] = S.bbest;
         corner[sl * 32] = S.prev;
+        sbest = __vmaxs2(sbest, S.bbest);
         S.best2 = __vmaxs2(S.best2, S.bbest);
         S.bbest = NEG_G2;
       }
     }
     S.best2 = __vmaxs2(S.best2, S.bbest);
+    if (TB) A.lanebest[(grp * A.strips_max + st) * 32 + lane] = sbest;
     __syncwarp();
   }
 #pragma unroll
@@ -278,63 +282,24 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
 }
 
 // ---------------------------------------------------------------- traceback
-// Two problems per warp (the pair group of the forward pass): lanes 0-15 serve
-// problem 2g, lanes 16-31 problem 2g+1. A 32-row block is recomputed by 16 lanes,
-// lane hl holding block rows hl+1 (low half) and hl+17 (high half) in one s16x2
-// register: the two halves are independent given the checkpoint row between them.
-//
-// The checkpoints are staircases: forward lane l (rows 8l+1..8l+8 of its strip)
-// stored its column at 32 s - l. Block (blk, slab) therefore covers, for the
-// rows of forward lane l = L0 + m (L0 = 4 (blk mod 8), m = 0..3), the columns
-// j = D + c - m, c = 1..32, D = 32 slab - L0: a 32 x 32 square in the sheared
-// column c. Inside one forward lane the recurrence keeps its shape; at the first
-// row of lanes L0+1 and L0+3 (block rows 9 and 25: lane hl = 8 of each half) the
-// row above sits one sheared column to the left, so "up" arrives one wavefront
-// step later and the diagonal of the first column is the corner word the
-// forward lane stored next to its checkpoint.
-// Hp[t][c+1] packs (H of block row t, H of block row 16+t), c = -1..32. Row 0
-// holds the checkpoint rows aligned with rows 1 and 17 (shear 0 and 2), column
-// c = 0 the checkpoint columns, column c = -1 of row 8 the corners.
-constexpr int kPS = kSlab + 2;        // packed row stride (words)
-constexpr int kPW = 17 * kPS + 14;    // words per packed block (592 = 16 mod 32: the halves hit disjoint banks)
-
-struct PackedView {
-  const Sw16Args* A;
-  int64_t grp;
-  int half, la, lb;
-  __device__ __forceinline__ int top_h(int band, int j) const {  // H at row 16*band, column j (0 off the table)
-    if (band == 0 || j <= 0 || j > lb) return 0;
-    const int b = band - 1;
-    const int st = b / kBandsPerStrip, bi = b % kBandsPerStrip;
-    const uint32_t v = A->rowck[((grp * A->strips_max + st) * kBandsPerStrip + bi) * A->max_lb + (j - 1)];
-    return half16(v, half) + A->gap;
-  }
-  // H at row i, at its forward lane's checkpoint slab-1 (column 32 slab - lane)
-  __device__ __forceinline__ int left_h(int i, int slab) const {
-    if (slab == 0) return 0;
-    const int st = (i - 1) / kStrip, ri = (i - 1) % kStrip;
-    const uint32_t v = A->colck[((grp * A->strips_max + st) * A->nslab_max + (slab - 1)) * kStrip + ri];
-    return half16(v, half) + A->gap;
-  }
-  // H of the row above forward lane `ln` (strip st) at its checkpoint slab-1
-  __device__ __forceinline__ int corner_h(int st, int ln, int slab) const {
-    if (slab == 0) return 0;
-    const uint32_t v = A->corner[((grp * A->strips_max + st) * A->nslab_max + (slab - 1)) * 32 + ln];
-    return half16(v, half) + A->gap;
-  }
-};
-
-__device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(uint16_t)lo | ((uint32_t)(uint16_t)hi << 16); }
-// H of packed row t (0..16) of half hf at sheared column c (-1..32)
-__device__ __forceinline__ int hp_at(const uint32_t* Hp, int hf, int t, int c) {
-  const uint32_t v = Hp[t * kPS + c + 1];
-  return hf ? hi16(v) : lo16(v);
-}
-// shear of packed row t of half hf (row 0 is aligned with row 1)
-__device__ __forceinline__ int shear_of(int hf, int t) { return 2 * hf + (t >= 1 ? (t - 1) >> 3 : 0); }
-
-constexpr int kDeadCode = 31;   // residue code whose sigma row/column is kDead (alphabets < 32)
-constexpr int kBPadLo = 64, kBPadHi = 96;  // dead residues staged around b (the sheared sweep reads past both ends)
+// k_sw16_tb3: one warp serves 8 forward pairs (problems 2g, 2g+1), one pair per
+// 4-lane group. A traceback "block" is 32 rows (forward lanes L0..L0+3 of one
+// strip, L0 = 4 (blk mod 8)) x one slab: forward lane L0+m covered columns
+// j = D + c - m, c = 1..32, D = 32 slab - L0, at forward steps 32 slab + c - 1.
+// So in the sheared column c all four lanes are at the SAME forward step and
+// group lane m re-runs forward lane L0+m (8 rows) for 32 steps exactly as the
+// sweep did (no ramp): the left column is its checkpoint, its first diagonal the
+// corner word, lane 0's "up" the band checkpoint row above the block. The two
+// s16x2 halves carry the pair's two problems, each with its own block. The G of
+// the block go to shared memory column-major; the canonical walk (diag > up >
+// left, stop at H = 0) then runs on one lane per problem, 16 walkers per warp.
+// The end cell (first row-major maximum) comes from the per-lane strip maxima,
+// then the slabs of that lane whose maximum equals the score.
+constexpr int kCS = 36;                  // words per block column: row t (-1..31) at t + 4
+constexpr int kGS = 34 * kCS + 4;        // words per group buffer (columns c = -1..32); = 4 mod 8
+constexpr int kBS = 40;                  // staged b residues per half (columns D-3 .. D+32)
+constexpr int kDeadCode = 31;            // residue code whose sigma row/column is kDead (alphabets < 32)
+constexpr int kOpsCap = 512;             // ops staged in shared memory per problem (longer paths spill to the row tail)
 
 __device__ __forceinline__ int lds_s8(uint32_t a) {
   int v;
@@ -346,213 +311,398 @@ __device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
   asm("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
   return v;
 }
+__device__ __forceinline__ uint32_t join(uint32_t lo_src, uint32_t hi_src) { return prmt(lo_src, hi_src, 0x7610u); }
+__device__ __forceinline__ void prefetch_l2(const void* p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
 
-// Recompute this problem's block (blk, slab) into Hp; `on` = this half-warp has a
-// block to do. sig32 = shared sigma with row stride 32 (kDead outside the
-// alphabet); b is staged with kDeadCode padding, so columns j <= 0 evaluate to
-// exactly H = 0 (the table border) without masks, and columns past lb (never
-// read by the walk or the end-cell search) need none either.
-__device__ void packed_block(const PackedView& V, const uint8_t* a, const uint8_t* b, int blk, int slab, bool on,
-                             uint32_t* Hp, uint32_t sig32, int g, int hl) {
-  const int R0 = blk * kBlk, st = R0 / kStrip, L0 = (R0 % kStrip) / kRows;
-  const int D = slab * kSlab - L0;
-  const int band0 = R0 / kBand;
-  if (on) {
-    for (int c = hl; c <= kSlab; c += 16)
-      Hp[c + 1] = pk(V.top_h(band0, D + c), V.top_h(band0 + 1, D + c - 2));
-  }
-  const int mL = hl >> 3, mH = 2 + (hl >> 3);
-  const int iL = R0 + hl + 1, iH = R0 + hl + 17;
-  const bool okL = on && iL <= V.la, okH = on && iH <= V.la;
-  uint32_t left = pk(okL ? V.left_h(iL, slab) : 0, okH ? V.left_h(iH, slab) : 0);
-  if (on) Hp[(hl + 1) * kPS + 1] = left;
-  const bool shear = hl == 8;
-  uint32_t corner = 0;
-  if (shear && on) {
-    corner = pk(V.corner_h(st, L0 + 1, slab), V.corner_h(st, L0 + 3, slab));
-    Hp[8 * kPS] = corner;
-  }
-  __syncwarp();
-  const uint32_t sLa = sig32 + 32 * (okL ? a[iL - 1] : kDeadCode);
-  const uint32_t sHa = sig32 + 32 * (okH ? a[iH - 1] : kDeadCode);
-  const uint32_t bsh = (uint32_t)__cvta_generic_to_shared(b);
-  const uint32_t bL = bsh + (D - mL - 1), bH = bsh + (D - mH - 1);  // residue of sheared column c at +c
-  const uint32_t NEG_G2 = (uint32_t)(uint16_t)(-g) * 0x10001u;
-  uint32_t* hrow = Hp + (hl + 1) * kPS + 1;
-  uint32_t diag = __shfl_up_sync(0xffffffffu, left, 1, 16);
-  if (hl == 0) diag = on ? Hp[1] : 0u;
-  if (shear) diag = corner;
-  uint32_t last = left, fprev = 0;
-  const bool top = hl == 0;
-#pragma unroll 4
-  for (int s = 0; s < kSlab + 15; ++s) {
-    const int c = s - hl + 1;
-    const uint32_t from = __shfl_up_sync(0xffffffffu, last, 1, 16);
-    const bool in = (unsigned)(c - 1) < (unsigned)kSlab;
-    const uint32_t up = top ? Hp[c + 1] : (shear ? fprev : from);
-    fprev = from;
-    const uint32_t sg = prmt((uint32_t)lds_s8(sLa + lds_u8(bL + c)), (uint32_t)lds_s8(sHa + lds_u8(bH + c)), 0xC480u);
-    const uint32_t h = __viaddmax_s16x2_relu(diag, sg, __vadd2(__vmaxs2(up, left), NEG_G2));
-    if (in) hrow[c] = h;
-    diag = in ? up : diag;
-    left = in ? h : left;
-    last = in ? h : last;
-  }
-  __syncwarp();
-}
+struct TbHalf {       // one problem of the pair (uniform within its group)
+  int64_t p;          // problem id
+  const uint8_t *a, *b;
+  int la, lb, best;
+  int mode;           // 0 done / idle, 1 end-cell search, 2 walk
+  int band;           // search: first lane band (strip*32 + lane) reaching the score
+  int scur, cand;     // search: next slab to probe, candidate slab (-1 none)
+  long long found;    // search: row-major key (i << 32 | j) of the first maximum
+  int i, j, h, n;     // walk state
+  int ei, ej;         // end cell
+  int blk, sl, on;    // this round's block
+};
 
-__global__ void __launch_bounds__(128) k_sw16_tb2(Sw16Args A, int64_t first, int64_t count, uint8_t* out,
-                                                   int64_t stride, int32_t* out_len, int32_t* coords, int seq_bytes) {
+__global__ void __launch_bounds__(32) k_sw16_tb3(Sw16Args A, int64_t first, int64_t count, uint8_t* out,
+                                                  int64_t stride, int32_t* out_len, int32_t* coords) {
   extern __shared__ __align__(16) uint8_t tsm[];
-  __shared__ int8_t sig_s[32 * 32];  // row stride 32, kDead outside the alphabet
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (int q = threadIdx.x; q < 32 * 32; q += blockDim.x) {
+  int8_t* sig_s = reinterpret_cast<int8_t*>(tsm);                 // [32][32], kDead outside the alphabet
+  const int lane = threadIdx.x, gq = lane >> 2, m = lane & 3;
+  for (int q = lane; q < 32 * 32; q += 32) {
     const int x = q >> 5, y = q & 31;
     sig_s[q] = (x < A.asz && y < A.asz) ? A.sigma[x * A.asz + y] : (int8_t)kDead;
   }
-  __syncthreads();
+  uint32_t* Hs = reinterpret_cast<uint32_t*>(tsm + 1024) + gq * kGS;
+  uint8_t* bS = tsm + 1024 + 8 * kGS * 4 + gq * 2 * kBS;           // [2][kBS] staged b residues
+  uint8_t* aS = tsm + 1024 + 8 * kGS * 4 + 8 * 2 * kBS + gq * 2 * kBlk;  // [2][32] staged a residues
+  uint8_t* opsS = tsm + 1024 + 8 * kGS * 4 + 8 * 2 * kBS + 8 * 2 * kBlk + gq * 2 * kOpsCap;  // [2][cap] ops
   const uint32_t sig32 = (uint32_t)__cvta_generic_to_shared(sig_s);
-  const int half = lane >> 4, hl = lane & 15;
-  const int64_t g0 = first >> 1;
-  const int64_t grp = g0 + (int64_t)blockIdx.x * 4 + warp;
-  const int64_t p = 2 * grp + half;
-  const bool mine = p >= first && p < first + count;  // this half's problem is requested
-  if (2 * grp >= first + count) return;                  // warp-uniform
-  const int64_t qidx = p - first;
-  PackedView V;
-  V.A = &A; V.grp = grp; V.half = half;
-  V.la = mine ? (int)(A.a_off[p + 1] - A.a_off[p]) : 0;
-  V.lb = mine ? (int)(A.b_off[p + 1] - A.b_off[p]) : 0;
-  const int la = V.la, lb = V.lb, asz = A.asz, g = A.gap;
-  uint8_t* wsm = tsm + (size_t)warp * (2 * (kPW * 4 + 2 * seq_bytes));
-  uint32_t* Hp = reinterpret_cast<uint32_t*>(wsm) + half * kPW;  // the halves start 16 words apart mod 32
-  uint8_t* a = wsm + 2 * kPW * 4 + half * 2 * seq_bytes;
-  uint8_t* ops = a + seq_bytes;  // the path, end -> start, staged in shared memory
-  uint8_t* b = a + ((la + 15) & ~15) + kBPadLo;
-  for (int q = hl; q < la; q += 16) a[q] = A.a_cat[A.a_off[p] + q];
-  for (int q = hl - kBPadLo; q < lb + kBPadHi; q += 16) b[q] = (q >= 0 && q < lb) ? A.b_cat[A.b_off[p] + q] : kDeadCode;
-  __syncwarp();
-  const int best = mine ? A.scores[p] : 0;
-  bool active = mine && best > 0 && la > 0 && lb > 0;
-  uint8_t* o = out + (mine ? qidx : 0) * stride;
-  const int ops_cap = seq_bytes;
-  // 1) first lane band (row-major) whose slab maxima reach the best value (per half)
-  int band8 = -1;
-  const int strips = (max(la, 1) + kStrip - 1) / kStrip;
-  const int nsl = (max(lb, 1) + 31 + kSlab - 1) / kSlab;  // slabs holding this problem's columns
-  const int strips_w = max(__shfl_sync(0xffffffffu, strips, 0), __shfl_sync(0xffffffffu, strips, 16));
-  for (int st = 0; st < strips_w; ++st) {
-    for (int l2 = 0; l2 < 2; ++l2) {  // the half's 16 lanes cover the 32 lane bands in two rounds
-      const int ln = hl + 16 * l2;
-      bool hit = false;
-      if (active && band8 < 0 && st < strips) {
-        const uint32_t* sb = A.slabbest + ((grp * A.strips_max + st) * A.nslab_max) * 32 + ln;
-        for (int s0 = 0; s0 < nsl; s0 += 8) {  // eight independent loads in flight
-          uint32_t v[8];
+  const uint32_t hs32 = (uint32_t)__cvta_generic_to_shared(Hs);
+  const uint32_t bs32 = (uint32_t)__cvta_generic_to_shared(bS);
+  const unsigned full = 0xffffffffu;
+  const int g = A.gap;
+  const uint32_t NEG_G2 = (uint32_t)(uint16_t)(-g) * 0x10001u;
+  const int64_t grp = (first >> 1) + (int64_t)blockIdx.x * 8 + gq;
+  const int64_t SM = A.strips_max, NS = A.nslab_max;
+  PhaseClock clk;
+  clk.dbg = A.dbg;
+  clk.start();
+
+  TbHalf H[2];
 #pragma unroll
-          for (int q = 0; q < 8; ++q) v[q] = (s0 + q < nsl) ? __ldg(sb + (s0 + q) * 32) : 0u;
-#pragma unroll
-          for (int q = 0; q < 8; ++q) hit |= (s0 + q < nsl) && half16(v[q], half) + g == best;
-        }
-      }
-      const unsigned m = __ballot_sync(0xffffffffu, hit) >> (16 * half) & 0xffffu;
-      if (band8 < 0 && m) band8 = st * 32 + 16 * l2 + __ffs(m) - 1;
-    }
+  for (int hf = 0; hf < 2; ++hf) {
+    TbHalf& X = H[hf];
+    X.p = 2 * grp + hf;
+    const bool mine = X.p >= first && X.p < first + count;
+    X.la = mine ? (int)(A.a_off[X.p + 1] - A.a_off[X.p]) : 0;
+    X.lb = mine ? (int)(A.b_off[X.p + 1] - A.b_off[X.p]) : 0;
+    X.a = mine ? A.a_cat + A.a_off[X.p] : A.a_cat;
+    X.b = mine ? A.b_cat + A.b_off[X.p] : A.b_cat;
+    X.best = mine ? A.scores[X.p] : 0;
+    X.mode = (mine && X.best > 0 && X.la > 0 && X.lb > 0) ? 1 : 0;
+    X.band = -1; X.scur = 0; X.cand = -1; X.found = -1;
+    X.i = X.j = X.h = X.n = 0; X.ei = X.ej = 0;
+    X.blk = X.sl = X.on = 0;
   }
-  // 2) first cell with H == best among the slabs of band8 holding the best (both halves together)
-  const int lane8 = band8 >= 0 ? band8 % 32 : 0, st8 = band8 >= 0 ? band8 / 32 : 0;
-  const int blk = (st8 * kStrip + lane8 * kRows) / kBlk;
-  const int L0b = lane8 & ~3;
-  int myr = 1 << 30, myc = 1 << 30;  // my best (row, col) candidate inside the block, row-major
-  const int nsl_w = max(__shfl_sync(0xffffffffu, nsl, 0), __shfl_sync(0xffffffffu, nsl, 16));
-  for (int sl = 0; sl < nsl_w; ++sl) {
-    const bool cand = active && sl < nsl &&
-        half16(A.slabbest[((grp * A.strips_max + st8) * A.nslab_max + sl) * 32 + lane8], half) + g == best;
-    if (!__any_sync(0xffffffffu, cand)) continue;
-    packed_block(V, a, b, blk, sl, cand, Hp, sig32, g, hl);
-    if (cand) {
-      const int D = sl * kSlab - L0b;
-      for (int rr = 0; rr < 2; ++rr) {  // rows hl+1 and hl+17
-        const int row = hl + 1 + 16 * rr, i = blk * kBlk + row, m = (row - 1) >> 3;
-        if (i > la || row > myr) continue;
-        for (int c = 1; c <= kSlab; ++c) {
-          const int j = D + c - m;
-          if (j >= 1 && j <= lb && hp_at(Hp, rr, hl + 1, c) == best) {
-            if (row < myr || (row == myr && j < myc)) { myr = row; myc = j; }
-            break;
+  // 1) first lane band (row-major: strip, lane) whose strip maximum reaches the score
+  {
+    int stw = max((H[0].la + kStrip - 1) / kStrip, (H[1].la + kStrip - 1) / kStrip);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) stw = max(stw, __shfl_xor_sync(full, stw, o));
+    for (int st = 0; st < stw; ++st) {
+      uint32_t w[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        w[q] = (H[0].mode | H[1].mode) && grp < (A.n + 1) / 2 && st < SM
+                   ? __ldcg(A.lanebest + (grp * SM + st) * 32 + 8 * m + q) : 0u;
+#pragma unroll
+      for (int hf = 0; hf < 2; ++hf) {
+        TbHalf& X = H[hf];
+        const bool want = X.mode == 1 && X.band < 0 && st * kStrip < X.la;
+        int firstl = 32;
+#pragma unroll
+        for (int q = 7; q >= 0; --q)
+          if (want && half16(w[q], hf) + g == X.best) firstl = 8 * m + q;
+        firstl = min(firstl, __shfl_xor_sync(full, firstl, 1));
+        firstl = min(firstl, __shfl_xor_sync(full, firstl, 2));
+        if (want && firstl < 32) X.band = st * 32 + firstl;
+      }
+    }
+#pragma unroll
+    for (int hf = 0; hf < 2; ++hf)
+      if (H[hf].mode == 1 && H[hf].band < 0) H[hf].mode = 0;  // cannot happen: the maxima name the score
+  }
+  __syncwarp();
+  clk.lap(0);
+
+  int guard = 8 * (int)((A.max_la + A.max_lb) / 16 + 8);
+  while (__any_sync(full, (H[0].mode | H[1].mode) != 0) && --guard > 0) {
+    // 2) searching halves: next candidate slab of their lane band (32 slabs per probe)
+    for (;;) {
+      bool need[2];
+#pragma unroll
+      for (int hf = 0; hf < 2; ++hf) need[hf] = H[hf].mode == 1 && H[hf].cand < 0;
+      if (!__any_sync(full, need[0] || need[1])) break;
+#pragma unroll
+      for (int hf = 0; hf < 2; ++hf) {
+        TbHalf& X = H[hf];
+        const int nsl = (X.lb + 31 + kSlab - 1) / kSlab;
+        const int st8 = X.band >> 5, ln8 = X.band & 31;
+        uint32_t bits = 0;
+        if (need[hf]) {
+          const uint32_t* sb = A.slabbest + ((grp * SM + st8) * NS) * 32 + ln8;
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const int s = X.scur + m + 4 * q;
+            if (s < nsl && half16(__ldcg(sb + (int64_t)s * 32), hf) + g == X.best) bits |= 1u << (m + 4 * q);
+          }
+        }
+        bits |= __shfl_xor_sync(full, bits, 1);
+        bits |= __shfl_xor_sync(full, bits, 2);
+        if (need[hf]) {
+          if (bits) {
+            X.cand = X.scur + __ffs(bits) - 1;
+          } else {
+            X.scur += 32;
+            if (X.scur >= nsl) {  // candidates exhausted: walk from the first maximum
+              if (X.found >= 0) {
+                X.mode = 2;
+                X.i = X.ei = (int)(X.found >> 32);
+                X.j = X.ej = (int)(X.found & 0xffffffffll);
+                X.h = X.best;
+              } else {
+                X.mode = 0;  // cannot happen
+              }
+            }
           }
         }
       }
     }
-    __syncwarp();
-  }
-  // smallest (row, col) over the half's lanes
-  for (int o2 = 8; o2 > 0; o2 >>= 1) {
-    const int orr = __shfl_xor_sync(0xffffffffu, myr, o2, 16), occ = __shfl_xor_sync(0xffffffffu, myc, o2, 16);
-    if (orr < myr || (orr == myr && occ < myc)) { myr = orr; myc = occ; }
-  }
-  if (myr == (1 << 30)) active = false;  // cannot happen: the slab maxima name a cell holding the best
-  const int ei = active ? blk * kBlk + myr : 0, ej = active ? myc : 0;
-  // 3) walk back block by block; the two halves walk concurrently (leaders hl == 0)
-  int i = ei, j = ej, h = active ? best : 0;
-  int n = 0;
-  bool overflow = false;
-  while (__any_sync(0xffffffffu, h > 0)) {
-    const bool on = h > 0;
-    int bg = 0, sl = 0;
-    if (on) {
-      bg = (i - 1) / kBlk;
-      const int ln = ((i - 1) % kStrip) / kRows;  // forward lane of row i
-      sl = (j + ln - 1) / kSlab;
-    }
-    packed_block(V, a, b, bg, sl, on, Hp, sig32, g, hl);
-    if (hl == 0 && on) {
-      // walk in the block's sheared coordinates: packed row t (1..16) of half hf, column c
-      const int R0 = bg * kBlk, D = sl * kSlab - (R0 % kStrip) / kRows;
-      const int ri = i - R0;
-      int hf = ri > 16 ? 1 : 0, t = ri - 16 * hf;
-      int c = j - D + ((ri - 1) >> 3);
-      int sh = 16 * hf;
-      while (h > 0 && t >= 1 && c >= 1) {
-        // branch-free step: all three neighbours are read, the move is selected
-        const int tm = t - 1, cu = c - (t == 9 ? 1 : 0);  // row above: one column left at a forward-lane start
-        const uint32_t* up_row = Hp + tm * kPS;
-        const int dV = (int)(int16_t)(up_row[cu] >> sh), uV = (int)(int16_t)(up_row[cu + 1] >> sh);
-        const int lV = (int)(int16_t)(Hp[t * kPS + c] >> sh);
-        const int ra = a[i - 1], rb = b[j - 1];
-        const int sub = sig_s[ra * 32 + rb];
-        const bool isD = h == dV + sub;
-        const bool isU = !isD && h == uV - g;
-        const bool mvI = isD || isU;  // the row index moves
-        const uint8_t op = isD ? (ra == rb ? 'M' : 'X') : (isU ? 'D' : 'I');
-        h = isD ? dV : (isU ? uV : lV);
-        i -= mvI ? 1 : 0;
-        j -= isU ? 0 : 1;
-        c = isD ? cu - 1 : (isU ? cu : c - 1);
-        t = mvI ? tm : t;
-        if (n < ops_cap) ops[n] = op;
-        ++n;
-        if (t == 0 && hf == 1) { hf = 0; sh = 0; t = 16; --c; }  // row 16: continue in the low half (shear 1)
+    clk.lap(1);
+    if (clk.dbg) clk.acc[7] += 1;
+    // 3) this round's block per half
+#pragma unroll
+    for (int hf = 0; hf < 2; ++hf) {
+      TbHalf& X = H[hf];
+      X.on = 0;
+      if (X.mode == 1 && X.cand >= 0) {
+        const int st8 = X.band >> 5, ln8 = X.band & 31;
+        X.blk = st8 * (kStrip / kBlk) + ln8 / 4;
+        X.sl = X.cand;
+        X.on = 1;
+      } else if (X.mode == 2) {
+        const int ln = ((X.i - 1) % kStrip) / kRows;
+        X.blk = (X.i - 1) / kBlk;
+        X.sl = (X.j + ln - 1) / kSlab;
+        X.on = 1;
       }
     }
-    i = __shfl_sync(0xffffffffu, i, 16 * half);
-    j = __shfl_sync(0xffffffffu, j, 16 * half);
-    h = __shfl_sync(0xffffffffu, h, 16 * half);
+    // 3b) walking halves: the block after this one is above, above-left or left of it;
+    // pull their checkpoints into L2 now so the next round's loads do not go to DRAM.
+#pragma unroll
+    for (int hf = 0; hf < 2; ++hf) {
+      const TbHalf& X = H[hf];
+      if (X.mode != 2) continue;
+#pragma unroll
+      for (int q = 0; q < 3; ++q) {
+        const int nb = X.blk - (q < 2 ? 1 : 0), ns = X.sl - (q > 0 ? 1 : 0);
+        if (nb < 0 || ns < 1) continue;
+        const int r0 = nb * kBlk, st = r0 / kStrip, L0 = (r0 % kStrip) / kRows;
+        const int64_t base = (grp * SM + st) * NS + (ns - 1);
+        prefetch_l2(A.colck + base * kStrip + (L0 + m) * kRows);
+        if (m == 0) prefetch_l2(A.corner + base * 32 + L0);
+        if (r0 > 0) {
+          const int bnd = r0 / kBand - 1, j0 = max(1, ns * kSlab - L0 + 16 * m);
+          if (j0 <= X.lb)
+            prefetch_l2(A.rowck + ((grp * SM + bnd / kBandsPerStrip) * kBandsPerStrip + bnd % kBandsPerStrip) * A.max_lb +
+                        (j0 - 1));
+        }
+      }
+    }
+    // 4) recompute both blocks. Every global load of the round is issued before any
+    // shared-memory store (checkpoint column, corner, a and b residues, top row).
+    int R0[2], D[2];
+    uint32_t sa[2][kRows];
+    uint32_t Gs[kRows], prev;
+    {
+      uint32_t w[2][kRows], cw[2], av[2][kRows], bv[2][kBS / 4], tv[2][9];
+#pragma unroll
+      for (int hf = 0; hf < 2; ++hf) {
+        TbHalf& X = H[hf];
+        R0[hf] = X.blk * kBlk;
+        const int st = R0[hf] / kStrip, L0 = (R0[hf] % kStrip) / kRows, l = L0 + m;
+        D[hf] = X.sl * kSlab - L0;
+        const bool ck = X.on && X.sl > 0;
+        const int64_t base = (grp * SM + st) * NS + (ck ? X.sl - 1 : 0);
+        const uint4* cp = reinterpret_cast<const uint4*>(A.colck + base * kStrip + l * kRows);
+        const uint4 v0 = ck ? __ldcg(cp) : make_uint4(NEG_G2, NEG_G2, NEG_G2, NEG_G2);
+        const uint4 v1 = ck ? __ldcg(cp + 1) : make_uint4(NEG_G2, NEG_G2, NEG_G2, NEG_G2);
+        w[hf][0] = v0.x; w[hf][1] = v0.y; w[hf][2] = v0.z; w[hf][3] = v0.w;
+        w[hf][4] = v1.x; w[hf][5] = v1.y; w[hf][6] = v1.z; w[hf][7] = v1.w;
+        cw[hf] = ck ? __ldcg(A.corner + base * 32 + l) : NEG_G2;
+#pragma unroll
+        for (int r = 0; r < kRows; ++r) {
+          const int i = R0[hf] + 8 * m + r + 1;
+          av[hf][r] = (X.on && i <= X.la) ? __ldg(X.a + i - 1) : (uint32_t)kDeadCode;
+        }
+#pragma unroll
+        for (int k = 0; k < kBS / 4; ++k) {  // b residues of columns D-3 .. D+36 (x = j - D + 3)
+          const int j = D[hf] + m + 4 * k - 3;
+          bv[hf][k] = (X.on && j >= 1 && j <= X.lb) ? __ldg(X.b + j - 1) : (uint32_t)kDeadCode;
+        }
+        // top row (G of row R0, columns D + c, c = 0..32): the band checkpoint above the block
+        const int bnd = R0[hf] / kBand - 1;
+        const uint32_t* rk = A.rowck + ((grp * SM + (bnd >= 0 ? bnd / kBandsPerStrip : 0)) * kBandsPerStrip +
+                                        (bnd >= 0 ? bnd % kBandsPerStrip : 0)) * A.max_lb - 1;
+#pragma unroll
+        for (int k = 0; k < 9; ++k) {
+          const int c = m + 4 * k, j = D[hf] + c;
+          tv[hf][k] = (X.on && bnd >= 0 && c <= kSlab && j >= 1 && j <= X.lb) ? __ldcg(rk + j) : NEG_G2;
+        }
+      }
+#pragma unroll
+      for (int hf = 0; hf < 2; ++hf) {
+#pragma unroll
+        for (int r = 0; r < kRows; ++r) {
+          sa[hf][r] = sig32 + 32 * av[hf][r];
+          aS[hf * kBlk + 8 * m + r] = (uint8_t)av[hf][r];
+        }
+#pragma unroll
+        for (int k = 0; k < kBS / 4; ++k) bS[hf * kBS + m + 4 * k] = (uint8_t)bv[hf][k];
+      }
+#pragma unroll
+      for (int k = 0; k < 9; ++k)
+        if (m + 4 * k <= kSlab) Hs[(m + 4 * k + 1) * kCS + 3] = join(tv[0][k], tv[1][k]);
+#pragma unroll
+      for (int r = 0; r < kRows; ++r) Gs[r] = join(w[0][r], w[1][r]);
+      prev = join(cw[0], cw[1]);
+      uint4* col0 = reinterpret_cast<uint4*>(Hs + kCS + 8 * m + 4);
+      col0[0] = make_uint4(Gs[0], Gs[1], Gs[2], Gs[3]);
+      col0[1] = make_uint4(Gs[4], Gs[5], Gs[6], Gs[7]);
+      if (m > 0) Hs[8 * m + 3] = prev;  // corner: row 8m-1, column c = -1
+    }
+    __syncwarp();
+    clk.lap(2);
+    {
+      const uint32_t bA = bs32 + (3 - m), bB = bs32 + kBS + (3 - m);
+#pragma unroll 4
+      for (int c = 1; c <= kSlab; ++c) {
+        const uint32_t topv = Hs[(c + 1) * kCS + 3];
+        const uint32_t fa = __shfl_up_sync(full, Gs[kRows - 1], 1, 4);
+        const uint32_t Gu = m == 0 ? topv : fa;
+        const uint32_t Gd = prev;
+        prev = Gu;
+        const uint32_t ca = lds_u8(bA + c), cb = lds_u8(bB + c);
+        uint32_t Xv[kRows];
+#pragma unroll
+        for (int r = 0; r < kRows; ++r) {
+          const uint32_t sg = prmt((uint32_t)lds_s8(sa[0][r] + ca), (uint32_t)lds_s8(sa[1][r] + cb), 0x5410u);
+          Xv[r] = __viaddmax_s16x2(r == 0 ? Gd : Gs[r - 1], sg, __viaddmax_s16x2(Gs[r], NEG_G2, NEG_G2));
+        }
+        uint32_t gg = Gu;
+#pragma unroll
+        for (int r = 0; r < kRows; ++r) {
+          gg = __viaddmax_s16x2(gg, NEG_G2, Xv[r]);
+          Gs[r] = gg;
+        }
+        uint4* col = reinterpret_cast<uint4*>(Hs + (c + 1) * kCS + 8 * m + 4);
+        col[0] = make_uint4(Gs[0], Gs[1], Gs[2], Gs[3]);
+        col[1] = make_uint4(Gs[4], Gs[5], Gs[6], Gs[7]);
+      }
+    }
+    __syncwarp();
+    clk.lap(3);
+    // 5) searching halves: first row-major cell of the lane band holding the score
+#pragma unroll
+    for (int hf = 0; hf < 2; ++hf) {
+      TbHalf& X = H[hf];
+      const bool srch = X.mode == 1 && X.on;
+      const int m8 = (X.band & 31) & 3;
+      int key = 1 << 30;  // r * 64 + c
+      if (srch) {
+        const int target = X.best - g;
+        for (int c = m + 1; c <= kSlab; c += 4) {
+          const uint4* col = reinterpret_cast<const uint4*>(Hs + (c + 1) * kCS + 8 * m8 + 4);
+          const uint4 v0 = col[0], v1 = col[1];
+          const uint32_t vv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+#pragma unroll
+          for (int r = kRows - 1; r >= 0; --r) {
+            const int i = R0[hf] + 8 * m8 + r + 1, j = D[hf] + c - m8;
+            if (half16(vv[r], hf) == target && i <= X.la && j >= 1 && j <= X.lb) key = min(key, r * 64 + c);
+          }
+        }
+      }
+      key = min(key, __shfl_xor_sync(full, key, 1));
+      key = min(key, __shfl_xor_sync(full, key, 2));
+      if (srch) {
+        if (key < (1 << 30)) {
+          const int r = key >> 6, c = key & 63;
+          const long long k2 = ((long long)(R0[hf] + 8 * m8 + r + 1) << 32) | (long long)(D[hf] + c - m8);
+          if (X.found < 0 || k2 < X.found) X.found = k2;
+        }
+        X.scur = X.cand + 1;
+        X.cand = -1;
+      }
+    }
+    clk.lap(4);
+    // 6) walking halves: lane m == half walks its problem through the block
+    if (m < 2) {
+      const int hf = m;
+      int mode = hf ? H[1].mode : H[0].mode;
+      if (mode == 2) {
+        int i = hf ? H[1].i : H[0].i, j = hf ? H[1].j : H[0].j, h = hf ? H[1].h : H[0].h, n = hf ? H[1].n : H[0].n;
+        const int r0 = hf ? R0[1] : R0[0], d0 = hf ? D[1] : D[0];
+        const int64_t p = hf ? H[1].p : H[0].p;
+        uint8_t* o = out + (p - first) * stride;
+        const uint8_t* as = aS + hf * kBlk - r0 - 1;   // as[i] = a[i - 1] for rows of the block
+        const uint8_t* bs = bS + hf * kBS - d0 + 3;    // bs[j] = b[j - 1] for columns D-3 .. D+36
+        uint8_t* ops = opsS + hf * kOpsCap;
+        const int sh16 = 16 * hf;
+        int t = i - r0 - 1;
+        int c = j - d0 + (t >> 3);
+        while (h > 0 && t >= 0 && c >= 1) {
+          const int cu = c - ((t > 0 && (t & 7) == 0) ? 1 : 0);  // row above: one column left at a lane start
+          const uint32_t* up_col = Hs + (cu + 1) * kCS + t + 3;     // (t-1, cu)
+          const int uV = (int)(int16_t)(up_col[0] >> sh16) + g;
+          const int dV = (int)(int16_t)(up_col[-kCS] >> sh16) + g;
+          const int lV = (int)(int16_t)(Hs[c * kCS + t + 4] >> sh16) + g;
+          const int ra = as[i], rb = bs[j];
+          const int sub = sig_s[ra * 32 + rb];
+          const bool isD = h == dV + sub;
+          const bool isU = !isD && h == uV - g;
+          const bool mvI = isD || isU;
+          const uint8_t op = isD ? (ra == rb ? 'M' : 'X') : (isU ? 'D' : 'I');
+          h = isD ? dV : (isU ? uV : lV);
+          i -= mvI ? 1 : 0;
+          j -= isU ? 0 : 1;
+          c = isD ? cu - 1 : (isU ? cu : c - 1);
+          t -= mvI ? 1 : 0;
+          if (n < kOpsCap) ops[n] = op;
+          else if (n < stride) o[stride - 1 - n] = op;  // long paths: the row's tail, moved at the end
+          ++n;
+        }
+        if (hf) { H[1].i = i; H[1].j = j; H[1].h = h; H[1].n = n; if (h <= 0) H[1].mode = 0; }
+        else { H[0].i = i; H[0].j = j; H[0].h = h; H[0].n = n; if (h <= 0) H[0].mode = 0; }
+      }
+    }
+    // the walkers' state to their groups
+#pragma unroll
+    for (int hf = 0; hf < 2; ++hf) {
+      const int src = (lane & ~3) | hf;
+      TbHalf& X = H[hf];
+      X.i = __shfl_sync(full, X.i, src);
+      X.j = __shfl_sync(full, X.j, src);
+      X.h = __shfl_sync(full, X.h, src);
+      X.n = __shfl_sync(full, X.n, src);
+      X.mode = __shfl_sync(full, X.mode, src);
+    }
+    __syncwarp();
+    clk.lap(5);
   }
-  // path start -> end, written by the half's 16 lanes
-  n = __shfl_sync(0xffffffffu, n, 16 * half);
-  overflow = n > stride || n > ops_cap;
+  // 7) outputs, start -> end: op q (walk order) goes to position n-1-q. Ops q < cap are in
+  // shared memory; longer paths left ops q >= cap at the row's tail (position stride-1-q),
+  // which is shifted left first (ordered 4-byte chunks: every read precedes the overlapping writes).
   __syncwarp();
-  if (mine && !overflow)
-    for (int64_t u = hl; u < n; u += 16) o[u] = ops[n - 1 - u];
-  if (hl == 0 && mine) {
-    out_len[qidx] = overflow ? -1 : (int32_t)n;
-    if (coords) {
-      coords[4 * qidx] = active ? i : 0; coords[4 * qidx + 1] = active ? j : 0;
-      coords[4 * qidx + 2] = ei; coords[4 * qidx + 3] = ej;
+#pragma unroll
+  for (int hf = 0; hf < 2; ++hf) {
+    const TbHalf& X = H[hf];
+    const bool mine = X.p >= first && X.p < first + count;
+    const int64_t q = X.p - first;
+    const bool active = X.best > 0 && X.la > 0 && X.lb > 0;
+    const int n = active ? X.n : 0;
+    const bool overflow = n > stride;
+    uint8_t* o = out + (mine ? q : 0) * stride;
+    if (mine && !overflow && n > kOpsCap) {
+      const int64_t s0 = stride - n;
+      for (int64_t u0 = 0; u0 < n - kOpsCap; u0 += 4) {
+        const int64_t u = u0 + m;
+        const uint8_t v = u < n - kOpsCap ? o[s0 + u] : 0;
+        __syncwarp(0xfu << (lane & ~3));
+        if (u < n - kOpsCap) o[u] = v;
+        __syncwarp(0xfu << (lane & ~3));
+      }
+    }
+    if (mine && !overflow) {
+      const uint8_t* ops = opsS + hf * kOpsCap;
+      for (int u = max(0, n - kOpsCap) + m; u < n; u += 4) o[u] = ops[n - 1 - u];
+    }
+    if (mine && m == 0) {
+      out_len[q] = overflow ? -1 : (int32_t)n;
+      if (coords) {
+        coords[4 * q] = active ? X.i : 0; coords[4 * q + 1] = active ? X.j : 0;
+        coords[4 * q + 2] = active ? X.ei : 0; coords[4 * q + 3] = active ? X.ej : 0;
+      }
     }
   }
+  clk.lap(6);
+  clk.flush(lane);
 }
+
+size_t tb3_smem_bytes() { return 1024 + 8 * kGS * 4 + 8 * 2 * kBS + 8 * 2 * kBlk + 8 * 2 * kOpsCap; }
 
 }  // namespace
 
@@ -576,7 +726,7 @@ void sw16_state_words(int64_t n, int64_t max_la, int64_t max_lb, int64_t* strips
   const int64_t groups = (n + 1) / 2;
   *rowck = groups * *strips * kBandsPerStrip * max_lb;
   *colck = groups * *strips * *nslab * kStrip;
-  *slabbest = 2 * groups * *strips * *nslab * 32;  // slab maxima, then corners
+  *slabbest = 2 * groups * *strips * *nslab * 32 + groups * *strips * 32;  // slab maxima, corners, strip maxima
 }
 
 cudaError_t sw16_solve(const Sw16Args& A, bool tb, cudaStream_t s, int64_t* launches) {
@@ -598,16 +748,14 @@ cudaError_t sw16_solve(const Sw16Args& A, bool tb, cudaStream_t s, int64_t* laun
 cudaError_t sw16_traceback(const Sw16Args& A, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                            int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches) {
   if (count == 0) return cudaSuccess;
-  const int seq_bytes = (int)(((A.max_la + 15) & ~15) + ((A.max_lb + 15) & ~15) + kBPadLo + kBPadHi);
   ++*launches;
-  const size_t smem = 4 * (2 * ((size_t)kPW * 4 + 2 * (size_t)seq_bytes));
-  cudaError_t e = cudaFuncSetAttribute(k_sw16_tb2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const size_t smem = tb3_smem_bytes();
+  cudaError_t e = cudaFuncSetAttribute(k_sw16_tb3, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_sw16_tb2, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  e = cudaFuncSetAttribute(k_sw16_tb3, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
   if (e != cudaSuccess) return e;
   const int64_t groups = ((first + count - 1) >> 1) - (first >> 1) + 1;
-  k_sw16_tb2<<<(unsigned)((groups + 3) / 4), 128, smem, s>>>(A, first, count, out, stride, out_len, coords,
-                                                             seq_bytes);
+  k_sw16_tb3<<<(unsigned)((groups + 7) / 8), 32, smem, s>>>(A, first, count, out, stride, out_len, coords);
   return cudaGetLastError();
 }
 
