@@ -29,6 +29,7 @@
 // with the split search spread over a warp.
 #include <algorithm>
 #include <cstdint>
+#include <type_traits>
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
@@ -174,6 +175,24 @@ __device__ __forceinline__ uint32_t pair_bits(const uint8_t* x, const uint8_t* p
   return bits;
 }
 
+__device__ __forceinline__ uint32_t opaque(uint32_t x) {
+  uint32_t y;
+  asm volatile("mov.b32 %0, %1;" : "=r"(y) : "r"(x));
+  return y;
+}
+__device__ __forceinline__ uint4 lds_v4(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ int lds_s16(uint32_t a) {
+  int16_t v;
+  asm volatile("ld.shared.s16 %0, [%1];" : "=h"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ void sts_u16(uint32_t a, int v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"((int16_t)v) : "memory");
+}
 __device__ __forceinline__ uint32_t pk16(int lo, int hi) { return (uint32_t)(uint16_t)lo | ((uint32_t)(uint16_t)hi << 16); }
 
 // Phase B: finalise tile (I,J) from C (max of the middle products), write its UT/L records.
@@ -248,38 +267,70 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
   int below_prev = __shfl_down_sync(full, left, 1);                // X[r+1][c-1]
   if (r == T - 1) below_prev = corner;
   if (diag) below_prev = 0;
-  const uint4* arow = reinterpret_cast<const uint4*>(B.as + r * kAS);
+  // 32-bit shared addresses, computed once (the loop is issue-bound)
+  // (opaque copies: otherwise the compiler rematerialises the shared base from SR_CgaCtaId
+  // inside the loop under the 128-register cap)
+  const uint32_t as_s = opaque((uint32_t)__cvta_generic_to_shared(B.as) + r * (kAS * 2));
+  const uint32_t bc_s = opaque((uint32_t)__cvta_generic_to_shared(B.bc));
+  const uint32_t cc_s = opaque((uint32_t)__cvta_generic_to_shared(B.cc) + r * (kCC * 2));
   const int lo = diag ? T + 1 + r : r + 1;
-  const int qlo = lo >> 3;
-  for (int dl = diag ? 1 : -(T - 1); dl <= T - 1; ++dl) {
-    const int c = r + dl;
-    const bool live = c >= 0 && c < T;
-    const int cc = live ? c : 0;
-    int below = __shfl_down_sync(full, v, 1);
-    if (r == T - 1) below = diag ? 0 : (int)B.bc[cc * kAS + (T - 1)];
-    if (diag && dl == 1) below = 0;
-    const uint4* bcol = reinterpret_cast<const uint4*>(B.bc + cc * kAS);
-    const int nq = diag ? ((dl + 5) >> 3) + 1 : ((37 + dl) >> 3) + 1;  // covers [qlo, q_hi] of every live lane
-    uint32_t a0 = 0, a1 = 0, a2 = 0, a3 = 0;  // four independent max chains (0 is neutral: gamma >= 0)
-    for (int t = 0; t < nq; ++t) {
-      const uint4 av = arow[qlo + t], bv = bcol[qlo + t];
-      a0 = __viaddmax_s16x2(av.x, bv.x, a0);
-      a1 = __viaddmax_s16x2(av.y, bv.y, a1);
-      a2 = __viaddmax_s16x2(av.z, bv.z, a2);
-      a3 = __viaddmax_s16x2(av.w, bv.w, a3);
+  const uint32_t a_q0 = opaque(as_s + (lo >> 3) * 16);
+  const uint32_t b_off = (lo >> 3) * 16;
+  const uint32_t st_bc = (uint32_t)((diag ? T + r - 1 : r - 1) * 2);  // my X[r][c] as a B entry of column c
+  // One step of the wavefront with NQ chunks (NQ covers [qlo, q_hi] of every live lane of
+  // local anti-diagonal dl); the steps run in segments of constant NQ, fully unrolled.
+  auto seg = [&](auto nqc, int dlA, int dlB) {
+    constexpr int NQ = decltype(nqc)::value;
+#pragma unroll 1
+    for (int dl = dlA; dl <= dlB; ++dl) {
+      const int c = r + dl;
+      const bool live = c >= 0 && c < T;
+      const int cc = live ? c : 0;
+      const uint32_t bcol = opaque(bc_s + cc * (kAS * 2));
+      int below = __shfl_down_sync(full, v, 1);
+      if (r == T - 1) below = diag ? 0 : lds_s16(bcol + (T - 1) * 2);
+      if (diag && dl == 1) below = 0;
+      uint32_t a0 = 0, a1 = 0, a2 = 0, a3 = 0;  // four independent max chains (0 is neutral: gamma >= 0)
+      const uint32_t pb = bcol + b_off;
+#pragma unroll
+      for (int t = 0; t < NQ; ++t) {
+        const uint4 av = lds_v4(a_q0 + 16 * t), bv = lds_v4(pb + 16 * t);
+        a0 = __viaddmax_s16x2(av.x, bv.x, a0);
+        a1 = __viaddmax_s16x2(av.y, bv.y, a1);
+        a2 = __viaddmax_s16x2(av.z, bv.z, a2);
+        a3 = __viaddmax_s16x2(av.w, bv.w, a3);
+      }
+      const uint32_t acc = __vmaxs2(__vmaxs2(a0, a1), __vmaxs2(a2, a3));
+      int val = max((int)(int16_t)(acc & 0xffffu), (int)(int16_t)(acc >> 16));
+      val = max(val, lds_s16(cc_s + cc * 2));
+      val = max(val, max(below, v));
+      if ((pairbits >> cc) & 1u) val = max(val, below_prev + 1);
+      if (live) {
+        sts_u16(as_s + (T + c) * 2, val);
+        if (r >= 1) sts_u16(bcol + st_bc, val);
+        v = val;
+        below_prev = below;
+      }
+      __syncwarp();
     }
-    const uint32_t acc = __vmaxs2(__vmaxs2(a0, a1), __vmaxs2(a2, a3));
-    int val = max((int)(int16_t)(acc & 0xffffu), (int)(int16_t)(acc >> 16));
-    val = max(val, (int)B.cc[r * kCC + cc]);
-    val = max(val, max(below, v));
-    if ((pairbits >> cc) & 1u) val = max(val, below_prev + 1);
-    if (live) {
-      B.as[r * kAS + T + c] = (int16_t)val;
-      if (r >= 1) B.bc[c * kAS + (diag ? T + r - 1 : r - 1)] = (int16_t)val;
-      v = val;
-      below_prev = below;
-    }
-    __syncwarp();
+  };
+  using std::integral_constant;
+  if (diag) {  // NQ = ((dl + 5) >> 3) + 1
+    seg(integral_constant<int, 1>(), 1, 2);
+    seg(integral_constant<int, 2>(), 3, 10);
+    seg(integral_constant<int, 3>(), 11, 18);
+    seg(integral_constant<int, 4>(), 19, 26);
+    seg(integral_constant<int, 5>(), 27, 31);
+  } else {     // NQ = ((37 + dl) >> 3) + 1
+    seg(integral_constant<int, 1>(), -31, -30);
+    seg(integral_constant<int, 2>(), -29, -22);
+    seg(integral_constant<int, 3>(), -21, -14);
+    seg(integral_constant<int, 4>(), -13, -6);
+    seg(integral_constant<int, 5>(), -5, 2);
+    seg(integral_constant<int, 6>(), 3, 10);
+    seg(integral_constant<int, 7>(), 11, 18);
+    seg(integral_constant<int, 8>(), 19, 26);
+    seg(integral_constant<int, 9>(), 27, 31);
   }
   // ---- records: UT[c][r] = X[r][c], L[k][c] = X[k+1][c] (k < 31), L[31][c] = X[32][c]
   {
