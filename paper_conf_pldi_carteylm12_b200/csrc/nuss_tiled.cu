@@ -31,6 +31,7 @@
 #include <cstdint>
 #include <type_traits>
 #include <cooperative_groups.h>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "dp_internal.h"
@@ -195,74 +196,13 @@ __device__ __forceinline__ void sts_u16(uint32_t a, int v) {
 }
 __device__ __forceinline__ uint32_t pk16(int lo, int hi) { return (uint32_t)(uint16_t)lo | ((uint32_t)(uint16_t)hi << 16); }
 
-// Phase B: finalise tile (I,J) from C (max of the middle products), write its UT/L records.
-// One cell per lane (lane = row r) per local anti-diagonal; the neighbours come from the
-// lane's own previous cell (left) and lane r+1's (below, and the pair's inner cell one step
-// later); the in-tile split points are the uniform-length AS x BC reduction above.
-__device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, InTileBuf& B, const uint8_t* x,
-                        const uint8_t* pm, int n, int h, int lane) {
+// The in-tile wavefront over staged AS / BC / CC (see InTileBuf): 63 local anti-diagonals
+// (31 on a diagonal tile), one cell per lane. left = gamma(i0+r, j0-1), corner =
+// gamma(i0+32, j0-1); on return AS[r][32+c] holds X[r][c] (kNeg for c <= r on diagonal
+// tiles) and BC[c][...] the column entries.
+__device__ __forceinline__ void wavefront(InTileBuf& B, bool diag, int left, int corner, uint32_t pairbits, int lane) {
   const unsigned full = 0xffffffffu;
-  const bool diag = I == J;
-  const int i0 = I * T, j0 = J * T, r = lane;
-  int16_t* ut = tab.UT(I, J);
-  int16_t* l = tab.L(I, J);
-  // ---- staging (all global loads before the shared stores of each part)
-  {
-    int16_t v[T];
-    if (!diag) {
-      const int16_t* utii = tab.UT(I, I);
-#pragma unroll
-      for (int p = 0; p < T; ++p) v[p] = utii[p * T + r];  // U(I,I)[r][p] = gamma(i0+r, i0+p)
-    }
-    uint4* row = reinterpret_cast<uint4*>(B.as + r * kAS);
-#pragma unroll
-    for (int w = 0; w < kAS / 8; ++w) {
-      uint32_t q[4];
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int p0 = 8 * w + 2 * e;
-        const int lo = (!diag && p0 < T && p0 > r) ? v[p0 < T ? p0 : 0] : kNeg;
-        const int hi = (!diag && p0 + 1 < T && p0 + 1 > r) ? v[p0 + 1 < T ? p0 + 1 : 0] : kNeg;
-        q[e] = pk16(lo, hi);
-      }
-      row[w] = make_uint4(q[0], q[1], q[2], q[3]);
-    }
-  }
-  {
-    const int c = lane;
-    int16_t v[T];
-    if (!diag) {
-      const int16_t* ljj = tab.L(J, J);
-#pragma unroll
-      for (int k = 0; k < T; ++k) v[k] = ljj[k * T + c];  // L(J,J)[k][c] = gamma(j0+k+1, j0+c)
-    }
-    const int below = diag ? 0 : (int)tab.UT(I + 1, J)[c * T + 0];  // X[32][c] = gamma(i0+32, j0+c)
-    uint4* col = reinterpret_cast<uint4*>(B.bc + c * kAS);
-#pragma unroll
-    for (int w = 0; w < kAS / 8; ++w) {
-      uint32_t q[4];
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int p0 = 8 * w + 2 * e;
-        auto val = [&](int p) -> int {
-          if (p == T - 1) return below;
-          if (p >= T && p < 2 * T) return diag ? 0 : (int)v[p - T < T && p >= T ? p - T : 0];
-          return 0;
-        };
-        q[e] = pk16(val(p0), val(p0 + 1));
-      }
-      col[w] = make_uint4(q[0], q[1], q[2], q[3]);
-    }
-    int cv[T];
-#pragma unroll
-    for (int rr = 0; rr < T; ++rr) cv[rr] = has_c ? __ldcg(C + rr * T + c) : 0;
-#pragma unroll
-    for (int rr = 0; rr < T; ++rr) B.cc[rr * kCC + c] = (int16_t)cv[rr];
-  }
-  const int left = diag ? 0 : (int)tab.UT(I, J - 1)[(T - 1) * T + r];  // gamma(i0+r, j0-1)
-  const int corner = (!diag && I + 1 <= J - 1) ? (int)tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
-  const uint32_t pairbits = pair_bits(x, pm, n, i0, j0, h, lane);
-  __syncwarp();
+  const int r = lane;
   int v = left;                                                    // X[r][c-1]
   int below_prev = __shfl_down_sync(full, left, 1);                // X[r+1][c-1]
   if (r == T - 1) below_prev = corner;
@@ -332,6 +272,77 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
     seg(integral_constant<int, 8>(), 19, 26);
     seg(integral_constant<int, 9>(), 27, 31);
   }
+}
+
+// Phase B: finalise tile (I,J) from C (max of the middle products), write its UT/L records.
+// One cell per lane (lane = row r) per local anti-diagonal; the neighbours come from the
+// lane's own previous cell (left) and lane r+1's (below, and the pair's inner cell one step
+// later); the in-tile split points are the uniform-length AS x BC reduction above.
+__device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, InTileBuf& B, const uint8_t* x,
+                        const uint8_t* pm, int n, int h, int lane) {
+  const unsigned full = 0xffffffffu;
+  const bool diag = I == J;
+  const int i0 = I * T, j0 = J * T, r = lane;
+  int16_t* ut = tab.UT(I, J);
+  int16_t* l = tab.L(I, J);
+  // ---- staging (all global loads before the shared stores of each part)
+  {
+    int16_t v[T];
+    if (!diag) {
+      const int16_t* utii = tab.UT(I, I);
+#pragma unroll
+      for (int p = 0; p < T; ++p) v[p] = utii[p * T + r];  // U(I,I)[r][p] = gamma(i0+r, i0+p)
+    }
+    uint4* row = reinterpret_cast<uint4*>(B.as + r * kAS);
+#pragma unroll
+    for (int w = 0; w < kAS / 8; ++w) {
+      uint32_t q[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const int p0 = 8 * w + 2 * e;
+        const int lo = (!diag && p0 < T && p0 > r) ? v[p0 < T ? p0 : 0] : kNeg;
+        const int hi = (!diag && p0 + 1 < T && p0 + 1 > r) ? v[p0 + 1 < T ? p0 + 1 : 0] : kNeg;
+        q[e] = pk16(lo, hi);
+      }
+      row[w] = make_uint4(q[0], q[1], q[2], q[3]);
+    }
+  }
+  {
+    const int c = lane;
+    int16_t v[T];
+    if (!diag) {
+      const int16_t* ljj = tab.L(J, J);
+#pragma unroll
+      for (int k = 0; k < T; ++k) v[k] = ljj[k * T + c];  // L(J,J)[k][c] = gamma(j0+k+1, j0+c)
+    }
+    const int below = diag ? 0 : (int)tab.UT(I + 1, J)[c * T + 0];  // X[32][c] = gamma(i0+32, j0+c)
+    uint4* col = reinterpret_cast<uint4*>(B.bc + c * kAS);
+#pragma unroll
+    for (int w = 0; w < kAS / 8; ++w) {
+      uint32_t q[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const int p0 = 8 * w + 2 * e;
+        auto val = [&](int p) -> int {
+          if (p == T - 1) return below;
+          if (p >= T && p < 2 * T) return diag ? 0 : (int)v[p - T < T && p >= T ? p - T : 0];
+          return 0;
+        };
+        q[e] = pk16(val(p0), val(p0 + 1));
+      }
+      col[w] = make_uint4(q[0], q[1], q[2], q[3]);
+    }
+    int cv[T];
+#pragma unroll
+    for (int rr = 0; rr < T; ++rr) cv[rr] = has_c ? __ldcg(C + rr * T + c) : 0;
+#pragma unroll
+    for (int rr = 0; rr < T; ++rr) B.cc[rr * kCC + c] = (int16_t)cv[rr];
+  }
+  const int left = diag ? 0 : (int)tab.UT(I, J - 1)[(T - 1) * T + r];  // gamma(i0+r, j0-1)
+  const int corner = (!diag && I + 1 <= J - 1) ? (int)tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
+  const uint32_t pairbits = pair_bits(x, pm, n, i0, j0, h, lane);
+  __syncwarp();
+  wavefront(B, diag, left, corner, pairbits, lane);
   // ---- records: UT[c][r] = X[r][c], L[k][c] = X[k+1][c] (k < 31), L[31][c] = X[32][c]
   {
     const uint4* xr = reinterpret_cast<const uint4*>(B.as + r * kAS + T);
@@ -366,7 +377,8 @@ __device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, 
 // split on a stack in global memory. One step costs one round trip: lanes 0-3 load
 // gamma(i,j), gamma(i+1,j), gamma(i,j-1), gamma(i+1,j-1) while all lanes load the
 // first 32 split candidates.
-__device__ void warp_traceback(const Tab& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
+template <class TabT>
+__device__ void warp_traceback(const TabT& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
                                int2* stk, int lane) {
   for (int k = lane; k < n; k += 32) db[k] = '.';
   if (n <= 1) return;
@@ -490,6 +502,201 @@ __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(Nu
   clk.flush(lane);
 }
 
+// ------------------------------------------------------------------ batch driver (one warp per problem)
+// k_nuss_batch: every warp owns one problem at a time (no CTA barriers; 1-warp CTAs, as many
+// per SM as shared memory allows) and sweeps its tile-diagonals itself:
+//   per tile (I,J): issue the phase-B operand rows (cp.async) -> phase A over K = I+1..J-1
+//   with double-buffered cp.async staging, C accumulated in registers -> C to shared ->
+//   wavefront -> records.
+// Records (global, one slot per warp): UTd[k][r] = gamma(32I+r, 32J+k) duplicated into both
+// halves of a 32-bit word (the micro-kernel's A operand as stored, so staging is a plain
+// copy), L[k][c] = gamma(32I+k+1, 32J+c) (B operand); per diagonal tile also the phase-B
+// rows ASd[r][p] = U(I,I)[r][p] (kNeg for p <= r) and BCd[c][k] = L(I,I)[k][c].
+constexpr int kRecW = T * T + T * T / 2;  // 32-bit words per tile record (UTd 4 KB + L 2 KB)
+constexpr int kDiagW = T * T;             // 32-bit words per diagonal extra (ASd 2 KB + BCd 2 KB)
+constexpr int kStageB = 6144;             // bytes per phase-A stage (A 4 KB + B 2 KB)
+
+struct Tab2 {
+  uint32_t* base;
+  int nt;
+  __device__ __forceinline__ uint32_t* UTd(int I, int J) const { return base + tile_id(I, J, nt) * kRecW; }
+  __device__ __forceinline__ int16_t* L(int I, int J) const { return reinterpret_cast<int16_t*>(UTd(I, J) + T * T); }
+  __device__ __forceinline__ int16_t* ASd(int I) const {
+    return reinterpret_cast<int16_t*>(base + tiles_of(nt) * kRecW + (int64_t)I * kDiagW);
+  }
+  __device__ __forceinline__ int16_t* BCd(int I) const { return ASd(I) + T * T; }
+  __device__ __forceinline__ int g16(int I, int J, int k, int r) const {  // UTd(I,J)[k][r] low half
+    return (int)(int16_t)(__ldcg(UTd(I, J) + k * T + r) & 0xffffu);
+  }
+  __device__ __forceinline__ int gamma(int i, int j) const {
+    if (j - i < 1) return 0;
+    return g16(i / T, j / T, j % T, i % T);
+  }
+};
+
+__device__ __forceinline__ void cp16(uint32_t s, const void* g) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s), "l"(g) : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+__device__ __forceinline__ void stage_async(const Tab2& tab, int I, int K, int J, uint32_t st, int lane) {
+  const uint32_t* a = tab.UTd(I, K);
+  const int16_t* b = tab.L(K, J);
+#pragma unroll
+  for (int t = 0; t < 8; ++t) cp16(st + (lane + 32 * t) * 16, a + (lane + 32 * t) * 4);
+#pragma unroll
+  for (int t = 0; t < 4; ++t) cp16(st + 4096 + (lane + 32 * t) * 16, b + (lane + 32 * t) * 8);
+}
+
+__device__ void batch_tile(const Tab2& tab, int I, int J, uint8_t* stg, InTileBuf& B, const uint8_t* x,
+                           const uint8_t* pm, int n, int h, int lane) {
+  const bool diag = I == J;
+  const int r = lane;
+  const uint32_t stg_s = (uint32_t)__cvta_generic_to_shared(stg);
+  // scalar neighbours of the wavefront (loads in flight during phase A)
+  const int below = diag ? 0 : tab.g16(I + 1, J, lane, 0);                              // X[32][c], c = lane
+  const int left = diag ? 0 : tab.g16(I, J - 1, T - 1, r);                              // gamma(i0+r, j0-1)
+  const int corner = (!diag && I + 1 <= J - 1) ? tab.g16(I + 1, J - 1, T - 1, 0) : 0;  // gamma(i0+32, j0-1)
+  // phase A: C = max over K = I+1..J-1 of UTd(I,K) (x) L(K,J), double-buffered
+  uint32_t acc[16];
+#pragma unroll
+  for (int q = 0; q < 16; ++q) acc[q] = 0;  // gamma >= 0, so 0 is a neutral start
+  const int K0 = I + 1, K1 = J;
+  if (K0 < K1) {
+    stage_async(tab, I, K0, J, stg_s, lane);
+    cp_commit();
+    for (int K = K0; K < K1; ++K) {
+      const int b = (K - K0) & 1;
+      if (K + 1 < K1) {
+        stage_async(tab, I, K + 1, J, stg_s + (b ^ 1) * kStageB, lane);
+        cp_commit();
+        cp_wait<1>();
+      } else {
+        cp_wait<0>();
+      }
+      __syncwarp();
+      micro(reinterpret_cast<const uint32_t*>(stg + b * kStageB),
+            reinterpret_cast<const uint16_t*>(stg + b * kStageB + 4096), acc, lane);
+      __syncwarp();
+    }
+  }
+  // phase B rows (the staging buffers alias them: phase A is done), C to shared (int16 [r][c])
+  __syncwarp();
+  if (!diag) {
+    const uint32_t as_s = (uint32_t)__cvta_generic_to_shared(B.as + r * kAS);
+    const uint32_t bc_s = (uint32_t)__cvta_generic_to_shared(B.bc + r * kAS + T);
+    const int16_t* asd = tab.ASd(I) + r * T;
+    const int16_t* bcd = tab.BCd(J) + r * T;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) { cp16(as_s + 16 * q, asd + 8 * q); cp16(bc_s + 16 * q, bcd + 8 * q); }
+    cp_commit();
+  }
+  {
+    const int ty = lane >> 2, tx = lane & 3;
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr)
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        *reinterpret_cast<uint32_t*>(B.cc + (4 * ty + rr) * kCC + 8 * tx + 2 * q) = acc[rr * 4 + q];
+    const uint32_t NEG2 = pk16(kNeg, kNeg);
+    uint4* ar = reinterpret_cast<uint4*>(B.as + r * kAS);
+    uint4* bc = reinterpret_cast<uint4*>(B.bc + r * kAS);
+    const uint4 negs = make_uint4(NEG2, NEG2, NEG2, NEG2), zero = make_uint4(0, 0, 0, 0);
+#pragma unroll
+    for (int q = 4; q < 9; ++q) ar[q] = negs;               // X[r][*] not computed yet, pad
+    if (diag) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) { ar[q] = negs; bc[4 + q] = zero; }
+    }
+#pragma unroll
+    for (int q = 0; q < 3; ++q) bc[q] = zero;
+    bc[3] = make_uint4(0, 0, 0, pk16(0, below));            // BC[c][31] = X[32][c]
+    bc[8] = zero;
+  }
+  cp_wait<0>();
+  const uint32_t pairbits = pair_bits(x, pm, n, I * T, J * T, h, lane);
+  __syncwarp();
+  wavefront(B, diag, left, corner, pairbits, lane);
+  // records
+  {
+    const uint4* xr = reinterpret_cast<const uint4*>(B.as + r * kAS + T);
+    uint4 w[4], raw[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      raw[q] = w[q] = xr[q];
+      if (diag) {  // entries with c <= r are gamma(i, j <= i) = 0 (held as kNeg)
+        w[q].x = __vmaxs2(w[q].x, 0u); w[q].y = __vmaxs2(w[q].y, 0u);
+        w[q].z = __vmaxs2(w[q].z, 0u); w[q].w = __vmaxs2(w[q].w, 0u);
+      }
+    }
+    const uint32_t ww[16] = {w[0].x, w[0].y, w[0].z, w[0].w, w[1].x, w[1].y, w[1].z, w[1].w,
+                             w[2].x, w[2].y, w[2].z, w[2].w, w[3].x, w[3].y, w[3].z, w[3].w};
+    uint32_t* ut = tab.UTd(I, J);
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const uint32_t lo = ww[q] & 0xffffu, hi = ww[q] >> 16;
+      ut[(2 * q) * T + r] = lo | (lo << 16);
+      ut[(2 * q + 1) * T + r] = hi | (hi << 16);
+    }
+    int16_t* l = tab.L(I, J);
+    if (r >= 1) {
+      uint4* lr = reinterpret_cast<uint4*>(l + (r - 1) * T);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) lr[q] = w[q];
+    }
+    l[(T - 1) * T + lane] = B.bc[lane * kAS + (T - 1)];
+    if (diag) {
+      uint4* asd = reinterpret_cast<uint4*>(tab.ASd(I) + r * T);
+      uint4* bcd = reinterpret_cast<uint4*>(tab.BCd(I) + r * T);
+      const uint4* bcr = reinterpret_cast<const uint4*>(B.bc + r * kAS + T);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) { asd[q] = raw[q]; bcd[q] = bcr[q]; }
+    }
+  }
+  __syncwarp();
+}
+
+constexpr size_t kBatchBuf = 2 * kStageB > sizeof(InTileBuf) ? 2 * kStageB : ((sizeof(InTileBuf) + 15) & ~size_t(15));
+size_t batch_warp_bytes(int64_t max_len) { return kBatchBuf + ((max_len + 15) & ~int64_t(15)) + 16; }
+
+__global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_words) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int lane = threadIdx.x;
+  uint8_t* stg = smem;
+  InTileBuf& IB = *reinterpret_cast<InTileBuf*>(smem);  // aliases the phase-A stages
+  uint8_t* xs = smem + kBatchBuf;
+  uint8_t* pm = xs + ((A.max_len + 15) & ~int64_t(15));
+  if (lane < 16) pm[lane] = A.pair_mask[lane];
+  Tab2 tab;
+  tab.base = reinterpret_cast<uint32_t*>(A.scratch) + (int64_t)blockIdx.x * slot_words;
+  const int ntm = (int)((A.max_len + T - 1) / T);
+  int2* stack = reinterpret_cast<int2*>(tab.base + tiles_of(ntm) * kRecW + (int64_t)ntm * kDiagW);
+  PhaseClock clk;
+  clk.dbg = A.dbg;
+  clk.start();
+  for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
+    const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+    __syncwarp();
+    for (int q = lane; q < n; q += 32) xs[q] = A.x_cat[A.x_off[p] + q];
+    const int nt = (n + T - 1) / T;
+    tab.nt = nt;
+    __syncwarp();
+    clk.lap(0);
+    for (int D = 0; D < nt; ++D)
+      for (int t = 0; t + D < nt; ++t) batch_tile(tab, t, t + D, stg, IB, xs, pm, n, A.hairpin, lane);
+    clk.lap(4);
+    if (lane == 0) {
+      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
+      if (A.db) A.db_len[p] = n;
+    }
+    if (A.db) warp_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, lane);
+    clk.lap(6);
+  }
+  clk.flush(lane);
+}
+
 // ------------------------------------------------------------------ grid driver (one large problem)
 __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_tiled_grid(NussArgs A, int64_t p) {
   cg::grid_group grid = cg::this_grid();
@@ -587,6 +794,22 @@ int num_sms_t(int device) {
   return v > 0 ? v : 148;
 }
 
+int64_t batch_slot_words(int64_t max_len) {
+  const int nt = (int)((max_len + T - 1) / T);
+  return tiles_of(nt) * kRecW + (int64_t)nt * kDiagW + 2 * (2 * max_len + 8);
+}
+
+int batch_ctas_per_sm(int64_t max_len) {
+  const size_t smem = batch_warp_bytes(max_len);
+  cudaFuncSetAttribute(k_nuss_batch, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncSetAttribute(k_nuss_batch, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  int per_sm = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_nuss_batch, 32, smem);
+  return per_sm > 0 ? per_sm : 1;
+}
+
+bool use_v1() { return getenv("DP_NUSS_V1") != nullptr; }
+
 }  // namespace
 
 bool nuss_tiled_supported(int64_t max_len) { return max_len <= 65536; }
@@ -597,8 +820,12 @@ int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
   if (n == 1 && max_len > kGridMin) {
     return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
   }
-  const int64_t grid = std::min<int64_t>(n, kCtaPerSm * (int64_t)num_sms_t(device));
-  return grid * (tiles_of(nt) * kRec * 2 + (int64_t)kCtaWarps * T * T * 4 + stack_bytes) + 256;
+  if (use_v1()) {
+    const int64_t grid = std::min<int64_t>(n, kCtaPerSm * (int64_t)num_sms_t(device));
+    return grid * (tiles_of(nt) * kRec * 2 + (int64_t)kCtaWarps * T * T * 4 + stack_bytes) + 256;
+  }
+  const int64_t grid = std::min<int64_t>(n, (int64_t)batch_ctas_per_sm(max_len) * num_sms_t(device));
+  return grid * batch_slot_words(max_len) * 4 + 256;
 }
 
 cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
@@ -622,6 +849,13 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
     return cudaLaunchCooperativeKernel((void*)k_nuss_tiled_grid, sms, kGridWarps * 32, args, smem, s);
   }
   if (A.max_len > 4096) return cudaErrorInvalidValue;  // batch path keeps the sequence in shared memory
+  if (!use_v1()) {
+    const int per_sm = batch_ctas_per_sm(A.max_len);
+    const int64_t grid = std::min<int64_t>(A.n, (int64_t)per_sm * sms);
+    ++*launches;
+    k_nuss_batch<<<(unsigned)grid, 32, batch_warp_bytes(A.max_len), s>>>(A, batch_slot_words(A.max_len));
+    return cudaGetLastError();
+  }
   const size_t smem = kCtaWarps * warp_bytes();
   cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
