@@ -390,7 +390,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         unsigned long long h[8];
         cudaStreamSynchronize(s);
         cudaMemcpy(h, dbg, sizeof(h), cudaMemcpyDeviceToHost);
-        const char* nm[8] = {"stage", "clearC", "phaseA", "waitA", "phaseB", "waitB", "traceback", "-"};
+        const char* nm[8] = {"stage", "phaseA", "stageB", "wavefront", "records", "score", "traceback", "-"};
         double tot = 0;
         for (int q = 0; q < 7; ++q) tot += (double)h[q];
         for (int q = 0; q < 7; ++q) fprintf(stderr, "nuss %-9s %16llu %5.1f%%\n", nm[q], h[q], 100.0 * h[q] / (tot > 0 ? tot : 1));

@@ -213,9 +213,12 @@ __device__ __forceinline__ void wavefront(InTileBuf& B, bool diag, int left, int
   const uint32_t as_s = opaque((uint32_t)__cvta_generic_to_shared(B.as) + r * (kAS * 2));
   const uint32_t bc_s = opaque((uint32_t)__cvta_generic_to_shared(B.bc));
   const uint32_t cc_s = opaque((uint32_t)__cvta_generic_to_shared(B.cc) + r * (kCC * 2));
-  const int lo = diag ? T + 1 + r : r + 1;
-  const uint32_t a_q0 = opaque(as_s + (lo >> 3) * 16);
-  const uint32_t b_off = (lo >> 3) * 16;
+  // first chunk: r >> 3 (off-diagonal) or 4 + (r >> 3) (diagonal), the same for the 8 lanes of
+  // a quarter-warp so their 16-byte loads stay conflict-free (chunks below a lane's range are
+  // masked by kNeg on the A side)
+  const int qlo = diag ? 4 + (r >> 3) : (r >> 3);
+  const uint32_t a_q0 = opaque(as_s + qlo * 16);
+  const uint32_t b_off = qlo * 16;
   const uint32_t st_bc = (uint32_t)((diag ? T + r - 1 : r - 1) * 2);  // my X[r][c] as a B entry of column c
   // One step of the wavefront with NQ chunks (NQ covers [qlo, q_hi] of every live lane of
   // local anti-diagonal dl); the steps run in segments of constant NQ, fully unrolled.
@@ -255,22 +258,22 @@ __device__ __forceinline__ void wavefront(InTileBuf& B, bool diag, int left, int
     }
   };
   using std::integral_constant;
-  if (diag) {  // NQ = ((dl + 5) >> 3) + 1
-    seg(integral_constant<int, 1>(), 1, 2);
-    seg(integral_constant<int, 2>(), 3, 10);
-    seg(integral_constant<int, 3>(), 11, 18);
-    seg(integral_constant<int, 4>(), 19, 26);
-    seg(integral_constant<int, 5>(), 27, 31);
-  } else {     // NQ = ((37 + dl) >> 3) + 1
-    seg(integral_constant<int, 1>(), -31, -30);
-    seg(integral_constant<int, 2>(), -29, -22);
-    seg(integral_constant<int, 3>(), -21, -14);
-    seg(integral_constant<int, 4>(), -13, -6);
-    seg(integral_constant<int, 5>(), -5, 2);
-    seg(integral_constant<int, 6>(), 3, 10);
-    seg(integral_constant<int, 7>(), 11, 18);
-    seg(integral_constant<int, 8>(), 19, 26);
-    seg(integral_constant<int, 9>(), 27, 31);
+  if (diag) {  // NQ = ((38 + dl) >> 3) - 3
+    seg(integral_constant<int, 1>(), 1, 1);
+    seg(integral_constant<int, 2>(), 2, 9);
+    seg(integral_constant<int, 3>(), 10, 17);
+    seg(integral_constant<int, 4>(), 18, 25);
+    seg(integral_constant<int, 5>(), 26, 31);
+  } else {     // NQ = ((38 + dl) >> 3) + 1
+    seg(integral_constant<int, 1>(), -31, -31);
+    seg(integral_constant<int, 2>(), -30, -23);
+    seg(integral_constant<int, 3>(), -22, -15);
+    seg(integral_constant<int, 4>(), -14, -7);
+    seg(integral_constant<int, 5>(), -6, 1);
+    seg(integral_constant<int, 6>(), 2, 9);
+    seg(integral_constant<int, 7>(), 10, 17);
+    seg(integral_constant<int, 8>(), 18, 25);
+    seg(integral_constant<int, 9>(), 26, 31);
   }
 }
 
@@ -426,6 +429,66 @@ __device__ void warp_traceback(const TabT& tab, const uint8_t* x, const uint8_t*
   }
 }
 
+// The same canonical traceback with the table in global memory (far from L2) and fewer
+// round trips: an 8x8 window of gamma (rows i..i+7, columns j-7..j) is fetched in one round
+// trip into shared memory and the unpaired / pair steps run out of it (a step moves i up or
+// j down by at most one, so a window serves up to 7 steps); split points cost one round
+// trip per 32 candidates. The interval stack lives in shared memory (kStk entries), deeper
+// entries in global memory.
+constexpr int kStk = 64;
+template <class TabT>
+__device__ void warp_traceback_win(const TabT& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
+                                   int2* stk, int* win, int2* sstk, int lane) {
+  for (int k = lane; k < n; k += 32) db[k] = '.';
+  if (n <= 1) return;
+  const unsigned full = 0xffffffffu;
+  int sp = 1;
+  if (lane == 0) sstk[0] = make_int2(0, n - 1);
+  __syncwarp();
+  int wi = -(1 << 20), wj = -(1 << 20);
+  int guard = 4 * n + 8;
+  while (sp > 0 && --guard > 0) {
+    --sp;
+    const int2 iv = sp < kStk ? sstk[sp] : stk[sp];
+    int i = iv.x, j = iv.y;
+    __syncwarp();
+    while (j - i >= 1 && --guard > 0) {
+      if (!(i >= wi && i + 1 <= wi + 7 && j <= wj && j - 1 >= wj - 7)) {
+        wi = i; wj = j;
+        const int a0 = tab.gamma(i + (lane >> 3), j - 7 + (lane & 7));
+        const int a1 = tab.gamma(i + 4 + (lane >> 3), j - 7 + (lane & 7));
+        __syncwarp();
+        win[lane] = a0;
+        win[lane + 32] = a1;
+        __syncwarp();
+      }
+      const int* wr = win + (i - wi) * 8 + (j - wj + 7);
+      const int v = wr[0], g1 = wr[8], g2 = wr[-1], g3 = wr[7];
+      if (v == g1) { i += 1; continue; }
+      if (v == g2) { j -= 1; continue; }
+      if (pairable(x, pm, n, i, j, h) && v == g3 + 1) {
+        if (lane == 0) { db[i] = '('; db[j] = ')'; }
+        i += 1; j -= 1;
+        continue;
+      }
+      int kk = -1;
+      for (int k0 = i + 1; kk < 0 && k0 < j; k0 += 32) {
+        const int kq = k0 + lane;
+        const unsigned m = __ballot_sync(full, kq < j && v == tab.gamma(i, kq) + tab.gamma(kq + 1, j));
+        if (m) kk = k0 + __ffs(m) - 1;
+      }
+      if (kk < 0) break;  // inconsistent table: cannot happen
+      if (lane == 0) {
+        if (sp < kStk) sstk[sp] = make_int2(kk + 1, j);  // right part later, left part now
+        else stk[sp] = make_int2(kk + 1, j);
+      }
+      ++sp;
+      __syncwarp();
+      j = kk;
+    }
+  }
+}
+
 // ------------------------------------------------------------------ batch driver
 __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
   extern __shared__ __align__(16) uint8_t smem[];
@@ -551,7 +614,7 @@ __device__ __forceinline__ void stage_async(const Tab2& tab, int I, int K, int J
 }
 
 __device__ void batch_tile(const Tab2& tab, int I, int J, uint8_t* stg, InTileBuf& B, const uint8_t* x,
-                           const uint8_t* pm, int n, int h, int lane) {
+                           const uint8_t* pm, int n, int h, int lane, PhaseClock& clk) {
   const bool diag = I == J;
   const int r = lane;
   const uint32_t stg_s = (uint32_t)__cvta_generic_to_shared(stg);
@@ -584,6 +647,7 @@ __device__ void batch_tile(const Tab2& tab, int I, int J, uint8_t* stg, InTileBu
   }
   // phase B rows (the staging buffers alias them: phase A is done), C to shared (int16 [r][c])
   __syncwarp();
+  clk.lap(1);
   if (!diag) {
     const uint32_t as_s = (uint32_t)__cvta_generic_to_shared(B.as + r * kAS);
     const uint32_t bc_s = (uint32_t)__cvta_generic_to_shared(B.bc + r * kAS + T);
@@ -618,7 +682,9 @@ __device__ void batch_tile(const Tab2& tab, int I, int J, uint8_t* stg, InTileBu
   cp_wait<0>();
   const uint32_t pairbits = pair_bits(x, pm, n, I * T, J * T, h, lane);
   __syncwarp();
+  clk.lap(2);
   wavefront(B, diag, left, corner, pairbits, lane);
+  clk.lap(3);
   // records
   {
     const uint4* xr = reinterpret_cast<const uint4*>(B.as + r * kAS + T);
@@ -656,10 +722,11 @@ __device__ void batch_tile(const Tab2& tab, int I, int J, uint8_t* stg, InTileBu
     }
   }
   __syncwarp();
+  clk.lap(4);
 }
 
 constexpr size_t kBatchBuf = 2 * kStageB > sizeof(InTileBuf) ? 2 * kStageB : ((sizeof(InTileBuf) + 15) & ~size_t(15));
-size_t batch_warp_bytes(int64_t max_len) { return kBatchBuf + ((max_len + 15) & ~int64_t(15)) + 16; }
+size_t batch_warp_bytes(int64_t max_len) { return kBatchBuf + ((max_len + 15) & ~int64_t(15)) + 16 + 256 + 8 * kStk; }
 
 __global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_words) {
   extern __shared__ __align__(16) uint8_t smem[];
@@ -668,6 +735,8 @@ __global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_
   InTileBuf& IB = *reinterpret_cast<InTileBuf*>(smem);  // aliases the phase-A stages
   uint8_t* xs = smem + kBatchBuf;
   uint8_t* pm = xs + ((A.max_len + 15) & ~int64_t(15));
+  int* win = reinterpret_cast<int*>(pm + 16);
+  int2* sstk = reinterpret_cast<int2*>(pm + 16 + 256);
   if (lane < 16) pm[lane] = A.pair_mask[lane];
   Tab2 tab;
   tab.base = reinterpret_cast<uint32_t*>(A.scratch) + (int64_t)blockIdx.x * slot_words;
@@ -685,13 +754,13 @@ __global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_
     __syncwarp();
     clk.lap(0);
     for (int D = 0; D < nt; ++D)
-      for (int t = 0; t + D < nt; ++t) batch_tile(tab, t, t + D, stg, IB, xs, pm, n, A.hairpin, lane);
-    clk.lap(4);
+      for (int t = 0; t + D < nt; ++t) batch_tile(tab, t, t + D, stg, IB, xs, pm, n, A.hairpin, lane, clk);
+    clk.lap(5);
     if (lane == 0) {
       A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
       if (A.db) A.db_len[p] = n;
     }
-    if (A.db) warp_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, lane);
+    if (A.db) warp_traceback_win(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, win, sstk, lane);
     clk.lap(6);
   }
   clk.flush(lane);
