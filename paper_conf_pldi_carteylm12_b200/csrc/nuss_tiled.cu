@@ -613,38 +613,56 @@ __device__ __forceinline__ void stage_async(const Tab2& tab, int I, int K, int J
   for (int t = 0; t < 4; ++t) cp16(st + 4096 + (lane + 32 * t) * 16, b + (lane + 32 * t) * 8);
 }
 
+// Phase A over K in [K0, K1): acc (micro-kernel lane layout) = max(acc, UTd(I,K) (x) L(K,J)),
+// operands staged by double-buffered cp.async.
+__device__ __forceinline__ void products_async(const Tab2& tab, int I, int J, int K0, int K1, uint8_t* stg,
+                                               uint32_t (&acc)[16], int lane) {
+  if (K0 >= K1) return;
+  const uint32_t stg_s = (uint32_t)__cvta_generic_to_shared(stg);
+  stage_async(tab, I, K0, J, stg_s, lane);
+  cp_commit();
+  for (int K = K0; K < K1; ++K) {
+    const int b = (K - K0) & 1;
+    if (K + 1 < K1) {
+      stage_async(tab, I, K + 1, J, stg_s + (b ^ 1) * kStageB, lane);
+      cp_commit();
+      cp_wait<1>();
+    } else {
+      cp_wait<0>();
+    }
+    __syncwarp();
+    micro(reinterpret_cast<const uint32_t*>(stg + b * kStageB),
+          reinterpret_cast<const uint16_t*>(stg + b * kStageB + 4096), acc, lane);
+    __syncwarp();
+  }
+}
+
+// Phase B of tile (I,J) from C in registers (acc), then its records.
+__device__ void tile_finish(const Tab2& tab, int I, int J, const uint32_t (&acc)[16], int below, int left, int corner,
+                            InTileBuf& B, const uint8_t* x, const uint8_t* pm, int n, int h, int lane,
+                            PhaseClock& clk);
+
 __device__ void batch_tile(const Tab2& tab, int I, int J, uint8_t* stg, InTileBuf& B, const uint8_t* x,
                            const uint8_t* pm, int n, int h, int lane, PhaseClock& clk) {
   const bool diag = I == J;
   const int r = lane;
-  const uint32_t stg_s = (uint32_t)__cvta_generic_to_shared(stg);
   // scalar neighbours of the wavefront (loads in flight during phase A)
   const int below = diag ? 0 : tab.g16(I + 1, J, lane, 0);                              // X[32][c], c = lane
   const int left = diag ? 0 : tab.g16(I, J - 1, T - 1, r);                              // gamma(i0+r, j0-1)
   const int corner = (!diag && I + 1 <= J - 1) ? tab.g16(I + 1, J - 1, T - 1, 0) : 0;  // gamma(i0+32, j0-1)
-  // phase A: C = max over K = I+1..J-1 of UTd(I,K) (x) L(K,J), double-buffered
+  // phase A: C = max over K = I+1..J-1 of UTd(I,K) (x) L(K,J)
   uint32_t acc[16];
 #pragma unroll
   for (int q = 0; q < 16; ++q) acc[q] = 0;  // gamma >= 0, so 0 is a neutral start
-  const int K0 = I + 1, K1 = J;
-  if (K0 < K1) {
-    stage_async(tab, I, K0, J, stg_s, lane);
-    cp_commit();
-    for (int K = K0; K < K1; ++K) {
-      const int b = (K - K0) & 1;
-      if (K + 1 < K1) {
-        stage_async(tab, I, K + 1, J, stg_s + (b ^ 1) * kStageB, lane);
-        cp_commit();
-        cp_wait<1>();
-      } else {
-        cp_wait<0>();
-      }
-      __syncwarp();
-      micro(reinterpret_cast<const uint32_t*>(stg + b * kStageB),
-            reinterpret_cast<const uint16_t*>(stg + b * kStageB + 4096), acc, lane);
-      __syncwarp();
-    }
-  }
+  products_async(tab, I, J, I + 1, J, stg, acc, lane);
+  tile_finish(tab, I, J, acc, below, left, corner, B, x, pm, n, h, lane, clk);
+}
+
+__device__ void tile_finish(const Tab2& tab, int I, int J, const uint32_t (&acc)[16], int below, int left, int corner,
+                            InTileBuf& B, const uint8_t* x, const uint8_t* pm, int n, int h, int lane,
+                            PhaseClock& clk) {
+  const bool diag = I == J;
+  const int r = lane;
   // phase B rows (the staging buffers alias them: phase A is done), C to shared (int16 [r][c])
   __syncwarp();
   clk.lap(1);
@@ -764,6 +782,116 @@ __global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_
     clk.lap(6);
   }
   clk.flush(lane);
+}
+
+// ------------------------------------------------------------------ grid driver v2 (one large problem)
+// k_nuss_grid2: the tile-diagonal sweep of one table over the whole grid (cooperative launch),
+// on the batch kernel's records (duplicated-A UTd, L, diagonal ASd/BCd) and cp.async staging.
+// Round D: phase-B warps (warp % 4 == 0, tiles spread over the SMs) add the two boundary
+// K-steps I+1 and J-1 in registers, merge the interior products from global C and finish the
+// tile; the other warps compute the interior K-steps of diagonal D+1 (split-K, atomicMax into
+// global C). One grid-wide barrier per tile-diagonal.
+__global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, int64_t p) {
+  cg::grid_group grid = cg::this_grid();
+  extern __shared__ __align__(16) uint8_t smem[];
+  __shared__ uint8_t pm[16];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
+  __syncthreads();
+  uint8_t* stg = smem + warp * kBatchBuf;
+  InTileBuf& IB = *reinterpret_cast<InTileBuf*>(stg);
+  const uint8_t* x = A.x_cat + A.x_off[p];
+  const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+  const int nt = (n + T - 1) / T;
+  Tab2 tab;
+  tab.base = reinterpret_cast<uint32_t*>(A.scratch);
+  tab.nt = nt;
+  int* Cg = reinterpret_cast<int*>(tab.base + tiles_of(nt) * kRecW + (int64_t)nt * kDiagW);  // 2 x nt x 1024
+  int2* stack = reinterpret_cast<int2*>(Cg + 2 * (int64_t)nt * T * T);
+  PhaseClock clk;
+  clk.dbg = nullptr;
+  const int ty = lane >> 2, tx = lane & 3;
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T;
+       q += (int64_t)gridDim.x * blockDim.x)
+    Cg[q] = 0;
+  grid.sync();
+  for (int D = 0; D < nt; ++D) {
+    if (A.round_ns && blockIdx.x == 0 && threadIdx.x == 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      A.round_ns[D] = t;
+    }
+    const int nT = nt - D;
+    int* C = Cg + (int64_t)(D & 1) * nt * T * T;        // diagonal D (interior products already in)
+    int* Cn = Cg + (int64_t)((D + 1) & 1) * nt * T * T; // diagonal D+1
+    if ((warp & 3) == 0) {
+      for (int64_t tt = blockIdx.x + (int64_t)gridDim.x * (warp >> 2); tt < nT;
+           tt += (int64_t)gridDim.x * (kGridWarps / 4)) {
+        const int t = (int)tt, I = t, J = t + D;
+        const bool diag = D == 0;
+        int* Ct = C + (int64_t)t * T * T;
+        const int below = diag ? 0 : tab.g16(I + 1, J, lane, 0);
+        const int left = diag ? 0 : tab.g16(I, J - 1, T - 1, lane);
+        const int corner = (!diag && I + 1 <= J - 1) ? tab.g16(I + 1, J - 1, T - 1, 0) : 0;
+        uint32_t acc[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) acc[q] = 0;
+        if (D >= 2) products_async(tab, I, J, I + 1, I + 2, stg, acc, lane);
+        if (D >= 3) products_async(tab, I, J, J - 1, J, stg, acc, lane);
+        if (D >= 4) {  // interior K = I+2 .. J-2 from the other warps (complete at the last grid barrier)
+#pragma unroll
+          for (int rr = 0; rr < 4; ++rr)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const int* cp = Ct + (4 * ty + rr) * T + 8 * tx + 2 * q;
+              acc[rr * 4 + q] = __vmaxs2(acc[rr * 4 + q], pk16(__ldcg(cp), __ldcg(cp + 1)));
+            }
+        }
+        tile_finish(tab, I, J, acc, below, left, corner, IB, x, pm, n, A.hairpin, lane, clk);
+        if (D >= 4)  // this C slot is reused by diagonal D+2
+          for (int q = lane; q < T * T; q += 32) Ct[q] = 0;
+      }
+    } else if (D + 1 < nt && D >= 3) {
+      // interior K-steps of diagonal D+1: tiles t' (I = t', J = t' + D + 1), K in [I+2, J-2]
+      const int nT1 = nt - (D + 1), ks = D - 2;
+      const int64_t total = (int64_t)nT1 * ks;
+      const int64_t nwA = (int64_t)gridDim.x * (kGridWarps - kGridWarps / 4);
+      const int64_t wA = (int64_t)blockIdx.x * (kGridWarps - kGridWarps / 4) + (warp - (warp >> 2) - 1);
+      const int64_t per = (total + nwA - 1) / nwA;
+      const int64_t b0 = wA * per, b1 = min(total, b0 + per);
+      int64_t it = b0;
+      while (it < b1) {
+        const int t = (int)(it / ks), kk = (int)(it % ks);
+        const int64_t e = min(b1, (int64_t)(t + 1) * ks);
+        const int I = t, J = t + D + 1;
+        uint32_t acc[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) acc[q] = 0;
+        products_async(tab, I, J, I + 2 + kk, I + 2 + kk + (int)(e - it), stg, acc, lane);
+        int* Ct = Cn + (int64_t)t * T * T;
+#pragma unroll
+        for (int rr = 0; rr < 4; ++rr)
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const uint32_t v = acc[rr * 4 + q];
+            int* c = Ct + (4 * ty + rr) * T + 8 * tx + 2 * q;
+            atomicMax(c, (int)(int16_t)(v & 0xffffu));
+            atomicMax(c + 1, (int)(int16_t)(v >> 16));
+          }
+        it = e;
+      }
+    }
+    grid.sync();
+  }
+  if (blockIdx.x == 0 && warp == 0) {
+    if (lane == 0) {
+      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
+      if (A.db) A.db_len[p] = n;
+    }
+    if (A.db)
+      warp_traceback_win(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, stack, reinterpret_cast<int*>(stg),
+                         reinterpret_cast<int2*>(stg + 256), lane);
+  }
 }
 
 // ------------------------------------------------------------------ grid driver (one large problem)
@@ -887,7 +1015,8 @@ int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
   const int nt = (int)((max_len + T - 1) / T);
   const int64_t stack_bytes = (4 * max_len + 8) * 4;
   if (n == 1 && max_len > kGridMin) {
-    return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
+    if (use_v1()) return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
+    return (tiles_of(nt) * kRecW + (int64_t)nt * kDiagW + 2 * (int64_t)nt * T * T) * 4 + stack_bytes + 256;
   }
   if (use_v1()) {
     const int64_t grid = std::min<int64_t>(n, kCtaPerSm * (int64_t)num_sms_t(device));
@@ -903,6 +1032,20 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
   cudaGetDevice(&dev);
   const int sms = num_sms_t(dev);
   const int nt = (int)((A.max_len + T - 1) / T);
+  if (A.n == 1 && A.max_len > kGridMin && !use_v1()) {
+    const size_t smem = kGridWarps * kBatchBuf;
+    cudaError_t e = cudaFuncSetAttribute(k_nuss_grid2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_nuss_grid2, kGridWarps * 32, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) return cudaErrorInvalidConfiguration;
+    NussArgs a2 = A;
+    int64_t p = 0;
+    void* args[2] = {&a2, &p};
+    ++*launches;
+    return cudaLaunchCooperativeKernel((void*)k_nuss_grid2, sms, kGridWarps * 32, args, smem, s);
+  }
   if (A.n == 1 && A.max_len > kGridMin) {
     const size_t smem = kGridWarps * warp_bytes();
     cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_grid, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
