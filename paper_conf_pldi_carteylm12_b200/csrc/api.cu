@@ -382,6 +382,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       if (e != cudaSuccess) break;
       A.scratch = p->scratch.ptr;
       unsigned long long* rounds = nullptr;
+      if (getenv("DP_NUSS_TBW")) A.tbw = atoi(getenv("DP_NUSS_TBW"));
       if (getenv("DP_NUSS_ROUNDS") && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), A.round_ns = rounds;
       unsigned long long* dbg = nullptr;
       if (getenv("DP_NUSS_TIMING") && tiled) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
@@ -402,6 +403,8 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         cudaMemcpy(h, rounds, sizeof(h), cudaMemcpyDeviceToHost);
         const int nt = (int)((A.max_len + 31) / 32);
         for (int d = 0; d + 1 < nt; ++d) fprintf(stderr, "round %d %.1f us\n", d, (h[d + 1] - h[d]) * 1e-3);
+        fprintf(stderr, "last round + score %.1f us\n", (h[nt] - h[nt - 1]) * 1e-3);
+        if (h[nt + 1] > h[nt]) fprintf(stderr, "traceback %.1f us\n", (h[nt + 1] - h[nt]) * 1e-3);
         cudaFree(rounds);
       }
       break;

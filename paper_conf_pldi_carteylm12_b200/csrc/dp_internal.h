@@ -90,6 +90,7 @@ struct NussArgs {
   int64_t scratch_bytes;
   unsigned long long* round_ns;  // optional: %globaltimer at each tile-diagonal round (grid sweep)
   unsigned long long* dbg = nullptr;  // DP_NUSS_TIMING: batch-kernel phase cycles (8 counters)
+  int tbw = 0;                        // grid traceback window (8/16/32; DP_NUSS_TBW), 0 = default
 };
 int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device);
 bool nuss_tiled_supported(int64_t max_len);

@@ -436,58 +436,94 @@ __device__ void warp_traceback(const TabT& tab, const uint8_t* x, const uint8_t*
 // trip per 32 candidates. The interval stack lives in shared memory (kStk entries), deeper
 // entries in global memory.
 constexpr int kStk = 64;
-template <class TabT>
+// Trace one interval [i, j] (canonical order); the right part of every split is handed to
+// push(k+1, j) and the walk continues on the left part. W x W window (rows i..i+W-1, columns
+// j-W+1..j; W*W/32 values per lane per round trip); KC split candidates per lane per round trip.
+template <int W, int KC, class TabT, class Push>
+__device__ __forceinline__ void trace_interval(const TabT& tab, const uint8_t* x, const uint8_t* pm, int n, int h,
+                                               uint8_t* db, int i, int j, int* win, int& guard, Push&& push,
+                                               int lane) {
+  const unsigned full = 0xffffffffu;
+  int wi = -(1 << 20), wj = -(1 << 20);
+  while (j - i >= 1 && --guard > 0) {
+    if (!(i >= wi && i + 1 <= wi + W - 1 && j <= wj && j - 1 >= wj - W + 1)) {
+      wi = i; wj = j;
+      int a[W * W / 32];
+#pragma unroll
+      for (int q = 0; q < W * W / 32; ++q) {
+        const int cell = lane + 32 * q;
+        a[q] = tab.gamma(i + cell / W, j - W + 1 + cell % W);
+      }
+      __syncwarp();
+#pragma unroll
+      for (int q = 0; q < W * W / 32; ++q) win[lane + 32 * q] = a[q];
+      __syncwarp();
+    }
+    const int* wr = win + (i - wi) * W + (j - wj + W - 1);
+    const int v = wr[0], g1 = wr[W], g2 = wr[-1], g3 = wr[W - 1];
+    if (v == g1) { i += 1; continue; }
+    if (v == g2) { j -= 1; continue; }
+    if (pairable(x, pm, n, i, j, h) && v == g3 + 1) {
+      if (lane == 0) { db[i] = '('; db[j] = ')'; }
+      i += 1; j -= 1;
+      continue;
+    }
+    int kk = -1;
+    for (int k0 = i + 1; kk < 0 && k0 < j; k0 += 32 * KC) {
+      int s[KC];
+#pragma unroll
+      for (int u = 0; u < KC; ++u) {
+        const int kq = k0 + lane + 32 * u;
+        s[u] = kq < j ? tab.gamma(i, kq) + tab.gamma(kq + 1, j) : -1;
+      }
+#pragma unroll
+      for (int u = 0; u < KC; ++u) {
+        const unsigned m = __ballot_sync(full, s[u] == v);
+        if (kk < 0 && m) kk = k0 + 32 * u + __ffs(m) - 1;
+      }
+    }
+    if (kk < 0) break;  // inconsistent table: cannot happen
+    push(kk + 1, j);    // right part later (or elsewhere), left part now
+    j = kk;
+  }
+}
+
+// One warp, interval stack in shared memory (kStk entries, deeper ones in global memory).
+template <int W, int KC, class TabT>
 __device__ void warp_traceback_win(const TabT& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
                                    int2* stk, int* win, int2* sstk, int lane) {
   for (int k = lane; k < n; k += 32) db[k] = '.';
   if (n <= 1) return;
-  const unsigned full = 0xffffffffu;
   int sp = 1;
   if (lane == 0) sstk[0] = make_int2(0, n - 1);
   __syncwarp();
-  int wi = -(1 << 20), wj = -(1 << 20);
   int guard = 4 * n + 8;
+  auto push = [&](int a, int b) {
+    if (lane == 0) {
+      if (sp < kStk) sstk[sp] = make_int2(a, b);
+      else stk[sp] = make_int2(a, b);
+    }
+    ++sp;
+    __syncwarp();
+  };
   while (sp > 0 && --guard > 0) {
     --sp;
     const int2 iv = sp < kStk ? sstk[sp] : stk[sp];
-    int i = iv.x, j = iv.y;
     __syncwarp();
-    while (j - i >= 1 && --guard > 0) {
-      if (!(i >= wi && i + 1 <= wi + 7 && j <= wj && j - 1 >= wj - 7)) {
-        wi = i; wj = j;
-        const int a0 = tab.gamma(i + (lane >> 3), j - 7 + (lane & 7));
-        const int a1 = tab.gamma(i + 4 + (lane >> 3), j - 7 + (lane & 7));
-        __syncwarp();
-        win[lane] = a0;
-        win[lane + 32] = a1;
-        __syncwarp();
-      }
-      const int* wr = win + (i - wi) * 8 + (j - wj + 7);
-      const int v = wr[0], g1 = wr[8], g2 = wr[-1], g3 = wr[7];
-      if (v == g1) { i += 1; continue; }
-      if (v == g2) { j -= 1; continue; }
-      if (pairable(x, pm, n, i, j, h) && v == g3 + 1) {
-        if (lane == 0) { db[i] = '('; db[j] = ')'; }
-        i += 1; j -= 1;
-        continue;
-      }
-      int kk = -1;
-      for (int k0 = i + 1; kk < 0 && k0 < j; k0 += 32) {
-        const int kq = k0 + lane;
-        const unsigned m = __ballot_sync(full, kq < j && v == tab.gamma(i, kq) + tab.gamma(kq + 1, j));
-        if (m) kk = k0 + __ffs(m) - 1;
-      }
-      if (kk < 0) break;  // inconsistent table: cannot happen
-      if (lane == 0) {
-        if (sp < kStk) sstk[sp] = make_int2(kk + 1, j);  // right part later, left part now
-        else stk[sp] = make_int2(kk + 1, j);
-      }
-      ++sp;
-      __syncwarp();
-      j = kk;
-    }
+    trace_interval<W, KC>(tab, x, pm, n, h, db, iv.x, iv.y, win, guard, push, lane);
   }
 }
+
+// Work queue of intervals for the grid-wide traceback (one large problem): tickets from
+// hdr[0] (head), slots published with a flag after a fence (hdr[1] = tail); hdr[2] counts
+// intervals not yet finished, so a warp waiting on an unpublished slot stops when it is zero.
+struct GridQueue {
+  int* hdr;
+  int* flag;
+  int2* item;
+  int cap;
+};
+__host__ __device__ __forceinline__ int grid_queue_cap(int64_t max_len) { return (int)max_len + 8192; }
 
 // ------------------------------------------------------------------ batch driver
 __global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
@@ -778,7 +814,7 @@ __global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_
       A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
       if (A.db) A.db_len[p] = n;
     }
-    if (A.db) warp_traceback_win(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, win, sstk, lane);
+    if (A.db) warp_traceback_win<8, 1>(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, win, sstk, lane);
     clk.lap(6);
   }
   clk.flush(lane);
@@ -807,13 +843,17 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   tab.base = reinterpret_cast<uint32_t*>(A.scratch);
   tab.nt = nt;
   int* Cg = reinterpret_cast<int*>(tab.base + tiles_of(nt) * kRecW + (int64_t)nt * kDiagW);  // 2 x nt x 1024
-  int2* stack = reinterpret_cast<int2*>(Cg + 2 * (int64_t)nt * T * T);
+  GridQueue Q;
+  Q.hdr = Cg + 2 * (int64_t)nt * T * T;
+  Q.cap = grid_queue_cap(A.max_len);
+  Q.flag = Q.hdr + 4;
+  Q.item = reinterpret_cast<int2*>(Q.flag + Q.cap + (Q.cap & 1));
   PhaseClock clk;
   clk.dbg = nullptr;
   const int ty = lane >> 2, tx = lane & 3;
-  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T;
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T + 4 + Q.cap;
        q += (int64_t)gridDim.x * blockDim.x)
-    Cg[q] = 0;
+    Cg[q] = 0;  // C buffers, queue counters and flags
   grid.sync();
   for (int D = 0; D < nt; ++D) {
     if (A.round_ns && blockIdx.x == 0 && threadIdx.x == 0) {
@@ -883,14 +923,76 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
     }
     grid.sync();
   }
-  if (blockIdx.x == 0 && warp == 0) {
-    if (lane == 0) {
-      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
-      if (A.db) A.db_len[p] = n;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (A.round_ns) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      A.round_ns[nt] = t;
     }
-    if (A.db)
-      warp_traceback_win(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, stack, reinterpret_cast<int*>(stg),
-                         reinterpret_cast<int2*>(stg + 256), lane);
+    A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
+    if (A.db) A.db_len[p] = n;
+  }
+  if (!A.db) return;
+  // canonical traceback by the whole grid: intervals in a work queue (see TbQueue)
+  uint8_t* db = A.db + p * A.db_stride;
+  const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, gthreads = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t q = gtid; q < n; q += gthreads) db[q] = '.';
+  if (gtid == 0 && n > 1) {
+    Q.item[0] = make_int2(0, n - 1);
+    Q.flag[0] = 1;
+    Q.hdr[1] = 1;  // tail
+    Q.hdr[2] = 1;  // outstanding
+  }
+  grid.sync();
+  const unsigned full = 0xffffffffu;
+  int* win = reinterpret_cast<int*>(stg);
+  int guard = 4 * n + 8;
+  auto push = [&](int a, int b) {
+    if (lane == 0) {
+      atomicAdd(&Q.hdr[2], 1);
+      const int t = atomicAdd(&Q.hdr[1], 1);
+      if (t < Q.cap) {
+        Q.item[t] = make_int2(a, b);
+        __threadfence();
+        atomicExch(&Q.flag[t], 1);
+      }
+    }
+    __syncwarp();
+  };
+  for (;;) {
+    int idx = 0;
+    if (lane == 0) idx = atomicAdd(&Q.hdr[0], 1);
+    idx = __shfl_sync(full, idx, 0);
+    int got = 0;
+    for (;;) {
+      int f = 0, o = 0;
+      if (lane == 0) {
+        f = idx < Q.cap ? *reinterpret_cast<volatile int*>(&Q.flag[idx]) : 0;
+        o = *reinterpret_cast<volatile int*>(&Q.hdr[2]);
+      }
+      f = __shfl_sync(full, f, 0);
+      o = __shfl_sync(full, o, 0);
+      if (f) { got = 1; break; }
+      if (o <= 0) break;
+      __nanosleep(128);
+    }
+    if (!got) break;
+    __threadfence();
+    const int2 iv = __ldcg(&Q.item[idx]);
+    trace_interval<8, 1>(tab, x, pm, n, A.hairpin, db, iv.x, iv.y, win, guard, push, lane);
+    __syncwarp();
+    if (lane == 0) {
+      __threadfence();
+      atomicSub(&Q.hdr[2], 1);
+    }
+  }
+  if (A.round_ns) {
+    grid.sync();
+    if (gtid == 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      A.round_ns[nt + 1] = t;
+    }
   }
 }
 
@@ -1016,7 +1118,8 @@ int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
   const int64_t stack_bytes = (4 * max_len + 8) * 4;
   if (n == 1 && max_len > kGridMin) {
     if (use_v1()) return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
-    return (tiles_of(nt) * kRecW + (int64_t)nt * kDiagW + 2 * (int64_t)nt * T * T) * 4 + stack_bytes + 256;
+    return (tiles_of(nt) * kRecW + (int64_t)nt * kDiagW + 2 * (int64_t)nt * T * T) * 4 +
+           (4 + 3 * (int64_t)grid_queue_cap(max_len) + 2) * 4 + 256;
   }
   if (use_v1()) {
     const int64_t grid = std::min<int64_t>(n, kCtaPerSm * (int64_t)num_sms_t(device));
