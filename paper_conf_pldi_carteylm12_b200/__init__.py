@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libdp.so")
+LIB_PATH = os.environ.get("DP_LIB") or os.path.join(_PKG, "libdp.so")  # DP_LIB: experiment builds only
 
 EDIT, SW_LINEAR, NUSSINOV, HMM_FORWARD, HMM_VITERBI, SW_AFFINE = range(6)
 KIND_NAMES = {EDIT: "edit", SW_LINEAR: "sw_linear", NUSSINOV: "nussinov", HMM_FORWARD: "hmm_forward",

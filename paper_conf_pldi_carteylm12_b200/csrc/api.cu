@@ -143,6 +143,8 @@ cudaError_t sw16_args(dp_plan* p, int64_t n, const uint8_t* a_cat, const int64_t
   A->lanebest = A->corner + slab_words;
   A->strips_max = strips;
   A->nslab_max = nslab > 0 ? nslab : 1;
+  A->tb_ctr = reinterpret_cast<unsigned long long*>(
+      (reinterpret_cast<uintptr_t>(A->rowck + rw + cw + bw) + 15) & ~static_cast<uintptr_t>(15));
   p->last_scores = scores;
   return cudaSuccess;
 }
@@ -219,7 +221,7 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) { st = DP_E_TOO_LARGE; break; }
       e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
       p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
-      p->packed16 = dpk::sw16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap) &&
+      p->packed16 = dpk::sw16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap, d->want_traceback != 0) &&
                     getenv("DP_FORCE_INT32") == nullptr;
       break;
     case DP_SW_AFFINE:

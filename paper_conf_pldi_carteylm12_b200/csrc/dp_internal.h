@@ -11,12 +11,18 @@ namespace dpk {
 // one predicated branch per lap.
 struct PhaseClock {
   unsigned long long* dbg;
-  long long t, acc[8];
-  __device__ __forceinline__ void start() { if (dbg) { t = clock64(); for (int q = 0; q < 8; ++q) acc[q] = 0; } }
-  __device__ __forceinline__ void lap(int q) { if (dbg) { const long long u = clock64(); acc[q] += u - t; t = u; } }
-  __device__ __forceinline__ void flush(int lane) {
-    if (dbg && lane == 0) for (int q = 0; q < 8; ++q) atomicAdd(dbg + q, (unsigned long long)acc[q]);
+  long long t;
+  __device__ __forceinline__ void start() { if (dbg) t = clock64(); }
+  // off (dbg == nullptr) only the pointer stays live; on, lane 0 of every warp adds its lap
+  __device__ __forceinline__ void lap(int q) {
+    if (dbg) {
+      const long long u = clock64();
+      if ((threadIdx.x & 31) == 0) atomicAdd(dbg + q, (unsigned long long)(u - t));
+      t = u;
+    }
   }
+  __device__ __forceinline__ void count(int q) { if (dbg && (threadIdx.x & 31) == 0) atomicAdd(dbg + q, 1ull); }
+  __device__ __forceinline__ void flush(int) {}
 };
 
 constexpr int kWarps = 8;  // warps per CTA for the warp-per-problem kernels
@@ -64,9 +70,10 @@ struct Sw16Args {
   uint32_t* corner;      // [groups][strips][nslab][32]           G of the row above the lane at its checkpoint column
   uint32_t* lanebest;    // [groups][strips][32]                  per-lane best G over the strip
   int64_t strips_max, nslab_max;
+  unsigned long long* tb_ctr;  // traceback work queues (two 64-bit counters, zeroed per launch)
   unsigned long long* dbg = nullptr;  // DP_SW_TIMING: traceback phase cycles (8 counters), else nullptr
 };
-bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap);
+bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap, bool want_tb);
 int sw16_smem_per_warp(int asz, int64_t max_la, int64_t max_lb);
 void sw16_state_words(int64_t n, int64_t max_la, int64_t max_lb, int64_t* strips, int64_t* nslab, int64_t* rowck,
                       int64_t* colck, int64_t* slabbest);

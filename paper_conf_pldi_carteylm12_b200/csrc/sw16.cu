@@ -20,10 +20,11 @@
 // every column) and, after every block of 32 steps, every lane's 8 rows at the
 // column it is on (a staircase, column 32 s - lane: warp-uniform, coalesced,
 // no per-step branch), the G above it there and its best G over the block
-// (0.25 B/cell), plus every lane's maximum over the strip. k_sw16_tb3 recomputes
-// only the 32x32 (sheared) blocks the canonical traceback needs and walks them
-// with the oracle's tie-break (diag > up > left, stop at H = 0; end cell = first
-// maximum in row-major order).
+// (0.25 B/cell), plus every lane's maximum over the strip. k_sw16_tb5 recomputes
+// only the 32x32 (sheared) blocks the canonical traceback needs, as 2-bit
+// direction codes that carry the oracle's tie-break (stop at H = 0, then
+// diag > up > left; end cell = first maximum in row-major order), and walks them.
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cuda_runtime.h>
@@ -282,237 +283,272 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
 }
 
 // ---------------------------------------------------------------- traceback
-// k_sw16_tb3: one warp serves 8 forward pairs (problems 2g, 2g+1), one pair per
-// 4-lane group. A traceback "block" is 32 rows (forward lanes L0..L0+3 of one
-// strip, L0 = 4 (blk mod 8)) x one slab: forward lane L0+m covered columns
+// k_sw16_tb5: persistent warps of 8 four-lane groups; CTAs of kTbWarps warps
+// share the sigma table. Each group carries two problems, one per s16x2 half:
+// the low half serves even problems, the high half odd ones (the forward packed
+// problems 2g, 2g+1 into the halves of its checkpoints), and each half takes its
+// next problem from its own queue (an atomic counter) as soon as it is done, so
+// warps stay full until the queues drain.
+//
+// A traceback "block" is 32 rows (forward lanes L0..L0+3 of one strip,
+// L0 = 4 (blk mod 8)) x one slab: forward lane L0+m covered columns
 // j = D + c - m, c = 1..32, D = 32 slab - L0, at forward steps 32 slab + c - 1.
 // So in the sheared column c all four lanes are at the SAME forward step and
 // group lane m re-runs forward lane L0+m (8 rows) for 32 steps exactly as the
 // sweep did (no ramp): the left column is its checkpoint, its first diagonal the
-// corner word, lane 0's "up" the band checkpoint row above the block. The two
-// s16x2 halves carry the pair's two problems, each with its own block. The G of
-// the block go to shared memory column-major; the canonical walk (diag > up >
-// left, stop at H = 0) then runs on one lane per problem, 16 walkers per warp.
-// The end cell (first row-major maximum) comes from the per-lane strip maxima,
-// then the slabs of that lane whose maximum equals the score.
-constexpr int kCS = 36;                  // words per block column: row t (-1..31) at t + 4
-constexpr int kGS = 34 * kCS + 4;        // words per group buffer (columns c = -1..32); = 4 mod 8
-constexpr int kBS = 40;                  // staged b residues per half (columns D-3 .. D+32)
-constexpr int kDeadCode = 31;            // residue code whose sigma row/column is kDead (alphabets < 32)
-constexpr int kOpsCap = 512;             // ops staged in shared memory per problem (longer paths spill to the row tail)
+// corner word, lane 0's "up" the band checkpoint row above the block.
+//
+// The re-run computes KEYS K = 4 G + code instead of G: every candidate of the
+// cell carries its traceback priority in the two low bits (Z: H = 0 -> 3,
+// diagonal 2, up 1, left 0; sigma is tabulated as 4 sigma + 2), so the max that
+// the recurrence takes anyway also takes the oracle's tie-break (stop at H = 0,
+// then diag > up > left). Only the codes are kept: 2 bits per cell and problem,
+// one 32-bit word per lane and column (8 rows x 2 halves), 512 B per group, and
+// the walk reads one word per step. Keys stay in s16 while 4 x the score bound
+// fits (plan check). The end cell (first row-major maximum) comes from the
+// per-lane strip maxima, then the slabs of that lane whose maximum equals the
+// score, then a compare inside the re-run (taken only on a hit).
+constexpr int kTbWarps = 4;              // warps per CTA
+#ifndef TB5_MINB
+#define TB5_MINB 5                       // CTAs per SM (register cap)
+#endif
+constexpr int kCW = 4 * kSlab;           // code words per group: [c - 1][m]
+constexpr int kTS = 36;                  // top-row keys per group, c = 0..32
+constexpr int kBS = 40;                  // staged b residues per half (columns D-3 .. D+36)
+constexpr int kDeadCode = 31;            // residue code whose sigma row/column is kDead4 (alphabets < 32)
+constexpr int kDead4 = -4000;            // keyed sigma outside a problem
+constexpr uint32_t kClean = 0xfffcfffcu, kCodeBits = 0x00030003u;
 
-__device__ __forceinline__ int lds_s8(uint32_t a) {
-  int v;
-  asm("ld.shared.s8 %0, [%1];" : "=r"(v) : "r"(a));
-  return v;
-}
+enum : int { kIdle = 0, kSearch = 1, kWalk = 2, kFinish = 3, kDone = 4 };
+struct TbState {      // one problem in one half of a group (shared memory; written by one lane)
+  long long p;        // problem id
+  long long found;    // search: row-major key (i << 32 | j) of the first maximum, -1 none
+  const uint8_t *a, *b;  // residues
+  int la, lb, best;
+  int mode;
+  int band;           // search: first lane band (strip * 32 + lane) whose maximum is the score
+  int scur, cand;     // search: next slab to probe, candidate slab (-1 none)
+  int i, j, n;        // walk: current cell, ops written
+  int ei, ej;         // end cell
+};
+constexpr int kGroupBytes = 4 * kCW + 4 * kTS + 2 * kBS + 2 * kBlk + 2 * (int)sizeof(TbState);
+constexpr int kTbWarpBytes = 8 * kGroupBytes;
+
 __device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
   uint32_t v;
   asm("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
   return v;
 }
+__device__ __forceinline__ uint32_t lds_s16w(uint32_t a) {
+  int v;
+  asm("ld.shared.s16 %0, [%1];" : "=r"(v) : "r"(a));
+  return (uint32_t)v;
+}
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
 __device__ __forceinline__ uint32_t join(uint32_t lo_src, uint32_t hi_src) { return prmt(lo_src, hi_src, 0x7610u); }
+__device__ __forceinline__ uint32_t key4(uint32_t g2) { return (g2 << 2) & kClean; }  // 4 G per half
+__device__ __forceinline__ uint32_t pack2(int v) { return (uint32_t)(uint16_t)(int16_t)v * 0x10001u; }
 __device__ __forceinline__ void prefetch_l2(const void* p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
 
-struct TbHalf {       // one problem of the pair (uniform within its group)
-  int64_t p;          // problem id
-  const uint8_t *a, *b;
-  int la, lb, best;
-  int mode;           // 0 done / idle, 1 end-cell search, 2 walk
-  int band;           // search: first lane band (strip*32 + lane) reaching the score
-  int scur, cand;     // search: next slab to probe, candidate slab (-1 none)
-  long long found;    // search: row-major key (i << 32 | j) of the first maximum
-  int i, j, h, n;     // walk state
-  int ei, ej;         // end cell
-  int blk, sl, on;    // this round's block
-};
-
-__global__ void __launch_bounds__(32) k_sw16_tb3(Sw16Args A, int64_t first, int64_t count, uint8_t* out,
-                                                  int64_t stride, int32_t* out_len, int32_t* coords) {
+__global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A, int64_t first, int64_t count,
+                                                                       uint8_t* out, int64_t stride, int32_t* out_len,
+                                                                       int32_t* coords) {
   extern __shared__ __align__(16) uint8_t tsm[];
-  int8_t* sig_s = reinterpret_cast<int8_t*>(tsm);                 // [32][32], kDead outside the alphabet
-  const int lane = threadIdx.x, gq = lane >> 2, m = lane & 3;
-  for (int q = lane; q < 32 * 32; q += 32) {
+  int16_t* sig_s = reinterpret_cast<int16_t*>(tsm);  // [32][32] 4 sigma + 2, kDead4 outside the alphabet
+  for (int q = threadIdx.x; q < 32 * 32; q += blockDim.x) {
     const int x = q >> 5, y = q & 31;
-    sig_s[q] = (x < A.asz && y < A.asz) ? A.sigma[x * A.asz + y] : (int8_t)kDead;
+    sig_s[q] = (x < A.asz && y < A.asz) ? (int16_t)(4 * A.sigma[x * A.asz + y] + 2) : (int16_t)kDead4;
   }
-  uint32_t* Hs = reinterpret_cast<uint32_t*>(tsm + 1024) + gq * kGS;
-  uint8_t* bS = tsm + 1024 + 8 * kGS * 4 + gq * 2 * kBS;           // [2][kBS] staged b residues
-  uint8_t* aS = tsm + 1024 + 8 * kGS * 4 + 8 * 2 * kBS + gq * 2 * kBlk;  // [2][32] staged a residues
-  uint8_t* opsS = tsm + 1024 + 8 * kGS * 4 + 8 * 2 * kBS + 8 * 2 * kBlk + gq * 2 * kOpsCap;  // [2][cap] ops
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, gq = lane >> 2, m = lane & 3;
+  uint8_t* wb = tsm + 2048 + warp * kTbWarpBytes;
+  uint32_t* Cs = reinterpret_cast<uint32_t*>(wb) + gq * kCW;
+  uint32_t* Ts = reinterpret_cast<uint32_t*>(wb + 8 * 4 * kCW) + gq * kTS;
+  uint8_t* bS = wb + 8 * 4 * (kCW + kTS) + gq * 2 * kBS;                  // [2][kBS] staged b residues
+  uint8_t* aS = wb + 8 * 4 * (kCW + kTS) + 8 * 2 * kBS + gq * 2 * kBlk;  // [2][32] staged a residues
+  TbState* St = reinterpret_cast<TbState*>(wb + 8 * (4 * (kCW + kTS) + 2 * kBS + 2 * kBlk)) + 2 * gq;
   const uint32_t sig32 = (uint32_t)__cvta_generic_to_shared(sig_s);
-  const uint32_t hs32 = (uint32_t)__cvta_generic_to_shared(Hs);
+  const uint32_t cs32 = (uint32_t)__cvta_generic_to_shared(Cs);
+  const uint32_t ts32 = (uint32_t)__cvta_generic_to_shared(Ts);
   const uint32_t bs32 = (uint32_t)__cvta_generic_to_shared(bS);
-  const unsigned full = 0xffffffffu;
+  const uint32_t aS32 = (uint32_t)__cvta_generic_to_shared(aS);
+  const unsigned full = 0xffffffffu, gmask = 0xfu << (lane & ~3);
   const int g = A.gap;
-  const uint32_t NEG_G2 = (uint32_t)(uint16_t)(-g) * 0x10001u;
-  const int64_t grp = (first >> 1) + (int64_t)blockIdx.x * 8 + gq;
+  const uint32_t NEG_G2 = pack2(-g), NEG4 = pack2(-4 * g), NEG4U = pack2(-4 * g + 1), ZC = pack2(-4 * g + 3);
   const int64_t SM = A.strips_max, NS = A.nslab_max;
+  // queues: half hf serves problems p = 2 k + hf in [first, first + count)
+  const int64_t k0[2] = {(first + 1) >> 1, first >> 1};
+  const int64_t kn[2] = {((first + count + 1) >> 1) - k0[0], ((first + count) >> 1) - k0[1]};
+  if (m == 0) { St[0].mode = kIdle; St[1].mode = kIdle; }
+  __syncthreads();
   PhaseClock clk;
   clk.dbg = A.dbg;
   clk.start();
 
-  TbHalf H[2];
+  for (;;) {
+    // A) idle halves take their next problem; a problem with score 0 finishes at once
 #pragma unroll
-  for (int hf = 0; hf < 2; ++hf) {
-    TbHalf& X = H[hf];
-    X.p = 2 * grp + hf;
-    const bool mine = X.p >= first && X.p < first + count;
-    X.la = mine ? (int)(A.a_off[X.p + 1] - A.a_off[X.p]) : 0;
-    X.lb = mine ? (int)(A.b_off[X.p + 1] - A.b_off[X.p]) : 0;
-    X.a = mine ? A.a_cat + A.a_off[X.p] : A.a_cat;
-    X.b = mine ? A.b_cat + A.b_off[X.p] : A.b_cat;
-    X.best = mine ? A.scores[X.p] : 0;
-    X.mode = (mine && X.best > 0 && X.la > 0 && X.lb > 0) ? 1 : 0;
-    X.band = -1; X.scur = 0; X.cand = -1; X.found = -1;
-    X.i = X.j = X.h = X.n = 0; X.ei = X.ej = 0;
-    X.blk = X.sl = X.on = 0;
-  }
-  // 1) first lane band (row-major: strip, lane) whose strip maximum reaches the score
-  {
-    int stw = max((H[0].la + kStrip - 1) / kStrip, (H[1].la + kStrip - 1) / kStrip);
+    for (int hf = 0; hf < 2; ++hf) {
+      if (St[hf].mode != kIdle) continue;
+      int64_t q = 0;
+      if (m == 0) q = atomicAdd(reinterpret_cast<unsigned long long*>(A.tb_ctr) + hf, 1ull);
+      q = __shfl_sync(gmask, q, lane & ~3);
+      if (m == 0) {
+        TbState& S = St[hf];
+        if (q >= kn[hf]) {
+          S.mode = kDone;
+        } else {
+          const int64_t p = 2 * (k0[hf] + q) + hf;
+          S.p = p;
+          const int64_t ao = A.a_off[p], bo = A.b_off[p];
+          S.a = A.a_cat + ao;
+          S.b = A.b_cat + bo;
+          S.la = (int)(A.a_off[p + 1] - ao);
+          S.lb = (int)(A.b_off[p + 1] - bo);
+          S.best = A.scores[p];
+          S.mode = (S.best > 0 && S.la > 0 && S.lb > 0) ? kSearch : kFinish;
+          S.band = -1; S.scur = 0; S.cand = -1; S.found = -1;
+          S.i = S.j = S.n = S.ei = S.ej = 0;
+        }
+      }
+      __syncwarp(gmask);
+      // prologue: first lane band (row-major: strip, lane) whose strip maximum reaches the score
+      if (St[hf].mode == kSearch) {
+        const int64_t grp = St[hf].p >> 1;
+        const int best = St[hf].best, la = St[hf].la;
+        int band = -1;
+        for (int st = 0; st * kStrip < la && band < 0; ++st) {
+          int firstl = 32;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) stw = max(stw, __shfl_xor_sync(full, stw, o));
-    for (int st = 0; st < stw; ++st) {
-      uint32_t w[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q)
-        w[q] = (H[0].mode | H[1].mode) && grp < (A.n + 1) / 2 && st < SM
-                   ? __ldcg(A.lanebest + (grp * SM + st) * 32 + 8 * m + q) : 0u;
-#pragma unroll
-      for (int hf = 0; hf < 2; ++hf) {
-        TbHalf& X = H[hf];
-        const bool want = X.mode == 1 && X.band < 0 && st * kStrip < X.la;
-        int firstl = 32;
-#pragma unroll
-        for (int q = 7; q >= 0; --q)
-          if (want && half16(w[q], hf) + g == X.best) firstl = 8 * m + q;
-        firstl = min(firstl, __shfl_xor_sync(full, firstl, 1));
-        firstl = min(firstl, __shfl_xor_sync(full, firstl, 2));
-        if (want && firstl < 32) X.band = st * 32 + firstl;
+          for (int q8 = 7; q8 >= 0; --q8)
+            if (half16(__ldcg(A.lanebest + (grp * SM + st) * 32 + 8 * m + q8), hf) + g == best) firstl = 8 * m + q8;
+          firstl = min(firstl, __shfl_xor_sync(gmask, firstl, 1));
+          firstl = min(firstl, __shfl_xor_sync(gmask, firstl, 2));
+          if (firstl < 32) band = st * 32 + firstl;
+        }
+        __syncwarp(gmask);
+        if (m == 0) {
+          St[hf].band = band;
+          if (band < 0) St[hf].mode = kFinish;  // cannot happen: the maxima name the score
+        }
+        __syncwarp(gmask);
       }
     }
+    if (!__any_sync(full, St[0].mode != kDone || St[1].mode != kDone)) break;
+    clk.lap(0);
+    // B) searching halves: next candidate slab of their lane band (32 slabs per probe)
 #pragma unroll
-    for (int hf = 0; hf < 2; ++hf)
-      if (H[hf].mode == 1 && H[hf].band < 0) H[hf].mode = 0;  // cannot happen: the maxima name the score
-  }
-  __syncwarp();
-  clk.lap(0);
-
-  int guard = 8 * (int)((A.max_la + A.max_lb) / 16 + 8);
-  while (__any_sync(full, (H[0].mode | H[1].mode) != 0) && --guard > 0) {
-    // 2) searching halves: next candidate slab of their lane band (32 slabs per probe)
-    for (;;) {
-      bool need[2];
-#pragma unroll
-      for (int hf = 0; hf < 2; ++hf) need[hf] = H[hf].mode == 1 && H[hf].cand < 0;
-      if (!__any_sync(full, need[0] || need[1])) break;
-#pragma unroll
-      for (int hf = 0; hf < 2; ++hf) {
-        TbHalf& X = H[hf];
-        const int nsl = (X.lb + 31 + kSlab - 1) / kSlab;
-        const int st8 = X.band >> 5, ln8 = X.band & 31;
+    for (int hf = 0; hf < 2; ++hf) {
+      while (St[hf].mode == kSearch && St[hf].cand < 0) {
+        const TbState& S = St[hf];
+        const int64_t grp = S.p >> 1;
+        const int nsl = (S.lb + 31 + kSlab - 1) / kSlab, scur = S.scur, best = S.best;
+        const uint32_t* sb = A.slabbest + ((grp * SM + (S.band >> 5)) * NS) * 32 + (S.band & 31);
         uint32_t bits = 0;
-        if (need[hf]) {
-          const uint32_t* sb = A.slabbest + ((grp * SM + st8) * NS) * 32 + ln8;
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const int s = X.scur + m + 4 * q;
-            if (s < nsl && half16(__ldcg(sb + (int64_t)s * 32), hf) + g == X.best) bits |= 1u << (m + 4 * q);
-          }
+        for (int q = 0; q < 8; ++q) {
+          const int s = scur + m + 4 * q;
+          if (s < nsl && half16(__ldcg(sb + (int64_t)s * 32), hf) + g == best) bits |= 1u << (m + 4 * q);
         }
-        bits |= __shfl_xor_sync(full, bits, 1);
-        bits |= __shfl_xor_sync(full, bits, 2);
-        if (need[hf]) {
+        bits |= __shfl_xor_sync(gmask, bits, 1);
+        bits |= __shfl_xor_sync(gmask, bits, 2);
+        __syncwarp(gmask);
+        if (m == 0) {
+          TbState& W = St[hf];
           if (bits) {
-            X.cand = X.scur + __ffs(bits) - 1;
+            W.cand = scur + __ffs(bits) - 1;
           } else {
-            X.scur += 32;
-            if (X.scur >= nsl) {  // candidates exhausted: walk from the first maximum
-              if (X.found >= 0) {
-                X.mode = 2;
-                X.i = X.ei = (int)(X.found >> 32);
-                X.j = X.ej = (int)(X.found & 0xffffffffll);
-                X.h = X.best;
+            W.scur = scur + 32;
+            if (W.scur >= nsl) {  // candidates exhausted: walk from the first maximum
+              if (W.found >= 0) {
+                W.mode = kWalk;
+                W.i = W.ei = (int)(W.found >> 32);
+                W.j = W.ej = (int)(W.found & 0xffffffffll);
               } else {
-                X.mode = 0;  // cannot happen
+                W.mode = kFinish;  // cannot happen
               }
             }
           }
         }
+        __syncwarp(gmask);
       }
     }
+    __syncwarp();
     clk.lap(1);
-    if (clk.dbg) clk.acc[7] += 1;
-    // 3) this round's block per half
-#pragma unroll
-    for (int hf = 0; hf < 2; ++hf) {
-      TbHalf& X = H[hf];
-      X.on = 0;
-      if (X.mode == 1 && X.cand >= 0) {
-        const int st8 = X.band >> 5, ln8 = X.band & 31;
-        X.blk = st8 * (kStrip / kBlk) + ln8 / 4;
-        X.sl = X.cand;
-        X.on = 1;
-      } else if (X.mode == 2) {
-        const int ln = ((X.i - 1) % kStrip) / kRows;
-        X.blk = (X.i - 1) / kBlk;
-        X.sl = (X.j + ln - 1) / kSlab;
-        X.on = 1;
-      }
-    }
-    // 3b) walking halves: the block after this one is above, above-left or left of it;
-    // pull their checkpoints into L2 now so the next round's loads do not go to DRAM.
-#pragma unroll
-    for (int hf = 0; hf < 2; ++hf) {
-      const TbHalf& X = H[hf];
-      if (X.mode != 2) continue;
-#pragma unroll
-      for (int q = 0; q < 3; ++q) {
-        const int nb = X.blk - (q < 2 ? 1 : 0), ns = X.sl - (q > 0 ? 1 : 0);
-        if (nb < 0 || ns < 1) continue;
-        const int r0 = nb * kBlk, st = r0 / kStrip, L0 = (r0 % kStrip) / kRows;
-        const int64_t base = (grp * SM + st) * NS + (ns - 1);
-        prefetch_l2(A.colck + base * kStrip + (L0 + m) * kRows);
-        if (m == 0) prefetch_l2(A.corner + base * 32 + L0);
-        if (r0 > 0) {
-          const int bnd = r0 / kBand - 1, j0 = max(1, ns * kSlab - L0 + 16 * m);
-          if (j0 <= X.lb)
-            prefetch_l2(A.rowck + ((grp * SM + bnd / kBandsPerStrip) * kBandsPerStrip + bnd % kBandsPerStrip) * A.max_lb +
-                        (j0 - 1));
-        }
-      }
-    }
-    // 4) recompute both blocks. Every global load of the round is issued before any
-    // shared-memory store (checkpoint column, corner, a and b residues, top row).
+    clk.count(7);
+    // C) this round's block per half, D) prefetch, E) checkpoints as keys. Every global
+    // load of the round is issued before any shared-memory store.
     int R0[2], D[2];
     uint32_t sa[2][kRows];
-    uint32_t Gs[kRows], prev;
+    uint32_t Kc[kRows], prev;
+    uint32_t T4m1 = 0x7fff7fffu;  // search target 4 (best - g) - 1 in lane m8's half, else never exceeded
     {
       uint32_t w[2][kRows], cw[2], av[2][kRows], bv[2][kBS / 4], tv[2][9];
 #pragma unroll
       for (int hf = 0; hf < 2; ++hf) {
-        TbHalf& X = H[hf];
-        R0[hf] = X.blk * kBlk;
+        const TbState& S = St[hf];
+        const int mode = S.mode;
+        const bool srch = mode == kSearch && S.cand >= 0;
+        const bool on = srch || mode == kWalk;
+        const int64_t grp = S.p >> 1;
+        int blk = 0, sl = 0;
+        if (srch) {
+          blk = (S.band >> 5) * (kStrip / kBlk) + (S.band & 31) / 4;
+          sl = S.cand;
+          if (m == ((S.band & 31) & 3)) {
+            const uint32_t t = (uint32_t)(uint16_t)(int16_t)(4 * (S.best - g) - 1);
+            T4m1 = hf ? ((T4m1 & 0xffffu) | (t << 16)) : ((T4m1 & 0xffff0000u) | t);
+          }
+        } else if (mode == kWalk) {
+          const int ln = ((S.i - 1) % kStrip) / kRows;
+          blk = (S.i - 1) / kBlk;
+          sl = (S.j + ln - 1) / kSlab;
+          // the block after this one is above, above-left or left of it: pull their checkpoints into L2
+#pragma unroll
+          for (int q = 0; q < 3; ++q) {
+            const int nb = blk - (q < 2 ? 1 : 0), ns = sl - (q > 0 ? 1 : 0);
+            if (nb < 0 || ns < 1) continue;
+            const int r0 = nb * kBlk, st = r0 / kStrip, L0 = (r0 % kStrip) / kRows;
+            const int64_t base = (grp * SM + st) * NS + (ns - 1);
+            prefetch_l2(A.colck + base * kStrip + (L0 + m) * kRows);
+            if (m == 0) prefetch_l2(A.corner + base * 32 + L0);
+            if (r0 > 0) {
+              const int bnd = r0 / kBand - 1, j0 = max(1, ns * kSlab - L0 + 16 * m);
+              if (j0 <= S.lb)
+                prefetch_l2(A.rowck + ((grp * SM + bnd / kBandsPerStrip) * kBandsPerStrip + bnd % kBandsPerStrip) *
+                                          A.max_lb + (j0 - 1));
+            }
+          }
+        }
+        R0[hf] = blk * kBlk;
         const int st = R0[hf] / kStrip, L0 = (R0[hf] % kStrip) / kRows, l = L0 + m;
-        D[hf] = X.sl * kSlab - L0;
-        const bool ck = X.on && X.sl > 0;
-        const int64_t base = (grp * SM + st) * NS + (ck ? X.sl - 1 : 0);
+        D[hf] = sl * kSlab - L0;
+        const bool ck = on && sl > 0;
+        const int64_t base = (grp * SM + st) * NS + (ck ? sl - 1 : 0);
         const uint4* cp = reinterpret_cast<const uint4*>(A.colck + base * kStrip + l * kRows);
         const uint4 v0 = ck ? __ldcg(cp) : make_uint4(NEG_G2, NEG_G2, NEG_G2, NEG_G2);
         const uint4 v1 = ck ? __ldcg(cp + 1) : make_uint4(NEG_G2, NEG_G2, NEG_G2, NEG_G2);
         w[hf][0] = v0.x; w[hf][1] = v0.y; w[hf][2] = v0.z; w[hf][3] = v0.w;
         w[hf][4] = v1.x; w[hf][5] = v1.y; w[hf][6] = v1.z; w[hf][7] = v1.w;
         cw[hf] = ck ? __ldcg(A.corner + base * 32 + l) : NEG_G2;
+        const uint8_t* ap = S.a;
+        const uint8_t* bp = S.b;
+        const int la = S.la, lb = S.lb;
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
           const int i = R0[hf] + 8 * m + r + 1;
-          av[hf][r] = (X.on && i <= X.la) ? __ldg(X.a + i - 1) : (uint32_t)kDeadCode;
+          av[hf][r] = (on && i <= la) ? __ldg(ap + i - 1) : (uint32_t)kDeadCode;
         }
 #pragma unroll
         for (int k = 0; k < kBS / 4; ++k) {  // b residues of columns D-3 .. D+36 (x = j - D + 3)
           const int j = D[hf] + m + 4 * k - 3;
-          bv[hf][k] = (X.on && j >= 1 && j <= X.lb) ? __ldg(X.b + j - 1) : (uint32_t)kDeadCode;
+          bv[hf][k] = (on && j >= 1 && j <= lb) ? __ldg(bp + j - 1) : (uint32_t)kDeadCode;
         }
         // top row (G of row R0, columns D + c, c = 0..32): the band checkpoint above the block
         const int bnd = R0[hf] / kBand - 1;
@@ -521,14 +557,14 @@ __global__ void __launch_bounds__(32) k_sw16_tb3(Sw16Args A, int64_t first, int6
 #pragma unroll
         for (int k = 0; k < 9; ++k) {
           const int c = m + 4 * k, j = D[hf] + c;
-          tv[hf][k] = (X.on && bnd >= 0 && c <= kSlab && j >= 1 && j <= X.lb) ? __ldcg(rk + j) : NEG_G2;
+          tv[hf][k] = (on && bnd >= 0 && c <= kSlab && j >= 1 && j <= lb) ? __ldcg(rk + j) : NEG_G2;
         }
       }
 #pragma unroll
       for (int hf = 0; hf < 2; ++hf) {
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
-          sa[hf][r] = sig32 + 32 * av[hf][r];
+          sa[hf][r] = sig32 + 64 * av[hf][r];
           aS[hf * kBlk + 8 * m + r] = (uint8_t)av[hf][r];
         }
 #pragma unroll
@@ -536,181 +572,163 @@ __global__ void __launch_bounds__(32) k_sw16_tb3(Sw16Args A, int64_t first, int6
       }
 #pragma unroll
       for (int k = 0; k < 9; ++k)
-        if (m + 4 * k <= kSlab) Hs[(m + 4 * k + 1) * kCS + 3] = join(tv[0][k], tv[1][k]);
+        if (m + 4 * k <= kSlab) Ts[m + 4 * k] = key4(join(tv[0][k], tv[1][k]));
 #pragma unroll
-      for (int r = 0; r < kRows; ++r) Gs[r] = join(w[0][r], w[1][r]);
-      prev = join(cw[0], cw[1]);
-      uint4* col0 = reinterpret_cast<uint4*>(Hs + kCS + 8 * m + 4);
-      col0[0] = make_uint4(Gs[0], Gs[1], Gs[2], Gs[3]);
-      col0[1] = make_uint4(Gs[4], Gs[5], Gs[6], Gs[7]);
-      if (m > 0) Hs[8 * m + 3] = prev;  // corner: row 8m-1, column c = -1
+      for (int r = 0; r < kRows; ++r) Kc[r] = key4(join(w[0][r], w[1][r]));
+      prev = key4(join(cw[0], cw[1]));
     }
+    const bool anys = __any_sync(full, T4m1 != 0x7fff7fffu);
     __syncwarp();
     clk.lap(2);
+    // F) re-run the 32 forward steps of both blocks in keys; codes to shared memory
+    int hkey[2] = {1 << 30, 1 << 30};  // search: first hit r * 64 + c per half
     {
       const uint32_t bA = bs32 + (3 - m), bB = bs32 + kBS + (3 - m);
+      const uint32_t cw0 = cs32 + 4 * m;
 #pragma unroll 4
       for (int c = 1; c <= kSlab; ++c) {
-        const uint32_t topv = Hs[(c + 1) * kCS + 3];
-        const uint32_t fa = __shfl_up_sync(full, Gs[kRows - 1], 1, 4);
-        const uint32_t Gu = m == 0 ? topv : fa;
-        const uint32_t Gd = prev;
-        prev = Gu;
-        const uint32_t ca = lds_u8(bA + c), cb = lds_u8(bB + c);
+        const uint32_t topv = lds_u32(ts32 + 4 * c);
+        const uint32_t fa = __shfl_up_sync(full, Kc[kRows - 1], 1, 4);
+        const uint32_t Ku = m == 0 ? topv : fa;
+        const uint32_t Kd = prev;
+        prev = Ku;
+        const uint32_t ca = 2 * lds_u8(bA + c), cb = 2 * lds_u8(bB + c);
         uint32_t Xv[kRows];
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
-          const uint32_t sg = prmt((uint32_t)lds_s8(sa[0][r] + ca), (uint32_t)lds_s8(sa[1][r] + cb), 0x5410u);
-          Xv[r] = __viaddmax_s16x2(r == 0 ? Gd : Gs[r - 1], sg, __viaddmax_s16x2(Gs[r], NEG_G2, NEG_G2));
+          const uint32_t sg = prmt(lds_s16w(sa[0][r] + ca), lds_s16w(sa[1][r] + cb), 0x5410u);
+          Xv[r] = __viaddmax_s16x2(r == 0 ? Kd : Kc[r - 1], sg, __viaddmax_s16x2(Kc[r], NEG4, ZC));
         }
-        uint32_t gg = Gu;
+        uint32_t kk = Ku, code = 0;
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
-          gg = __viaddmax_s16x2(gg, NEG_G2, Xv[r]);
-          Gs[r] = gg;
+          const uint32_t K = __viaddmax_s16x2(kk, NEG4U, Xv[r]);
+          kk = K & kClean;
+          Kc[r] = kk;
+          code = code * 4u + (K & kCodeBits);
         }
-        uint4* col = reinterpret_cast<uint4*>(Hs + (c + 1) * kCS + 8 * m + 4);
-        col[0] = make_uint4(Gs[0], Gs[1], Gs[2], Gs[3]);
-        col[1] = make_uint4(Gs[4], Gs[5], Gs[6], Gs[7]);
+        sts_u32(cw0 + 16 * (c - 1), code);
+        if (anys) {
+          uint32_t mx = __vimax3_s16x2(Kc[0], Kc[1], Kc[2]);
+          mx = __vimax3_s16x2(mx, Kc[3], Kc[4]);
+          mx = __vimax3_s16x2(mx, Kc[5], Kc[6]);
+          mx = __vmaxs2(mx, Kc[7]);
+          if (__vmaxs2(mx, T4m1) != T4m1) {  // rare: a cell of this lane reaches the score
+#pragma unroll
+            for (int hf = 0; hf < 2; ++hf) {
+              const int th = half16(T4m1, hf), la = St[hf].la, lb = St[hf].lb;
+#pragma unroll
+              for (int r = 0; r < kRows; ++r) {
+                const int i = R0[hf] + 8 * m + r + 1, j = D[hf] + c - m;
+                if (half16(Kc[r], hf) > th && i <= la && j >= 1 && j <= lb) hkey[hf] = min(hkey[hf], r * 64 + c);
+              }
+            }
+          }
+        }
       }
     }
     __syncwarp();
     clk.lap(3);
-    // 5) searching halves: first row-major cell of the lane band holding the score
+    // G) searching halves: first row-major cell of the lane band holding the score
 #pragma unroll
     for (int hf = 0; hf < 2; ++hf) {
-      TbHalf& X = H[hf];
-      const bool srch = X.mode == 1 && X.on;
-      const int m8 = (X.band & 31) & 3;
-      int key = 1 << 30;  // r * 64 + c
-      if (srch) {
-        const int target = X.best - g;
-        for (int c = m + 1; c <= kSlab; c += 4) {
-          const uint4* col = reinterpret_cast<const uint4*>(Hs + (c + 1) * kCS + 8 * m8 + 4);
-          const uint4 v0 = col[0], v1 = col[1];
-          const uint32_t vv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
-#pragma unroll
-          for (int r = kRows - 1; r >= 0; --r) {
-            const int i = R0[hf] + 8 * m8 + r + 1, j = D[hf] + c - m8;
-            if (half16(vv[r], hf) == target && i <= X.la && j >= 1 && j <= X.lb) key = min(key, r * 64 + c);
-          }
-        }
-      }
+      int key = hkey[hf];
       key = min(key, __shfl_xor_sync(full, key, 1));
       key = min(key, __shfl_xor_sync(full, key, 2));
-      if (srch) {
+      TbState& S = St[hf];
+      if (m == 0 && S.mode == kSearch && S.cand >= 0) {
         if (key < (1 << 30)) {
-          const int r = key >> 6, c = key & 63;
+          const int m8 = (S.band & 31) & 3, r = key >> 6, c = key & 63;
           const long long k2 = ((long long)(R0[hf] + 8 * m8 + r + 1) << 32) | (long long)(D[hf] + c - m8);
-          if (X.found < 0 || k2 < X.found) X.found = k2;
+          if (S.found < 0 || k2 < S.found) S.found = k2;
         }
-        X.scur = X.cand + 1;
-        X.cand = -1;
+        S.scur = S.cand + 1;
+        S.cand = -1;
       }
     }
     clk.lap(4);
-    // 6) walking halves: lane m == half walks its problem through the block
+    // H) walking halves: lane m == half walks its problem through the block's codes
     if (m < 2) {
       const int hf = m;
-      int mode = hf ? H[1].mode : H[0].mode;
-      if (mode == 2) {
-        int i = hf ? H[1].i : H[0].i, j = hf ? H[1].j : H[0].j, h = hf ? H[1].h : H[0].h, n = hf ? H[1].n : H[0].n;
-        const int r0 = hf ? R0[1] : R0[0], d0 = hf ? D[1] : D[0];
-        const int64_t p = hf ? H[1].p : H[0].p;
-        uint8_t* o = out + (p - first) * stride;
-        const uint8_t* as = aS + hf * kBlk - r0 - 1;   // as[i] = a[i - 1] for rows of the block
-        const uint8_t* bs = bS + hf * kBS - d0 + 3;    // bs[j] = b[j - 1] for columns D-3 .. D+36
-        uint8_t* ops = opsS + hf * kOpsCap;
-        const int sh16 = 16 * hf;
+      TbState& S = St[hf];
+      if (S.mode == kWalk) {
+        int i = S.i, j = S.j;
+        const int r0 = R0[hf], d0 = D[hf];
+        uint8_t* const o0 = out + (S.p - first) * stride;
+        uint8_t* o = o0 + S.n;                            // ops end -> start (stride >= la + lb: no overflow)
+        const uint32_t as32 = aS32 + hf * kBlk - r0 - 1;  // a[i - 1] of the block's rows at as32 + i
+        const uint32_t bsx = bs32 + hf * kBS - d0 + 3;    // b[j - 1] of columns D-3 .. D+36 at bsx + j
+        const uint32_t cw = cs32 - 16;                    // code word (c, lane mm) at cw + 16 c + 4 mm
+        const int sh = 16 * hf + 14;
         int t = i - r0 - 1;
         int c = j - d0 + (t >> 3);
-        while (h > 0 && t >= 0 && c >= 1) {
-          const int cu = c - ((t > 0 && (t & 7) == 0) ? 1 : 0);  // row above: one column left at a lane start
-          const uint32_t* up_col = Hs + (cu + 1) * kCS + t + 3;     // (t-1, cu)
-          const int uV = (int)(int16_t)(up_col[0] >> sh16) + g;
-          const int dV = (int)(int16_t)(up_col[-kCS] >> sh16) + g;
-          const int lV = (int)(int16_t)(Hs[c * kCS + t + 4] >> sh16) + g;
-          const int ra = as[i], rb = bs[j];
-          const int sub = sig_s[ra * 32 + rb];
-          const bool isD = h == dV + sub;
-          const bool isU = !isD && h == uV - g;
+        bool stop = false;
+        while (t >= 0 && c >= 1) {
+          const uint32_t wd = lds_u32(cw + 16 * c + 4 * (t >> 3));
+          const uint32_t ra = lds_u8(as32 + i), rb = lds_u8(bsx + j);
+          const int code = (int)(wd >> (sh - 2 * (t & 7))) & 3;
+          if (code == 3) { stop = true; break; }      // H = 0: the alignment starts here
+          const bool isD = code == 2, isU = code == 1;
+          *o++ = isD ? (ra == rb ? 'M' : 'X') : (isU ? 'D' : 'I');
+          const int cu = c - ((t & 7) == 0 && t > 0 ? 1 : 0);  // row above: one column left at a lane start
           const bool mvI = isD || isU;
-          const uint8_t op = isD ? (ra == rb ? 'M' : 'X') : (isU ? 'D' : 'I');
-          h = isD ? dV : (isU ? uV : lV);
           i -= mvI ? 1 : 0;
           j -= isU ? 0 : 1;
           c = isD ? cu - 1 : (isU ? cu : c - 1);
           t -= mvI ? 1 : 0;
-          if (n < kOpsCap) ops[n] = op;
-          else if (n < stride) o[stride - 1 - n] = op;  // long paths: the row's tail, moved at the end
-          ++n;
+          if (i == 0 || j == 0) { stop = true; break; }  // table boundary: H = 0
         }
-        if (hf) { H[1].i = i; H[1].j = j; H[1].h = h; H[1].n = n; if (h <= 0) H[1].mode = 0; }
-        else { H[0].i = i; H[0].j = j; H[0].h = h; H[0].n = n; if (h <= 0) H[0].mode = 0; }
+        S.i = i; S.j = j; S.n = (int)(o - o0);
+        if (stop) S.mode = kFinish;
       }
-    }
-    // the walkers' state to their groups
-#pragma unroll
-    for (int hf = 0; hf < 2; ++hf) {
-      const int src = (lane & ~3) | hf;
-      TbHalf& X = H[hf];
-      X.i = __shfl_sync(full, X.i, src);
-      X.j = __shfl_sync(full, X.j, src);
-      X.h = __shfl_sync(full, X.h, src);
-      X.n = __shfl_sync(full, X.n, src);
-      X.mode = __shfl_sync(full, X.mode, src);
     }
     __syncwarp();
     clk.lap(5);
-  }
-  // 7) outputs, start -> end: op q (walk order) goes to position n-1-q. Ops q < cap are in
-  // shared memory; longer paths left ops q >= cap at the row's tail (position stride-1-q),
-  // which is shifted left first (ordered 4-byte chunks: every read precedes the overlapping writes).
-  __syncwarp();
+    // I) finished halves: lengths and coordinates (k_sw16_rev reverses the ops afterwards)
 #pragma unroll
-  for (int hf = 0; hf < 2; ++hf) {
-    const TbHalf& X = H[hf];
-    const bool mine = X.p >= first && X.p < first + count;
-    const int64_t q = X.p - first;
-    const bool active = X.best > 0 && X.la > 0 && X.lb > 0;
-    const int n = active ? X.n : 0;
-    const bool overflow = n > stride;
-    uint8_t* o = out + (mine ? q : 0) * stride;
-    if (mine && !overflow && n > kOpsCap) {
-      const int64_t s0 = stride - n;
-      for (int64_t u0 = 0; u0 < n - kOpsCap; u0 += 4) {
-        const int64_t u = u0 + m;
-        const uint8_t v = u < n - kOpsCap ? o[s0 + u] : 0;
-        __syncwarp(0xfu << (lane & ~3));
-        if (u < n - kOpsCap) o[u] = v;
-        __syncwarp(0xfu << (lane & ~3));
+    for (int hf = 0; hf < 2; ++hf) {
+      TbState& S = St[hf];
+      if (m == 0 && S.mode == kFinish) {
+        const int64_t q = S.p - first;
+        out_len[q] = S.n;
+        if (coords) {
+          coords[4 * q] = S.i; coords[4 * q + 1] = S.j;
+          coords[4 * q + 2] = S.ei; coords[4 * q + 3] = S.ej;
+        }
+        S.mode = kIdle;
       }
     }
-    if (mine && !overflow) {
-      const uint8_t* ops = opsS + hf * kOpsCap;
-      for (int u = max(0, n - kOpsCap) + m; u < n; u += 4) o[u] = ops[n - 1 - u];
-    }
-    if (mine && m == 0) {
-      out_len[q] = overflow ? -1 : (int32_t)n;
-      if (coords) {
-        coords[4 * q] = active ? X.i : 0; coords[4 * q + 1] = active ? X.j : 0;
-        coords[4 * q + 2] = active ? X.ei : 0; coords[4 * q + 3] = active ? X.ej : 0;
-      }
-    }
+    __syncwarp();
+    clk.lap(6);
   }
-  clk.lap(6);
-  clk.flush(lane);
 }
 
-size_t tb3_smem_bytes() { return 1024 + 8 * kGS * 4 + 8 * 2 * kBS + 8 * 2 * kBlk + 8 * 2 * kOpsCap; }
+// The walk writes each alignment end -> start; one warp per row puts it in order.
+__global__ void __launch_bounds__(256) k_sw16_rev(int64_t count, uint8_t* out, int64_t stride, const int32_t* out_len) {
+  const int64_t q = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (q >= count) return;
+  const int n = out_len[q];
+  uint8_t* o = out + q * stride;
+  for (int u0 = 0; u0 < n / 2; u0 += 32) {
+    const int u = u0 + lane;
+    uint8_t x = 0, y = 0;
+    if (u < n / 2) { x = o[u]; y = o[n - 1 - u]; }
+    __syncwarp();
+    if (u < n / 2) { o[u] = y; o[n - 1 - u] = x; }
+  }
+}
+
+size_t tb5_smem_bytes() { return 2048 + (size_t)kTbWarps * kTbWarpBytes; }
 
 }  // namespace
 
-bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap) {
+bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap, bool want_tb) {
   int smax = 0, smin = 0;
   for (int q = 0; q < asz * asz; ++q) { smax = max(smax, (int)sigma_host[q]); smin = min(smin, (int)sigma_host[q]); }
   const int64_t bound = (int64_t)smax * (max_la < max_lb ? max_la : max_lb) + gap;
-  return asz < 32 && bound < 32000 && smax <= 127 && smin >= -99 && gap >= 1 && gap < 1000 && (asz + 1) * kStrip <= 65535;
+  // the traceback re-run works on keys 4 G + code (s16): 4 x the bound must fit too
+  return asz < 32 && bound < (want_tb ? 7900 : 32000) && smax <= 127 && smin >= -99 && gap >= 1 && gap < 1000 && (asz + 1) * kStrip <= 65535;
 }
 
 int sw16_smem_per_warp(int asz, int64_t max_la, int64_t max_lb) {
@@ -748,14 +766,29 @@ cudaError_t sw16_solve(const Sw16Args& A, bool tb, cudaStream_t s, int64_t* laun
 cudaError_t sw16_traceback(const Sw16Args& A, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                            int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches) {
   if (count == 0) return cudaSuccess;
+  const size_t smem = tb5_smem_bytes();
+  cudaError_t e = cudaFuncSetAttribute(k_sw16_tb5, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(k_sw16_tb5, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  if (e != cudaSuccess) return e;
+  // persistent grid: as many CTAs as fit, fewer if the queues are short
+  static int per_sm = 0, sms = 0;
+  if (per_sm == 0) {
+    int dev = 0;
+    if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+    if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sw16_tb5, kTbWarps * 32, smem)) != cudaSuccess)
+      return e;
+    if (per_sm < 1) per_sm = 1;
+  }
+  const int64_t per_queue = (count + 1) / 2, per_cta = 8 * kTbWarps;
+  const int64_t ctas = std::min<int64_t>((per_queue + per_cta - 1) / per_cta, (int64_t)per_sm * sms);
+  if ((e = cudaMemsetAsync(A.tb_ctr, 0, 2 * sizeof(unsigned long long), s)) != cudaSuccess) return e;
   ++*launches;
-  const size_t smem = tb3_smem_bytes();
-  cudaError_t e = cudaFuncSetAttribute(k_sw16_tb3, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  e = cudaFuncSetAttribute(k_sw16_tb3, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-  if (e != cudaSuccess) return e;
-  const int64_t groups = ((first + count - 1) >> 1) - (first >> 1) + 1;
-  k_sw16_tb3<<<(unsigned)((groups + 7) / 8), 32, smem, s>>>(A, first, count, out, stride, out_len, coords);
+  k_sw16_tb5<<<(unsigned)ctas, kTbWarps * 32, smem, s>>>(A, first, count, out, stride, out_len, coords);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  ++*launches;
+  k_sw16_rev<<<(unsigned)((count + 7) / 8), 256, 0, s>>>(count, out, stride, out_len);
   return cudaGetLastError();
 }
 
