@@ -497,9 +497,12 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         const bool srch = mode == kSearch && S.cand >= 0;
         const bool on = srch || mode == kWalk;
         const int64_t grp = S.p >> 1;
-        int blk = 0, sl = 0;
+        // block rows R0+1 .. R0+32 = forward lanes L0..L0+3 of one strip, L0 even (the top row is
+        // a band checkpoint). A walker's block puts it in lane L0+2 or L0+3, so it runs through
+        // at least 16 rows before leaving upwards.
+        int r0 = 0, sl = 0;
         if (srch) {
-          blk = (S.band >> 5) * (kStrip / kBlk) + (S.band & 31) / 4;
+          r0 = (S.band >> 5) * kStrip + kBlk * ((S.band & 31) / 4);
           sl = S.cand;
           if (m == ((S.band & 31) & 3)) {
             const uint32_t t = (uint32_t)(uint16_t)(int16_t)(4 * (S.best - g) - 1);
@@ -507,27 +510,27 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
           }
         } else if (mode == kWalk) {
           const int ln = ((S.i - 1) % kStrip) / kRows;
-          blk = (S.i - 1) / kBlk;
+          r0 = (S.i - 1) / kStrip * kStrip + kRows * (ln < 2 ? 0 : ((ln - 2) & ~1));
           sl = (S.j + ln - 1) / kSlab;
-          // the block after this one is above, above-left or left of it: pull their checkpoints into L2
+          // the next block is left (same rows or 16 up) or 32 rows up: pull their checkpoints into L2
 #pragma unroll
           for (int q = 0; q < 3; ++q) {
-            const int nb = blk - (q < 2 ? 1 : 0), ns = sl - (q > 0 ? 1 : 0);
-            if (nb < 0 || ns < 1) continue;
-            const int r0 = nb * kBlk, st = r0 / kStrip, L0 = (r0 % kStrip) / kRows;
+            const int nr = r0 - (q == 0 ? 0 : (q == 1 ? 16 : 32)), ns = sl - (q < 2 ? 1 : 0);
+            if (nr < 0 || ns < 1) continue;
+            const int st = nr / kStrip, L0 = (nr % kStrip) / kRows;
             const int64_t base = (grp * SM + st) * NS + (ns - 1);
             prefetch_l2(A.colck + base * kStrip + (L0 + m) * kRows);
             if (m == 0) prefetch_l2(A.corner + base * 32 + L0);
-            if (r0 > 0) {
-              const int bnd = r0 / kBand - 1, j0 = max(1, ns * kSlab - L0 + 16 * m);
+            if (nr > 0) {
+              const int bnd = nr / kBand - 1, j0 = max(1, ns * kSlab - L0 + 16 * m);
               if (j0 <= S.lb)
                 prefetch_l2(A.rowck + ((grp * SM + bnd / kBandsPerStrip) * kBandsPerStrip + bnd % kBandsPerStrip) *
                                           A.max_lb + (j0 - 1));
             }
           }
         }
-        R0[hf] = blk * kBlk;
-        const int st = R0[hf] / kStrip, L0 = (R0[hf] % kStrip) / kRows, l = L0 + m;
+        R0[hf] = r0;
+        const int st = r0 / kStrip, L0 = (r0 % kStrip) / kRows, l = L0 + m;
         D[hf] = sl * kSlab - L0;
         const bool ck = on && sl > 0;
         const int64_t base = (grp * SM + st) * NS + (ck ? sl - 1 : 0);
