@@ -39,7 +39,6 @@ constexpr int kStrip = 32 * kRows;    // rows per strip
 constexpr int kBand = 16;             // checkpoint band height (two lanes)
 constexpr int kLanesPerBand = kBand / kRows;
 constexpr int kBandsPerStrip = kStrip / kBand;
-constexpr int kBlk = 32;              // traceback recompute block height (two independent bands)
 constexpr int kSlab = 32;             // checkpoint column spacing
 constexpr int kDead = -100;           // profile value for rows/columns outside a problem
 constexpr int kPad = 32;              // dead columns on each side of the residue array
@@ -309,10 +308,16 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
 // per-lane strip maxima, then the slabs of that lane whose maximum equals the
 // score, then a compare inside the re-run (taken only on a hit).
 constexpr int kTbWarps = 4;              // warps per CTA
+#ifndef TB_GL
+#define TB_GL 4                          // lanes per group = forward lanes per traceback block (2 measured slower)
+#endif
+constexpr int kGL = TB_GL;               // 2: blocks of 16 rows (one checkpoint band), 4: 32 rows
+constexpr int kGroups = 32 / kGL;        // groups per warp
+constexpr int kBlk = kRows * kGL;        // traceback block height
 #ifndef TB5_MINB
 #define TB5_MINB 5                       // CTAs per SM (register cap)
 #endif
-constexpr int kCW = 4 * kSlab;           // code words per group: [c - 1][m]
+constexpr int kCW = kGL * kSlab;         // code words per group: [c - 1][m]
 constexpr int kTS = 36;                  // top-row keys per group, c = 0..32
 constexpr int kBS = 40;                  // staged b residues per half (columns D-3 .. D+36)
 constexpr int kDeadCode = 31;            // residue code whose sigma row/column is kDead4 (alphabets < 32)
@@ -332,7 +337,7 @@ struct TbState {      // one problem in one half of a group (shared memory; writ
   int ei, ej;         // end cell
 };
 constexpr int kGroupBytes = 4 * kCW + 4 * kTS + 2 * kBS + 2 * kBlk + 2 * (int)sizeof(TbState);
-constexpr int kTbWarpBytes = 8 * kGroupBytes;
+constexpr int kTbWarpBytes = kGroups * kGroupBytes;
 
 __device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
   uint32_t v;
@@ -366,19 +371,19 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
     const int x = q >> 5, y = q & 31;
     sig_s[q] = (x < A.asz && y < A.asz) ? (int16_t)(4 * A.sigma[x * A.asz + y] + 2) : (int16_t)kDead4;
   }
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, gq = lane >> 2, m = lane & 3;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, gq = lane / kGL, m = lane % kGL;
   uint8_t* wb = tsm + 2048 + warp * kTbWarpBytes;
   uint32_t* Cs = reinterpret_cast<uint32_t*>(wb) + gq * kCW;
-  uint32_t* Ts = reinterpret_cast<uint32_t*>(wb + 8 * 4 * kCW) + gq * kTS;
-  uint8_t* bS = wb + 8 * 4 * (kCW + kTS) + gq * 2 * kBS;                  // [2][kBS] staged b residues
-  uint8_t* aS = wb + 8 * 4 * (kCW + kTS) + 8 * 2 * kBS + gq * 2 * kBlk;  // [2][32] staged a residues
-  TbState* St = reinterpret_cast<TbState*>(wb + 8 * (4 * (kCW + kTS) + 2 * kBS + 2 * kBlk)) + 2 * gq;
+  uint32_t* Ts = reinterpret_cast<uint32_t*>(wb + kGroups * 4 * kCW) + gq * kTS;
+  uint8_t* bS = wb + kGroups * 4 * (kCW + kTS) + gq * 2 * kBS;                  // [2][kBS] staged b residues
+  uint8_t* aS = wb + kGroups * (4 * (kCW + kTS) + 2 * kBS) + gq * 2 * kBlk;  // [2][kBlk] staged a residues
+  TbState* St = reinterpret_cast<TbState*>(wb + kGroups * (4 * (kCW + kTS) + 2 * kBS + 2 * kBlk)) + 2 * gq;
   const uint32_t sig32 = (uint32_t)__cvta_generic_to_shared(sig_s);
   const uint32_t cs32 = (uint32_t)__cvta_generic_to_shared(Cs);
   const uint32_t ts32 = (uint32_t)__cvta_generic_to_shared(Ts);
   const uint32_t bs32 = (uint32_t)__cvta_generic_to_shared(bS);
   const uint32_t aS32 = (uint32_t)__cvta_generic_to_shared(aS);
-  const unsigned full = 0xffffffffu, gmask = 0xfu << (lane & ~3);
+  const unsigned full = 0xffffffffu, gmask = ((1u << kGL) - 1) << (lane & ~(kGL - 1));
   const int g = A.gap;
   const uint32_t NEG_G2 = pack2(-g), NEG4 = pack2(-4 * g), NEG4U = pack2(-4 * g + 1), ZC = pack2(-4 * g + 3);
   const int64_t SM = A.strips_max, NS = A.nslab_max;
@@ -398,7 +403,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
       if (St[hf].mode != kIdle) continue;
       int64_t q = 0;
       if (m == 0) q = atomicAdd(reinterpret_cast<unsigned long long*>(A.tb_ctr) + hf, 1ull);
-      q = __shfl_sync(gmask, q, lane & ~3);
+      q = __shfl_sync(gmask, q, lane & ~(kGL - 1));
       if (m == 0) {
         TbState& S = St[hf];
         if (q >= kn[hf]) {
@@ -426,10 +431,11 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         for (int st = 0; st * kStrip < la && band < 0; ++st) {
           int firstl = 32;
 #pragma unroll
-          for (int q8 = 7; q8 >= 0; --q8)
-            if (half16(__ldcg(A.lanebest + (grp * SM + st) * 32 + 8 * m + q8), hf) + g == best) firstl = 8 * m + q8;
-          firstl = min(firstl, __shfl_xor_sync(gmask, firstl, 1));
-          firstl = min(firstl, __shfl_xor_sync(gmask, firstl, 2));
+          for (int q8 = 32 / kGL - 1; q8 >= 0; --q8)
+            if (half16(__ldcg(A.lanebest + (grp * SM + st) * 32 + (32 / kGL) * m + q8), hf) + g == best)
+              firstl = (32 / kGL) * m + q8;
+#pragma unroll
+          for (int o = 1; o < kGL; o <<= 1) firstl = min(firstl, __shfl_xor_sync(gmask, firstl, o));
           if (firstl < 32) band = st * 32 + firstl;
         }
         __syncwarp(gmask);
@@ -452,12 +458,12 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         const uint32_t* sb = A.slabbest + ((grp * SM + (S.band >> 5)) * NS) * 32 + (S.band & 31);
         uint32_t bits = 0;
 #pragma unroll
-        for (int q = 0; q < 8; ++q) {
-          const int s = scur + m + 4 * q;
-          if (s < nsl && half16(__ldcg(sb + (int64_t)s * 32), hf) + g == best) bits |= 1u << (m + 4 * q);
+        for (int q = 0; q < 32 / kGL; ++q) {
+          const int s = scur + m + kGL * q;
+          if (s < nsl && half16(__ldcg(sb + (int64_t)s * 32), hf) + g == best) bits |= 1u << (m + kGL * q);
         }
-        bits |= __shfl_xor_sync(gmask, bits, 1);
-        bits |= __shfl_xor_sync(gmask, bits, 2);
+#pragma unroll
+        for (int o = 1; o < kGL; o <<= 1) bits |= __shfl_xor_sync(gmask, bits, o);
         __syncwarp(gmask);
         if (m == 0) {
           TbState& W = St[hf];
@@ -489,7 +495,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
     uint32_t Kc[kRows], prev;
     uint32_t T4m1 = 0x7fff7fffu;  // search target 4 (best - g) - 1 in lane m8's half, else never exceeded
     {
-      uint32_t w[2][kRows], cw[2], av[2][kRows], bv[2][kBS / 4], tv[2][9];
+      uint32_t w[2][kRows], cw[2];
 #pragma unroll
       for (int hf = 0; hf < 2; ++hf) {
         const TbState& S = St[hf];
@@ -502,15 +508,15 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         // at least 16 rows before leaving upwards.
         int r0 = 0, sl = 0;
         if (srch) {
-          r0 = (S.band >> 5) * kStrip + kBlk * ((S.band & 31) / 4);
+          r0 = (S.band >> 5) * kStrip + kBlk * ((S.band & 31) / kGL);
           sl = S.cand;
-          if (m == ((S.band & 31) & 3)) {
+          if (m == (S.band & 31) % kGL) {
             const uint32_t t = (uint32_t)(uint16_t)(int16_t)(4 * (S.best - g) - 1);
             T4m1 = hf ? ((T4m1 & 0xffffu) | (t << 16)) : ((T4m1 & 0xffff0000u) | t);
           }
         } else if (mode == kWalk) {
           const int ln = ((S.i - 1) % kStrip) / kRows;
-          r0 = (S.i - 1) / kStrip * kStrip + kRows * (ln < 2 ? 0 : ((ln - 2) & ~1));
+          r0 = (S.i - 1) / kStrip * kStrip + kRows * (kGL == 2 ? (ln & ~1) : (ln < 2 ? 0 : ((ln - 2) & ~1)));
           sl = (S.j + ln - 1) / kSlab;
           // the next block is left (same rows or 16 up) or 32 rows up: pull their checkpoints into L2
 #pragma unroll
@@ -522,7 +528,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
             prefetch_l2(A.colck + base * kStrip + (L0 + m) * kRows);
             if (m == 0) prefetch_l2(A.corner + base * 32 + L0);
             if (nr > 0) {
-              const int bnd = nr / kBand - 1, j0 = max(1, ns * kSlab - L0 + 16 * m);
+              const int bnd = nr / kBand - 1, j0 = max(1, ns * kSlab - L0 + (32 / kGL) * m);
               if (j0 <= S.lb)
                 prefetch_l2(A.rowck + ((grp * SM + bnd / kBandsPerStrip) * kBandsPerStrip + bnd % kBandsPerStrip) *
                                           A.max_lb + (j0 - 1));
@@ -543,39 +549,39 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         const uint8_t* ap = S.a;
         const uint8_t* bp = S.b;
         const int la = S.la, lb = S.lb;
+        uint32_t av[kRows], bv[kBS / kGL], tv[(kSlab + kGL) / kGL];
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
-          const int i = R0[hf] + 8 * m + r + 1;
-          av[hf][r] = (on && i <= la) ? __ldg(ap + i - 1) : (uint32_t)kDeadCode;
+          const int i = R0[hf] + kRows * m + r + 1;
+          av[r] = (on && i <= la) ? __ldg(ap + i - 1) : (uint32_t)kDeadCode;
         }
 #pragma unroll
-        for (int k = 0; k < kBS / 4; ++k) {  // b residues of columns D-3 .. D+36 (x = j - D + 3)
-          const int j = D[hf] + m + 4 * k - 3;
-          bv[hf][k] = (on && j >= 1 && j <= lb) ? __ldg(bp + j - 1) : (uint32_t)kDeadCode;
+        for (int k = 0; k < kBS / kGL; ++k) {  // b residues of columns D-3 .. D+36 (x = j - D + 3)
+          const int j = D[hf] + m + kGL * k - 3;
+          bv[k] = (on && j >= 1 && j <= lb) ? __ldg(bp + j - 1) : (uint32_t)kDeadCode;
         }
         // top row (G of row R0, columns D + c, c = 0..32): the band checkpoint above the block
         const int bnd = R0[hf] / kBand - 1;
         const uint32_t* rk = A.rowck + ((grp * SM + (bnd >= 0 ? bnd / kBandsPerStrip : 0)) * kBandsPerStrip +
                                         (bnd >= 0 ? bnd % kBandsPerStrip : 0)) * A.max_lb - 1;
 #pragma unroll
-        for (int k = 0; k < 9; ++k) {
-          const int c = m + 4 * k, j = D[hf] + c;
-          tv[hf][k] = (on && bnd >= 0 && c <= kSlab && j >= 1 && j <= lb) ? __ldcg(rk + j) : NEG_G2;
+        for (int k = 0; k < (kSlab + kGL) / kGL; ++k) {
+          const int c = m + kGL * k, j = D[hf] + c;
+          tv[k] = (on && bnd >= 0 && c <= kSlab && j >= 1 && j <= lb) ? __ldcg(rk + j) : NEG_G2;
         }
-      }
-#pragma unroll
-      for (int hf = 0; hf < 2; ++hf) {
+        // this half's residues and top-row keys to shared memory
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
-          sa[hf][r] = sig32 + 64 * av[hf][r];
-          aS[hf * kBlk + 8 * m + r] = (uint8_t)av[hf][r];
+          sa[hf][r] = sig32 + 64 * av[r];
+          aS[hf * kBlk + kRows * m + r] = (uint8_t)av[r];
         }
 #pragma unroll
-        for (int k = 0; k < kBS / 4; ++k) bS[hf * kBS + m + 4 * k] = (uint8_t)bv[hf][k];
-      }
+        for (int k = 0; k < kBS / kGL; ++k) bS[hf * kBS + m + kGL * k] = (uint8_t)bv[k];
+        int16_t* ts16 = reinterpret_cast<int16_t*>(Ts) + hf;
 #pragma unroll
-      for (int k = 0; k < 9; ++k)
-        if (m + 4 * k <= kSlab) Ts[m + 4 * k] = key4(join(tv[0][k], tv[1][k]));
+        for (int k = 0; k < (kSlab + kGL) / kGL; ++k)
+          if (m + kGL * k <= kSlab) ts16[2 * (m + kGL * k)] = (int16_t)(4 * half16(tv[k], hf));
+      }
 #pragma unroll
       for (int r = 0; r < kRows; ++r) Kc[r] = key4(join(w[0][r], w[1][r]));
       prev = key4(join(cw[0], cw[1]));
@@ -591,7 +597,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
 #pragma unroll 4
       for (int c = 1; c <= kSlab; ++c) {
         const uint32_t topv = lds_u32(ts32 + 4 * c);
-        const uint32_t fa = __shfl_up_sync(full, Kc[kRows - 1], 1, 4);
+        const uint32_t fa = __shfl_up_sync(full, Kc[kRows - 1], 1, kGL);
         const uint32_t Ku = m == 0 ? topv : fa;
         const uint32_t Kd = prev;
         prev = Ku;
@@ -610,7 +616,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
           Kc[r] = kk;
           code = code * 4u + (K & kCodeBits);
         }
-        sts_u32(cw0 + 16 * (c - 1), code);
+        sts_u32(cw0 + 4 * kGL * (c - 1), code);
         if (anys) {
           uint32_t mx = __vimax3_s16x2(Kc[0], Kc[1], Kc[2]);
           mx = __vimax3_s16x2(mx, Kc[3], Kc[4]);
@@ -622,7 +628,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
               const int th = half16(T4m1, hf), la = St[hf].la, lb = St[hf].lb;
 #pragma unroll
               for (int r = 0; r < kRows; ++r) {
-                const int i = R0[hf] + 8 * m + r + 1, j = D[hf] + c - m;
+                const int i = R0[hf] + kRows * m + r + 1, j = D[hf] + c - m;
                 if (half16(Kc[r], hf) > th && i <= la && j >= 1 && j <= lb) hkey[hf] = min(hkey[hf], r * 64 + c);
               }
             }
@@ -636,13 +642,13 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
 #pragma unroll
     for (int hf = 0; hf < 2; ++hf) {
       int key = hkey[hf];
-      key = min(key, __shfl_xor_sync(full, key, 1));
-      key = min(key, __shfl_xor_sync(full, key, 2));
+#pragma unroll
+      for (int o = 1; o < kGL; o <<= 1) key = min(key, __shfl_xor_sync(full, key, o));
       TbState& S = St[hf];
       if (m == 0 && S.mode == kSearch && S.cand >= 0) {
         if (key < (1 << 30)) {
-          const int m8 = (S.band & 31) & 3, r = key >> 6, c = key & 63;
-          const long long k2 = ((long long)(R0[hf] + 8 * m8 + r + 1) << 32) | (long long)(D[hf] + c - m8);
+          const int m8 = (S.band & 31) % kGL, r = key >> 6, c = key & 63;
+          const long long k2 = ((long long)(R0[hf] + kRows * m8 + r + 1) << 32) | (long long)(D[hf] + c - m8);
           if (S.found < 0 || k2 < S.found) S.found = k2;
         }
         S.scur = S.cand + 1;
@@ -661,13 +667,13 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         uint8_t* o = o0 + S.n;                            // ops end -> start (stride >= la + lb: no overflow)
         const uint32_t as32 = aS32 + hf * kBlk - r0 - 1;  // a[i - 1] of the block's rows at as32 + i
         const uint32_t bsx = bs32 + hf * kBS - d0 + 3;    // b[j - 1] of columns D-3 .. D+36 at bsx + j
-        const uint32_t cw = cs32 - 16;                    // code word (c, lane mm) at cw + 16 c + 4 mm
+        const uint32_t cw = cs32 - 4 * kGL;               // code word (c, lane mm) at cw + 4 kGL c + 4 mm
         const int sh = 16 * hf + 14;
         int t = i - r0 - 1;
         int c = j - d0 + (t >> 3);
         bool stop = false;
         while (t >= 0 && c >= 1) {
-          const uint32_t wd = lds_u32(cw + 16 * c + 4 * (t >> 3));
+          const uint32_t wd = lds_u32(cw + 4 * kGL * c + 4 * (t >> 3));
           const uint32_t ra = lds_u8(as32 + i), rb = lds_u8(bsx + j);
           const int code = (int)(wd >> (sh - 2 * (t & 7))) & 3;
           if (code == 3) { stop = true; break; }      // H = 0: the alignment starts here
@@ -784,7 +790,7 @@ cudaError_t sw16_traceback(const Sw16Args& A, int64_t first, int64_t count, uint
       return e;
     if (per_sm < 1) per_sm = 1;
   }
-  const int64_t per_queue = (count + 1) / 2, per_cta = 8 * kTbWarps;
+  const int64_t per_queue = (count + 1) / 2, per_cta = kGroups * kTbWarps;
   const int64_t ctas = std::min<int64_t>((per_queue + per_cta - 1) / per_cta, (int64_t)per_sm * sms);
   if ((e = cudaMemsetAsync(A.tb_ctr, 0, 2 * sizeof(unsigned long long), s)) != cudaSuccess) return e;
   ++*launches;
