@@ -214,24 +214,45 @@ def run_ours(args, rank, world, local_rank):
                      "nuss": "dp_traceback (copy)", "hmm": "k_viterbi_tb (traceback)"}[W["kind"]]])
     ev_phase = [[] for _ in phase_names]
 
-    def ev():
+    # HMM: the forward (tensor cores, latency-bound on ~n/128 SMs) and Viterbi (ALU) are
+    # independent passes over the same sequences; the forward runs on a side stream so the
+    # Viterbi kernel fills the SMs the forward leaves idle.
+    side = torch.cuda.Stream(device=dev) if W["kind"] == "hmm" else None
+
+    def ev(st=None):
         e = torch.cuda.Event(enable_timing=True)
-        e.record(stream)
+        e.record(st or stream)
         return e
 
     def step(timed):
         with torch.cuda.stream(stream):
             marks = [ev()] if timed else None
-            for k, p in enumerate(plans):
-                p.solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=W.get("max_lb", 0), out=scores[k],
-                              stream=stream)
+            if side is not None:
+                side.wait_event(ev())
+                f0 = ev(side) if timed else None
+                plans[0].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[0], stream=side)
+                f1 = ev(side)
+                v0 = ev() if timed else None
+                plans[1].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[1], stream=stream)
                 if timed:
-                    marks.append(ev())
+                    marks = [f0, f1, v0, ev()]
+            else:
+                for k, p in enumerate(plans):
+                    p.solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=W.get("max_lb", 0), out=scores[k],
+                                  stream=stream)
+                    if timed:
+                        marks.append(ev())
             tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
+            if side is not None:
+                stream.wait_event(f1)
             if timed:
                 marks.append(ev())
+                if side is not None:  # forward, Viterbi, traceback (the first two overlap)
+                    pairs = [(marks[0], marks[1]), (marks[2], marks[3]), (marks[3], marks[4])]
+                else:
+                    pairs = [(marks[q], marks[q + 1]) for q in range(len(phase_names))]
                 for q in range(len(phase_names)):
-                    ev_phase[q].append((marks[q], marks[q + 1]))
+                    ev_phase[q].append(pairs[q])
             if world > 1:
                 dist.all_gather_into_tensor(gathered, scores[-1] if W["kind"] != "hmm" else scores[1])
                 # tracebacks go to rank 0 only
