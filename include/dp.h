@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define DP_ABI_VERSION 2
+#define DP_ABI_VERSION 3
 #define DP_MAX_DIM 4
 
 typedef enum dp_status {
@@ -88,6 +88,30 @@ typedef struct dp_dep {
 dp_status dp_schedule_derive(int ndim, const int64_t extent[], int triangular, int ndeps, const dp_dep deps[],
                              int coeff_bound, const int32_t* user_coeff, int32_t coeff_out[], int64_t* p_lo,
                              int64_t* p_hi, int32_t* window);
+
+/*
+ * dp_schedule_conditional — §4.7 conditional parallelisation (L379–L402), pure
+ * CPU. "Different problem sizes may therefore require different schedules"
+ * (L380–L381): for each of the ndim! orders of the dimensions, the valid a in
+ * [-coeff_bound, coeff_bound]^ndim (criteria as dp_schedule_derive) that
+ * minimises |a| dimension by dimension in that order (L398–L401; magnitudes per
+ * DESIGN.md R-SCHED-COND), sign ties to the lexicographically smallest a.
+ * Distinct results (each minimal for some extents) go to coeffs_out as
+ * count x ndim int32, identity order first. max_out bounds the output
+ * (DP_E_TOO_LARGE if exceeded; ndim! <= 24 always suffices).
+ * Returns DP_E_NO_SCHEDULE (count 0) when no valid a exists, DP_E_INVALID on
+ * bad arguments. Example (L386–L388): f(x-1, y-1) -> {(0,1), (1,0)}.
+ */
+dp_status dp_schedule_conditional(int ndim, int ndeps, const dp_dep deps[], int coeff_bound, int max_out,
+                                  int32_t coeffs_out[], int* count);
+
+/*
+ * dp_schedule_select — the run-time half of §4.7 (L384–L386): index of the
+ * candidate (coeffs: count x ndim, from dp_schedule_conditional) with the
+ * smallest box range sum_i |a_i| (extent_i - 1) (eq.4) for one problem's
+ * extents; the first on ties. -1 on bad arguments.
+ */
+int dp_schedule_select(int ndim, int count, const int32_t coeffs[], const int64_t extent[]);
 
 /*
  * Plan description. POD; set struct_size = sizeof(dp_desc). All pointers are

@@ -16,7 +16,12 @@ edge of the instance.
   * ties: the first solution in lexicographic order of a (DESIGN.md R-SCHED-TIE);
   * partitions are enumerated over the exact domain (Fig.9/10 L278-L282);
   * sliding window: max over edges of S(c1) - S(c2) when all call sites are
-    uniform (§4.8), else None.
+    uniform (§4.8 L409-L418), else None;
+  * conditional schedules (§4.7): for each of the n! orders of the
+    dimensions, the valid a minimising |a| dimension by dimension in that order
+    ("the first lexicographical solution with respect to the permutation of
+    dimensions", L398-L401; |a_i| per DESIGN.md R-SCHED-COND), then at run time
+    the candidate with the smallest box range for the problem's extents.
 """
 from __future__ import annotations
 
@@ -65,6 +70,25 @@ def derive(domain, calls, extents, bound=10):
     a = best[0]
     vals = [schedule_value(a, x) for x in domain]
     return {"a": tuple(a), "goal": best[1], "p_lo": min(vals), "p_hi": max(vals)}
+
+
+def conditional(domain, calls, ndim, bound=10):
+    """§4.7: distinct per-permutation solutions, in itertools.permutations order (identity first)."""
+    edges = edges_of(list(domain), calls)
+    valid = [a for a in itertools.product(range(-bound, bound + 1), repeat=ndim) if is_valid(a, edges)]
+    out = []
+    for perm in itertools.permutations(range(ndim)):
+        if not valid:
+            break
+        a = min(valid, key=lambda v: (tuple(abs(v[i]) for i in perm), v))
+        if a not in out:
+            out.append(a)
+    return out
+
+
+def select(candidates, extents):
+    """Run-time half of §4.7 (L384-L386): the candidate with the smallest box range (first on ties)."""
+    return min(range(len(candidates)), key=lambda k: (box_range(candidates[k], extents), k))
 
 
 def partitions(domain, a):

@@ -68,6 +68,11 @@ def lib():
                                          ctypes.POINTER(Dep), ctypes.c_int, ctypes.POINTER(i32),
                                          ctypes.POINTER(i32), ctypes.POINTER(i64), ctypes.POINTER(i64),
                                          ctypes.POINTER(i32)]
+        L.dp_schedule_conditional.restype = ctypes.c_int
+        L.dp_schedule_conditional.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.POINTER(Dep), ctypes.c_int,
+                                              ctypes.c_int, ctypes.POINTER(i32), ctypes.POINTER(ctypes.c_int)]
+        L.dp_schedule_select.restype = ctypes.c_int
+        L.dp_schedule_select.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.POINTER(i32), ctypes.POINTER(i64)]
         L.dp_plan_create.restype = ctypes.c_int
         L.dp_plan_create.argtypes = [ctypes.POINTER(Desc), ctypes.POINTER(vp)]
         L.dp_plan_destroy.restype = None
@@ -89,7 +94,8 @@ def lib():
     return _lib
 
 
-EXPORTS = ["dp_abi_version", "dp_status_string", "dp_schedule_derive", "dp_plan_create", "dp_plan_destroy",
+EXPORTS = ["dp_abi_version", "dp_status_string", "dp_schedule_derive", "dp_schedule_conditional",
+           "dp_schedule_select", "dp_plan_create", "dp_plan_destroy",
            "dp_plan_get_schedule", "dp_solve_batch", "dp_solve", "dp_solve_batch_host", "dp_traceback",
            "dp_plan_launch_count"]
 
@@ -116,6 +122,36 @@ def schedule_derive(extent, deps, triangular=False, coeff_bound=10, user_coeff=N
     _check(lib().dp_schedule_derive(nd, ext, int(bool(triangular)), len(deps), arr, int(coeff_bound), uc, out,
                                     ctypes.byref(lo), ctypes.byref(hi), ctypes.byref(w)), "dp_schedule_derive")
     return {"a": tuple(out[i] for i in range(nd)), "p_lo": lo.value, "p_hi": hi.value, "window": w.value}
+
+
+def _deps_array(deps):
+    arr = (Dep * max(1, len(deps)))()
+    for k, (off, axis, lo, hi) in enumerate(deps):
+        for i, v in enumerate(off):
+            arr[k].offset[i] = int(v)
+        arr[k].ranged_axis = -1 if axis is None else int(axis)
+        arr[k].lo, arr[k].hi = int(lo), int(hi)
+    return arr
+
+
+def schedule_conditional(ndim, deps, coeff_bound=10):
+    """§4.7 candidates (dp_schedule_conditional): list of coefficient tuples, identity order
+    first; raises DPError (DP_E_NO_SCHEDULE) when infeasible."""
+    out = (ctypes.c_int32 * (24 * MAX_DIM))()
+    cnt = ctypes.c_int()
+    _check(lib().dp_schedule_conditional(int(ndim), len(deps), _deps_array(deps), int(coeff_bound), 24, out,
+                                         ctypes.byref(cnt)), "dp_schedule_conditional")
+    return [tuple(out[c * ndim + i] for i in range(ndim)) for c in range(cnt.value)]
+
+
+def schedule_select(candidates, extent):
+    """Index of the candidate with the smallest box range for these extents (dp_schedule_select)."""
+    nd = len(extent)
+    flat = (ctypes.c_int32 * (len(candidates) * nd))(*[int(v) for a in candidates for v in a])
+    k = lib().dp_schedule_select(nd, len(candidates), flat, (ctypes.c_int64 * nd)(*extent))
+    if k < 0:
+        raise DPError(1, "dp_schedule_select")
+    return k
 
 
 def _ptr(t):

@@ -7,6 +7,9 @@
 #include <cstdint>
 #include <cstdlib>
 #include <climits>
+#include <algorithm>
+#include <vector>
+#include <array>
 
 #include "dp.h"
 
@@ -128,4 +131,76 @@ extern "C" dp_status dp_schedule_derive(int ndim, const int64_t extent[], int tr
   if (p_hi) *p_hi = hi;
   if (window) *window = window_of(ndim, best, ndeps, deps);
   return DP_OK;
+}
+
+/*
+ * §4.7 conditional parallelisation (L379–L402). For each order pi of the
+ * dimensions (ndim! of them, identity first, std::next_permutation order) the
+ * valid a in [-B, B]^ndim minimising |a_pi1|, then |a_pi2|, ... (each
+ * dimension minimised in turn with the constraints of the earlier ones
+ * propagated; R-SCHED-COND); among the valid a with that tuple of
+ * magnitudes the lexicographically smallest. Distinct results are candidates,
+ * each minimal for some extents vector; dp_schedule_select picks one per problem.
+ */
+extern "C" dp_status dp_schedule_conditional(int ndim, int ndeps, const dp_dep deps[], int coeff_bound, int max_out,
+                                             int32_t coeffs_out[], int* count) {
+  if (ndim < 1 || ndim > DP_MAX_DIM || ndeps < 0 || (ndeps > 0 && !deps) || max_out < 1 || !coeffs_out || !count)
+    return DP_E_INVALID;
+  for (int d = 0; d < ndeps; ++d)
+    if (deps[d].ranged_axis >= ndim || (deps[d].ranged_axis >= 0 && deps[d].lo > deps[d].hi)) return DP_E_INVALID;
+  const int B = coeff_bound > 0 ? coeff_bound : 10;
+  // the valid coefficient vectors (eq.3 per family)
+  std::vector<std::array<int32_t, DP_MAX_DIM>> valid;
+  {
+    std::array<int32_t, DP_MAX_DIM> a{};
+    for (int i = 0; i < ndim; ++i) a[i] = -B;
+    for (;;) {
+      if (satisfies(ndim, a.data(), ndeps, deps)) valid.push_back(a);
+      int k = ndim - 1;
+      while (k >= 0 && a[k] == B) { a[k] = -B; --k; }
+      if (k < 0) break;
+      ++a[k];
+    }
+  }
+  *count = 0;
+  if (valid.empty()) return DP_E_NO_SCHEDULE;
+  int perm[DP_MAX_DIM];
+  for (int i = 0; i < ndim; ++i) perm[i] = i;
+  do {
+    // minimise |a_perm[k]| in turn, keeping only the vectors that attain each minimum
+    std::vector<const std::array<int32_t, DP_MAX_DIM>*> cand;
+    for (const auto& a : valid) cand.push_back(&a);
+    for (int k = 0; k < ndim; ++k) {
+      int32_t m = INT32_MAX;
+      for (const auto* a : cand) m = std::min(m, std::abs((*a)[perm[k]]));
+      std::vector<const std::array<int32_t, DP_MAX_DIM>*> keep;
+      for (const auto* a : cand)
+        if (std::abs((*a)[perm[k]]) == m) keep.push_back(a);
+      cand.swap(keep);
+    }
+    // sign ties: the lexicographically smallest (valid is in lexicographic order)
+    const auto& best = *cand.front();
+    bool dup = false;
+    for (int c = 0; c < *count && !dup; ++c)
+      dup = std::equal(best.begin(), best.begin() + ndim, coeffs_out + (size_t)c * ndim);
+    if (!dup) {
+      if (*count == max_out) return DP_E_TOO_LARGE;
+      std::copy(best.begin(), best.begin() + ndim, coeffs_out + (size_t)(*count) * ndim);
+      ++*count;
+    }
+  } while (std::next_permutation(perm, perm + ndim));
+  return DP_OK;
+}
+
+/* Run-time half of §4.7 (L384–L386): the candidate with the smallest box range
+ * sum |a_i| (extent_i - 1) for this problem (eq.4); the first on ties. */
+extern "C" int dp_schedule_select(int ndim, int count, const int32_t coeffs[], const int64_t extent[]) {
+  if (ndim < 1 || ndim > DP_MAX_DIM || count < 1 || !coeffs || !extent) return -1;
+  int best = 0;
+  int64_t bg = INT64_MAX;
+  for (int c = 0; c < count; ++c) {
+    const int64_t g = box_goal(ndim, coeffs + (size_t)c * ndim, extent);
+    if (g < bg) { bg = g; best = c; }
+  }
+  return best;
 }

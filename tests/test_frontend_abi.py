@@ -30,7 +30,7 @@ def test_exports_match_header(dp):
     L = dp.lib()
     for name in declared:
         assert hasattr(L, name), name
-    assert L.dp_abi_version() == 2
+    assert L.dp_abi_version() == 3
     for code in range(8):
         assert L.dp_status_string(code)
 
@@ -129,3 +129,69 @@ def test_bad_arguments(dp):
     with pytest.raises(dp.DPError) as e:
         dp.schedule_derive((0, 3), [U(-1, 0)])
     assert e.value.code == 1
+
+
+# ---------------------------------------------------------------- §4.7 conditional schedules
+def test_conditional_diagonal_only(dp):
+    """§4.7: f(x-1, y-1) -> candidates (0,1), (1,0); S = x when nx < ny."""
+    g = GOLD["diagonal_only"]
+    cands = dp.schedule_conditional(2, [U(-1, -1)])
+    dom, calls, ext = sch.diagonal_instance(5, 6)
+    assert cands == sch.conditional(dom, calls, 2)
+    assert sorted(cands) == sorted([tuple(g["nx_lt_ny"]), tuple(g["nx_gt_ny"])])
+    assert cands[dp.schedule_select(cands, (4, 9))] == tuple(g["nx_lt_ny"])
+    assert cands[dp.schedule_select(cands, (9, 4))] == tuple(g["nx_gt_ny"])
+    for a in g["valid_never_minimal"]:
+        assert tuple(a) not in cands
+        assert dp.schedule_derive((5, 6), [U(-1, -1)], user_coeff=tuple(a))["a"] == tuple(a)  # valid (L326)
+
+
+def test_conditional_case_studies_single(dp):
+    """The case studies' recurrences have one candidate each, equal to dp_schedule_derive's."""
+    nuss = [U(1, 0), U(0, -1), U(1, -1), ((0, 0), 1, -63, -1), ((0, 0), 0, 1, 63)]
+    for nd, deps, ext in [(2, [U(-1, 0), U(0, -1), U(-1, -1)], (257, 257)),
+                          (2, [((-63, -1), 0, 0, 126)], (64, 1001)),
+                          (2, nuss, (64, 64))]:
+        cands = dp.schedule_conditional(nd, deps)
+        assert cands == [dp.schedule_derive(ext, deps)["a"]]
+    with pytest.raises(dp.DPError) as e:
+        dp.schedule_conditional(1, [U(-1), U(1)])
+    assert e.value.code == 2
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_conditional_matches_bruteforce(dp, seed):
+    """Random uniform dependency sets in 2-D and 3-D: the symbolic front-end's candidates
+    equal the brute force over the explicit call graph of a concrete instance, and each
+    is dp_schedule_derive's choice for extents skewed in its permutation's order."""
+    import itertools
+    import random
+    rnd = random.Random(seed)
+    nd = 2 if seed < 6 else 3
+    B = 3
+    offs = []
+    while len(offs) < rnd.randint(1, 3):
+        o = tuple(rnd.randint(-2, 1) for _ in range(nd))
+        if any(o) and o not in offs:
+            offs.append(o)
+    deps = [U(*o) for o in offs]
+    side = 4 if nd == 3 else 6
+    dom = list(itertools.product(range(side), repeat=nd))
+
+    def calls(c):
+        return [tuple(ci + oi for ci, oi in zip(c, o)) for o in offs]
+
+    want = sch.conditional(dom, calls, nd, bound=B)
+    if not want:
+        with pytest.raises(dp.DPError):
+            dp.schedule_conditional(nd, deps, coeff_bound=B)
+        return
+    got = dp.schedule_conditional(nd, deps, coeff_bound=B)
+    assert got == want
+    for perm in itertools.permutations(range(nd)):
+        ext = [0] * nd
+        for rank, d in enumerate(perm):
+            ext[d] = [10 ** 6, 10 ** 4, 10 ** 2][rank]
+        a = dp.schedule_derive(tuple(ext), deps, coeff_bound=B)["a"]
+        assert a in got
+        assert got[dp.schedule_select(got, tuple(ext))] == a
