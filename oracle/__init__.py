@@ -65,6 +65,9 @@ def lib():
         L.orc_sw_affine_traceback_batch.argtypes = [i64, i64, u8p, i64p, u8p, i64p, i8p, ctypes.c_int, i64, i64,
                                                     u8p, i64, i64p]
         L.orc_nussinov.restype = i64
+        L.orc_lcsubstr.restype = i64
+        L.orc_lcsubstr.argtypes = [u8p, i64, u8p, i64]
+        L.orc_lcsubstr_batch.argtypes = [i64, i64, u8p, i64p, u8p, i64p, i64p]
         L.orc_nussinov.argtypes = [u8p, i64, u8p, ctypes.c_int]
         L.orc_nussinov_traceback.restype = i64
         L.orc_nussinov_traceback.argtypes = [u8p, i64, u8p, ctypes.c_int, u8p]
@@ -166,6 +169,12 @@ def sw_affine_traceback_batch(a_cat, a_off, b_cat, b_off, sigma, go, ge, stride,
     return ops, lens
 
 
+def lcsubstr(s, t) -> int:
+    """Diagonal-only recurrence of §4.7 (L386-L388) as the longest common substring."""
+    s, t = _u8(s), _u8(t)
+    return int(lib().orc_lcsubstr(s, len(s), t, len(t)))
+
+
 def nussinov(x, pair_mask, h) -> int:
     x = _u8(x)
     return int(lib().orc_nussinov(x, len(x), _u8(pair_mask).reshape(-1).copy(), int(h)))
@@ -236,6 +245,16 @@ def sw_traceback_batch(a_cat, a_off, b_cat, b_off, sigma, g, stride, threads=1):
     _parallel(n, lambda f, c: lib().orc_sw_traceback_batch(f, c, a_cat, a_off, b_cat, b_off, sig, sig.shape[0],
                                                            int(g), ops.reshape(-1), stride, lens), threads)
     return ops, lens
+
+
+def lcsubstr_batch(a_cat, a_off, b_cat, b_off, threads=1) -> np.ndarray:
+    """Diagonal-only recurrence (§4.7 example; longest common substring) over a packed batch."""
+    n = len(a_off) - 1
+    out = np.zeros(n, dtype=np.int64)
+    a_cat, b_cat = _u8(a_cat), _u8(b_cat)
+    a_off, b_off = np.ascontiguousarray(a_off, np.int64), np.ascontiguousarray(b_off, np.int64)
+    _parallel(n, lambda f, c: lib().orc_lcsubstr_batch(f, c, a_cat, a_off, b_cat, b_off, out), threads)
+    return out
 
 
 def nussinov_batch(x_cat, x_off, pair_mask, h, threads=1) -> np.ndarray:
