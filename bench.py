@@ -145,6 +145,16 @@ def workload(name, rank, world):
                 "cells": int((lens * (lens - 1) // 2).sum()),
                 "inner": int((lens * (lens - 1) * (lens - 2) // 6).sum()), "tb_stride": 512,
                 "workload": "BASELINE config 5: RNAs of length U[128,512], Nussinov batch, with tracebacks"}
+    if name == "diag":
+        n = 20_000
+        a_cat, a_off, b_cat, b_off = dpgen.diag_pairs(n, first=rank * n)
+        la, lb = np.diff(a_off), np.diff(b_off)
+        return {"kind": "diag", "n": n, "a_cat": a_cat, "a_off": a_off, "b_cat": b_cat, "b_off": b_off,
+                "max_la": int(la.max()), "max_lb": int(lb.max()), "cells": int((la * lb).sum()), "ops_per_cell": 3,
+                "tb_stride": None,
+                "workload": "SURVEY 8(f) NEXT 2 (conditional schedules, §4.7): the diagonal-only recurrence "
+                            "(longest common substring) over 20k DNA pairs, |a| and |b| log-uniform in "
+                            "[32, 4096], schedule chosen per problem"}
     if name == "hmm":
         n = 10_000
         d = dpgen.config3_hmm(n_seqs=n)
@@ -181,6 +191,9 @@ def run_ours(args, rank, world, local_rank):
         plans.append(dp.Plan(dp.SW_AFFINE, W["max_la"], W["max_lb"], sigma=dpgen.blosum62(),
                              gap_open=dpgen.SW_GAP_OPEN, gap_extend=dpgen.SW_GAP_EXTEND, want_traceback=True))
         dev_in = (cu(W["a_cat"]), cu(W["a_off"]), cu(W["b_cat"]), cu(W["b_off"]))
+    elif W["kind"] == "diag":
+        plans.append(dp.Plan(dp.DIAG_LCS, W["max_la"], W["max_lb"]))
+        dev_in = (cu(W["a_cat"]), cu(W["a_off"]), cu(W["b_cat"]), cu(W["b_off"]))
     elif W["kind"] == "nuss":
         plans.append(dp.Plan(dp.NUSSINOV, W["max_la"], pair_mask=dpgen.rna_pair_mask(),
                              min_hairpin=dpgen.NUSS_HAIRPIN, want_traceback=True))
@@ -194,8 +207,8 @@ def run_ours(args, rank, world, local_rank):
     n = W["n"]
     scores = [torch.empty(n, dtype=torch.float32 if (W["kind"] == "hmm" and k == 0) else torch.int32, device=dev)
               for k in range(len(plans))]
-    tb_plan = plans[-1]
-    stride = W["tb_stride"]
+    tb_plan = plans[-1] if W["tb_stride"] else None
+    stride = W["tb_stride"] or 0
     tb_out = torch.empty((n, stride), dtype=torch.uint8, device=dev)
     tb_len = torch.empty(n, dtype=torch.int32, device=dev)
     tb_co = torch.empty((n, 4), dtype=torch.int32, device=dev) if W["kind"] in ("sw", "swa") else None
@@ -207,11 +220,12 @@ def run_ours(args, rank, world, local_rank):
     # CUDA events (on the launching stream) around each phase of the step: every solve
     # launch and the traceback launch; the dominant one carries the roofline
     phase_names = ([{"sw": "k_sw16 (partition sweep)", "swa": "k_align_affine (partition sweep)",
-                     "nuss": "k_nuss (fill + in-kernel traceback)",
+                     "nuss": "k_nuss (fill + in-kernel traceback)", "diag": "k_diag (conditional schedule)",
                      "hmm": "k_forward_tc (tcgen05 forward)"}[W["kind"]]] +
                    (["k_viterbi (max-plus)"] if W["kind"] == "hmm" else []) +
-                   [{"sw": "k_sw16_tb (traceback)", "swa": "k_align_affine_tb (traceback)",
-                     "nuss": "dp_traceback (copy)", "hmm": "k_viterbi_tb (traceback)"}[W["kind"]]])
+                   ([{"sw": "k_sw16_tb (traceback)", "swa": "k_align_affine_tb (traceback)",
+                      "nuss": "dp_traceback (copy)", "hmm": "k_viterbi_tb (traceback)"}[W["kind"]]]
+                    if tb_plan is not None else []))
     ev_phase = [[] for _ in phase_names]
 
     # HMM: the forward (tensor cores, latency-bound on ~n/128 SMs) and Viterbi (ALU) are
@@ -242,11 +256,13 @@ def run_ours(args, rank, world, local_rank):
                                   stream=stream)
                     if timed:
                         marks.append(ev())
-            tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
+            if tb_plan is not None:
+                tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
             if side is not None:
                 stream.wait_event(f1)
             if timed:
-                marks.append(ev())
+                if tb_plan is not None:
+                    marks.append(ev())
                 if side is not None:  # forward, Viterbi, traceback (the first two overlap)
                     pairs = [(marks[0], marks[1]), (marks[2], marks[3]), (marks[3], marks[4])]
                 else:
@@ -256,7 +272,9 @@ def run_ours(args, rank, world, local_rank):
             if world > 1:
                 dist.all_gather_into_tensor(gathered, scores[-1] if W["kind"] != "hmm" else scores[1])
                 # tracebacks go to rank 0 only
-                if rank == 0:
+                if tb_plan is None:
+                    pass
+                elif rank == 0:
                     bufs = [torch.empty_like(tb_out) for _ in range(world)]
                     dist.gather(tb_out, gather_list=bufs, dst=0)
                 else:
@@ -293,6 +311,22 @@ def run_ours(args, rank, world, local_rank):
     dom = max(range(len(phase_ms)), key=lambda q: phase_ms[q])
     k_ms = phase_ms[0]
 
+    # ---- §4.7 evidence (diag): the same steps with each candidate schedule forced for every problem
+    fixed = None
+    if W["kind"] == "diag":
+        fixed = {}
+        for k, a in enumerate(dp.schedule_conditional(2, [((-1, -1), None, 0, 0)])):  # the plan's candidates
+            os.environ["DP_DIAG_FORCE"] = str(k)
+            step(False)
+            f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            f0.record(stream)
+            for _ in range(max(1, min(args.steps, 3))):
+                step(False)
+            f1.record(stream)
+            torch.cuda.synchronize(dev)
+            fixed[str(tuple(a))] = round(f0.elapsed_time(f1) / max(1, min(args.steps, 3)), 4)
+        os.environ.pop("DP_DIAG_FORCE", None)
+
     # ---- end to end through the C ABI with host buffers (pinned), same work per step
     e2e = e2e_host(args, W, plans, dev, stream, world)
 
@@ -308,7 +342,8 @@ def run_ours(args, rank, world, local_rank):
         "higher_is_better": True,
         "scaling": "weak",
         "vs_baseline": None,
-        "dtype": {"sw": "int32", "swa": "int32", "nuss": "int16 table / int32 arithmetic", "hmm": "f32 (forward) + int32 (Viterbi)"}[W["kind"]],
+        "dtype": {"sw": "int32", "swa": "int32", "nuss": "int16 table / int32 arithmetic", "diag": "uint16 table / int32",
+                  "hmm": "f32 (forward) + int32 (Viterbi)"}[W["kind"]],
         "data": "synthetic (seeded, dpgen)",
         "config": {"workload": W["workload"], "config": args.config, "problems_per_gpu": n,
                    "cells_per_gpu": W["cells"], "l2": "flushed between steps (256 MiB write outside step events)",
@@ -318,6 +353,7 @@ def run_ours(args, rank, world, local_rank):
         "dominant_phase": phase_names[dom],
         "roofline": roof,
         "gpu_launches": int(launches),
+        **({"fixed_schedule_ms": fixed, "conditional_schedule_ms": round(ms_step, 4)} if fixed else {}),
         "e2e": e2e,
         "clocks": clk.summary(),
     }
@@ -360,6 +396,10 @@ def roofline(W, phase_ms, pk):
         # bounded to 16 bits by the plan check) -> the s32 peak
         return alu("k_align_affine", W["cells"] * W["ops_per_cell"], phase_ms[0], peak32,
                    "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz")
+    if W["kind"] == "diag":
+        # compare-select, +1, running max: 3 int32 ops per cell -> the s32 ALU peak
+        return alu("k_diag", W["cells"] * W["ops_per_cell"], phase_ms[0], peak32,
+                   "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (3 int ops per cell)")
     if W["kind"] == "nuss":
         return alu("k_nuss_tiled (fill + traceback)", W["inner"], phase_ms[0], peak16,
                    "ubench_r01 VIADDMNMX.S16x2 x 148 SMs x sm_max_mhz (one split evaluation = one max-plus)")
@@ -391,7 +431,7 @@ def e2e_host(args, W, plans, dev, stream, world):
     a_cat, a_off = pin(W["a_cat"]), pin(W["a_off"])
     b_cat = pin(W["b_cat"]) if "b_cat" in W else None
     b_off = pin(W["b_off"]) if "b_off" in W else None
-    n, stride = W["n"], W["tb_stride"]
+    n, stride = W["n"], W["tb_stride"] or 0
     outs = []
     for k, p in enumerate(plans):
         sc = pin(np.empty(n, np.float32 if (W["kind"] == "hmm" and k == 0) else np.int32))
@@ -468,6 +508,13 @@ def oracle_sample(config, W, budget_s):
             oracle.nussinov_traceback(x, dpgen.rna_pair_mask(), 3)
         dt = time.perf_counter() - t
         return reps * W["cells"] / dt, f"config 1 x{reps} repetitions (score + traceback), 1 core", 1
+    if config == "diag":
+        k = 150
+        a_cat, a_off, b_cat, b_off = dpgen.diag_pairs(k)
+        t = time.perf_counter()
+        oracle.lcsubstr_batch(a_cat, a_off, b_cat, b_off, threads=cores)
+        dt = time.perf_counter() - t
+        return int((np.diff(a_off) * np.diff(b_off)).sum()) / dt, f"first {k} pairs of the diag workload", cores
     if config in ("nuss4", "nuss5"):
         ids = dpgen.config5_sample_ids(k=2000 if config == "nuss5" else 200)
         cat, off = dpgen.config5_rna_batch(ids=ids)
@@ -525,7 +572,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="sw", choices=["sw", "swa", "nuss1", "hmm", "nuss4", "nuss5"])
+    ap.add_argument("--config", default="sw", choices=["sw", "swa", "nuss1", "hmm", "nuss4", "nuss5", "diag"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))

@@ -136,6 +136,24 @@ def config2_protein_pairs(n_pairs: int = 100_000, length: int = 256, first: int 
     return a.reshape(-1).copy(), off, b.reshape(-1).copy(), off.copy()
 
 
+def diag_pairs(n_pairs: int = 20_000, lo: int = 32, hi: int = 4096, first: int = 0):
+    """Mixed-shape batch for the diagonal-only recurrence (§4.7 example):
+    DNA pairs (codes 0..3) whose lengths |a|, |b| are drawn independently and log-uniformly
+    from [lo, hi], so about half the pairs are taller than wide; seed 20120611+8.
+    Returns (a_cat, a_off, b_cat, b_off); `first` skips that many pairs of the stream."""
+    g = rng(8)
+    total = first + n_pairs
+    la = np.exp(g.uniform(np.log(lo), np.log(hi + 1), total)).astype(np.int64).clip(lo, hi)
+    lb = np.exp(g.uniform(np.log(lo), np.log(hi + 1), total)).astype(np.int64).clip(lo, hi)
+    a = g.integers(0, 4, int(la.sum()), dtype=np.uint8)
+    b = g.integers(0, 4, int(lb.sum()), dtype=np.uint8)
+    ao = np.concatenate([[0], np.cumsum(la)]).astype(np.int64)
+    bo = np.concatenate([[0], np.cumsum(lb)]).astype(np.int64)
+    a, b = a[ao[first]:], b[bo[first]:]
+    ao, bo = ao[first:] - ao[first], bo[first:] - bo[first]
+    return a.copy(), ao, b.copy(), bo
+
+
 def hmm_params(g: np.random.Generator, S: int = HMM_STATES, K: int = 4):
     """Rows of pi (1xS), A (SxS), E (SxK) ~ Dirichlet(1), float64."""
     pi = g.dirichlet(np.ones(S))

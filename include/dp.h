@@ -55,7 +55,10 @@ typedef enum dp_kind {
   DP_HMM_FORWARD = 3, /* Fig.11a, natural-log likelihood, float32 */
   DP_HMM_VITERBI = 4, /* max-variant of Fig.11a (L463–L464), int32 milli-bit score */
   DP_SW_AFFINE = 5    /* SURVEY §8(f) NEXT 1 (Gotoh, L509–L520; mutual recursion = Further Work L585–L589):
-                         local alignment, gap of length k costs gap_open + k * gap_extend, int32 score */
+                         local alignment, gap of length k costs gap_open + k * gap_extend, int32 score */,
+  DP_DIAG_LCS = 6     /* the §4.7 example f(x,y) = ... f(x-1,y-1) ... (L386–L388) as the
+                         longest common substring, int32; its schedule is chosen per problem among the
+                         conditional candidates (S = i when |a| < |b|, else S = j); no traceback (ABI 3) */
 } dp_kind;
 
 /*

@@ -15,7 +15,7 @@ import numpy as np
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("DP_LIB") or os.path.join(_PKG, "libdp.so")  # DP_LIB: experiment builds only
 
-EDIT, SW_LINEAR, NUSSINOV, HMM_FORWARD, HMM_VITERBI, SW_AFFINE = range(6)
+EDIT, SW_LINEAR, NUSSINOV, HMM_FORWARD, HMM_VITERBI, SW_AFFINE, DIAG_LCS = range(7)
 KIND_NAMES = {EDIT: "edit", SW_LINEAR: "sw_linear", NUSSINOV: "nussinov", HMM_FORWARD: "hmm_forward",
               HMM_VITERBI: "hmm_viterbi", SW_AFFINE: "sw_affine"}
 STATUS = {0: "DP_OK", 1: "DP_E_INVALID", 2: "DP_E_NO_SCHEDULE", 3: "DP_E_UNSUPPORTED", 4: "DP_E_TOO_LARGE",
@@ -257,7 +257,7 @@ class Plan:
             max_len_a = int((a_off[1:] - a_off[:-1]).max().item()) if n > 0 else 0
         if max_len_b is None:
             max_len_b = int((b_off[1:] - b_off[:-1]).max().item()) if (b_off is not None and n > 0) else 0
-        limit = 4 if self.kind == NUSSINOV else self.alphabet_size
+        limit = 4 if self.kind == NUSSINOV else (256 if self.kind == DIAG_LCS else self.alphabet_size)
         self._debug_codes(a_cat, limit)
         self._debug_codes(b_cat, limit)
         if out is None:

@@ -47,6 +47,8 @@ struct dp_plan {
   int64_t p_lo = 0, p_hi = 0;
   int64_t ext[2] = {1, 1};
   int32_t window = -1;
+  int32_t cand[24][2] = {};  // DP_DIAG_LCS: §4.7 candidate schedules
+  int ncand = 0, force = -1;
   // device parameters
   int8_t* d_sigma = nullptr;
   std::vector<int8_t> h_sigma;
@@ -112,6 +114,10 @@ int families(int kind, int64_t la, int64_t lb, int S, int64_t ext[2], int* trian
       deps[4].ranged_axis = 0; deps[4].lo = 1; deps[4].hi = n - 1;      // (k + 1 - i, 0)
       return 5;
     }
+    case DP_DIAG_LCS:  // f(x-1, y-1) only (§4.7)
+      ext[0] = la + 1; ext[1] = lb + 1;
+      deps[0].offset[0] = -1; deps[0].offset[1] = -1;
+      return 1;
     case DP_HMM_FORWARD:
     case DP_HMM_VITERBI:  // F(t.start, i-1) for t in s.transitionsto: any state (§5.2)
       ext[0] = S; ext[1] = la + 1;
@@ -195,7 +201,7 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
   if (!d || !out) return DP_E_INVALID;
   *out = nullptr;
   if (d->struct_size != sizeof(dp_desc)) return DP_E_INVALID;
-  if (d->kind < DP_EDIT || d->kind > DP_SW_AFFINE) return DP_E_INVALID;
+  if (d->kind < DP_EDIT || d->kind > DP_DIAG_LCS) return DP_E_INVALID;
   if (d->max_len_a < 0 || d->max_len_b < 0) return DP_E_INVALID;
   dp_plan* p = new (std::nothrow) dp_plan();
   if (!p) return DP_E_NOMEM;
@@ -233,6 +239,10 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
       p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
       break;
+    case DP_DIAG_LCS:
+      if (p->want_tb) { st = DP_E_UNSUPPORTED; break; }
+      if (d->max_len_a > 40000 || d->max_len_b > 40000) st = DP_E_TOO_LARGE;  // uint16 window rows in smem
+      break;
     case DP_NUSSINOV:
       if (!d->pair_mask || d->min_hairpin < 0) { st = DP_E_INVALID; break; }
       if (d->max_len_a > 32767 * 2) { st = DP_E_TOO_LARGE; break; }
@@ -268,8 +278,19 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
     p->ndim = 2;
     st = dp_schedule_derive(2, p->ext, tri, nd, deps, d->coeff_bound, d->user_coeff, p->coeff, &p->p_lo, &p->p_hi,
                             &p->window);
+    if (st == DP_OK && d->kind == DP_DIAG_LCS) {
+      // §4.7: every candidate schedule; the kernel picks one per problem. A (valid) user
+      // schedule must be one of them and is then used for every problem.
+      int32_t c[24 * 2];
+      st = dp_schedule_conditional(2, nd, deps, d->coeff_bound, 24, c, &p->ncand);
+      for (int k = 0; st == DP_OK && k < p->ncand; ++k) {
+        p->cand[k][0] = c[2 * k]; p->cand[k][1] = c[2 * k + 1];
+        if (d->user_coeff && c[2 * k] == d->user_coeff[0] && c[2 * k + 1] == d->user_coeff[1]) p->force = k;
+      }
+      if (st == DP_OK && d->user_coeff && p->force < 0) st = DP_E_UNSUPPORTED;
+    }
   }
-  if (st == DP_OK) {
+  if (st == DP_OK && d->kind != DP_DIAG_LCS) {
     // The kernels implement the derived schedule; a user schedule that is valid
     // but differs would need another kernel (conditional schedules, §4.7: NEXT).
     // Coefficients of a dimension of extent 1 do not change the partitions.
@@ -303,7 +324,8 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
                          void* stream) {
   if (!p || n < 0) return DP_E_INVALID;
   if (n > 0 && (!a_off || !scores_out)) return DP_E_INVALID;
-  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE;
+  const bool align =
+      p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE || p->kind == DP_DIAG_LCS;
   if (align && n > 0 && !b_off) return DP_E_INVALID;
   if (max_len_a < 0 || max_len_b < 0) return DP_E_INVALID;
   if (max_len_a > p->max_la || (align && max_len_b > p->max_lb)) return DP_E_TOO_LARGE;
@@ -316,6 +338,17 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
   p->last_a = a_cat; p->last_b = b_cat; p->last_aoff = a_off; p->last_boff = b_off;
   p->last_max_la = max_len_a; p->last_max_lb = max_len_b;
   switch (p->kind) {
+    case DP_DIAG_LCS: {
+      dpk::DiagArgs A{};
+      A.n = n; A.a_cat = a_cat; A.b_cat = b_cat; A.a_off = a_off; A.b_off = b_off;
+      A.max_len = std::max<int64_t>(1, std::max(max_len_a, max_len_b));
+      A.scores = static_cast<int32_t*>(scores_out);
+      A.ncand = p->ncand;
+      for (int k = 0; k < p->ncand; ++k) { A.cand[k][0] = p->cand[k][0]; A.cand[k][1] = p->cand[k][1]; }
+      A.force = getenv("DP_DIAG_FORCE") ? atoi(getenv("DP_DIAG_FORCE")) : p->force;  // env: diagnostic
+      e = dpk::diag_solve(A, s, &p->launches);
+      break;
+    }
     case DP_SW_LINEAR:
       if (p->packed16) {
         dpk::Sw16Args A{};
@@ -558,7 +591,8 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
                               const uint8_t* b_cat, const int64_t* b_off, void* scores_out, uint8_t* tb_out,
                               int64_t tb_stride, int32_t* tb_len, int32_t* tb_coords, void* stream) {
   if (!p || n < 0 || (n > 0 && (!a_off || !a_cat || !scores_out))) return DP_E_INVALID;
-  const bool align = p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE;
+  const bool align =
+      p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE || p->kind == DP_DIAG_LCS;
   if (align && n > 0 && (!b_off || !b_cat)) return DP_E_INVALID;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   int64_t max_la = 0, max_lb = 0;

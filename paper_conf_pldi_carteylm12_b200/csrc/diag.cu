@@ -1,0 +1,101 @@
+// The §4.7 example recurrence f(x, y) = ... f(x-1, y-1) ... (L386-L388), as the
+// longest common substring (DESIGN.md R-DIAG):
+//   L(i,j) = a_i == b_j ? L(i-1,j-1) + 1 : 0,   score = max L.
+// Its only dependency family is (-1,-1), so both S = i (a = (1,0)) and S = j
+// (a = (0,1)) are valid and each is minimal for some extents: "when nx < ny then
+// Sf(x,y) = x otherwise Sf(x,y) = y" (L386-L388). The plan holds the candidates
+// dp_schedule_conditional derives; the kernel evaluates the run-time condition
+// per problem (L384-L386) — the candidate with the smallest box range for
+// (|a|, |b|) — and sweeps that schedule's partitions: one CTA per problem
+// (persistent over the batch), one partition per iteration with every thread
+// on a strided slice of it, one barrier between partitions (Fig.8), the window
+// of one partition (§4.8: w = 1) double-buffered in shared memory as uint16.
+// Choosing the schedule with fewer, longer partitions is what keeps the CTA
+// busy: a 64 x 4096 pair takes 64 barriers instead of 4096.
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "dp_internal.h"
+
+namespace dpk {
+namespace {
+
+constexpr int kDT = 256;  // threads per CTA
+
+__global__ void __launch_bounds__(kDT) k_diag(DiagArgs A) {
+  extern __shared__ __align__(16) uint8_t dsm[];
+  const int64_t cap = A.max_len;
+  uint16_t* row0 = reinterpret_cast<uint16_t*>(dsm);
+  uint16_t* row1 = row0 + cap + 8;
+  uint8_t* qs = reinterpret_cast<uint8_t*>(row1 + cap + 8);
+  __shared__ int red[kDT / 32];
+  const int tid = threadIdx.x;
+  for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
+    const int64_t la = A.a_off[p + 1] - A.a_off[p], lb = A.b_off[p + 1] - A.b_off[p];
+    // run-time schedule choice (§4.7): the candidate with the smallest box range sum |a_i| (n_i - 1)
+    int k = 0;
+    if (A.force >= 0 && A.force < A.ncand) {
+      k = A.force;
+    } else {
+      int64_t bg = INT64_MAX;
+      for (int c = 0; c < A.ncand; ++c) {
+        const int64_t g = (int64_t)abs(A.cand[c][0]) * (la > 0 ? la - 1 : 0) + (int64_t)abs(A.cand[c][1]) * (lb > 0 ? lb - 1 : 0);
+        if (g < bg) { bg = g; k = c; }
+      }
+    }
+    // S = i: the partitions are the rows i = 1..|a| (cells along j); S = j: the columns.
+    // L is symmetric in (a, b), so the column sweep is the row sweep of the swapped pair.
+    const bool by_row = A.cand[k][0] != 0;
+    const uint8_t* P = by_row ? A.a_cat + A.a_off[p] : A.b_cat + A.b_off[p];
+    const uint8_t* Q = by_row ? A.b_cat + A.b_off[p] : A.a_cat + A.a_off[p];
+    const int np = (int)(by_row ? la : lb), nq = (int)(by_row ? lb : la);
+    __syncthreads();  // the previous problem's buffers are free
+    for (int y = tid; y < nq; y += kDT) qs[y] = Q[y];
+    for (int y = tid; y <= nq; y += kDT) { row0[y] = 0; row1[y] = 0; }
+    __syncthreads();
+    int best = 0;
+    uint16_t* prev = row0;
+    uint16_t* cur = row1;
+    for (int x = 1; x <= np; ++x) {  // partition x: every cell (x, y) at once, then a barrier
+      const uint8_t px = __ldg(P + x - 1);
+      for (int y = tid + 1; y <= nq; y += kDT) {
+        const int v = qs[y - 1] == px ? prev[y - 1] + 1 : 0;
+        cur[y] = (uint16_t)v;
+        best = max(best, v);
+      }
+      __syncthreads();
+      uint16_t* t = prev; prev = cur; cur = t;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
+    if ((tid & 31) == 0) red[tid >> 5] = best;
+    __syncthreads();
+    if (tid == 0) {
+      int b = 0;
+      for (int w = 0; w < kDT / 32; ++w) b = max(b, red[w]);
+      A.scores[p] = b;
+    }
+  }
+}
+
+}  // namespace
+
+size_t diag_smem_bytes(int64_t max_len) { return (size_t)(2 * (max_len + 8) * 2 + ((max_len + 15) & ~int64_t(15))); }
+
+cudaError_t diag_solve(const DiagArgs& A, cudaStream_t s, int64_t* launches) {
+  if (A.n == 0) return cudaSuccess;
+  const size_t smem = diag_smem_bytes(A.max_len);
+  cudaError_t e = cudaFuncSetAttribute(k_diag, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int dev = 0, sms = 0, per_sm = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_diag, kDT, smem)) != cudaSuccess) return e;
+  if (per_sm < 1) return cudaErrorInvalidConfiguration;
+  const int64_t grid = A.n < (int64_t)per_sm * sms ? A.n : (int64_t)per_sm * sms;
+  ++*launches;
+  k_diag<<<(unsigned)grid, kDT, smem, s>>>(A);
+  return cudaGetLastError();
+}
+
+}  // namespace dpk

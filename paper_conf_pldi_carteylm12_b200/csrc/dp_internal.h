@@ -81,6 +81,20 @@ cudaError_t sw16_solve(const Sw16Args& a, bool tb, cudaStream_t s, int64_t* laun
 cudaError_t sw16_traceback(const Sw16Args& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                            int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
 
+// ---------------------------------------------------------------- diagonal-only (§4.7)
+struct DiagArgs {
+  int64_t n;
+  const uint8_t *a_cat, *b_cat;
+  const int64_t *a_off, *b_off;
+  int64_t max_len;       // max over the batch of max(|a|, |b|)
+  int32_t* scores;
+  int32_t cand[24][2];   // §4.7 candidate schedules (dp_schedule_conditional)
+  int ncand;
+  int force;             // -1: run-time choice per problem; else that candidate (diagnostic)
+};
+size_t diag_smem_bytes(int64_t max_len);
+cudaError_t diag_solve(const DiagArgs& a, cudaStream_t s, int64_t* launches);
+
 // ---------------------------------------------------------------- Nussinov
 struct NussArgs {
   int64_t n;

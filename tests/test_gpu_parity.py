@@ -417,3 +417,58 @@ def test_host_entry_point(dp, orc):
         ops, co = orc.sw_traceback(a[q], b[q], sig, 4)
         assert sc[q] == s0 and bytes(tb[q, :tbl[q]]).decode() == ops and tuple(tbc[q]) == co
     plan.close()
+
+
+# ----------------------------------------------------------------------------- §4.7 diagonal-only
+def run_diag(dp, a_seqs, b_seqs, **kw):
+    a_cat, a_off = dpgen.pack(a_seqs)
+    b_cat, b_off = dpgen.pack(b_seqs)
+    la = max((len(s) for s in a_seqs), default=0)
+    lb = max((len(s) for s in b_seqs), default=0)
+    with dp.Plan(dp.DIAG_LCS, max(la, 1), max(lb, 1), **kw) as plan:
+        return host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=la, max_len_b=lb))
+
+
+@pytest.mark.parametrize("force", [None, "0", "1"])
+def test_diag_mixed_shapes(dp, orc, monkeypatch, force):
+    """Ragged tall and wide pairs, empty sides, length 1: bit-exact against the oracle under the
+    run-time schedule choice and under each candidate forced (the result cannot depend on it)."""
+    if force is not None:
+        monkeypatch.setenv("DP_DIAG_FORCE", force)
+    g = np.random.default_rng(800)
+    a = [g.integers(0, 4, int(g.integers(0, 700))).astype(np.uint8) for _ in range(150)]
+    b = [g.integers(0, 4, int(g.integers(0, 700))).astype(np.uint8) for _ in range(150)]
+    a[:4] = [np.zeros(0, np.uint8), np.ones(1, np.uint8), a[2], np.arange(300, dtype=np.uint8) % 4]
+    b[:4] = [b[0], np.zeros(0, np.uint8), a[2].copy(), np.arange(5, 900, dtype=np.uint8) % 4]
+    a[5], b[5] = np.full(257, 2, np.uint8), np.full(33, 2, np.uint8)   # a run: the answer is 33
+    got = run_diag(dp, a, b)
+    want = np.array([orc.lcsubstr(x, y) for x, y in zip(a, b)])
+    assert (got == want).all()
+    assert got[5] == 33
+
+
+def test_diag_workload_sampled(dp, orc):
+    """The bench workload's distribution (log-uniform 32..4096 per side), first 120 pairs."""
+    a_cat, a_off, b_cat, b_off = dpgen.diag_pairs(120)
+    la, lb = int(np.diff(a_off).max()), int(np.diff(b_off).max())
+    with dp.Plan(dp.DIAG_LCS, la, lb) as plan:
+        got = host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=la, max_len_b=lb))
+    want = orc.lcsubstr_batch(a_cat, a_off, b_cat, b_off, threads=THREADS)
+    assert (got == want).all()
+
+
+def test_diag_plan_schedules(dp):
+    """§4.7: the plan accepts a user schedule only if it is one of the conditional candidates
+    (L326, L386-L388); no traceback is retained for this kind."""
+    with dp.Plan(dp.DIAG_LCS, 100, 50) as p:
+        assert p.schedule()["a"] in ((0, 1), (1, 0))
+    for uc in ((1, 0), (0, 1)):
+        with dp.Plan(dp.DIAG_LCS, 100, 50, user_coeff=uc) as p:
+            assert p.schedule()["a"] == uc
+    for uc, code in (((2, 1), 3), ((1, -1), 2)):      # valid but never minimal / invalid
+        with pytest.raises(dp.DPError) as e:
+            dp.Plan(dp.DIAG_LCS, 100, 50, user_coeff=uc)
+        assert e.value.code == code
+    with pytest.raises(dp.DPError) as e:
+        dp.Plan(dp.DIAG_LCS, 100, 50, want_traceback=True)
+    assert e.value.code == 3
