@@ -42,6 +42,14 @@ namespace dpk {
 namespace {
 
 constexpr int T = 32;
+#ifndef NUSS_TBW_G
+#define NUSS_TBW_G 8   // traceback gamma window (W x W per round trip) and split-search width (32 KC) of the grid
+#define NUSS_TBK_G 1   // sweep (16 / 2 measured no faster)
+#endif
+#ifndef NUSS_TBW_B
+#define NUSS_TBW_B 8   // the same for the batch kernel
+#define NUSS_TBK_B 1
+#endif
 constexpr int kTileWords = T * T;      // int16 per tile record half
 constexpr int kRec = 2 * kTileWords;   // int16 per tile record (UT + L)
 constexpr int kCtaWarps = 2;   // batch driver: eight CTAs (eight sequences) per SM
@@ -474,7 +482,11 @@ __device__ __forceinline__ void trace_interval(const TabT& tab, const uint8_t* x
 #pragma unroll
       for (int u = 0; u < KC; ++u) {
         const int kq = k0 + lane + 32 * u;
-        s[u] = kq < j ? tab.gamma(i, kq) + tab.gamma(kq + 1, j) : -1;
+        // gamma(i, kq) along row i from the row-major L record of row i (L(I',K)[k][c] =
+        // gamma(32I'+k+1, 32K+c)): 32 consecutive k are 64 contiguous bytes instead of 32 lines
+        const int gik = kq >= j ? 0 : (i >= 1 ? (int)__ldcg(tab.L((i - 1) / T, kq / T) + ((i - 1) % T) * T + kq % T)
+                                              : tab.gamma(i, kq));
+        s[u] = kq < j ? gik + tab.gamma(kq + 1, j) : -1;
       }
 #pragma unroll
       for (int u = 0; u < KC; ++u) {
@@ -814,7 +826,7 @@ __global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_
       A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
       if (A.db) A.db_len[p] = n;
     }
-    if (A.db) warp_traceback_win<8, 1>(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, win, sstk, lane);
+    if (A.db) warp_traceback_win<NUSS_TBW_B, NUSS_TBK_B>(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, stack, win, sstk, lane);
     clk.lap(6);
   }
   clk.flush(lane);
@@ -849,7 +861,7 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   Q.flag = Q.hdr + 4;
   Q.item = reinterpret_cast<int2*>(Q.flag + Q.cap + (Q.cap & 1));
   PhaseClock clk;
-  clk.dbg = nullptr;
+  clk.dbg = A.dbg;  // DP_NUSS_TIMING: phase-B warps' per-tile phases (diagnostic)
   const int ty = lane >> 2, tx = lane & 3;
   for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T + 4 + Q.cap;
        q += (int64_t)gridDim.x * blockDim.x)
@@ -861,6 +873,7 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
       asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
       A.round_ns[D] = t;
     }
+    if ((warp & 3) == 0) clk.start();
     const int nT = nt - D;
     int* C = Cg + (int64_t)(D & 1) * nt * T * T;        // diagonal D (interior products already in)
     int* Cn = Cg + (int64_t)((D + 1) & 1) * nt * T * T; // diagonal D+1
@@ -873,6 +886,7 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
         const int below = diag ? 0 : tab.g16(I + 1, J, lane, 0);
         const int left = diag ? 0 : tab.g16(I, J - 1, T - 1, lane);
         const int corner = (!diag && I + 1 <= J - 1) ? tab.g16(I + 1, J - 1, T - 1, 0) : 0;
+        clk.start();
         uint32_t acc[16];
 #pragma unroll
         for (int q = 0; q < 16; ++q) acc[q] = 0;
@@ -890,6 +904,7 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
         tile_finish(tab, I, J, acc, below, left, corner, IB, x, pm, n, A.hairpin, lane, clk);
         if (D >= 4)  // this C slot is reused by diagonal D+2
           for (int q = lane; q < T * T; q += 32) Ct[q] = 0;
+        clk.lap(4);
       }
     } else if (D + 1 < nt && D >= 3) {
       // interior K-steps of diagonal D+1: tiles t' (I = t', J = t' + D + 1), K in [I+2, J-2]
@@ -922,6 +937,7 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
       }
     }
     grid.sync();
+    if ((warp & 3) == 0) clk.lap(5);  // barrier wait of the phase-B warps
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     if (A.round_ns) {
@@ -979,7 +995,7 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
     if (!got) break;
     __threadfence();
     const int2 iv = __ldcg(&Q.item[idx]);
-    trace_interval<8, 1>(tab, x, pm, n, A.hairpin, db, iv.x, iv.y, win, guard, push, lane);
+    trace_interval<NUSS_TBW_G, NUSS_TBK_G>(tab, x, pm, n, A.hairpin, db, iv.x, iv.y, win, guard, push, lane);
     __syncwarp();
     if (lane == 0) {
       __threadfence();
