@@ -7,9 +7,10 @@
 // dp_schedule_conditional derives; the kernel evaluates the run-time condition
 // per problem (L384-L386) — the candidate with the smallest box range for
 // (|a|, |b|) — and sweeps that schedule's partitions: one CTA per problem
-// (persistent over the batch), one partition per iteration with every thread
-// on a strided slice of it, one barrier between partitions (Fig.8), the window
-// of one partition (§4.8: w = 1) double-buffered in shared memory as uint16.
+// (persistent over the batch), one partition per iteration, one barrier
+// between partitions (Fig.8). Partitions of <= 4096 cells keep the window of
+// one partition (§4.8: w = 1) in registers (C = 1..16 consecutive cells per
+// thread); longer ones double-buffer it in shared memory as uint16.
 // Choosing the schedule with fewer, longer partitions is what keeps the CTA
 // busy: a 64 x 4096 pair takes 64 barriers instead of 4096.
 #include <cstdint>
@@ -22,13 +23,46 @@ namespace {
 
 constexpr int kDT = 256;  // threads per CTA
 
+// One partition per iteration with C cells per thread in registers: thread t owns cells
+// y = C t + 1 .. C t + C of every partition (nq <= 256 C). L(x, y) needs L(x-1, y-1): the
+// thread's own previous values shifted by one, and for its first cell the last cell of
+// thread t-1 (a shuffle; across warps through shared memory, double-buffered by parity).
+// Cells past the end compare against a code no residue has and stay 0.
+template <int C>
+__device__ __forceinline__ int sweep_regs(const uint8_t* P, const uint8_t* Q, int np, int nq, int* xw, int tid) {
+  const int lane = tid & 31, warp = tid >> 5;
+  int q[C], L[C];
+#pragma unroll
+  for (int c = 0; c < C; ++c) {
+    const int y = C * tid + c;  // 0-based column of cell c
+    q[c] = y < nq ? (int)Q[y] : 0x1000;
+    L[c] = 0;
+  }
+  int best = 0;
+  for (int x = 0; x < np; ++x) {
+    const int px = (int)P[x];
+    int nb = __shfl_up_sync(0xffffffffu, L[C - 1], 1);
+    if (lane == 0) nb = (warp > 0 && x > 0) ? xw[((x + 1) & 1) * (kDT / 32) + warp - 1] : 0;  // partition x-1's
+#pragma unroll
+    for (int c = C - 1; c >= 1; --c) L[c] = q[c] == px ? L[c - 1] + 1 : 0;
+    L[0] = q[0] == px ? nb + 1 : 0;
+#pragma unroll
+    for (int c = 0; c < C; ++c) best = max(best, L[c]);
+    if (lane == 31) xw[(x & 1) * (kDT / 32) + warp] = L[C - 1];
+    __syncthreads();
+  }
+  return best;
+}
+
 __global__ void __launch_bounds__(kDT) k_diag(DiagArgs A) {
   extern __shared__ __align__(16) uint8_t dsm[];
   const int64_t cap = A.max_len;
   uint16_t* row0 = reinterpret_cast<uint16_t*>(dsm);
   uint16_t* row1 = row0 + cap + 8;
   uint8_t* qs = reinterpret_cast<uint8_t*>(row1 + cap + 8);
+  uint8_t* ps = qs + ((cap + 15) & ~int64_t(15));
   __shared__ int red[kDT / 32];
+  __shared__ int xw[2 * (kDT / 32)];
   const int tid = threadIdx.x;
   for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
     const int64_t la = A.a_off[p + 1] - A.a_off[p], lb = A.b_off[p + 1] - A.b_off[p];
@@ -51,20 +85,32 @@ __global__ void __launch_bounds__(kDT) k_diag(DiagArgs A) {
     const int np = (int)(by_row ? la : lb), nq = (int)(by_row ? lb : la);
     __syncthreads();  // the previous problem's buffers are free
     for (int y = tid; y < nq; y += kDT) qs[y] = Q[y];
-    for (int y = tid; y <= nq; y += kDT) { row0[y] = 0; row1[y] = 0; }
+    for (int y = tid; y < np; y += kDT) ps[y] = P[y];
+    const bool regs = nq <= 16 * kDT;
+    if (!regs)
+      for (int y = tid; y <= nq; y += kDT) { row0[y] = 0; row1[y] = 0; }
     __syncthreads();
     int best = 0;
-    uint16_t* prev = row0;
-    uint16_t* cur = row1;
-    for (int x = 1; x <= np; ++x) {  // partition x: every cell (x, y) at once, then a barrier
-      const uint8_t px = __ldg(P + x - 1);
-      for (int y = tid + 1; y <= nq; y += kDT) {
-        const int v = qs[y - 1] == px ? prev[y - 1] + 1 : 0;
-        cur[y] = (uint16_t)v;
-        best = max(best, v);
+    if (regs) {
+      if (nq <= kDT) best = sweep_regs<1>(ps, qs, np, nq, xw, tid);
+      else if (nq <= 2 * kDT) best = sweep_regs<2>(ps, qs, np, nq, xw, tid);
+      else if (nq <= 4 * kDT) best = sweep_regs<4>(ps, qs, np, nq, xw, tid);
+      else if (nq <= 8 * kDT) best = sweep_regs<8>(ps, qs, np, nq, xw, tid);
+      else best = sweep_regs<16>(ps, qs, np, nq, xw, tid);
+    } else {
+      // long partitions: the window row in shared memory, every thread on a strided slice
+      uint16_t* prev = row0;
+      uint16_t* cur = row1;
+      for (int x = 1; x <= np; ++x) {  // partition x: every cell (x, y) at once, then a barrier
+        const uint8_t px = ps[x - 1];
+        for (int y = tid + 1; y <= nq; y += kDT) {
+          const int v = qs[y - 1] == px ? prev[y - 1] + 1 : 0;
+          cur[y] = (uint16_t)v;
+          best = max(best, v);
+        }
+        __syncthreads();
+        uint16_t* t = prev; prev = cur; cur = t;
       }
-      __syncthreads();
-      uint16_t* t = prev; prev = cur; cur = t;
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
@@ -80,7 +126,7 @@ __global__ void __launch_bounds__(kDT) k_diag(DiagArgs A) {
 
 }  // namespace
 
-size_t diag_smem_bytes(int64_t max_len) { return (size_t)(2 * (max_len + 8) * 2 + ((max_len + 15) & ~int64_t(15))); }
+size_t diag_smem_bytes(int64_t max_len) { return (size_t)(2 * (max_len + 8) * 2 + 2 * ((max_len + 15) & ~int64_t(15))); }
 
 cudaError_t diag_solve(const DiagArgs& A, cudaStream_t s, int64_t* launches) {
   if (A.n == 0) return cudaSuccess;

@@ -441,6 +441,8 @@ def test_diag_mixed_shapes(dp, orc, monkeypatch, force):
     a[:4] = [np.zeros(0, np.uint8), np.ones(1, np.uint8), a[2], np.arange(300, dtype=np.uint8) % 4]
     b[:4] = [b[0], np.zeros(0, np.uint8), a[2].copy(), np.arange(5, 900, dtype=np.uint8) % 4]
     a[5], b[5] = np.full(257, 2, np.uint8), np.full(33, 2, np.uint8)   # a run: the answer is 33
+    a[6], b[6] = g.integers(0, 4, 60).astype(np.uint8), g.integers(0, 4, 4500).astype(np.uint8)  # > 4096: smem path
+    a[7], b[7] = g.integers(0, 2, 5000).astype(np.uint8), g.integers(0, 2, 3000).astype(np.uint8)
     got = run_diag(dp, a, b)
     want = np.array([orc.lcsubstr(x, y) for x, y in zip(a, b)])
     assert (got == want).all()
