@@ -144,9 +144,14 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int asz = A.asz, gap = A.gap;
-  int8_t* sig_s = reinterpret_cast<int8_t*>(smem);
-  const int sig_bytes = (asz * asz + 15) & ~15;
-  for (int q = threadIdx.x; q < asz * asz; q += blockDim.x) sig_s[q] = A.sigma[q];
+  // sigma transposed, sigT[c][a] (32 x 32 int8): kDead outside the alphabet, so a = 31 is a
+  // dead residue and c = asz a dead column code
+  int8_t* sigT = reinterpret_cast<int8_t*>(smem);
+  constexpr int sig_bytes = 32 * 32;
+  for (int q = threadIdx.x; q < 32 * 32; q += blockDim.x) {
+    const int c = q >> 5, a = q & 31;
+    sigT[q] = (c < asz && a < asz) ? A.sigma[a * asz + c] : (int8_t)kDead;
+  }
   __syncthreads();
   const int64_t grp = (int64_t)blockIdx.x * kWarps + warp;
   const int64_t pA = 2 * grp, pB = 2 * grp + 1;
@@ -192,21 +197,39 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
 
   for (int st = 0; st < strips; ++st) {
     const int i0 = st * kStrip + lane * kRows;  // 0-based index of my first row
-    // profiles for my 8 rows: P[c][row] int8, one 8-byte word per lane per residue
-    int ra[kRows], rb[kRows];
+    // profiles for my 8 rows: P[c][row] int8, one 8-byte word per lane per residue. Each 4-row
+    // word is gathered from column c of sigT with byte permutes: residue a selects byte a & 7 of
+    // the 8-byte window a >> 3, one PRMT per window, merged under per-row window masks.
+    uint32_t sel[4], msk[4][4];  // [problem A rows 0-3, 4-7, problem B rows 0-3, 4-7]
 #pragma unroll
-    for (int r = 0; r < kRows; ++r) {
-      ra[r] = (i0 + r < laA) ? aA[i0 + r] : -1;
-      rb[r] = (i0 + r < laB) ? aB[i0 + r] : -1;
+    for (int g4 = 0; g4 < 4; ++g4) {
+      const uint8_t* src = g4 < 2 ? aA : aB;
+      const int la = g4 < 2 ? laA : laB;
+      uint32_t sl = 0, m[4] = {0, 0, 0, 0};
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int i = i0 + 4 * (g4 & 1) + k;
+        const int a = i < la ? src[i] : 31;  // dead rows read sigma = kDead
+        sl |= (uint32_t)(a & 7) << (4 * k);
+        m[a >> 3] |= 0xffu << (8 * k);
+      }
+      sel[g4] = sl;
+#pragma unroll
+      for (int w = 0; w < 4; ++w) msk[g4][w] = m[w];
     }
     for (int c = 0; c <= asz; ++c) {
-      uint32_t w[4] = {0, 0, 0, 0};
+      uint32_t col[8];  // sigT[c][0..31]
+      const uint4 c0 = *reinterpret_cast<const uint4*>(sigT + 32 * c);
+      const uint4 c1 = *reinterpret_cast<const uint4*>(sigT + 32 * c + 16);
+      col[0] = c0.x; col[1] = c0.y; col[2] = c0.z; col[3] = c0.w;
+      col[4] = c1.x; col[5] = c1.y; col[6] = c1.z; col[7] = c1.w;
+      uint32_t w[4];
 #pragma unroll
-      for (int r = 0; r < kRows; ++r) {
-        const int va = (ra[r] >= 0 && c < asz) ? sig_s[ra[r] * asz + c] : kDead;
-        const int vb = (rb[r] >= 0 && c < asz) ? sig_s[rb[r] * asz + c] : kDead;
-        w[r / 4] |= (uint32_t)(uint8_t)(int8_t)va << (8 * (r % 4));
-        w[2 + r / 4] |= (uint32_t)(uint8_t)(int8_t)vb << (8 * (r % 4));
+      for (int g4 = 0; g4 < 4; ++g4) {
+        uint32_t v = prmt(col[0], col[1], sel[g4]) & msk[g4][0];
+#pragma unroll
+        for (int win = 1; win < 4; ++win) v |= prmt(col[2 * win], col[2 * win + 1], sel[g4]) & msk[g4][win];
+        w[g4] = v;
       }
       *reinterpret_cast<uint2*>(profA + c * kStrip + lane * kRows) = make_uint2(w[0], w[1]);
       *reinterpret_cast<uint2*>(profB + c * kStrip + lane * kRows) = make_uint2(w[2], w[3]);
@@ -758,7 +781,7 @@ void sw16_state_words(int64_t n, int64_t max_la, int64_t max_lb, int64_t* strips
 
 cudaError_t sw16_solve(const Sw16Args& A, bool tb, cudaStream_t s, int64_t* launches) {
   if (A.n == 0) return cudaSuccess;
-  const size_t smem = ((A.asz * A.asz + 15) & ~15) + (size_t)kWarps * A.smem_per_warp;
+  const size_t smem = 32 * 32 + (size_t)kWarps * A.smem_per_warp;
   const bool multi = A.max_la > kStrip;
   auto kern = tb ? (multi ? k_sw16<true, true> : k_sw16<true, false>) : (multi ? k_sw16<false, true> : k_sw16<false, false>);
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
