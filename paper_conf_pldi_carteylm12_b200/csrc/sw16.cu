@@ -356,6 +356,7 @@ struct TbState {      // one problem in one half of a group (shared memory; writ
   int mode;
   int band;           // search: first lane band (strip * 32 + lane) whose maximum is the score
   int scur, cand;     // search: next slab to probe, candidate slab (-1 none)
+  unsigned cbits;     // search: candidate slabs scur + b of the current probe window still to visit
   int i, j, n;        // walk: current cell, ops written
   int ei, ej;         // end cell
 };
@@ -492,6 +493,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
           TbState& W = St[hf];
           if (bits) {
             W.cand = scur + __ffs(bits) - 1;
+            W.cbits = bits;
           } else {
             W.scur = scur + 32;
             if (W.scur >= nsl) {  // candidates exhausted: walk from the first maximum
@@ -674,8 +676,19 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
           const long long k2 = ((long long)(R0[hf] + kRows * m8 + r + 1) << 32) | (long long)(D[hf] + c - m8);
           if (S.found < 0 || k2 < S.found) S.found = k2;
         }
-        S.scur = S.cand + 1;
-        S.cand = -1;
+        const unsigned rest = S.cbits & ~(1u << (S.cand - S.scur));
+        const int nsl = (S.lb + 31 + kSlab - 1) / kSlab;
+        if (rest) {              // the next candidate of this probe window
+          S.cbits = rest;
+          S.cand = S.scur + __ffs(rest) - 1;
+        } else if (S.scur + 32 < nsl) {  // probe the next window
+          S.scur += 32;
+          S.cand = -1;
+        } else {                 // search complete: walk from the first maximum (this round if it is in
+          S.mode = kWalk;        // this block: its codes are in shared memory; phase H checks)
+          S.i = S.ei = (int)(S.found >> 32);
+          S.j = S.ej = (int)(S.found & 0xffffffffll);
+        }
       }
     }
     clk.lap(4);
@@ -695,6 +708,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         int t = i - r0 - 1;
         int c = j - d0 + (t >> 3);
         bool stop = false;
+        if (t >= kBlk || c > kSlab) t = -1;  // a search just ended outside this block: walk next round
         while (t >= 0 && c >= 1) {
           const uint32_t wd = lds_u32(cw + 4 * kGL * c + 4 * (t >> 3));
           const uint32_t ra = lds_u8(as32 + i), rb = lds_u8(bsx + j);
