@@ -278,8 +278,14 @@ __global__ void k_viterbi_tb(HmmArgs H, int64_t first, int64_t count, uint8_t* o
   const uint8_t* bp = H.bp + (p * H.max_len) * kMaxS;
   uint8_t* o = out + q * stride;
   int s = H.final_state[p];
+  // the walk is one dependent load per step; the rows it will read are known in advance, so
+  // pull them towards L2 kPf steps ahead (the back-pointers come straight from DRAM otherwise)
+  constexpr int kPf = 24;
+  for (int i = T - 1; i >= 1 && i >= T - kPf; --i)
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(bp + (int64_t)(i - 1) * kMaxS));
   for (int i = T; i >= 1; --i) {
     o[i - 1] = (uint8_t)s;
+    if (i - 1 - kPf >= 1) asm volatile("prefetch.global.L2 [%0];" ::"l"(bp + (int64_t)(i - 2 - kPf) * kMaxS));
     if (i > 1) s = bp[(int64_t)(i - 1) * kMaxS + s];
   }
   out_len[q] = T;
