@@ -114,6 +114,22 @@ def test_sw_packed_odd_batch_and_ties(dp, orc):
         assert r["scores"][q] == sc and r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
 
 
+def test_sw_long_columns_multiwindow_search(dp, orc):
+    """|b| > 993 (more than 32 checkpoint slabs: the end-cell search probes several slab
+    windows), several strips of rows, and a 3-letter alphabet so that the maximum recurs in
+    several slabs (the candidate list of one window is walked slab by slab)."""
+    g = np.random.default_rng(106)
+    sig = dpgen.blosum62()
+    a, _ = rand_batch(g, 24, 150, 600, 3)
+    b, _ = rand_batch(g, 24, 1000, 1600, 3)
+    a[0], b[0] = np.zeros(700, np.uint8), np.zeros(1500, np.uint8)   # one long run: ties everywhere
+    r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=3, asz=24)
+    for q in range(24):
+        sc, ei, ej = orc.sw(a[q], b[q], sig, 3)
+        ops, co = orc.sw_traceback(a[q], b[q], sig, 3)
+        assert r["scores"][q] == sc and r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+
+
 @pytest.mark.parametrize("maxlen,go,ge", [(40, 11, 1), (300, 11, 1), (300, 3, 2), (600, 0, 4)])
 def test_sw_affine_random_ragged(dp, orc, maxlen, go, ge):
     """Affine gaps (NEXT rank 1): ragged lengths across lane tiles and strips; scores
