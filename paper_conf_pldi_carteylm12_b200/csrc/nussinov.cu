@@ -28,6 +28,7 @@ namespace {
 
 constexpr int kNussThreads = 512;
 constexpr int64_t kSmemMaxN = 340;  // 2 n^2 bytes of int16 table <= 227 KiB
+constexpr int64_t kSmemStackN = 256;  // the traceback stack (4 n + 8 ints) also in shared memory up to here
 
 __host__ __device__ __forceinline__ int64_t ustart(int64_t i, int64_t n) { return i * n - (i * (i - 1)) / 2; }
 __host__ __device__ __forceinline__ int64_t lstart(int64_t j) { return (j * (j - 1)) / 2; }
@@ -37,26 +38,29 @@ __host__ __device__ __forceinline__ int64_t table_elems(int64_t n) { return (n *
 // Evaluate the cells of partition d assigned to this thread. `tid`/`nthr`
 // span the CTA (or the whole grid).
 __device__ __forceinline__ void nuss_partition(int16_t* U, int16_t* L, const uint8_t* x, int n, int d,
-                                               const uint8_t* pm, int h, int64_t tid, int64_t nthr) {
+                                               const uint8_t* pm, int h, int64_t tid64, int64_t nthr64) {
   const int ncells = n - d;
-  // group size G: power of two <= 32, about nthr / ncells lanes per cell, no more than the split count
-  int G = 1;
-  while (G < 32 && (int64_t)G * 2 * ncells <= nthr && G * 2 <= max(1, d - 1)) G *= 2;
-  const int64_t ngroups = nthr / G;
-  const int q = (int)(tid % G);
-  const int64_t grp = tid / G;
+  // group size G = 2^lg: power of two <= 32, about nthr / ncells lanes per cell, no more than the
+  // split count (32-bit index math, shifts: this runs once per partition per thread)
+  const int tid = (int)tid64, nthr = (int)nthr64;
+  int lg = 0;
+  while (lg < 5 && (2 << lg) * ncells <= nthr && (2 << lg) <= max(1, d - 1)) ++lg;
+  const int G = 1 << lg;
+  const int ngroups = nthr >> lg;
+  const int q = tid & (G - 1);
+  const int grp = tid >> lg;
   // every group runs the same number of iterations so the shuffles stay converged
-  const int64_t iters = (ncells + ngroups - 1) / ngroups;
-  for (int64_t it = 0; it < iters; ++it) {
-    const int64_t cidx = grp + it * ngroups;
-    const bool live = cidx < ncells && grp < ngroups;
-    const int i = live ? (int)cidx : 0;
+  const int iters = (ncells + ngroups - 1) / ngroups;
+  for (int it = 0; it < iters; ++it) {
+    const int cidx = grp + it * ngroups;
+    const bool live = cidx < ncells;
+    const int i = live ? cidx : 0;
     const int j = i + d;
     int best = 0;
     if (live) {
-      const int16_t* Ui = U + ustart(i, n);
+      const int16_t* Ui = U + ustart(i, n) - i;  // Ui[k] = gamma(i, k)
       const int16_t* Lj = L + lstart(j);
-      for (int k = i + 1 + q; k < j; k += G) best = max(best, (int)Ui[k - i] + (int)Lj[k]);
+      for (int k = i + 1 + q; k < j; k += G) best = max(best, (int)Ui[k] + (int)Lj[k]);
     }
     const unsigned mask = 0xffffffffu;
     if (G > 1) {
@@ -155,6 +159,8 @@ __global__ void __launch_bounds__(kNussThreads) k_nuss_cta(NussArgs A, int64_t s
   else tab = reinterpret_cast<int16_t*>(A.scratch) + (int64_t)blockIdx.x * slice_elems;
   int* stack = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * (SMEM ? 0 : slice_elems)) +
                (int64_t)blockIdx.x * (4 * A.max_len + 8);
+  if (SMEM && A.max_len <= kSmemStackN)  // the traceback's interval stack next to the table
+    stack = reinterpret_cast<int*>(tab + table_elems(A.max_len));
   for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
     const uint8_t* xg = A.x_cat + A.x_off[p];
     const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
@@ -249,12 +255,15 @@ cudaError_t nuss_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
   cudaGetDevice(&dev);
   const int sms = num_sms(dev);
   if (A.max_len <= kSmemMaxN) {
-    const size_t smem = ((A.max_len + 15) & ~15) + (size_t)table_elems(A.max_len) * 2;
+    const size_t smem = ((A.max_len + 15) & ~15) + (size_t)table_elems(A.max_len) * 2 +
+                        (A.max_len <= kSmemStackN ? (size_t)(4 * A.max_len + 8) * 4 : 0);
     cudaError_t e = cudaFuncSetAttribute(k_nuss_cta<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     const int64_t grid = std::min<int64_t>(A.n, (int64_t)sms * 4);
+    // a few short problems: a small CTA keeps the per-partition barrier cheap
+    const int threads = (A.n <= 2 * sms && A.max_len <= 128) ? 128 : kNussThreads;
     ++*launches;
-    k_nuss_cta<true><<<(unsigned)grid, kNussThreads, smem, s>>>(A, 0);
+    k_nuss_cta<true><<<(unsigned)grid, threads, smem, s>>>(A, 0);
     return cudaGetLastError();
   }
   if (A.n == 1) {
