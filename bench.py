@@ -569,12 +569,17 @@ def run_reference(args, rank, world):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=None,
+                    help="timed steps (default per config: ~0.15 s of steps, so the clock sampler sees the run)")
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="sw", choices=["sw", "swa", "nuss1", "hmm", "nuss4", "nuss5", "diag"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
+    if args.steps is None:  # ~0.15 s of timed steps per config (the nvidia-smi sampler runs at 20 ms)
+        args.steps = {"sw": 60, "swa": 20, "hmm": 30, "nuss1": 200, "nuss4": 15, "nuss5": 2, "diag": 25}[args.config]
+        if args.impl == "reference":
+            args.steps = 3
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
