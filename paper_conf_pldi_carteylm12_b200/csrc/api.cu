@@ -68,7 +68,7 @@ struct dp_plan {
   // chunk by chunk, overlapped with the solve of the neighbouring chunks
   DevBuf h_a, h_b, h_aoff, h_boff, h_scores, h_tb, h_tblen, h_coords;
   cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
-  static constexpr int kMaxChunks = 8;
+  static constexpr int kMaxChunks = 16;
   cudaEvent_t ev_start = nullptr, ev_in[kMaxChunks] = {}, ev_out[kMaxChunks] = {};
   int64_t launches = 0;
 };
@@ -634,8 +634,11 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   // byte q of a_cat lives at h_a + (q - a_off[0]), so the kernels take the
   // caller's (absolute) offsets with a rebased base pointer.
   // a chunk must still fill the GPU: ~3 waves of the sweep kernels
+  // (config 2, measured: 1 / 2 / 3 / 4 / 8 / 12 chunks -> 4.53 / 3.73 / 3.55 / 3.46 / 4.14 / 4.31 ms)
   const int64_t min_chunk = align ? 16384 : (p->kind == DP_NUSSINOV ? 65536 : 32768);
-  int nch = (int)std::min<int64_t>(dp_plan::kMaxChunks / 2, (n + min_chunk - 1) / min_chunk);
+  const int max_ch = getenv("DP_HOST_CHUNKS") ? std::max(1, std::min(dp_plan::kMaxChunks, atoi(getenv("DP_HOST_CHUNKS"))))
+                                              : 4;  // env: diagnostic
+  int nch = (int)std::min<int64_t>(max_ch, (n + min_chunk - 1) / min_chunk);
   if (nch < 1) nch = 1;
   const int64_t per = (n + nch - 1) / nch;
   uint8_t* da = static_cast<uint8_t*>(p->h_a.ptr);
