@@ -444,9 +444,24 @@ def e2e_host(args, W, plans, dev, stream, world):
     d2h = sum(o[0].nbytes + (o[1].nbytes + o[2].nbytes if o[1] is not None else 0) +
               (o[3].nbytes if o[3] is not None else 0) for o in outs)
 
+    streams = [stream] + [torch.cuda.Stream(device=dev) for _ in plans[1:]]
+
+    def run(k):
+        sc, tb, tl, tc = outs[k]
+        plans[k].solve_batch_host_into(a_cat, a_off, b_cat, b_off, sc, tb, stride, tl, tc, stream=streams[k])
+
     def one():
-        for p, (sc, tb, tl, tc) in zip(plans, outs):
-            p.solve_batch_host_into(a_cat, a_off, b_cat, b_off, sc, tb, stride, tl, tc, stream=stream)
+        # several plans over the same inputs (HMM forward + Viterbi) are independent calls: a user
+        # runs them from two host threads on two streams (ctypes releases the GIL)
+        if len(plans) == 1:
+            run(0)
+            return
+        import threading
+        ths = [threading.Thread(target=run, args=(k,)) for k in range(len(plans))]
+        for t in ths:
+            t.start()
+        for t in ths:
+            t.join()
 
     one()
     torch.cuda.synchronize(dev)
