@@ -192,7 +192,7 @@ def run_ours(args, rank, world, local_rank):
                              gap_open=dpgen.SW_GAP_OPEN, gap_extend=dpgen.SW_GAP_EXTEND, want_traceback=True))
         dev_in = (cu(W["a_cat"]), cu(W["a_off"]), cu(W["b_cat"]), cu(W["b_off"]))
     elif W["kind"] == "diag":
-        plans.append(dp.Plan(dp.DIAG_LCS, W["max_la"], W["max_lb"]))
+        plans.append(dp.Plan(dp.DIAG_LCS, W["max_la"], W["max_lb"], alphabet_size=4))  # DNA
         dev_in = (cu(W["a_cat"]), cu(W["a_off"]), cu(W["b_cat"]), cu(W["b_off"]))
     elif W["kind"] == "nuss":
         plans.append(dp.Plan(dp.NUSSINOV, W["max_la"], pair_mask=dpgen.rna_pair_mask(),

@@ -241,6 +241,7 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       break;
     case DP_DIAG_LCS:
       if (p->want_tb) { st = DP_E_UNSUPPORTED; break; }
+      p->asz = d->alphabet_size > 0 && d->alphabet_size <= 256 ? d->alphabet_size : 0;  // optional
       if (d->max_len_a > 40000 || d->max_len_b > 40000) st = DP_E_TOO_LARGE;  // uint16 window rows in smem
       break;
     case DP_NUSSINOV:
@@ -346,6 +347,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       A.ncand = p->ncand;
       for (int k = 0; k < p->ncand; ++k) { A.cand[k][0] = p->cand[k][0]; A.cand[k][1] = p->cand[k][1]; }
       A.force = getenv("DP_DIAG_FORCE") ? atoi(getenv("DP_DIAG_FORCE")) : p->force;  // env: diagnostic
+      A.asz = getenv("DP_DIAG_GENERIC") ? 0 : p->asz;  // env: diagnostic (the unpacked path)
       e = dpk::diag_solve(A, s, &p->launches);
       break;
     }

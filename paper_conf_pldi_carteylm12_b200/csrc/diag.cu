@@ -13,6 +13,7 @@
 // thread); longer ones double-buffer it in shared memory as uint16.
 // Choosing the schedule with fewer, longer partitions is what keeps the CTA
 // busy: a 64 x 4096 pair takes 64 barriers instead of 4096.
+#include <algorithm>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -22,6 +23,12 @@ namespace dpk {
 namespace {
 
 constexpr int kDT = 256;  // threads per CTA
+
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
+  uint32_t r;
+  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
+  return r;
+}
 
 // One partition per iteration with C cells per thread in registers: thread t owns cells
 // y = C t + 1 .. C t + C of every partition (nq <= 256 C). L(x, y) needs L(x-1, y-1): the
@@ -54,15 +61,56 @@ __device__ __forceinline__ int sweep_regs(const uint8_t* P, const uint8_t* Q, in
   return best;
 }
 
+// Small alphabets (asz <= 8): two cells per register (u16x2). Thread t owns cells
+// 2W t .. 2W t + 2W - 1; per partition it loads, for the partition's residue px, the
+// precomputed masks (0xffff in the half of a cell whose residue is px) and updates a word as
+//   L' = (shift-by-one-cell(L) + 1) & mask     (PRMT, add, LOP; no carry: values < 65535)
+// with a packed running max (VIMNMX.U16x2): ~2 ALU ops per cell instead of ~4.
+template <int W>
+__device__ __forceinline__ int sweep_packed(const uint8_t* P, const uint8_t* Q, int np, int nq, int asz,
+                                            uint32_t* msk, uint32_t* xw, int tid) {
+  const int lane = tid & 31, warp = tid >> 5;
+  // masks [code][w][tid] (conflict-free: consecutive threads, consecutive words)
+  for (int code = 0; code < asz; ++code)
+#pragma unroll
+    for (int w = 0; w < W; ++w) {
+      const int y0 = 2 * W * tid + 2 * w;
+      const uint32_t lo = (y0 < nq && Q[y0] == code) ? 0xffffu : 0u;
+      const uint32_t hi = (y0 + 1 < nq && Q[y0 + 1] == code) ? 0xffff0000u : 0u;
+      msk[(code * W + w) * kDT + tid] = lo | hi;
+    }
+  __syncthreads();
+  uint32_t L[W], acc = 0;
+#pragma unroll
+  for (int w = 0; w < W; ++w) L[w] = 0;
+  for (int x = 0; x < np; ++x) {
+    const int px = (int)P[x];
+    uint32_t m[W];
+#pragma unroll
+    for (int w = 0; w < W; ++w) m[w] = px < asz ? msk[(px * W + w) * kDT + tid] : 0u;
+    uint32_t nb = __shfl_up_sync(0xffffffffu, L[W - 1], 1);
+    if (lane == 0) nb = (warp > 0 && x > 0) ? xw[((x + 1) & 1) * (kDT / 32) + warp - 1] : 0u;  // partition x-1's
+#pragma unroll
+    for (int w = W - 1; w >= 1; --w) L[w] = (prmt(L[w - 1], L[w], 0x5432u) + 0x00010001u) & m[w];
+    L[0] = (prmt(nb, L[0], 0x5432u) + 0x00010001u) & m[0];
+#pragma unroll
+    for (int w = 0; w < W; ++w) acc = __vmaxu2(acc, L[w]);
+    if (lane == 31) xw[(x & 1) * (kDT / 32) + warp] = L[W - 1];
+    __syncthreads();
+  }
+  return (int)max(acc & 0xffffu, acc >> 16);
+}
+
 __global__ void __launch_bounds__(kDT) k_diag(DiagArgs A) {
   extern __shared__ __align__(16) uint8_t dsm[];
   const int64_t cap = A.max_len;
   uint16_t* row0 = reinterpret_cast<uint16_t*>(dsm);
   uint16_t* row1 = row0 + cap + 8;
-  uint8_t* qs = reinterpret_cast<uint8_t*>(row1 + cap + 8);
+  const size_t region = max((size_t)(2 * (cap + 8) * 2), (A.asz >= 1 && A.asz <= 8) ? (size_t)A.asz * 8 * kDT * 4 : 0);
+  uint8_t* qs = dsm + region;
   uint8_t* ps = qs + ((cap + 15) & ~int64_t(15));
   __shared__ int red[kDT / 32];
-  __shared__ int xw[2 * (kDT / 32)];
+  __shared__ uint32_t xw[2 * (kDT / 32)];
   const int tid = threadIdx.x;
   for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
     const int64_t la = A.a_off[p + 1] - A.a_off[p], lb = A.b_off[p + 1] - A.b_off[p];
@@ -86,17 +134,24 @@ __global__ void __launch_bounds__(kDT) k_diag(DiagArgs A) {
     __syncthreads();  // the previous problem's buffers are free
     for (int y = tid; y < nq; y += kDT) qs[y] = Q[y];
     for (int y = tid; y < np; y += kDT) ps[y] = P[y];
+    const bool packed = A.asz >= 1 && A.asz <= 8 && nq <= 16 * kDT;
     const bool regs = nq <= 16 * kDT;
     if (!regs)
       for (int y = tid; y <= nq; y += kDT) { row0[y] = 0; row1[y] = 0; }
     __syncthreads();
     int best = 0;
-    if (regs) {
-      if (nq <= kDT) best = sweep_regs<1>(ps, qs, np, nq, xw, tid);
-      else if (nq <= 2 * kDT) best = sweep_regs<2>(ps, qs, np, nq, xw, tid);
-      else if (nq <= 4 * kDT) best = sweep_regs<4>(ps, qs, np, nq, xw, tid);
-      else if (nq <= 8 * kDT) best = sweep_regs<8>(ps, qs, np, nq, xw, tid);
-      else best = sweep_regs<16>(ps, qs, np, nq, xw, tid);
+    if (packed) {
+      uint32_t* msk = reinterpret_cast<uint32_t*>(row0);  // the window rows are free on this path
+      if (nq <= 2 * kDT) best = sweep_packed<1>(ps, qs, np, nq, A.asz, msk, xw, tid);
+      else if (nq <= 4 * kDT) best = sweep_packed<2>(ps, qs, np, nq, A.asz, msk, xw, tid);
+      else if (nq <= 8 * kDT) best = sweep_packed<4>(ps, qs, np, nq, A.asz, msk, xw, tid);
+      else best = sweep_packed<8>(ps, qs, np, nq, A.asz, msk, xw, tid);
+    } else if (regs) {
+      if (nq <= kDT) best = sweep_regs<1>(ps, qs, np, nq, reinterpret_cast<int*>(xw), tid);
+      else if (nq <= 2 * kDT) best = sweep_regs<2>(ps, qs, np, nq, reinterpret_cast<int*>(xw), tid);
+      else if (nq <= 4 * kDT) best = sweep_regs<4>(ps, qs, np, nq, reinterpret_cast<int*>(xw), tid);
+      else if (nq <= 8 * kDT) best = sweep_regs<8>(ps, qs, np, nq, reinterpret_cast<int*>(xw), tid);
+      else best = sweep_regs<16>(ps, qs, np, nq, reinterpret_cast<int*>(xw), tid);
     } else {
       // long partitions: the window row in shared memory, every thread on a strided slice
       uint16_t* prev = row0;
@@ -126,11 +181,16 @@ __global__ void __launch_bounds__(kDT) k_diag(DiagArgs A) {
 
 }  // namespace
 
-size_t diag_smem_bytes(int64_t max_len) { return (size_t)(2 * (max_len + 8) * 2 + 2 * ((max_len + 15) & ~int64_t(15))); }
+size_t diag_smem_bytes(int64_t max_len, int asz) {
+  // window rows (generic path) or, aliased, the masks of the packed path (asz x 8 words x 256)
+  const size_t rows = (size_t)(2 * (max_len + 8) * 2);
+  const size_t masks = (asz >= 1 && asz <= 8) ? (size_t)asz * 8 * kDT * 4 : 0;
+  return std::max(rows, masks) + 2 * ((max_len + 15) & ~int64_t(15));
+}
 
 cudaError_t diag_solve(const DiagArgs& A, cudaStream_t s, int64_t* launches) {
   if (A.n == 0) return cudaSuccess;
-  const size_t smem = diag_smem_bytes(A.max_len);
+  const size_t smem = diag_smem_bytes(A.max_len, A.asz);
   cudaError_t e = cudaFuncSetAttribute(k_diag, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0, per_sm = 0;

@@ -91,8 +91,9 @@ struct DiagArgs {
   int32_t cand[24][2];   // §4.7 candidate schedules (dp_schedule_conditional)
   int ncand;
   int force;             // -1: run-time choice per problem; else that candidate (diagnostic)
+  int asz;               // alphabet size if known (<= 8: packed two-cells-per-register path), else 0
 };
-size_t diag_smem_bytes(int64_t max_len);
+size_t diag_smem_bytes(int64_t max_len, int asz);
 cudaError_t diag_solve(const DiagArgs& a, cudaStream_t s, int64_t* launches);
 
 // ---------------------------------------------------------------- Nussinov

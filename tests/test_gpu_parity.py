@@ -445,10 +445,11 @@ def run_diag(dp, a_seqs, b_seqs, **kw):
         return host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=la, max_len_b=lb))
 
 
-@pytest.mark.parametrize("force", [None, "0", "1"])
-def test_diag_mixed_shapes(dp, orc, monkeypatch, force):
+@pytest.mark.parametrize("force,asz", [(None, 0), ("0", 0), ("1", 0), (None, 4), ("0", 4), ("1", 4)])
+def test_diag_mixed_shapes(dp, orc, monkeypatch, force, asz):
     """Ragged tall and wide pairs, empty sides, length 1: bit-exact against the oracle under the
-    run-time schedule choice and under each candidate forced (the result cannot depend on it)."""
+    run-time schedule choice and under each candidate forced (the result cannot depend on it),
+    with the alphabet unknown (one cell per register) and given (asz = 4: two per register)."""
     if force is not None:
         monkeypatch.setenv("DP_DIAG_FORCE", force)
     g = np.random.default_rng(800)
@@ -459,7 +460,7 @@ def test_diag_mixed_shapes(dp, orc, monkeypatch, force):
     a[5], b[5] = np.full(257, 2, np.uint8), np.full(33, 2, np.uint8)   # a run: the answer is 33
     a[6], b[6] = g.integers(0, 4, 60).astype(np.uint8), g.integers(0, 4, 4500).astype(np.uint8)  # > 4096: smem path
     a[7], b[7] = g.integers(0, 2, 5000).astype(np.uint8), g.integers(0, 2, 3000).astype(np.uint8)
-    got = run_diag(dp, a, b)
+    got = run_diag(dp, a, b, alphabet_size=asz)
     want = np.array([orc.lcsubstr(x, y) for x, y in zip(a, b)])
     assert (got == want).all()
     assert got[5] == 33
@@ -469,10 +470,12 @@ def test_diag_workload_sampled(dp, orc):
     """The bench workload's distribution (log-uniform 32..4096 per side), first 120 pairs."""
     a_cat, a_off, b_cat, b_off = dpgen.diag_pairs(120)
     la, lb = int(np.diff(a_off).max()), int(np.diff(b_off).max())
-    with dp.Plan(dp.DIAG_LCS, la, lb) as plan:
-        got = host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=la, max_len_b=lb))
     want = orc.lcsubstr_batch(a_cat, a_off, b_cat, b_off, threads=THREADS)
-    assert (got == want).all()
+    for asz in (0, 4):
+        with dp.Plan(dp.DIAG_LCS, la, lb, alphabet_size=asz) as plan:
+            got = host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=la,
+                                        max_len_b=lb))
+        assert (got == want).all(), asz
 
 
 def test_diag_plan_schedules(dp):
