@@ -6,6 +6,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <new>
+#include <utility>
 #include <vector>
 #include <cuda_runtime.h>
 
@@ -58,6 +59,8 @@ struct dp_plan {
   int32_t *d_lpi = nullptr, *d_lA = nullptr, *d_lE = nullptr;
   // retained state of the most recent solve
   DevBuf tb_state, tb_aux, tb_aux2, scratch;
+  DevBuf tb_state_alt;             // host entry point: the other chunk's retained state (packed SW)
+  cudaStream_t s_cmp = nullptr;    // host entry point: second compute stream (packed SW)
   int64_t last_n = -1;
   int64_t last_max_la = 0, last_max_lb = 0;
   const uint8_t *last_a = nullptr, *last_b = nullptr;
@@ -187,6 +190,8 @@ void dp_plan_destroy(dp_plan_t p) {
                     &p->h_aoff, &p->h_boff, &p->h_scores, &p->h_tb, &p->h_tblen, &p->h_coords};
   for (DevBuf* b : bufs) b->release();
   if (p->s_h2d) cudaStreamDestroy(p->s_h2d);
+  if (p->s_cmp) cudaStreamDestroy(p->s_cmp);
+  p->tb_state_alt.release();
   if (p->s_d2h) cudaStreamDestroy(p->s_d2h);
   if (p->ev_start) cudaEventDestroy(p->ev_start);
   for (int k = 0; k < dp_plan::kMaxChunks; ++k) {
@@ -652,29 +657,48 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   if (e == cudaSuccess) e = cudaMemcpyAsync(dao, a_off, (n + 1) * 8, cudaMemcpyHostToDevice, p->s_h2d);
   if (e == cudaSuccess && align) e = cudaMemcpyAsync(dbo, b_off, (n + 1) * 8, cudaMemcpyHostToDevice, p->s_h2d);
   if (e != cudaSuccess) return cuda_status(e);
+  // Packed SW keeps all of a solve's retained state in tb_state, so consecutive chunks can
+  // alternate between two compute streams and two state buffers: chunk c+1's sweep then fills the
+  // SMs while chunk c's traceback drains (other kinds stay on the caller's stream).
+  const bool two = p->kind == DP_SW_LINEAR && p->packed16 && nch > 1;
+  if (two && !p->s_cmp) {
+    e = cudaStreamCreateWithFlags(&p->s_cmp, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(p->s_cmp, p->ev_start, 0);
+    if (e != cudaSuccess) return cuda_status(e);
+  } else if (two) {
+    e = cudaStreamWaitEvent(p->s_cmp, p->ev_start, 0);
+    if (e != cudaSuccess) return cuda_status(e);
+  }
+  int installed = 0;  // which state buffer is in p->tb_state
   for (int c = 0; c < nch; ++c) {
     const int64_t k0 = c * per, k1 = std::min(n, k0 + per), nk = k1 - k0;
     if (nk <= 0) break;
+    const cudaStream_t sc = (two && (c & 1)) ? p->s_cmp : s;
+    void* const scv = reinterpret_cast<void*>(sc);
+    if (two && (c & 1) != installed) {
+      std::swap(p->tb_state, p->tb_state_alt);
+      installed = c & 1;
+    }
     e = cudaMemcpyAsync(da + (a_off[k0] - a_off[0]), a_cat + a_off[k0], a_off[k1] - a_off[k0],
                         cudaMemcpyHostToDevice, p->s_h2d);
     if (e == cudaSuccess && align)
       e = cudaMemcpyAsync(db + (b_off[k0] - b_off[0]), b_cat + b_off[k0], b_off[k1] - b_off[k0],
                           cudaMemcpyHostToDevice, p->s_h2d);
     if (e == cudaSuccess) e = cudaEventRecord(p->ev_in[c], p->s_h2d);
-    if (e == cudaSuccess) e = cudaStreamWaitEvent(s, p->ev_in[c], 0);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(sc, p->ev_in[c], 0);
     if (e != cudaSuccess) return cuda_status(e);
     int32_t* dsc = static_cast<int32_t*>(p->h_scores.ptr) + k0;
     dp_status st = dp_solve_batch(p, nk, da - a_off[0], dao + k0, align ? db - b_off[0] : nullptr,
-                                  align ? dbo + k0 : nullptr, max_la, max_lb, dsc, stream);
+                                  align ? dbo + k0 : nullptr, max_la, max_lb, dsc, scv);
     if (st != DP_OK) return st;
     uint8_t* dtb = tb ? static_cast<uint8_t*>(p->h_tb.ptr) + k0 * tb_stride : nullptr;
     int32_t* dtl = tb ? static_cast<int32_t*>(p->h_tblen.ptr) + k0 : nullptr;
     int32_t* dco = (tb && tb_coords) ? static_cast<int32_t*>(p->h_coords.ptr) + 4 * k0 : nullptr;
     if (tb) {
-      st = dp_traceback(p, 0, nk, dtb, tb_stride, dtl, dco, stream);
+      st = dp_traceback(p, 0, nk, dtb, tb_stride, dtl, dco, scv);
       if (st != DP_OK) return st;
     }
-    e = cudaEventRecord(p->ev_out[c], s);
+    e = cudaEventRecord(p->ev_out[c], sc);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(p->s_d2h, p->ev_out[c], 0);
     if (e == cudaSuccess)
       e = cudaMemcpyAsync(static_cast<uint8_t*>(scores_out) + 4 * k0, dsc, nk * 4, cudaMemcpyDeviceToHost, p->s_d2h);
@@ -686,6 +710,7 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   }
   e = cudaStreamSynchronize(p->s_d2h);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e == cudaSuccess && two) e = cudaStreamSynchronize(p->s_cmp);
   return cuda_status(e);
 }
 

@@ -435,6 +435,30 @@ def test_host_entry_point(dp, orc):
     plan.close()
 
 
+def test_host_entry_point_chunked(dp, orc):
+    """A batch large enough for several chunks (packed SW alternates two compute streams and two
+    retained-state buffers): the host path equals the device path everywhere and the oracle on a
+    sample spread over the chunks."""
+    import torch
+    n = 70_000
+    a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(n)
+    sig = dpgen.blosum62()
+    plan = dp.Plan(dp.SW_LINEAR, 256, 256, sigma=sig, gap=dpgen.SW_GAP, want_traceback=True)
+    sc, tb, tbl, tbc = plan.solve_batch_host(a_cat, a_off, b_cat, b_off, tb_stride=513)
+    dsc = host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=256, max_len_b=256))
+    out, ln, co = plan.traceback(0, n, 513)
+    torch.cuda.synchronize()
+    assert (sc == dsc).all()
+    assert (tbl == host(ln)).all() and (tbc == host(co)).all()
+    used = np.arange(513)[None, :] < tbl[:, None]  # bytes past a row's length are unspecified
+    assert (tb[used] == host(out)[used]).all()
+    for q in range(0, n, 1750):
+        x, y = a_cat[a_off[q]:a_off[q + 1]], b_cat[b_off[q]:b_off[q + 1]]
+        ops, c = orc.sw_traceback(x, y, sig, dpgen.SW_GAP)
+        assert sc[q] == orc.sw(x, y, sig, dpgen.SW_GAP)[0] and bytes(tb[q, :tbl[q]]).decode() == ops
+    plan.close()
+
+
 # ----------------------------------------------------------------------------- §4.7 diagonal-only
 def run_diag(dp, a_seqs, b_seqs, **kw):
     a_cat, a_off = dpgen.pack(a_seqs)
