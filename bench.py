@@ -126,14 +126,14 @@ def workload(name, rank, world):
         x = dpgen.config1_rna64()
         cat, off = dpgen.pack([x])
         n = 64
-        return {"kind": "nuss", "n": 1, "a_cat": cat, "a_off": off, "max_la": 64, "cells": n * (n - 1) // 2,
+        return {"kind": "nuss", "config": "nuss1", "n": 1, "a_cat": cat, "a_off": off, "max_la": 64, "cells": n * (n - 1) // 2,
                 "inner": sum((64 - d) * (d - 1) for d in range(1, 64)), "tb_stride": 64,
                 "workload": "BASELINE config 1: one 64-nt RNA, Nussinov (h=3, WC+GU), with traceback"}
     if name == "nuss4":
         x = dpgen.config4_rna8192()
         cat, off = dpgen.pack([x])
         n = 8192
-        return {"kind": "nuss", "n": 1, "a_cat": cat, "a_off": off, "max_la": n, "cells": n * (n - 1) // 2,
+        return {"kind": "nuss", "config": "nuss4", "n": 1, "a_cat": cat, "a_off": off, "max_la": n, "cells": n * (n - 1) // 2,
                 "inner": sum((n - d) * (d - 1) for d in range(1, n)), "tb_stride": n,
                 "workload": "BASELINE config 4: one 8192-nt RNA, Nussinov grid-wide hyperplane sweep, with traceback"}
     if name == "nuss5":
@@ -141,7 +141,7 @@ def workload(name, rank, world):
         nseq = int(os.environ.get("DP_NUSS5_N", nseq))
         cat, off = dpgen.config5_rna_batch(nseq)
         lens = np.diff(off)
-        return {"kind": "nuss", "n": nseq, "a_cat": cat, "a_off": off, "max_la": int(lens.max()),
+        return {"kind": "nuss", "config": "nuss5", "n": nseq, "a_cat": cat, "a_off": off, "max_la": int(lens.max()),
                 "cells": int((lens * (lens - 1) // 2).sum()),
                 "inner": int((lens * (lens - 1) * (lens - 2) // 6).sum()), "tb_stride": 512,
                 "workload": "BASELINE config 5: RNAs of length U[128,512], Nussinov batch, with tracebacks"}
@@ -401,7 +401,8 @@ def roofline(W, phase_ms, pk):
         return alu("k_diag", W["cells"] * W["ops_per_cell"], phase_ms[0], peak32,
                    "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (3 int ops per cell)")
     if W["kind"] == "nuss":
-        return alu("k_nuss_tiled (fill + traceback)", W["inner"], phase_ms[0], peak16,
+        kname = {"nuss1": "k_nuss_cta", "nuss4": "k_nuss_grid2", "nuss5": "k_nuss_batch"}.get(W.get("config"), "k_nuss")
+        return alu(kname + " (fill + traceback)", W["inner"], phase_ms[0], peak16,
                    "ubench_r01 VIADDMNMX.S16x2 x 148 SMs x sm_max_mhz (one split evaluation = one max-plus)")
     # HMM: Viterbi (max-plus, SIMT) vs the tcgen05 forward
     vit = alu("k_viterbi", W["inner"], phase_ms[1], peak32,

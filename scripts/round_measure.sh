@@ -5,12 +5,12 @@ nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > gp
 python -m pytest tests -m gpu -q 2>&1 | tail -3 > gpurun_out/gpu_tests.log
 python bench.py 2>gpurun_out/bench_sw.err | tail -1 > gpurun_out/bench_sw.json
 python bench.py --impl reference --steps 3 --warmup 1 2>/dev/null | tail -1 > gpurun_out/bench_ref.json
-python bench.py --config swa --steps 5 --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_swa.json
-python bench.py --config hmm --steps 5 --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_hmm.json
-python bench.py --config nuss1 --steps 20 --warmup 5 2>/dev/null | tail -1 > gpurun_out/bench_nuss1.json
-python bench.py --config nuss4 --steps 3 --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_nuss4.json
+python bench.py --config swa --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_swa.json
+python bench.py --config hmm --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_hmm.json
+python bench.py --config nuss1 --warmup 5 2>/dev/null | tail -1 > gpurun_out/bench_nuss1.json
+python bench.py --config nuss4 --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_nuss4.json
 python bench.py --config nuss5 --steps 2 --warmup 3 2>gpurun_out/bench_nuss5.err | tail -1 > gpurun_out/bench_nuss5.json
-python bench.py --config diag --steps 5 --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_diag.json
+python bench.py --config diag --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_diag.json
 ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_sw.csv python bench.py --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
 ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_hmm.csv python bench.py --config hmm --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
 ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_nuss4.csv python bench.py --config nuss4 --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
