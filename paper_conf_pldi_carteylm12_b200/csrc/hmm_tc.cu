@@ -22,7 +22,9 @@
 // Operands live in shared memory (alpha hi/lo 2 x 16 KB, transitions 16 KB);
 // the accumulator lives in TMEM (128 columns). DP_HMM_TIMING=1 prints per-phase
 // step times of CTA 0 (diagnostic).
+#include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
@@ -291,7 +293,10 @@ bool hmm_forward_tc_supported(int S) { return S <= kS && getenv("DP_HMM_SIMT") =
 
 cudaError_t hmm_forward_tc(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
   if (H.n == 0) return cudaSuccess;
-  const size_t smem = sizeof(TcSmem) + 1024;
+  // The step is a latency chain (MMA -> epilogue -> MMA): reserving the SM's shared memory keeps
+  // other kernels' CTAs (e.g. a concurrent Viterbi) off the SMs running it. DP_HMM_TC_SHARE=1: no.
+  const size_t need = sizeof(TcSmem) + 1024;
+  const size_t smem = getenv("DP_HMM_TC_SHARE") ? need : std::max(need, (size_t)200 * 1024);
   cudaError_t e = cudaFuncSetAttribute(k_forward_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   ++*launches;
