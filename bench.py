@@ -242,16 +242,14 @@ def run_ours(args, rank, world, local_rank):
         with torch.cuda.stream(stream):
             marks = [ev()] if timed else None
             if side is not None:
-                # the forward is submitted first, on the main stream, so its CTAs are resident before
-                # Viterbi's flood the SMs (it reserves its SMs' shared memory: no co-resident CTAs)
-                f0 = marks[0] if timed else None
-                plans[0].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[0], stream=stream)
-                f1 = ev()
-                side.wait_event(marks[0] if timed else ev())
-                v0 = ev(side) if timed else None
-                plans[1].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[1], stream=side)
+                side.wait_event(ev())
+                f0 = ev(side) if timed else None
+                plans[0].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[0], stream=side)
+                f1 = ev(side)
+                v0 = ev() if timed else None
+                plans[1].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[1], stream=stream)
                 if timed:
-                    marks = [f0, f1, v0, ev(side)]
+                    marks = [f0, f1, v0, ev()]
             else:
                 for k, p in enumerate(plans):
                     p.solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=W.get("max_lb", 0), out=scores[k],
@@ -259,9 +257,9 @@ def run_ours(args, rank, world, local_rank):
                     if timed:
                         marks.append(ev())
             if tb_plan is not None:
-                tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=side if side is not None else stream)
+                tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
             if side is not None:
-                stream.wait_stream(side)
+                stream.wait_event(f1)
             if timed:
                 if tb_plan is not None:
                     marks.append(ev())
