@@ -54,7 +54,10 @@ constexpr int kTileWords = T * T;      // int16 per tile record half
 constexpr int kRec = 2 * kTileWords;   // int16 per tile record (UT + L)
 constexpr int kCtaWarps = 2;   // batch driver: eight CTAs (eight sequences) per SM
 constexpr int kCtaPerSm = 8;
-constexpr int kGridWarps = 16; // grid driver
+#ifndef NUSS_GRID_WARPS
+#define NUSS_GRID_WARPS 8   // 8 measured best for config 4 (16: 10.6 ms, 12: 9.7, 8: 8.75, 4: 9.3)
+#endif
+constexpr int kGridWarps = NUSS_GRID_WARPS;  // grid driver
 constexpr int kGridMin = 1024;         // single problems longer than this use the whole grid
 
 __host__ __device__ __forceinline__ int64_t tile_id(int I, int J, int nt) {
