@@ -1184,7 +1184,8 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
   }
   if (A.max_len > 4096) return cudaErrorInvalidValue;  // batch path keeps the sequence in shared memory
   if (!use_v1()) {
-    const int per_sm = batch_ctas_per_sm(A.max_len);
+    int per_sm = batch_ctas_per_sm(A.max_len);
+    if (getenv("DP_NUSS_BATCH_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(getenv("DP_NUSS_BATCH_PER_SM"))));  // diagnostic
     const int64_t grid = std::min<int64_t>(A.n, (int64_t)per_sm * sms);
     ++*launches;
     k_nuss_batch<<<(unsigned)grid, 32, batch_warp_bytes(A.max_len), s>>>(A, batch_slot_words(A.max_len));
