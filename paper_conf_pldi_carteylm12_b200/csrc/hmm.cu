@@ -20,7 +20,9 @@
 // packed keys key(p) = V(p) * 64 + (63 - p), so one VIADDMNMX per (p, s) yields
 // both the max and the argmax; V is renormalised by its max every 32 steps
 // (exact integer offset kept in int64) so keys never overflow.
+#include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "dp_internal.h"
@@ -301,9 +303,9 @@ int sms_of_current() {
 template <int NS>
 void* fwd_ptr(bool viterbi) { return viterbi ? (void*)k_viterbi<NS> : (void*)k_forward<NS>; }
 
-// Sequences per warp: minimise (waves of resident warps) x (NS + 2): the per-warp
-// time grows with NS plus a latency term (the per-step reduction and the
-// broadcast) that NS independent sequences share; ties go to the smaller NS.
+// Sequences per warp: minimise (waves of resident warps) x (NS + latency term): the per-warp
+// time grows with NS plus (forward) a latency term that NS independent sequences share;
+// ties go to the smaller NS.
 int pick_ns(int64_t n, bool viterbi, void** kern) {
   void* ks[8] = {fwd_ptr<1>(viterbi), fwd_ptr<2>(viterbi), fwd_ptr<3>(viterbi), fwd_ptr<4>(viterbi),
                  fwd_ptr<5>(viterbi), fwd_ptr<6>(viterbi), fwd_ptr<7>(viterbi), fwd_ptr<8>(viterbi)};
@@ -316,9 +318,12 @@ int pick_ns(int64_t n, bool viterbi, void** kern) {
       continue;
     const int64_t warps = (n + ns - 1) / ns;
     const int64_t wave = (int64_t)sms * per_sm * kHW;
-    const int64_t cost = ((warps + wave - 1) / wave) * (ns + 2);
+    // Viterbi: measured (10k x 1000, S = 64) NS = 1 / 2 / 3 / 4 -> 2.99 / 3.57 / 3.86 / 3.95 ms, so no
+    // latency term; the SIMT forward keeps it
+    const int64_t cost = ((warps + wave - 1) / wave) * (ns + (viterbi ? 0 : 2));
     if (cost < best_cost) { best_cost = cost; best = ns; }
   }
+  if (getenv("DP_HMM_NS")) best = std::max(1, std::min(8, atoi(getenv("DP_HMM_NS"))));  // diagnostic
   *kern = ks[best - 1];
   return best;
 }
