@@ -34,6 +34,9 @@
 namespace dpk {
 namespace {
 
+#ifndef SW16_UNROLL
+#define SW16_UNROLL 16  // steady-loop unroll (2 / 4 / 8 / 16 / 32: sweep 1.344 / 1.268 / 1.234 / 1.225 / 1.224 ms)
+#endif
 constexpr int kRows = 8;              // rows per lane
 constexpr int kStrip = 32 * kRows;    // rows per strip
 constexpr int kBand = 16;             // checkpoint band height (two lanes)
@@ -255,7 +258,7 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
     // the G above it there (corner), and its best G over the block.
     const uint32_t rec0 = sh_rec + kRec * (kPad - lane);
     const int K = lbm + 31;
-    constexpr int U = 4;
+    constexpr int U = SW16_UNROLL;
     for (int kb = 0, sl = 0; kb < K; kb += kSlab, ++sl) {
       const int ke = min(kb + kSlab, K);
       // steady range: lane 31 at j >= 1 and lane 0 at j <= lbm - 1
