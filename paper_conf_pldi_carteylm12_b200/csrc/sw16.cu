@@ -340,8 +340,12 @@ constexpr int kTbWarps = 4;              // warps per CTA
 constexpr int kGL = TB_GL;               // 2: blocks of 16 rows (one checkpoint band), 4: 32 rows
 constexpr int kGroups = 32 / kGL;        // groups per warp
 constexpr int kBlk = kRows * kGL;        // traceback block height
+#ifndef TB5_UNROLL
+#define TB5_UNROLL 1   // 1 / 2 / 4 / 8 / 32: traceback 1.06 / 1.10 / 1.16 / 1.22 / 1.63 ms (register pressure)
+#endif
+constexpr int kTbUnroll = TB5_UNROLL;   // re-run steps unrolled
 #ifndef TB5_MINB
-#define TB5_MINB 5                       // CTAs per SM (register cap)
+#define TB5_MINB 4                       // CTAs per SM (register cap; 4 / 5 / 6 with no unroll: 1.049 / 1.059 / 1.099 ms)
 #endif
 constexpr int kCW = kGL * kSlab;         // code words per group: [c - 1][m]
 constexpr int kTS = 36;                  // top-row keys per group, c = 0..32
@@ -622,7 +626,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
     {
       const uint32_t bA = bs32 + (3 - m), bB = bs32 + kBS + (3 - m);
       const uint32_t cw0 = cs32 + 4 * m;
-#pragma unroll 4
+#pragma unroll kTbUnroll
       for (int c = 1; c <= kSlab; ++c) {
         const uint32_t topv = lds_u32(ts32 + 4 * c);
         const uint32_t fa = __shfl_up_sync(full, Kc[kRows - 1], 1, kGL);
