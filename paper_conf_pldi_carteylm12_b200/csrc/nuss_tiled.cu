@@ -42,6 +42,10 @@ namespace dpk {
 namespace {
 
 constexpr int T = 32;
+#ifndef NUSS_MICRO_UNROLL
+#define NUSS_MICRO_UNROLL 8
+#endif
+constexpr int kMicroUnroll = NUSS_MICRO_UNROLL;  // phase-A micro-kernel k loop
 #ifndef NUSS_TBW_G
 #define NUSS_TBW_G 8   // traceback gamma window (W x W per round trip) and split-search width (32 KC) of the grid
 #define NUSS_TBK_G 1   // sweep (16 / 2 measured no faster)
@@ -108,7 +112,7 @@ __device__ __forceinline__ void stage(const int16_t* __restrict__ ut, const int1
 // acc[4 rows][4 pairs] = max(acc, A (x) B) over the 32 k of one staged K tile.
 __device__ __forceinline__ void micro(const uint32_t* As, const uint16_t* Bs, uint32_t (&acc)[16], int lane) {
   const int ty = lane >> 2, tx = lane & 3;
-#pragma unroll 8
+#pragma unroll kMicroUnroll
   for (int k = 0; k < T; ++k) {
     const uint4 a = *reinterpret_cast<const uint4*>(As + k * T + 4 * ty);
     const uint4 b = *reinterpret_cast<const uint4*>(Bs + k * T + 8 * tx);
