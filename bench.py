@@ -231,7 +231,8 @@ def run_ours(args, rank, world, local_rank):
     # HMM: the forward (tensor cores, latency-bound on ~n/128 SMs) and Viterbi (ALU) are
     # independent passes over the same sequences; the forward runs on a side stream so the
     # Viterbi kernel fills the SMs the forward leaves idle.
-    side = torch.cuda.Stream(device=dev) if W["kind"] == "hmm" else None  # (a high-priority side stream measured slower: 4.92 vs 4.77 ms)
+    side = torch.cuda.Stream(device=dev) if W["kind"] == "hmm" else None
+    fwd_first = os.environ.get("DP_BENCH_FWD_FIRST", "0") == "1"  # (a high-priority side stream measured slower: 4.92 vs 4.77 ms)
 
     def ev(st=None):
         e = torch.cuda.Event(enable_timing=True)
@@ -241,7 +242,18 @@ def run_ours(args, rank, world, local_rank):
     def step(timed):
         with torch.cuda.stream(stream):
             marks = [ev()] if timed else None
-            if side is not None:
+            if side is not None and fwd_first:
+                # forward submitted first on the main stream (its CTAs resident before Viterbi's flood
+                # the SMs; it reserves its SMs' shared memory), Viterbi + traceback on the side stream
+                f0 = marks[0] if timed else None
+                plans[0].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[0], stream=stream)
+                f1 = ev()
+                side.wait_event(marks[0] if timed else ev())
+                v0 = ev(side) if timed else None
+                plans[1].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[1], stream=side)
+                if timed:
+                    marks = [f0, f1, v0, ev(side)]
+            elif side is not None:
                 side.wait_event(ev())
                 f0 = ev(side) if timed else None
                 plans[0].solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=0, out=scores[0], stream=side)
@@ -257,9 +269,13 @@ def run_ours(args, rank, world, local_rank):
                     if timed:
                         marks.append(ev())
             if tb_plan is not None:
-                tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
+                tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co,
+                                       stream=side if (side is not None and fwd_first) else stream)
             if side is not None:
-                stream.wait_event(f1)
+                if fwd_first:
+                    stream.wait_stream(side)
+                else:
+                    stream.wait_event(f1)
             if timed:
                 if tb_plan is not None:
                     marks.append(ev())

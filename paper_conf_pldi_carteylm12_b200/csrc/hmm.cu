@@ -156,6 +156,9 @@ __global__ void __launch_bounds__(kHW * 32) k_forward(HmmArgs H) {
   }
 }
 
+#ifndef VIT_TB_PF
+#define VIT_TB_PF 24  // Viterbi traceback: back-pointer rows prefetched ahead (24 / 64 / 128: same)
+#endif
 constexpr int kNegKey = -(1 << 30);
 constexpr int kRenorm = 32;
 
@@ -282,7 +285,7 @@ __global__ void k_viterbi_tb(HmmArgs H, int64_t first, int64_t count, uint8_t* o
   int s = H.final_state[p];
   // the walk is one dependent load per step; the rows it will read are known in advance, so
   // pull them towards L2 kPf steps ahead (the back-pointers come straight from DRAM otherwise)
-  constexpr int kPf = 24;
+  constexpr int kPf = VIT_TB_PF;
   for (int i = T - 1; i >= 1 && i >= T - kPf; --i)
     asm volatile("prefetch.global.L2 [%0];" ::"l"(bp + (int64_t)(i - 1) * kMaxS));
   for (int i = T; i >= 1; --i) {
