@@ -420,7 +420,7 @@ def roofline(W, phase_ms, pk):
         return alu("k_diag", W["cells"] * W["ops_per_cell"], phase_ms[0], peak32,
                    "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (3 int ops per cell)")
     if W["kind"] == "nuss":
-        kname = {"nuss1": "k_nuss_cta", "nuss4": "k_nuss_grid2", "nuss5": "k_nuss_batch"}.get(W.get("config"), "k_nuss")
+        kname = {"nuss1": "k_nuss_batch", "nuss4": "k_nuss_grid2", "nuss5": "k_nuss_batch"}.get(W.get("config"), "k_nuss")
         return alu(kname + " (fill + traceback)", W["inner"], phase_ms[0], peak16,
                    "ubench_r01 VIADDMNMX.S16x2 x 148 SMs x sm_max_mhz (one split evaluation = one max-plus)")
     # HMM: Viterbi (max-plus, SIMT) vs the tcgen05 forward

@@ -416,7 +416,8 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       }
       // cell-level CTA kernel (table in shared memory) for short sequences, tiled
       // max-plus kernels above (SURVEY §8(a) A6b'); DP_NUSS_CELL=1 forces the cell level
-      const int64_t tiled_min = getenv("DP_NUSS_TILED_MIN") ? atoll(getenv("DP_NUSS_TILED_MIN")) : 128;
+      // (config 1, n = 64: tiled 0.097 ms per step vs 0.109 cell-level)
+      const int64_t tiled_min = getenv("DP_NUSS_TILED_MIN") ? atoll(getenv("DP_NUSS_TILED_MIN")) : 32;
       const bool tiled = A.max_len > tiled_min && getenv("DP_NUSS_CELL") == nullptr &&
                          (n == 1 || A.max_len <= 4096);
       A.scratch_bytes = tiled ? dpk::nuss_tiled_scratch_bytes(A.max_len, n, p->device)
