@@ -46,6 +46,10 @@ constexpr int T = 32;
 #define NUSS_MICRO_UNROLL 8
 #endif
 constexpr int kMicroUnroll = NUSS_MICRO_UNROLL;  // phase-A micro-kernel k loop
+#ifndef NUSS_WAVE_UNROLL
+#define NUSS_WAVE_UNROLL 1   // 1 / 2 / 4: config 5 subset 195 / 233 / 288 ms (registers)
+#endif
+constexpr int kWaveUnroll = NUSS_WAVE_UNROLL;    // in-tile wavefront steps
 #ifndef NUSS_TBW_G
 #define NUSS_TBW_G 8   // traceback gamma window (W x W per round trip) and split-search width (32 KC) of the grid
 #define NUSS_TBK_G 1   // sweep (16 / 2 measured no faster)
@@ -239,7 +243,7 @@ __device__ __forceinline__ void wavefront(InTileBuf& B, bool diag, int left, int
   // local anti-diagonal dl); the steps run in segments of constant NQ, fully unrolled.
   auto seg = [&](auto nqc, int dlA, int dlB) {
     constexpr int NQ = decltype(nqc)::value;
-#pragma unroll 1
+#pragma unroll kWaveUnroll
     for (int dl = dlA; dl <= dlB; ++dl) {
       const int c = r + dl;
       const bool live = c >= 0 && c < T;
