@@ -124,8 +124,10 @@ def config1_rna64() -> np.ndarray:
 def config2_protein_pairs(n_pairs: int = 100_000, length: int = 256, first: int = 0):
     """D2: n_pairs protein pairs of the given length, seed 20120611+2.
 
-    Returns (a_cat, a_off, b_cat, b_off). `first` skips that many pairs of the
-    same stream (so a bounded sample is a prefix-consistent slice)."""
+    Returns (a_cat, a_off, b_cat, b_off): pairs [first, first + n_pairs) of the
+    stream drawn for first + n_pairs pairs (all a rows, then all b rows). The a
+    sequences are prefix-consistent across totals, the b sequences are NOT: a
+    shard of a larger batch must be sliced from that batch (bench.py does)."""
     g = rng(2)
     total = first + n_pairs
     a = g.integers(0, 20, size=(total, length), dtype=np.uint8)

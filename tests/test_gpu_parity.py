@@ -1,6 +1,10 @@
 """GPU parity: the CUDA path (through the C ABI) against the oracle, element by
 element on seeded inputs. Integer scores and tracebacks bit-exact; forward
-log-likelihoods within relative 1e-5 (north_star)."""
+log-likelihoods within relative 1e-5 of log P (north_star; DESIGN.md §2
+"Tolerances"), the achieved error printed in nats."""
+import concurrent.futures
+import hashlib
+import json
 import os
 
 import numpy as np
@@ -98,6 +102,30 @@ def test_sw_int32_kernel_path(dp, orc, monkeypatch):
         assert r["scores"][q] == orc.sw(a[q], b[q], sig, 4)[0], q
         ops, co = orc.sw_traceback(a[q], b[q], sig, 4)
         assert r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+
+
+def test_sw_s16_guard_crosses_to_int32(dp, orc):
+    """a plan whose score bound does not fit the s16x2 keys takes the int32
+    kernels automatically (no environment override). Identical high-scoring sequences make the
+    real scores exceed the s16 traceback keys (4 x score > 32767) and, score-only, exceed int16."""
+    g = np.random.default_rng(107)
+    asz = 8
+    sig = np.full((asz, asz), -2, np.int8)
+    np.fill_diagonal(sig, 60)
+    a = [g.integers(0, asz, size=int(l)).astype(np.uint8) for l in (200, 150, 260, 40)]
+    b = [x.copy() for x in a]
+    b[1][70] = (b[1][70] + 1) % asz
+    r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=5, asz=asz)
+    assert r["scores"][0] == 60 * 200 > 7900
+    for q in range(4):
+        sc, _, _ = orc.sw(a[q], b[q], sig, 5)
+        ops, co = orc.sw_traceback(a[q], b[q], sig, 5)
+        assert r["scores"][q] == sc and r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+    sig2 = np.full((asz, asz), -2, np.int8)
+    np.fill_diagonal(sig2, 127)
+    a2 = [g.integers(0, asz, size=300).astype(np.uint8)]
+    r2 = run_align(dp, dp.SW_LINEAR, a2, [a2[0].copy()], sigma=sig2, gap=5, asz=asz, tb=False)
+    assert r2["scores"][0] == 127 * 300 == orc.sw(a2[0], a2[0], sig2, 5)[0] > 32767
 
 
 def test_sw_packed_odd_batch_and_ties(dp, orc):
@@ -293,23 +321,61 @@ def test_nussinov_grid_sweep(dp, orc):
     assert r["scores"][0] == sc and r["db"][0] == db
 
 
-def test_nussinov_config4_properties(dp):
-    """n = 8192 (oracle ~20+ min): the structure is valid and has score-many pairs."""
+def test_nussinov_config4_golden(dp):
+    """BASELINE config 4 (n = 8192, the grid-wide sweep, the bench's launch) bit-exact against the
+    oracle's verdict committed in tests/golden/config4.json (written by
+    scripts/make_golden_config4.py, which calls only oracle/): score and dot-bracket."""
     from tests import brute
+    with open(os.path.join(os.path.dirname(__file__), "golden", "config4.json")) as f:
+        gold = json.load(f)
     x = dpgen.config4_rna8192()
+    assert hashlib.sha256(x.tobytes()).hexdigest() == gold["input_sha256"]
     r = run_nuss(dp, [x])
+    assert r["scores"][0] == gold["score"]
+    assert hashlib.sha256(r["db"][0].encode()).hexdigest() == gold["dotbracket_sha256"]
+    assert r["db"][0] == gold["dotbracket"]
     pairs = brute.dotbracket_pairs(r["db"][0])
-    pm = dpgen.rna_pair_mask()
-    assert len(pairs) == r["scores"][0]
-    assert all(pm[x[i]][x[j]] and j - i - 1 >= 3 for i, j in pairs)
-    assert 0.25 * 8192 < r["scores"][0] <= (8192 - 3) // 2
+    assert len(pairs) == gold["score"]
 
 
 def test_nussinov_config5_sampled(dp, orc):
+    """BASELINE config 5 at full size (1M RNAs, U[128, 512]) in the bench's launch (scores and
+    tracebacks of the whole batch in one solve); scores and canonical dot-brackets of a seeded
+    sample (ids spread over the batch plus the first and last) bit-exact against the oracle."""
+    cat, off = dpgen.config5_rna_batch()
+    n = len(off) - 1
+    lens = np.diff(off)
+    ml = int(lens.max())
+    pm = dpgen.rna_pair_mask()
+    plan = dp.Plan(dp.NUSSINOV, ml, pair_mask=pm, min_hairpin=3, want_traceback=True)
+    sc = host(plan.solve_batch(cuda(cat), cuda(off), max_len_a=ml))
+    out, ln, _ = plan.traceback(0, n, 512, coords=False)
+    out, ln = host(out), host(ln)
+    plan.close()
+    ids = np.concatenate([[0, n - 1], np.sort(np.random.default_rng(141).choice(n, 62, replace=False))])
+    ids = np.concatenate([ids, [int(np.argmax(lens)), int(np.argmin(lens))]])
+
+    def one(q):
+        return orc.nussinov_traceback(cat[off[q]:off[q + 1]], pm, 3)
+
+    with concurrent.futures.ThreadPoolExecutor(THREADS) as ex:
+        want = list(ex.map(one, ids))
+    for q, (wsc, wdb) in zip(ids, want):
+        assert sc[q] == wsc, q
+        assert ln[q] == lens[q] and bytes(out[q, :ln[q]]).decode() == wdb, q
+    # scores of a larger seeded subset (oracle, scores only)
+    sub = dpgen.config5_sample_ids(k=400)
+    scat, soff = dpgen.config5_rna_batch(ids=sub)
+    assert (sc[sub] == orc.nussinov_batch(scat, soff, pm, 3, threads=THREADS)).all()
+
+
+def test_nussinov_batch_sampled_small(dp, orc):
     ids = dpgen.config5_sample_ids(k=400)
     cat, off = dpgen.config5_rna_batch(ids=ids)
     seqs = [cat[off[q]:off[q + 1]] for q in range(len(ids))]
-    r = run_nuss(dp, seqs, tb=False)
+    r = run_nuss(dp, seqs, tb=True)
+    for q in range(0, len(ids), 20):
+        assert (r["scores"][q], r["db"][q]) == orc.nussinov_traceback(seqs[q], dpgen.rna_pair_mask(), 3), q
     want = orc.nussinov_batch(cat, off, dpgen.rna_pair_mask(), 3, threads=THREADS)
     assert (r["scores"] == want).all()
 
@@ -322,8 +388,19 @@ def hmm_case(g, S, n, tlo, thi):
     return pi32, A32, E32, seqs
 
 
+def forward_errors(ll, want, label, capsys):
+    """Achieved error of log P: max |delta| in nats and max relative; printed into the test log
+    (the north_star bar is relative 1e-5 of log P, DESIGN.md §2 "Tolerances")."""
+    ll, want = np.asarray(ll, np.float64), np.asarray(want, np.float64)
+    d = np.abs(ll - want)
+    rel = d / np.maximum(np.abs(want), 1e-30)
+    with capsys.disabled():
+        print(f"\n[forward {label}] n={len(d)} max |dlogP| = {d.max():.3e} nats, max rel = {rel.max():.3e}")
+    return d, rel
+
+
 @pytest.mark.parametrize("S", [1, 5, 64])
-def test_forward_random(dp, orc, S):
+def test_forward_random(dp, orc, S, capsys):
     g = np.random.default_rng(120 + S)
     pi, A, E, seqs = hmm_case(g, S, 60, 0, 300)
     cat, off = dpgen.pack(seqs)
@@ -331,15 +408,16 @@ def test_forward_random(dp, orc, S):
     ll = host(plan.solve_batch(cuda(cat), cuda(off)))
     want = orc.forward_batch(cat, off, pi.astype(np.float64), A.astype(np.float64), E.astype(np.float64),
                              threads=THREADS)
-    for q in range(len(seqs)):
-        if len(seqs[q]) == 0:
-            assert ll[q] == 0.0
-        else:
-            assert abs(ll[q] - want[q]) <= 1e-5 * abs(want[q]), (q, ll[q], want[q])
+    live = np.array([len(x) > 0 for x in seqs])
+    assert (ll[~live] == 0.0).all()
+    d, rel = forward_errors(ll[live], want[live], f"tcgen05 S={S}", capsys)
+    assert rel.max() <= 1e-5
+    # absolute bar in nats: T <= 300 steps of fp32 rounding (DESIGN.md §2 "Tolerances")
+    assert d.max() <= 2e-3
 
 
 @pytest.mark.parametrize("S", [5, 64])
-def test_forward_simt_path(dp, orc, S, monkeypatch):
+def test_forward_simt_path(dp, orc, S, monkeypatch, capsys):
     """The SIMT forward kernel (used when the tensor-core path is disabled)."""
     monkeypatch.setenv("DP_HMM_SIMT", "1")
     g = np.random.default_rng(125 + S)
@@ -349,8 +427,8 @@ def test_forward_simt_path(dp, orc, S, monkeypatch):
     ll = host(plan.solve_batch(cuda(cat), cuda(off)))
     want = orc.forward_batch(cat, off, pi.astype(np.float64), A.astype(np.float64), E.astype(np.float64),
                              threads=THREADS)
-    for q in range(len(seqs)):
-        assert abs(ll[q] - want[q]) <= 1e-5 * max(abs(want[q]), 1e-30), (q, ll[q], want[q])
+    d, rel = forward_errors(ll, want, f"SIMT S={S}", capsys)
+    assert rel.max() <= 1e-5 and d.max() <= 2e-3
 
 
 @pytest.mark.parametrize("S", [1, 7, 64])
@@ -370,7 +448,7 @@ def test_viterbi_random(dp, orc, S):
         assert ln[q] == len(x) and (out[q, :len(x)] == path).all(), q
 
 
-def test_hmm_config3_sampled(dp, orc):
+def test_hmm_config3_sampled(dp, orc, capsys):
     """BASELINE config 3 at full size (10k x 1000, S = 64), sampled against the oracle."""
     d = dpgen.config3_hmm()
     seqs = d["seqs"]
@@ -387,8 +465,9 @@ def test_hmm_config3_sampled(dp, orc):
     sub_off = np.arange(len(ids) + 1, dtype=np.int64) * T
     sub = seqs[ids].reshape(-1)
     want = orc.forward_batch(sub, sub_off, *(d[k].astype(np.float64) for k in ("pi", "A", "E")), threads=THREADS)
+    d, rel = forward_errors(ll[ids], want, "config 3 (S=64, T=1000)", capsys)
+    assert rel.max() <= 1e-5 and d.max() <= 1e-2
     for k, q in enumerate(ids):
-        assert abs(ll[q] - want[k]) <= 1e-5 * abs(want[k])
         v, path = orc.viterbi(seqs[q], d["lpi"], d["lA"], d["lE"])
         assert vs[q] == v and (out[q] == path).all()
 
@@ -418,6 +497,55 @@ def test_errors_and_empty(dp):
         dp.Plan(dp.SW_LINEAR, 16, 16, sigma=sig, gap=4, user_coeff=(1, -1))
     assert ex.value.code == 2   # user schedule violates eq.(3)
     plan.close()
+
+
+def test_dp_solve_single_problem(dp, orc):
+    """dp_solve (one problem, device buffers): each kind against the oracle, and many calls on
+    two streams in flight at once (the per-call offset slots must not be shared)."""
+    import torch
+    sig = dpgen.blosum62()
+    g = np.random.default_rng(151)
+    pairs = [(g.integers(0, 20, int(g.integers(1, 300))).astype(np.uint8),
+              g.integers(0, 20, int(g.integers(1, 300))).astype(np.uint8)) for _ in range(40)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    with dp.Plan(dp.SW_LINEAR, 300, 300, sigma=sig, gap=4) as p:
+        outs = []
+        for k, (a, b) in enumerate(pairs):
+            st = streams[k % 2]
+            with torch.cuda.stream(st):
+                ta, tb = cuda(a), cuda(b)
+                outs.append((p.solve(ta, tb, stream=st), ta, tb))
+        torch.cuda.synchronize()
+        for (o, _, _), (a, b) in zip(outs, pairs):
+            assert int(o[0]) == orc.sw(a, b, sig, 4)[0]
+    # retained state belongs to the plan's most recent solve: traceback after dp_solve
+    a, b = pairs[-1]
+    with dp.Plan(dp.SW_LINEAR, 300, 300, sigma=sig, gap=4, want_traceback=True) as p:
+        p.solve(cuda(a), cuda(b))
+        out, ln, co = p.traceback(0, 1, 600)
+        ops, c = orc.sw_traceback(a, b, sig, 4)
+        assert bytes(host(out[0, :int(ln[0])])).decode() == ops and tuple(host(co[0])) == c
+    x = dpgen.config1_rna64()
+    with dp.Plan(dp.NUSSINOV, 64, pair_mask=dpgen.rna_pair_mask(), min_hairpin=3, want_traceback=True) as p:
+        assert int(p.solve(cuda(x))[0]) == orc.nussinov(x, dpgen.rna_pair_mask(), 3)
+    s, t = dpgen.encode("kitten", dpgen.EN), dpgen.encode("sitting", dpgen.EN)
+    with dp.Plan(dp.EDIT, 6, 7, alphabet_size=26) as p:
+        assert int(p.solve(cuda(s), cuda(t))[0]) == 3
+    with pytest.raises(dp.DPError) as ex:
+        with dp.Plan(dp.EDIT, 6, 7, alphabet_size=26) as p:
+            p.solve(cuda(np.zeros(9, np.uint8)), cuda(t))
+    assert ex.value.code == 4
+
+
+def test_plan_rejects_what_the_kernels_cannot_run(dp):
+    """Plan creation checks the kernels' shared-memory needs against the device limit
+    (DP_E_TOO_LARGE at dp_plan_create, not DP_E_CUDA at solve time)."""
+    sig = dpgen.blosum62()
+    for kind, kw in ((dp.SW_AFFINE, dict(gap_open=11, gap_extend=1)), (dp.EDIT, {})):
+        with pytest.raises(dp.DPError) as ex:
+            dp.Plan(kind, 200_000, 200_000, sigma=sig if kind == dp.SW_AFFINE else None, alphabet_size=24,
+                    want_traceback=False, **kw)
+        assert ex.value.code == 4
 
 
 def test_host_entry_point(dp, orc):

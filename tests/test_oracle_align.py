@@ -1,6 +1,6 @@
 """Pins for the oracle's edit distance (Fig.7) and Smith–Waterman (§6.1) functions.
 
-Brute force over every (local) alignment on tiny inputs, closed forms and
+Brute force over every (local) alignment for lengths <= 8, closed forms and
 textbook special cases."""
 import numpy as np
 import pytest
@@ -37,26 +37,29 @@ def test_edit_closed_forms(orc):
 
 
 def test_edit_brute_force(orc):
+    """d = the minimum over EVERY global alignment (lengths <= 8: up to D(8,8) = 265,729)."""
     g = np.random.default_rng(2)
-    for _ in range(60):
-        s = g.integers(0, 3, size=g.integers(0, 7)).astype(np.uint8)
-        t = g.integers(0, 3, size=g.integers(0, 7)).astype(np.uint8)
+    for k in range(60):
+        n, m = (8, 8) if k < 4 else (int(g.integers(0, 9)), int(g.integers(0, 9)))
+        s = g.integers(0, 3, size=n).astype(np.uint8)
+        t = g.integers(0, 3, size=m).astype(np.uint8)
+        assert orc.edit(s, t) == int(brute.global_alignment_costs(list(s), list(t)).min())
+    for _ in range(10):   # the pure-Python enumerator agrees on small cases
+        s = g.integers(0, 3, size=g.integers(0, 6)).astype(np.uint8)
+        t = g.integers(0, 3, size=g.integers(0, 6)).astype(np.uint8)
         assert orc.edit(s, t) == brute.brute_edit(list(s), list(t))
 
 
 def test_edit_traceback_canonical(orc):
     """Ops are an optimal alignment and the canonical one: the smallest reversed op
-    sequence under diag < up(D) < left(I) among all optimal alignments."""
+    sequence under diag < up(D) < left(I) among all optimal global alignments (lengths <= 8)."""
     g = np.random.default_rng(3)
-    rank = {"M": 0, "X": 0, "S": 0, "D": 1, "I": 2}
-    for _ in range(40):
-        s = list(g.integers(0, 3, size=g.integers(0, 6)))
-        t = list(g.integers(0, 3, size=g.integers(0, 6)))
+    for k in range(50):
+        n, m = (8, 8) if k < 3 else (int(g.integers(0, 9)), int(g.integers(0, 9)))
+        s = list(g.integers(0, 3, size=n))
+        t = list(g.integers(0, 3, size=m))
         ops = orc.edit_traceback(np.array(s, np.uint8), np.array(t, np.uint8))
         d = orc.edit(np.array(s, np.uint8), np.array(t, np.uint8))
-        cost = brute.score_alignment(s, t, ops.replace("M", "S").replace("X", "S"),
-                                     lambda a, b: -int(a != b), 1)
-        assert -cost == d
         i = j = 0
         for o in ops:  # M/X labels agree with the residues
             if o in "MX":
@@ -65,52 +68,53 @@ def test_edit_traceback_canonical(orc):
                 i += 1
             else:
                 j += 1
-        best = None
-        for al in brute.all_global_alignments(len(s), len(t)):
-            if -brute.score_alignment(s, t, al, lambda a, b: -int(a != b), 1) == d:
-                key = tuple(rank[o] for o in reversed(al))
-                best = key if best is None or key < best else best
-        assert tuple(rank[o] for o in reversed(ops)) == best
+        assert (i, j) == (n, m)
+        want, _ = brute.canonical_local_traceback(s, t, (n, m), -d, lambda a, b: -int(a != b), 0, 1, whole=True)
+        assert ops == want
 
 
 def test_sw_brute_force_cells_and_end(orc):
-    """Score and end cell equal the brute-force max over all local alignments."""
+    """Score and end cell equal the maximum over EVERY local alignment (lengths <= 8)."""
     g = np.random.default_rng(4)
     sig = dpgen.blosum62()
-    for _ in range(25):
-        s = list(g.integers(0, 24, size=g.integers(0, 5)))
-        t = list(g.integers(0, 24, size=g.integers(0, 5)))
+    sub = lambda a, b: int(sig[a][b])
+    for k in range(40):
+        n, m = (8, 8) if k < 4 else (int(g.integers(0, 9)), int(g.integers(0, 9)))
+        alpha = 24 if k % 2 else 4    # small alphabets: recurring maxima, end-cell ties
+        s = list(g.integers(0, alpha, size=n))
+        t = list(g.integers(0, alpha, size=m))
         gap = int(g.integers(1, 6))
-        _, best, (bi, bj) = brute.brute_local_cells(s, t, sig, gap)
+        _, best, (bi, bj) = brute.local_alignment_scores(s, t, sub, gap)
         sc, ei, ej = orc.sw(np.array(s, np.uint8), np.array(t, np.uint8), sig, gap)
         assert sc == best
         assert (ei, ej) == (bi, bj)
+    for _ in range(5):   # the pure-Python enumerator agrees on small cases
+        s = list(g.integers(0, 24, size=g.integers(0, 4)))
+        t = list(g.integers(0, 24, size=g.integers(0, 4)))
+        assert orc.sw(np.array(s, np.uint8), np.array(t, np.uint8), sig, 3)[0] == brute.brute_local_cells(s, t, sig, 3)[1]
 
 
 def test_sw_traceback_canonical(orc):
+    """The canonical local alignment (R-TB-SW): among every optimal local alignment ending at the
+    end cell, the smallest reversed op sequence under diag < up < left with stopping first
+    (lengths <= 8)."""
     g = np.random.default_rng(5)
     sig = dpgen.blosum62()
-    rank = {"S": 0, "M": 0, "X": 0, "D": 1, "I": 2}
-    for _ in range(25):
-        s = list(g.integers(0, 6, size=g.integers(0, 5)))
-        t = list(g.integers(0, 6, size=g.integers(0, 5)))
+    sub = lambda a, b: int(sig[a][b])
+    for k in range(60):
+        n, m = (8, 8) if k < 4 else (int(g.integers(0, 9)), int(g.integers(0, 9)))
+        s = list(g.integers(0, 6, size=n))
+        t = list(g.integers(0, 6, size=m))
         gap = int(g.integers(1, 5))
         sc, ei, ej = orc.sw(np.array(s, np.uint8), np.array(t, np.uint8), sig, gap)
         ops, (si, sj, ei2, ej2) = orc.sw_traceback(np.array(s, np.uint8), np.array(t, np.uint8), sig, gap)
         assert (ei2, ej2) == ((ei, ej) if sc > 0 else (0, 0))
-        sub = lambda a, b: int(sig[a][b])
         if sc == 0:
             assert ops == ""
             continue
         assert brute.score_alignment(s[si:ei], t[sj:ej], ops.replace("M", "S").replace("X", "S"), sub, gap) == sc
-        best = None
-        for i0 in range(ei + 1):
-            for j0 in range(ej + 1):
-                for al in brute.all_global_alignments(ei - i0, ej - j0):
-                    if brute.score_alignment(s[i0:ei], t[j0:ej], al, sub, gap) == sc:
-                        key = tuple(rank[o] for o in reversed(al))
-                        best = key if best is None or key < best else best
-        assert tuple(rank[o] for o in reversed(ops)) == best
+        want, start = brute.canonical_local_traceback(s, t, (ei, ej), sc, sub, 0, gap)
+        assert ops == want and (si, sj) == start
 
 
 def test_sw_longest_common_substring(orc):

@@ -17,14 +17,17 @@ def rand_hmm(g, S, K):
 
 
 def test_forward_brute_force(orc):
+    """log P(x) = log of the sum over EVERY state path (S <= 8, T <= 6: up to 262,144 paths)."""
     g = np.random.default_rng(20)
-    for _ in range(20):
-        S, K, T = int(g.integers(1, 5)), int(g.integers(2, 5)), int(g.integers(0, 6))
+    for k in range(30):
+        S, K, T = (8, 4, 6) if k < 3 else (int(g.integers(1, 7)), int(g.integers(2, 5)), int(g.integers(0, 7)))
         pi, A, E = rand_hmm(g, S, K)
         x = g.integers(0, K, size=T).astype(np.uint8)
-        want = brute.brute_forward(list(x), pi, A, E)
+        want = brute.brute_forward_np(list(x), pi, A, E)
         got = orc.forward(x, pi, A, E)
         assert abs(got - want) <= 1e-12 * max(1.0, abs(want))
+        if S <= 3 and T <= 4:   # the pure-Python enumerator agrees
+            assert abs(brute.brute_forward(list(x), pi, A, E) - want) <= 1e-12 * max(1.0, abs(want))
 
 
 def test_forward_sums_to_one(orc):
@@ -61,18 +64,20 @@ def test_viterbi_brute_force_and_canonical_path(orc):
     """Score = max over all paths; path = the optimal path whose reversal is
     lexicographically smallest (final state lowest, then predecessors lowest)."""
     g = np.random.default_rng(23)
-    for _ in range(30):
-        S, K, T = int(g.integers(1, 5)), int(g.integers(2, 4)), int(g.integers(1, 6))
+    for k in range(40):
+        S, K, T = (8, 3, 6) if k < 3 else (int(g.integers(1, 7)), int(g.integers(2, 4)), int(g.integers(1, 7)))
         pi, A, E = rand_hmm(g, S, K)
         # coarse scores so that ties actually occur
         lpi, lA, lE = (np.rint(dpgen.millibits(v) / 997.0).astype(np.int32) for v in (pi, A, E))
         x = g.integers(0, K, size=T).astype(np.uint8)
-        best, paths = brute.brute_viterbi(list(x), lpi, lA, lE)
+        best, canon = brute.brute_viterbi_np(list(x), lpi, lA, lE)
         sc, path = orc.viterbi(x, lpi, lA, lE)
         assert sc == best
         assert brute.viterbi_path_score(list(x), list(path), lpi, lA, lE) == best
-        canon = min(paths, key=lambda p: tuple(reversed(p)))
-        assert tuple(int(v) for v in path) == tuple(canon)
+        assert tuple(int(v) for v in path) == canon
+        if S <= 3 and T <= 4:   # the pure-Python enumerator agrees
+            b2, paths = brute.brute_viterbi(list(x), lpi, lA, lE)
+            assert b2 == best and min(paths, key=lambda p: tuple(reversed(p))) == canon
 
 
 def test_viterbi_closed_forms(orc):
