@@ -268,6 +268,17 @@ class Plan:
                                     int(max_len_b), _ptr(out), _stream_ptr(stream)), "dp_solve_batch")
         return out
 
+    def solve(self, a, b=None, *, out=None, stream=None):
+        """dp_solve: one problem from device tensors a (and b for the alignment kinds); returns a
+        1-element device tensor (int32, or float32 log-likelihood for HMM_FORWARD)."""
+        import torch
+        if out is None:
+            out = torch.empty(1, dtype=torch.float32 if self.kind == HMM_FORWARD else torch.int32, device=a.device)
+        self._last_inputs = (a, None, b, None)  # must outlive dp_traceback
+        _check(lib().dp_solve(self._h, _ptr(a), int(a.numel()), _ptr(b), int(b.numel()) if b is not None else 0,
+                              _ptr(out), _stream_ptr(stream)), "dp_solve")
+        return out
+
     def traceback(self, first, count, stride, *, coords=True, stream=None, device="cuda"):
         import torch
         out = torch.empty((count, stride), dtype=torch.uint8, device=device)

@@ -263,12 +263,17 @@ int pick_R(int64_t max_la) {
   return 8;
 }
 
+int64_t align_per_warp(int R, int asz, int64_t max_la, int64_t max_lb) {
+  const int64_t strips_max = (max_la + 32 * R - 1) / (32 * R);
+  int64_t per_warp = (int64_t)asz * 32 * R + ((max_lb + 15) & ~int64_t(15));
+  if (strips_max > 1) per_warp += (max_lb + 1) * 4;
+  return (per_warp + 15) & ~int64_t(15);
+}
+
 template <int R, bool LOCAL, bool TB>
 cudaError_t launch_align(const AlignArgs& A, cudaStream_t s) {
   const int strips_max = (int)((A.max_la + 32 * R - 1) / (32 * R));
-  int per_warp = A.asz * 32 * R + (int)((A.max_lb + 15) & ~15);
-  if (strips_max > 1) per_warp += (int)(A.max_lb + 1) * 4;
-  per_warp = (per_warp + 15) & ~15;
+  const int per_warp = (int)align_per_warp(R, A.asz, A.max_la, A.max_lb);
   const int sig_bytes = LOCAL ? ((A.asz * A.asz + 15) & ~15) : 0;
   const size_t smem = sig_bytes + (size_t)kWarps * per_warp;
   auto kern = k_align<R, LOCAL, TB>;
@@ -293,6 +298,12 @@ int64_t align_dir_words(int64_t max_la, int64_t max_lb) {
   const int64_t strips = (max_la + 32 * R - 1) / (32 * R);
   const int64_t wpl = (max_lb + cols_per_word(R) - 1) / cols_per_word(R);
   return strips * wpl * 32;
+}
+
+size_t align_smem_bytes(int asz, bool local, int64_t max_la, int64_t max_lb) {
+  const int R = pick_R(max_la);
+  const size_t sig_bytes = local ? (size_t)((asz * asz + 15) & ~15) : 0;
+  return sig_bytes + (size_t)kWarps * (size_t)align_per_warp(R, asz, max_la, max_lb);
 }
 
 cudaError_t align_solve(const AlignArgs& A, cudaStream_t s, int64_t* launches) {

@@ -234,12 +234,16 @@ int pick_R_affine(int64_t max_la) {
   return 8;
 }
 
+int64_t affine_per_warp(int R, int asz, int64_t max_la, int64_t max_lb) {
+  const int64_t strips_max = (max_la + 32 * R - 1) / (32 * R);
+  int64_t per_warp = (int64_t)asz * 32 * R + ((max_lb + 15) & ~int64_t(15));
+  if (strips_max > 1) per_warp += (max_lb + 1) * 8;
+  return (per_warp + 15) & ~int64_t(15);
+}
+
 template <int R, bool TB>
 cudaError_t launch_affine(const AlignArgs& A, cudaStream_t s) {
-  const int strips_max = (int)((A.max_la + 32 * R - 1) / (32 * R));
-  int per_warp = A.asz * 32 * R + (int)((A.max_lb + 15) & ~15);
-  if (strips_max > 1) per_warp += (int)(A.max_lb + 1) * 8;
-  per_warp = (per_warp + 15) & ~15;
+  const int per_warp = (int)affine_per_warp(R, A.asz, A.max_la, A.max_lb);
   const size_t smem = ((A.asz * A.asz + 15) & ~15) + (size_t)kWarps * per_warp;
   auto kern = k_align_affine<R, TB>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -255,6 +259,10 @@ int64_t align_affine_dir_words(int64_t max_la, int64_t max_lb) {
   const int64_t strips = (max_la + 32 * R - 1) / (32 * R);
   const int64_t wpl = (max_lb + acols_per_word(R) - 1) / acols_per_word(R);
   return strips * wpl * 32;
+}
+
+size_t align_affine_smem_bytes(int asz, int64_t max_la, int64_t max_lb) {
+  return (size_t)((asz * asz + 15) & ~15) + (size_t)kWarps * (size_t)affine_per_warp(pick_R_affine(max_la), asz, max_la, max_lb);
 }
 
 cudaError_t align_affine_solve(const AlignArgs& A, cudaStream_t s, int64_t* launches) {

@@ -34,6 +34,20 @@ struct DevBuf {
   }
 };
 
+// Makes the plan's device current for the lifetime of a call and restores the caller's on every
+// exit path (the plan binds the device that was current at dp_plan_create).
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
 }  // namespace
 
 struct dp_plan {
@@ -74,9 +88,43 @@ struct dp_plan {
   static constexpr int kMaxChunks = 16;
   cudaEvent_t ev_start = nullptr, ev_in[kMaxChunks] = {}, ev_out[kMaxChunks] = {};
   int64_t launches = 0;
+  // dp_solve: a ring of {0, len_a, 0, len_b} offset slots in device memory; a slot is reused only
+  // after the event recorded behind the solve that read it has completed
+  static constexpr int kSolveSlots = 16;
+  DevBuf solve_off;
+  cudaEvent_t solve_ev[kSolveSlots] = {};
+  int solve_next = 0;
+  // diagnostics (environment, read once at dp_plan_create; tests and experiments only)
+  struct {
+    bool force_int32 = false, nuss_cell = false, hmm_timing = false, nuss_timing = false, sw_timing = false;
+    bool nuss_rounds = false, diag_generic = false;
+    int64_t nuss_tiled_min = 32;
+    int nuss_tbw = 0, diag_force = -1, host_chunks = 4;
+  } env;
 };
 
 namespace {
+
+void read_env(dp_plan* p) {
+  auto on = [](const char* k) { return getenv(k) != nullptr; };
+  p->env.force_int32 = on("DP_FORCE_INT32");
+  p->env.nuss_cell = on("DP_NUSS_CELL");
+  p->env.hmm_timing = on("DP_HMM_TIMING");
+  p->env.nuss_timing = on("DP_NUSS_TIMING");
+  p->env.sw_timing = on("DP_SW_TIMING");
+  p->env.nuss_rounds = on("DP_NUSS_ROUNDS");
+  p->env.diag_generic = on("DP_DIAG_GENERIC");
+  if (on("DP_NUSS_TILED_MIN")) p->env.nuss_tiled_min = atoll(getenv("DP_NUSS_TILED_MIN"));
+  if (on("DP_NUSS_TBW")) p->env.nuss_tbw = atoi(getenv("DP_NUSS_TBW"));
+  if (on("DP_DIAG_FORCE")) p->env.diag_force = atoi(getenv("DP_DIAG_FORCE"));
+  if (on("DP_HOST_CHUNKS")) p->env.host_chunks = std::max(1, std::min(dp_plan::kMaxChunks, atoi(getenv("DP_HOST_CHUNKS"))));
+}
+
+int max_smem_optin(int dev) {
+  int v = 0;
+  if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) v = 0;
+  return v;
+}
 
 dp_status cuda_status(cudaError_t e) {
   if (e == cudaSuccess) return DP_OK;
@@ -192,6 +240,9 @@ void dp_plan_destroy(dp_plan_t p) {
   if (p->s_h2d) cudaStreamDestroy(p->s_h2d);
   if (p->s_cmp) cudaStreamDestroy(p->s_cmp);
   p->tb_state_alt.release();
+  p->solve_off.release();
+  for (int k = 0; k < dp_plan::kSolveSlots; ++k)
+    if (p->solve_ev[k]) cudaEventDestroy(p->solve_ev[k]);
   if (p->s_d2h) cudaStreamDestroy(p->s_d2h);
   if (p->ev_start) cudaEventDestroy(p->ev_start);
   for (int k = 0; k < dp_plan::kMaxChunks; ++k) {
@@ -215,6 +266,8 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
   p->max_lb = d->max_len_b;
   p->want_tb = d->want_traceback != 0;
   cudaGetDevice(&p->device);
+  read_env(p);
+  const int smem_limit = max_smem_optin(p->device);
   dp_status st = DP_OK;
   cudaError_t e = cudaSuccess;
   switch (d->kind) {
@@ -223,6 +276,9 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       if (p->asz > 32) st = DP_E_UNSUPPORTED;
       p->gap = 1;
       if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) st = DP_E_TOO_LARGE;
+      // the warp kernel keeps the column residues (and the strip boundary row) in shared memory
+      else if (smem_limit > 0 && dpk::align_smem_bytes(p->asz, false, d->max_len_a, d->max_len_b) > (size_t)smem_limit)
+        st = DP_E_TOO_LARGE;
       break;
     case DP_SW_LINEAR:
       p->asz = d->alphabet_size;
@@ -233,7 +289,11 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
       p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
       p->packed16 = dpk::sw16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap, d->want_traceback != 0) &&
-                    getenv("DP_FORCE_INT32") == nullptr;
+                    !p->env.force_int32 &&
+                    (smem_limit <= 0 || dpk::sw16_smem_bytes(p->asz, d->max_len_a, d->max_len_b) <= (size_t)smem_limit);
+      if (!p->packed16 && smem_limit > 0 &&
+          dpk::align_smem_bytes(p->asz, true, d->max_len_a, d->max_len_b) > (size_t)smem_limit)
+        st = DP_E_TOO_LARGE;
       break;
     case DP_SW_AFFINE:
       p->asz = d->alphabet_size;
@@ -241,6 +301,10 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       if (p->asz > 32) { st = DP_E_UNSUPPORTED; break; }
       p->gap_open = d->gap_open; p->gap_ext = d->gap_extend;
       if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) { st = DP_E_TOO_LARGE; break; }
+      if (smem_limit > 0 && dpk::align_affine_smem_bytes(p->asz, d->max_len_a, d->max_len_b) > (size_t)smem_limit) {
+        st = DP_E_TOO_LARGE;
+        break;
+      }
       e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
       p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
       break;
@@ -248,6 +312,9 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       if (p->want_tb) { st = DP_E_UNSUPPORTED; break; }
       p->asz = d->alphabet_size > 0 && d->alphabet_size <= 256 ? d->alphabet_size : 0;  // optional
       if (d->max_len_a > 40000 || d->max_len_b > 40000) st = DP_E_TOO_LARGE;  // uint16 window rows in smem
+      else if (smem_limit > 0 &&
+               dpk::diag_smem_bytes(std::max(d->max_len_a, d->max_len_b), p->asz) > (size_t)smem_limit)
+        st = DP_E_TOO_LARGE;
       break;
     case DP_NUSSINOV:
       if (!d->pair_mask || d->min_hairpin < 0) { st = DP_E_INVALID; break; }
@@ -336,9 +403,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
   if (max_len_a < 0 || max_len_b < 0) return DP_E_INVALID;
   if (max_len_a > p->max_la || (align && max_len_b > p->max_lb)) return DP_E_TOO_LARGE;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  int cur = 0;
-  cudaGetDevice(&cur);
-  if (cur != p->device) cudaSetDevice(p->device);
+  DeviceGuard guard(p->device);
   cudaError_t e = cudaSuccess;
   p->last_n = n;
   p->last_a = a_cat; p->last_b = b_cat; p->last_aoff = a_off; p->last_boff = b_off;
@@ -351,8 +416,8 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       A.scores = static_cast<int32_t*>(scores_out);
       A.ncand = p->ncand;
       for (int k = 0; k < p->ncand; ++k) { A.cand[k][0] = p->cand[k][0]; A.cand[k][1] = p->cand[k][1]; }
-      A.force = getenv("DP_DIAG_FORCE") ? atoi(getenv("DP_DIAG_FORCE")) : p->force;  // env: diagnostic
-      A.asz = getenv("DP_DIAG_GENERIC") ? 0 : p->asz;  // env: diagnostic (the unpacked path)
+      A.force = p->env.diag_force >= 0 ? p->env.diag_force : p->force;  // env: diagnostic
+      A.asz = p->env.diag_generic ? 0 : p->asz;  // env: diagnostic (the unpacked path)
       e = dpk::diag_solve(A, s, &p->launches);
       break;
     }
@@ -417,19 +482,17 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       // cell-level CTA kernel (table in shared memory) for short sequences, tiled
       // max-plus kernels above (SURVEY §8(a) A6b'); DP_NUSS_CELL=1 forces the cell level
       // (config 1, n = 64: tiled 0.097 ms per step vs 0.109 cell-level)
-      const int64_t tiled_min = getenv("DP_NUSS_TILED_MIN") ? atoll(getenv("DP_NUSS_TILED_MIN")) : 32;
-      const bool tiled = A.max_len > tiled_min && getenv("DP_NUSS_CELL") == nullptr &&
-                         (n == 1 || A.max_len <= 4096);
+      const bool tiled = A.max_len > p->env.nuss_tiled_min && !p->env.nuss_cell && (n == 1 || A.max_len <= 4096);
       A.scratch_bytes = tiled ? dpk::nuss_tiled_scratch_bytes(A.max_len, n, p->device)
                               : dpk::nuss_scratch_bytes(A.max_len, n, p->device);
       e = p->scratch.ensure((size_t)A.scratch_bytes);
       if (e != cudaSuccess) break;
       A.scratch = p->scratch.ptr;
       unsigned long long* rounds = nullptr;
-      if (getenv("DP_NUSS_TBW")) A.tbw = atoi(getenv("DP_NUSS_TBW"));
-      if (getenv("DP_NUSS_ROUNDS") && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), A.round_ns = rounds;
+      A.tbw = p->env.nuss_tbw;
+      if (p->env.nuss_rounds && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), A.round_ns = rounds;
       unsigned long long* dbg = nullptr;
-      if (getenv("DP_NUSS_TIMING") && tiled) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
+      if (p->env.nuss_timing && tiled) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
       e = tiled ? dpk::nuss_tiled_solve(A, s, &p->launches) : dpk::nuss_solve(A, s, &p->launches);
       if (dbg) {  // diagnostic: batch-kernel phase cycles summed over warps (stderr)
         unsigned long long h[8];
@@ -462,7 +525,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         H.ll_out = static_cast<float*>(scores_out);
         // the [batch x S] x [S x S] step on tcgen05 (SIMT fallback kernel via DP_HMM_SIMT=1)
         unsigned long long* dbg = nullptr;
-        if (getenv("DP_HMM_TIMING")) cudaMalloc(&dbg, 8 * 4 * 66), cudaMemset(dbg, 0, 8 * 4 * 66), H.dbg = dbg;
+        if (p->env.hmm_timing) cudaMalloc(&dbg, 8 * 4 * 66), cudaMemset(dbg, 0, 8 * 4 * 66), H.dbg = dbg;
         e = dpk::hmm_forward_tc_supported(p->S) ? dpk::hmm_forward_tc(H, s, &p->launches)
                                                  : dpk::hmm_forward(H, s, &p->launches);
         if (dbg) {  // diagnostic: CTA 0 step phases (ns): MMA issue, wait for MMA, epilogue, barrier
@@ -496,7 +559,6 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       break;
     }
   }
-  if (cur != p->device) cudaSetDevice(cur);
   if (e != cudaSuccess) {
     p->last_n = -1;
     return cuda_status(e);
@@ -506,16 +568,31 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
 
 dp_status dp_solve(dp_plan_t p, const uint8_t* a, int64_t len_a, const uint8_t* b, int64_t len_b, void* score_out,
                    void* stream) {
-  if (!p || len_a < 0 || len_b < 0) return DP_E_INVALID;
-  // offsets {0, len} live in plan workspace
+  if (!p || len_a < 0 || len_b < 0 || !score_out) return DP_E_INVALID;
+  const bool align =
+      p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE || p->kind == DP_DIAG_LCS;
+  if ((len_a > 0 && !a) || (align && len_b > 0 && !b)) return DP_E_INVALID;
+  if (len_a > p->max_la || (align && len_b > p->max_lb)) return DP_E_TOO_LARGE;
+  DeviceGuard guard(p->device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  cudaError_t e = p->tb_aux2.ensure(64);
+  // offsets {0, len_a, 0, len_b} in a slot of the plan's ring; the slot's previous reader has
+  // finished once its event has (host wait, normally long done), so calls on different streams
+  // never share a live slot
+  cudaError_t e = p->solve_off.ensure(dp_plan::kSolveSlots * 32);
+  const int slot = p->solve_next;
+  if (e == cudaSuccess && !p->solve_ev[slot]) e = cudaEventCreateWithFlags(&p->solve_ev[slot], cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventSynchronize(p->solve_ev[slot]);
   if (e != cudaSuccess) return cuda_status(e);
-  int64_t off[4] = {0, len_a, 0, len_b};
-  e = cudaMemcpyAsync(p->tb_aux2.ptr, off, sizeof(off), cudaMemcpyHostToDevice, s);
+  int64_t* d = static_cast<int64_t*>(p->solve_off.ptr) + 4 * slot;
+  const int64_t off[4] = {0, len_a, 0, len_b};
+  e = cudaMemcpyAsync(d, off, sizeof(off), cudaMemcpyHostToDevice, s);
   if (e != cudaSuccess) return cuda_status(e);
-  const int64_t* d = static_cast<const int64_t*>(p->tb_aux2.ptr);
-  return dp_solve_batch(p, 1, a, d, b, d + 2, len_a, len_b, score_out, stream);
+  const dp_status st = dp_solve_batch(p, 1, a, d, align ? b : nullptr, align ? d + 2 : nullptr, len_a,
+                                      align ? len_b : 0, score_out, stream);
+  e = cudaEventRecord(p->solve_ev[slot], s);
+  p->solve_next = (slot + 1) % dp_plan::kSolveSlots;
+  if (st != DP_OK) return st;
+  return cuda_status(e);
 }
 
 dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, int64_t stride, int32_t* out_len,
@@ -526,6 +603,7 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
   if (first < 0 || count < 0 || first + count > p->last_n || stride < 0) return DP_E_INVALID;
   if (count > 0 && (!out || !out_len)) return DP_E_INVALID;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  DeviceGuard guard(p->device);
   cudaError_t e = cudaSuccess;
   switch (p->kind) {
     case DP_SW_LINEAR:
@@ -535,7 +613,7 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
         e = sw16_args(p, p->last_n, p->last_a, p->last_aoff, p->last_b, p->last_boff, p->last_max_la,
                       p->last_max_lb, p->last_scores, &A);
         unsigned long long* dbg = nullptr;
-        if (getenv("DP_SW_TIMING")) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
+        if (p->env.sw_timing) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
         if (e == cudaSuccess) e = dpk::sw16_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
         if (dbg) {  // diagnostic: traceback phase cycles summed over warps
           unsigned long long h[8];
@@ -615,10 +693,15 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
       if (lb > max_lb) max_lb = lb;
     }
   }
-  if (max_la > p->max_la || max_lb > p->max_lb) return DP_E_TOO_LARGE;
+  if (max_la > p->max_la || (align && max_lb > p->max_lb)) return DP_E_TOO_LARGE;
   const int64_t abytes = n > 0 ? a_off[n] - a_off[0] : 0;
   const int64_t bbytes = (align && n > 0) ? b_off[n] - b_off[0] : 0;
   const bool tb = p->want_tb && tb_out && tb_len && p->kind != DP_HMM_FORWARD && n > 0;
+  if (tb) {  // the traceback's stride requirement, checked before anything is enqueued
+    const int64_t need = (p->kind == DP_NUSSINOV || p->kind == DP_HMM_VITERBI) ? max_la : max_la + max_lb;
+    if (tb_stride < need) return DP_E_TOO_LARGE;
+  }
+  DeviceGuard guard(p->device);
   cudaError_t e = p->h_a.ensure((size_t)abytes + 16);
   if (e == cudaSuccess) e = p->h_aoff.ensure((size_t)(n + 1) * 8);
   if (e == cudaSuccess && align) e = p->h_b.ensure((size_t)bbytes + 16);
@@ -644,8 +727,7 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   // a chunk must still fill the GPU: ~3 waves of the sweep kernels
   // (config 2, measured: 1 / 2 / 3 / 4 / 8 / 12 chunks -> 4.53 / 3.73 / 3.55 / 3.46 / 4.14 / 4.31 ms)
   const int64_t min_chunk = align ? 16384 : (p->kind == DP_NUSSINOV ? 65536 : 32768);
-  const int max_ch = getenv("DP_HOST_CHUNKS") ? std::max(1, std::min(dp_plan::kMaxChunks, atoi(getenv("DP_HOST_CHUNKS"))))
-                                              : 4;  // env: diagnostic
+  const int max_ch = p->env.host_chunks;  // env DP_HOST_CHUNKS: diagnostic
   int nch = (int)std::min<int64_t>(max_ch, (n + min_chunk - 1) / min_chunk);
   if (nch < 1) nch = 1;
   const int64_t per = (n + nch - 1) / nch;
@@ -653,11 +735,21 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   uint8_t* db = align ? static_cast<uint8_t*>(p->h_b.ptr) : nullptr;
   int64_t* dao = static_cast<int64_t*>(p->h_aoff.ptr);
   int64_t* dbo = align ? static_cast<int64_t*>(p->h_boff.ptr) : nullptr;
+  // Once anything is enqueued an error path must not return while copies into or out of the
+  // caller's host buffers may still run: drain every stream first (the call is synchronous).
+  const bool two_cmp = p->kind == DP_SW_LINEAR && p->packed16;
+  auto drain = [&](dp_status st) {
+    cudaStreamSynchronize(p->s_h2d);
+    cudaStreamSynchronize(s);
+    if (two_cmp && p->s_cmp) cudaStreamSynchronize(p->s_cmp);
+    cudaStreamSynchronize(p->s_d2h);
+    return st;
+  };
   e = cudaEventRecord(p->ev_start, s);  // buffers are free once earlier work on the caller's stream is done
   if (e == cudaSuccess) e = cudaStreamWaitEvent(p->s_h2d, p->ev_start, 0);
   if (e == cudaSuccess) e = cudaMemcpyAsync(dao, a_off, (n + 1) * 8, cudaMemcpyHostToDevice, p->s_h2d);
   if (e == cudaSuccess && align) e = cudaMemcpyAsync(dbo, b_off, (n + 1) * 8, cudaMemcpyHostToDevice, p->s_h2d);
-  if (e != cudaSuccess) return cuda_status(e);
+  if (e != cudaSuccess) return drain(cuda_status(e));
   // Packed SW keeps all of a solve's retained state in tb_state, so consecutive chunks can
   // alternate between two compute streams and two state buffers: chunk c+1's sweep then fills the
   // SMs while chunk c's traceback drains (other kinds stay on the caller's stream).
@@ -665,10 +757,10 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   if (two && !p->s_cmp) {
     e = cudaStreamCreateWithFlags(&p->s_cmp, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(p->s_cmp, p->ev_start, 0);
-    if (e != cudaSuccess) return cuda_status(e);
+    if (e != cudaSuccess) return drain(cuda_status(e));
   } else if (two) {
     e = cudaStreamWaitEvent(p->s_cmp, p->ev_start, 0);
-    if (e != cudaSuccess) return cuda_status(e);
+    if (e != cudaSuccess) return drain(cuda_status(e));
   }
   int installed = 0;  // which state buffer is in p->tb_state
   for (int c = 0; c < nch; ++c) {
@@ -687,17 +779,17 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
                           cudaMemcpyHostToDevice, p->s_h2d);
     if (e == cudaSuccess) e = cudaEventRecord(p->ev_in[c], p->s_h2d);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(sc, p->ev_in[c], 0);
-    if (e != cudaSuccess) return cuda_status(e);
+    if (e != cudaSuccess) return drain(cuda_status(e));
     int32_t* dsc = static_cast<int32_t*>(p->h_scores.ptr) + k0;
     dp_status st = dp_solve_batch(p, nk, da - a_off[0], dao + k0, align ? db - b_off[0] : nullptr,
                                   align ? dbo + k0 : nullptr, max_la, max_lb, dsc, scv);
-    if (st != DP_OK) return st;
+    if (st != DP_OK) return drain(st);
     uint8_t* dtb = tb ? static_cast<uint8_t*>(p->h_tb.ptr) + k0 * tb_stride : nullptr;
     int32_t* dtl = tb ? static_cast<int32_t*>(p->h_tblen.ptr) + k0 : nullptr;
     int32_t* dco = (tb && tb_coords) ? static_cast<int32_t*>(p->h_coords.ptr) + 4 * k0 : nullptr;
     if (tb) {
       st = dp_traceback(p, 0, nk, dtb, tb_stride, dtl, dco, scv);
-      if (st != DP_OK) return st;
+      if (st != DP_OK) return drain(st);
     }
     e = cudaEventRecord(p->ev_out[c], sc);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(p->s_d2h, p->ev_out[c], 0);
@@ -707,7 +799,7 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
                                                     cudaMemcpyDeviceToHost, p->s_d2h);
     if (e == cudaSuccess && tb) e = cudaMemcpyAsync(tb_len + k0, dtl, nk * 4, cudaMemcpyDeviceToHost, p->s_d2h);
     if (e == cudaSuccess && dco) e = cudaMemcpyAsync(tb_coords + 4 * k0, dco, nk * 16, cudaMemcpyDeviceToHost, p->s_d2h);
-    if (e != cudaSuccess) return cuda_status(e);
+    if (e != cudaSuccess) return drain(cuda_status(e));
   }
   e = cudaStreamSynchronize(p->s_d2h);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);

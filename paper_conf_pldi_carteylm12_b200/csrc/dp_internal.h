@@ -45,6 +45,8 @@ struct AlignArgs {
   int32_t* ends;         // n x 2 (end_i, end_j)
 };
 int64_t align_dir_words(int64_t max_la, int64_t max_lb);  // words per problem for `dirs`
+size_t align_smem_bytes(int asz, bool local, int64_t max_la, int64_t max_lb);  // k_align dynamic smem per CTA
+size_t align_affine_smem_bytes(int asz, int64_t max_la, int64_t max_lb);        // k_align_affine
 int64_t align_affine_dir_words(int64_t max_la, int64_t max_lb);  // affine: 4 bits per cell
 cudaError_t align_affine_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t align_affine_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
@@ -75,6 +77,7 @@ struct Sw16Args {
 };
 bool sw16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int gap, bool want_tb);
 int sw16_smem_per_warp(int asz, int64_t max_la, int64_t max_lb);
+size_t sw16_smem_bytes(int asz, int64_t max_la, int64_t max_lb);  // k_sw16 dynamic smem per CTA
 void sw16_state_words(int64_t n, int64_t max_la, int64_t max_lb, int64_t* strips, int64_t* nslab, int64_t* rowck,
                       int64_t* colck, int64_t* slabbest);
 cudaError_t sw16_solve(const Sw16Args& a, bool tb, cudaStream_t s, int64_t* launches);

@@ -790,6 +790,10 @@ int sw16_smem_per_warp(int asz, int64_t max_la, int64_t max_lb) {
   return (int)((2 * prof_bytes + rec + 15) & ~15);
 }
 
+size_t sw16_smem_bytes(int asz, int64_t max_la, int64_t max_lb) {
+  return 32 * 32 + (size_t)kWarps * (size_t)sw16_smem_per_warp(asz, max_la, max_lb);
+}
+
 void sw16_state_words(int64_t n, int64_t max_la, int64_t max_lb, int64_t* strips, int64_t* nslab, int64_t* rowck,
                       int64_t* colck, int64_t* slabbest) {
   *strips = (max_la + kStrip - 1) / kStrip;
