@@ -242,3 +242,77 @@ def config5_rna_batch(n_seqs: int = 1_000_000, lo: int = 128, hi: int = 512, ids
 def config5_sample_ids(n_seqs: int = 1_000_000, k: int = 10_000) -> np.ndarray:
     """The fixed 1% subset (seed +7) used for the on-box oracle timing."""
     return np.sort(rng(7).choice(n_seqs, size=k, replace=False))
+
+
+# ----------------------------------------------------------------------------- profile HMM (SURVEY §8(f) NEXT 3)
+# Transition slots of position j (0..L): from state X_j, X in (M, I, D) (M_0 is the begin state B,
+# D_0 does not exist), to (M_{j+1}, I_j, D_{j+1}) (M_{L+1} is the end state E, D_{L+1} does not
+# exist). tr[j][3 * from + to], from/to order (M, I, D) / (M_{j+1}, I_j, D_{j+1}).
+PROFILE_FROM = ("M", "I", "D")
+PROFILE_TO = ("M+1", "I", "D+1")
+
+
+def profile_hmm_params(g: np.random.Generator, L: int, K: int = 20):
+    """A Plan7-like profile HMM of L match positions (Durbin et al. ch. 5, the paper's ref [3];
+    PAPER.md §6.3), all nine transitions per position (M/I/D -> M/I/D):
+      tr : (L+1) x 9 float64, rows from M ~ Dir(90, 5, 5), from I ~ Dir(60, 35, 5),
+           from D ~ Dir(65, 5, 30); D_0 does not exist (its row is 0); at j = L the "to D_{L+1}"
+           slot is 0 and each row is renormalised over (E, I_L);
+      eM : (L+1) x K match emissions ~ Dir(0.4) (row 0 unused, zeros);
+      eI : (L+1) x K insert emissions ~ Dir(20) (close to background)."""
+    tr = np.zeros((L + 1, 9))
+    for j in range(L + 1):
+        tr[j, 0:3] = g.dirichlet([90, 5, 5])
+        tr[j, 3:6] = g.dirichlet([60, 35, 5])
+        tr[j, 6:9] = g.dirichlet([65, 5, 30]) if j > 0 else 0.0
+        if j == L:
+            for f in range(3):
+                row = tr[j, 3 * f:3 * f + 3].copy()
+                row[2] = 0.0
+                tr[j, 3 * f:3 * f + 3] = row / row.sum() if row.sum() > 0 else 0.0
+    eM = np.zeros((L + 1, K))
+    eM[1:] = g.dirichlet(np.full(K, 0.4), size=L)
+    eI = g.dirichlet(np.full(K, 20.0), size=L + 1)
+    return tr, eM, eI
+
+
+def sample_profile(g: np.random.Generator, tr, eM, eI, n: int, max_len: int = 1 << 30):
+    """n sequences emitted by walking the profile from B to E (M and I states emit)."""
+    L = tr.shape[0] - 1
+    K = eM.shape[1]
+    cM, cI = np.cumsum(eM, axis=1), np.cumsum(eI, axis=1)
+    out = []
+    while len(out) < n:
+        st, j, seq = 0, 0, []   # st: 0 = M (M_0 = B), 1 = I, 2 = D; at position j
+        while True:
+            row = tr[j, 3 * st:3 * st + 3]
+            to = min(int(np.searchsorted(np.cumsum(row), g.random(), side="right")), 2)
+            if to == 1:
+                st = 1
+                seq.append(min(int(np.searchsorted(cI[j], g.random(), side="right")), K - 1))
+            else:
+                j += 1
+                st = 0 if to == 0 else 2
+                if j == L + 1:
+                    break
+                if st == 0:
+                    seq.append(min(int(np.searchsorted(cM[j], g.random(), side="right")), K - 1))
+            if len(seq) > max_len:
+                break
+        if len(seq) <= max_len:
+            out.append(np.array(seq, dtype=np.uint8))
+    return out
+
+
+def profile_hmm_workload(n_seqs: int = 13_355, L: int = 256, K: int = 20):
+    """NEXT 3 workload: one L = 256 position protein profile (params seed +9), n sequences sampled
+    from it (seed +10; 13,355 = the database size of the paper's Fig.15). Both sides get the
+    float32 parameters (the oracle widens them to float64)."""
+    tr, eM, eI = profile_hmm_params(rng(9), L, K)
+    tr32, eM32, eI32 = (x.astype(np.float32) for x in (tr, eM, eI))
+    seqs = sample_profile(rng(10), tr, eM, eI, n_seqs, max_len=1023)
+    cat, off = pack(seqs)
+    return {"L": L, "K": K, "cat": cat, "off": off,
+            "model": {"trans": tr32, "emit_m": eM32, "emit_i": eI32},
+            "model64": {"trans": tr32.astype(np.float64), "emit_m": eM32.astype(np.float64),
+                        "emit_i": eI32.astype(np.float64)}}

@@ -73,6 +73,12 @@ def lib():
         L.orc_nussinov_traceback.argtypes = [u8p, i64, u8p, ctypes.c_int, u8p]
         L.orc_forward.restype = ctypes.c_double
         L.orc_forward.argtypes = [u8p, i64, ctypes.c_int, ctypes.c_int, f64p, f64p, f64p]
+        L.orc_silent_forward.restype = ctypes.c_double
+        L.orc_silent_forward.argtypes = [u8p, i64, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int, u8p, f64p,
+                                         f64p]
+        L.orc_silent_forward_batch.restype = None
+        L.orc_silent_forward_batch.argtypes = [i64, i64, u8p, i64p, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                               ctypes.c_int, u8p, f64p, f64p, f64p]
         L.orc_viterbi.restype = i64
         L.orc_viterbi.argtypes = [u8p, i64, ctypes.c_int, ctypes.c_int, i32p, i32p, i32p, u8p]
         L.orc_sw_batch.restype = None
@@ -194,6 +200,73 @@ def forward(x, pi, A, E) -> float:
     A = np.ascontiguousarray(A, dtype=np.float64)
     E = np.ascontiguousarray(E, dtype=np.float64)
     return float(lib().orc_forward(x, len(x), len(pi), E.shape[1], pi, A, E))
+
+
+def silent_forward(x, silent, A, E, begin, end) -> float:
+    """log P(x) (natural log, fp64) of a generic HMM with silent states (§5.2; DESIGN.md R-PHMM)."""
+    x = _u8(x)
+    sil = _u8(silent)
+    A = np.ascontiguousarray(A, dtype=np.float64)
+    E = np.ascontiguousarray(E, dtype=np.float64)
+    return float(lib().orc_silent_forward(x, len(x), len(sil), E.shape[1], int(begin), int(end), sil, A, E))
+
+
+def profile_as_hmm(trans, emit_m, emit_i):
+    """The profile HMM of L positions written as a generic HMM in the paper's extension (§5.2:
+    states, transitions, emissions, silent states), so its forward is §5.2's forward. State
+    order: B = M_0, then for j = 1..L: M_j, I_{j-1}, D_j; then I_L, then E (= M_{L+1}) — a
+    position-major total order (the paper's "arbitrary total order", L453-L455).
+    trans[j][3 f + t]: from (M_j, I_j, D_j)[f] to (M_{j+1}, I_j, D_{j+1})[t]."""
+    trans = np.asarray(trans, np.float64)
+    eM, eI = np.asarray(emit_m, np.float64), np.asarray(emit_i, np.float64)
+    L = trans.shape[0] - 1
+    K = eM.shape[1]
+    idx = {("M", 0): 0}
+    for j in range(1, L + 1):
+        idx[("M", j)] = len(idx)
+        idx[("I", j - 1)] = len(idx)
+        idx[("D", j)] = len(idx)
+    idx[("I", L)] = len(idx)
+    idx[("M", L + 1)] = len(idx)       # E
+    S = len(idx)
+    A = np.zeros((S, S))
+    E = np.zeros((S, K))
+    silent = np.zeros(S, np.uint8)
+    for (k, j), s in idx.items():
+        if k == "D" or (k == "M" and j in (0, L + 1)):
+            silent[s] = 1
+        elif k == "M":
+            E[s] = eM[j]
+        else:
+            E[s] = eI[j]
+    for j in range(L + 1):
+        for f, kf in enumerate("MID"):
+            src = idx.get((kf, j))
+            if src is None:
+                continue
+            for t, dst in enumerate((("M", j + 1), ("I", j), ("D", j + 1))):
+                p = trans[j][3 * f + t]
+                if p > 0 and dst in idx:
+                    A[src, idx[dst]] += p
+    return silent, A, E, idx[("M", 0)], idx[("M", L + 1)]
+
+
+def profile_forward(x, trans, emit_m, emit_i) -> float:
+    """log P(x) of the profile HMM, via the generic silent-state forward."""
+    silent, A, E, b, e = profile_as_hmm(trans, emit_m, emit_i)
+    return silent_forward(x, silent, A, E, b, e)
+
+
+def profile_forward_batch(cat, off, L, trans, emit_m, emit_i, threads=1) -> np.ndarray:
+    silent, A, E, b, e = profile_as_hmm(trans, emit_m, emit_i)
+    n = len(off) - 1
+    out = np.zeros(n, dtype=np.float64)
+    cat, off = _u8(cat), np.ascontiguousarray(off, np.int64)
+    A = np.ascontiguousarray(A)
+    E = np.ascontiguousarray(E)
+    _parallel(n, lambda f, c: lib().orc_silent_forward_batch(f, c, cat, off, len(silent), E.shape[1], int(b), int(e),
+                                                             silent, A, E, out), threads)
+    return out
 
 
 def viterbi(x, lpi, lA, lE) -> tuple[int, np.ndarray]:

@@ -504,3 +504,60 @@ def local_affine_best(s, t, sub, go, ge):
             if H[i, j] > best:
                 best, bi, bj = int(H[i, j]), i, j
     return best, (bi, bj)
+
+
+# ----------------------------------------------------------------------------- HMMs with silent states
+def brute_silent_hmm(x, silent, A, E, begin, end):
+    """log of the sum over EVERY state path begin -> ... -> end that emits exactly x (emitting
+    states consume one symbol each, silent ones none), each path's probability the product of its
+    transitions and emissions. Depth-first over (state, symbols emitted); silent cycles are not
+    allowed (a path through a silent cycle would not terminate)."""
+    T = len(x)
+    S = len(silent)
+    tot = 0.0
+    stack = [(begin, 0, 1.0, 0)]
+    while stack:
+        s, i, p, depth = stack.pop()
+        assert depth <= (T + 1) * S + 1, "silent cycle"
+        if s == end and i == T:
+            tot += p
+            continue
+        for t in range(S):
+            a = A[s][t]
+            if a <= 0:
+                continue
+            if silent[t]:
+                stack.append((t, i, p * a, depth + 1))
+            elif i < T:
+                e = E[t][x[i]]
+                if e > 0:
+                    stack.append((t, i + 1, p * a * e, depth + 1))
+    return math.log(tot) if tot > 0 else -math.inf
+
+
+def brute_profile(x, trans, emit_m, emit_i):
+    """log P(x) of a profile HMM by walking its states directly ((M,j), (I,j), (D,j); M_0 = begin,
+    M_{L+1} = end) over every path that emits exactly x — written from the profile's own
+    description, independent of any generic-HMM encoding."""
+    L = len(trans) - 1
+    T = len(x)
+    tot = 0.0
+    stack = [("M", 0, 0, 1.0)]
+    while stack:
+        k, j, i, p = stack.pop()
+        if k == "M" and j == L + 1:
+            if i == T:
+                tot += p
+            continue
+        f = "MID".index(k)
+        for t, (kt, jt) in enumerate((("M", j + 1), ("I", j), ("D", j + 1))):
+            a = trans[j][3 * f + t]
+            if a <= 0 or (kt == "D" and jt > L):
+                continue
+            if kt == "D" or (kt == "M" and jt == L + 1):
+                stack.append((kt, jt, i, p * a))
+            elif i < T:
+                e = (emit_m if kt == "M" else emit_i)[jt][x[i]]
+                if e > 0:
+                    stack.append((kt, jt, i + 1, p * a * e))
+    return math.log(tot) if tot > 0 else -math.inf
