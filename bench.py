@@ -49,7 +49,7 @@ MEASURED_UBENCH = {  # profiles/ubench_r01.jsonl, lane-ops per SM clock on B200 
     "viaddmnmx_s32": 64.0, "viaddmnmx_s16x2": 128.0, "ffma": 128.0, "lds_bytes": 128.0,
 }
 SMS = 148
-ALL_CONFIGS = ["sw", "nuss1", "hmm", "nuss4", "nuss5", "swa", "diag"]
+ALL_CONFIGS = ["sw", "nuss1", "hmm", "nuss4", "nuss5", "swa", "diag", "phmm"]
 # configs in the `configs` block at N > 1: the batched ones (the others are single tables: replicas only)
 SHARDED = {"sw", "hmm", "nuss5", "swa", "diag", "phmm"}
 
@@ -283,7 +283,7 @@ def workload(name, rank=0, world=1, scaling="strong"):
                 "workload": "BASELINE config 3: 64-state dense HMM, 10k DNA sequences x 1000, forward + Viterbi "
                             "with Viterbi tracebacks (cells = 2 tables x S x T x n)"}
     if name == "phmm":
-        n = 10_000
+        n = 13_355   # the database size of the paper's Fig.15 (L297)
         d = dpgen.profile_hmm_workload(n_seqs=n)
         ids = shard_ids(name, n, None, rank, world, scaling)
         cat, off = d["cat"], d["off"]
@@ -294,8 +294,8 @@ def workload(name, rank=0, world=1, scaling="strong"):
         return {"kind": "phmm", "n_total": n, "ids": ids, "a_cat": cat, "a_off": off, "max_la": int(np.diff(d["off"]).max()),
                 "phmm": d, "cells_total": int(3 * L * np.diff(d["off"]).sum()), "cells_local": int(3 * L * lens.sum()),
                 "inner_local": int(L * lens.sum()), "tb_stride": None,
-                "workload": f"SURVEY 8(f) NEXT 3: profile-HMM forward (§6.3), {L}-position model, 10k sequences "
-                            f"sampled from it (cells = 3 tables x L x T)"}
+                "workload": f"SURVEY 8(f) NEXT 3: profile-HMM forward (§6.3), {L}-position protein profile, 13,355 "
+                            f"sequences sampled from it (Fig.15's database size; cells = 3 tables x L x T)"}
     raise SystemExit(f"unknown config {name}")
 
 
@@ -314,7 +314,7 @@ def make_plans(dp, W):
                         want_traceback=True)]
     if W["kind"] == "phmm":
         d = W["phmm"]
-        return [dp.ProfilePlan(d["L"], W["max_la"], **d["model"])]
+        return [dp.Plan(dp.PROFILE_FORWARD, W["max_la"], **d["model"])]
     h = W["hmm"]
     return [dp.Plan(dp.HMM_FORWARD, W["max_la"], pi=h["pi"], A=h["A"], E=h["E"]),
             dp.Plan(dp.HMM_VITERBI, W["max_la"], lpi=h["lpi"], lA=h["lA"], lE=h["lE"], want_traceback=True)]
@@ -571,12 +571,13 @@ def roofline(W, name, phase_ms, alone, pk):
         return alu(kname, W["inner_local"], phase_ms[0], peak16,
                    "ubench_r01 VIADDMNMX.S16x2 x 148 SMs x sm_max_mhz (one split evaluation = one max-plus)")
     if W["kind"] == "phmm":
-        # forward: per cell (j, i): M = e (M + I + D)·t (3 FMA), I (3 FMA), D (2 FMA) -> 8 FFMA lane-ops per
-        # position-column pair; roofline = the FFMA SIMT peak
+        # forward: per (position j, index i) nine transition products and two emission products (M, I)
+        # = 11 fp32 FMA-pipe lane-ops; roofline = the FFMA SIMT peak
         peakf = MEASURED_UBENCH["ffma"] * SMS * clock_hz
-        r = alu("k_phmm_forward", 8 * W["inner_local"], phase_ms[0], peakf,
-                "ubench_r01 FFMA 128 lane-ops/clk/SM x 148 SMs x sm_max_mhz (8 FMA per profile position and residue)")
-        r["unit"] = "TFLOP-lane-ops/s"
+        r = alu("k_phmm_forward", 11 * W["inner_local"], phase_ms[0], peakf,
+                "ubench_r01 FFMA 128 lane-ops/clk/SM x 148 SMs x sm_max_mhz (11 FMA-pipe ops per position and "
+                "residue: 9 transition products + 2 emissions)")
+        r["unit"] = "Tops/s (fp32 FMA pipe)"
         return r
     # HMM: Viterbi (max-plus, SIMT, the step's critical path) and the tcgen05 forward on its own time
     vit_ms = alone.get("k_viterbi", phase_ms[1])

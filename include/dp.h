@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define DP_ABI_VERSION 3
+#define DP_ABI_VERSION 4
 #define DP_MAX_DIM 4
 
 typedef enum dp_status {
@@ -56,9 +56,13 @@ typedef enum dp_kind {
   DP_HMM_VITERBI = 4, /* max-variant of Fig.11a (L463–L464), int32 milli-bit score */
   DP_SW_AFFINE = 5    /* SURVEY §8(f) NEXT 1 (Gotoh, L509–L520; mutual recursion = Further Work L585–L589):
                          local alignment, gap of length k costs gap_open + k * gap_extend, int32 score */,
-  DP_DIAG_LCS = 6     /* the §4.7 example f(x,y) = ... f(x-1,y-1) ... (L386–L388) as the
+  DP_DIAG_LCS = 6,    /* the §4.7 example f(x,y) = ... f(x-1,y-1) ... (L386–L388) as the
                          longest common substring, int32; its schedule is chosen per problem among the
                          conditional candidates (S = i when |a| < |b|, else S = j); no traceback (ABI 3) */
+  DP_PROFILE_FORWARD = 7 /* profile-HMM forward (§6.3; Durbin ch.5, ref [3]):
+                         one profile of n_positions match positions against each sequence a, natural-log
+                         likelihood, float32; three tables (M, I, D) over (position, index), schedule (1,1);
+                         no traceback (ABI 4) */
 } dp_kind;
 
 /*
@@ -147,6 +151,13 @@ typedef struct dp_desc {
   /* affine gaps (DP_SW_AFFINE; ABI 2): gap of length k costs gap_open + k * gap_extend */
   int32_t gap_open;          /* >= 0 */
   int32_t gap_extend;        /* >= 1 */
+  /* profile HMM (DP_PROFILE_FORWARD; ABI 4). Positions j = 0..L (L = n_positions >= 1); state M_0 is the
+   * begin state, M_{L+1} the end state, D_0 does not exist. alphabet_size = K <= 32 emission codes. */
+  int32_t n_positions;       /* L */
+  const float* ptrans;       /* [(L+1) x 9]: ptrans[9 j + 3 f + t] = probability from (M_j, I_j, D_j)[f] to
+                                (M_{j+1}, I_j, D_{j+1})[t]; at j = L the "to M_{L+1}" slot is the end */
+  const float* pemit_m;      /* [(L+1) x K] match emissions e_{M_j}(c) (row 0 unused) */
+  const float* pemit_i;      /* [(L+1) x K] insert emissions e_{I_j}(c) */
 } dp_desc;
 
 typedef struct dp_plan* dp_plan_t;
@@ -167,8 +178,8 @@ dp_status dp_plan_get_schedule(dp_plan_t p, int32_t coeff[], int* ndim, int64_t*
  * dp_solve_batch — the `map` primitive. All pointers are DEVICE pointers:
  *   a_cat/a_off: n sequences concatenated (uint8 codes), a_off[n+1] int64;
  *   b_cat/b_off: second sequences (alignment kinds), else NULL;
- *   scores_out:  n x int32 (EDIT, SW, NUSSINOV, VITERBI) or n x float32 (FORWARD),
- *                in input order.
+ *   scores_out:  n x int32 (EDIT, SW, NUSSINOV, VITERBI) or n x float32 (HMM_FORWARD,
+ *                PROFILE_FORWARD: natural-log likelihood, -inf for P = 0), in input order.
  * Asynchronous on `stream` (a cudaStream_t; NULL = legacy default stream).
  * max_len_a/max_len_b of THIS batch must be supplied (<= the plan maxima);
  * they size the launch without reading device offsets on the host.

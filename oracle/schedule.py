@@ -143,6 +143,26 @@ def edit_instance(n, m):
     return dom, (lambda c: [(c[0] - 1, c[1]), (c[0], c[1] - 1), (c[0] - 1, c[1] - 1)]), (n + 1, m + 1)
 
 
+def profile_instance(L, T, position_major=True):
+    """Profile-HMM forward (§6.3) on cells (j, i), j = 0..L positions, i = 0..T: the cell holds
+    M, I, D of position j; M calls (j-1, i-1), I calls (j, i-1), the silent D calls (j-1, i) (all
+    three states of the called cell). position_major=False: the generic §5.2 reading over a flat
+    state axis s = 3 j + type where `t.start` may be ANY state (L466-L472) and a silent state
+    reads the same index: every state calls every state at i-1 (emitting) and at i (silent)."""
+    if position_major:
+        dom = [(j, i) for j in range(L + 1) for i in range(T + 1)]
+        return dom, (lambda c: [(c[0] - 1, c[1] - 1), (c[0], c[1] - 1), (c[0] - 1, c[1])]), (L + 1, T + 1)
+    S = 3 * (L + 1)
+    dom = [(s, i) for s in range(S) for i in range(T + 1)]
+
+    def calls(c):
+        s, i = c
+        same = [(q, i) for q in range(S) if q != s] if s % 3 == 2 else []   # silent delete states
+        return [(q, i - 1) for q in range(S)] + same
+
+    return dom, calls, (S, T + 1)
+
+
 def diagonal_instance(nx, ny):
     """f(x,y) = ... f(x-1,y-1) ... (§4.7)."""
     dom = [(x, y) for x in range(nx) for y in range(ny)]

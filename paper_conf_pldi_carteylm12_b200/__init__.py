@@ -15,9 +15,11 @@ import numpy as np
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("DP_LIB") or os.path.join(_PKG, "libdp.so")  # DP_LIB: experiment builds only
 
-EDIT, SW_LINEAR, NUSSINOV, HMM_FORWARD, HMM_VITERBI, SW_AFFINE, DIAG_LCS = range(7)
+EDIT, SW_LINEAR, NUSSINOV, HMM_FORWARD, HMM_VITERBI, SW_AFFINE, DIAG_LCS, PROFILE_FORWARD = range(8)
 KIND_NAMES = {EDIT: "edit", SW_LINEAR: "sw_linear", NUSSINOV: "nussinov", HMM_FORWARD: "hmm_forward",
-              HMM_VITERBI: "hmm_viterbi", SW_AFFINE: "sw_affine"}
+              HMM_VITERBI: "hmm_viterbi", SW_AFFINE: "sw_affine", DIAG_LCS: "diag_lcs",
+              PROFILE_FORWARD: "profile_forward"}
+FLOAT_KINDS = (HMM_FORWARD, PROFILE_FORWARD)
 STATUS = {0: "DP_OK", 1: "DP_E_INVALID", 2: "DP_E_NO_SCHEDULE", 3: "DP_E_UNSUPPORTED", 4: "DP_E_TOO_LARGE",
           5: "DP_E_NOMEM", 6: "DP_E_CUDA", 7: "DP_E_NO_TRACEBACK"}
 MAX_DIM = 4
@@ -45,6 +47,8 @@ class Desc(ctypes.Structure):
         ("lpi", ctypes.c_void_p), ("lA", ctypes.c_void_p), ("lE", ctypes.c_void_p),
         ("coeff_bound", ctypes.c_int32), ("user_coeff", ctypes.c_void_p), ("want_traceback", ctypes.c_int32),
         ("gap_open", ctypes.c_int32), ("gap_extend", ctypes.c_int32),
+        ("n_positions", ctypes.c_int32), ("ptrans", ctypes.c_void_p), ("pemit_m", ctypes.c_void_p),
+        ("pemit_i", ctypes.c_void_p),
     ]
 
 
@@ -174,7 +178,7 @@ class Plan:
 
     def __init__(self, kind, max_len_a, max_len_b=0, *, sigma=None, gap=0, alphabet_size=0, pair_mask=None,
                  min_hairpin=0, pi=None, A=None, E=None, lpi=None, lA=None, lE=None, want_traceback=False,
-                 coeff_bound=0, user_coeff=None, gap_open=0, gap_extend=0):
+                 coeff_bound=0, user_coeff=None, gap_open=0, gap_extend=0, trans=None, emit_m=None, emit_i=None):
         self.kind = kind
         self._keep = []
         d = Desc()
@@ -207,6 +211,12 @@ class Plan:
         d.pi, d.A, d.E = keep(pi, np.float32), keep(A, np.float32), keep(E, np.float32)
         d.lpi, d.lA, d.lE = keep(lpi, np.int32), keep(lA, np.int32), keep(lE, np.int32)
         d.user_coeff = keep(user_coeff, np.int32)
+        if trans is not None:  # profile HMM: (L+1) x 9 transitions, (L+1) x K emissions
+            d.n_positions = np.asarray(trans).shape[0] - 1
+            d.alphabet_size = np.asarray(emit_m).shape[1]
+            d.ptrans = keep(np.asarray(trans).reshape(-1), np.float32)
+            d.pemit_m = keep(np.asarray(emit_m).reshape(-1), np.float32)
+            d.pemit_i = keep(np.asarray(emit_i).reshape(-1), np.float32)
         self.alphabet_size = d.alphabet_size
         self.max_len_a, self.max_len_b = int(max_len_a), int(max_len_b)
         self.want_traceback = bool(want_traceback)
@@ -261,7 +271,7 @@ class Plan:
         self._debug_codes(a_cat, limit)
         self._debug_codes(b_cat, limit)
         if out is None:
-            dt = torch.float32 if self.kind == HMM_FORWARD else torch.int32
+            dt = torch.float32 if self.kind in FLOAT_KINDS else torch.int32
             out = torch.empty(max(n, 0), dtype=dt, device=a_off.device)
         self._last_inputs = (a_cat, a_off, b_cat, b_off)  # must outlive dp_traceback
         _check(lib().dp_solve_batch(self._h, n, _ptr(a_cat), _ptr(a_off), _ptr(b_cat), _ptr(b_off), int(max_len_a),
@@ -273,7 +283,7 @@ class Plan:
         1-element device tensor (int32, or float32 log-likelihood for HMM_FORWARD)."""
         import torch
         if out is None:
-            out = torch.empty(1, dtype=torch.float32 if self.kind == HMM_FORWARD else torch.int32, device=a.device)
+            out = torch.empty(1, dtype=torch.float32 if self.kind in FLOAT_KINDS else torch.int32, device=a.device)
         self._last_inputs = (a, None, b, None)  # must outlive dp_traceback
         _check(lib().dp_solve(self._h, _ptr(a), int(a.numel()), _ptr(b), int(b.numel()) if b is not None else 0,
                               _ptr(out), _stream_ptr(stream)), "dp_solve")
@@ -303,7 +313,7 @@ class Plan:
     def solve_batch_host(self, a_cat, a_off, b_cat=None, b_off=None, *, tb_stride=0, stream=None):
         """Host (numpy, ideally pinned) buffers in and out; synchronous (includes H2D/D2H)."""
         n = len(a_off) - 1
-        scores = np.empty(n, dtype=np.float32 if self.kind == HMM_FORWARD else np.int32)
+        scores = np.empty(n, dtype=np.float32 if self.kind in FLOAT_KINDS else np.int32)
         tb = tbl = tbc = None
         if self.want_traceback and tb_stride:
             tb = np.empty((n, tb_stride), dtype=np.uint8)

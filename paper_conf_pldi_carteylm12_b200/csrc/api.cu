@@ -71,6 +71,8 @@ struct dp_plan {
   uint8_t* d_pair = nullptr;
   float *d_pi = nullptr, *d_A = nullptr, *d_E = nullptr;
   int32_t *d_lpi = nullptr, *d_lA = nullptr, *d_lE = nullptr;
+  int L = 0;                                         // DP_PROFILE_FORWARD positions
+  float *d_ptr = nullptr, *d_pem = nullptr, *d_pei = nullptr;
   // retained state of the most recent solve
   DevBuf tb_state, tb_aux, tb_aux2, scratch;
   DevBuf tb_state_alt;             // host entry point: the other chunk's retained state (packed SW)
@@ -169,6 +171,12 @@ int families(int kind, int64_t la, int64_t lb, int S, int64_t ext[2], int* trian
       ext[0] = la + 1; ext[1] = lb + 1;
       deps[0].offset[0] = -1; deps[0].offset[1] = -1;
       return 1;
+    case DP_PROFILE_FORWARD:  // (j, i): M <- (-1,-1), I <- (0,-1), D <- (-1,0) (position-major state order)
+      ext[0] = S + 1; ext[1] = la + 1;
+      deps[0].offset[0] = -1; deps[0].offset[1] = -1;
+      deps[1].offset[1] = -1;
+      deps[2].offset[0] = -1;
+      return 3;
     case DP_HMM_FORWARD:
     case DP_HMM_VITERBI:  // F(t.start, i-1) for t in s.transitionsto: any state (§5.2)
       ext[0] = S; ext[1] = la + 1;
@@ -234,6 +242,7 @@ void dp_plan_destroy(dp_plan_t p) {
   cudaFree(p->d_sigma); cudaFree(p->d_pair);
   cudaFree(p->d_pi); cudaFree(p->d_A); cudaFree(p->d_E);
   cudaFree(p->d_lpi); cudaFree(p->d_lA); cudaFree(p->d_lE);
+  cudaFree(p->d_ptr); cudaFree(p->d_pem); cudaFree(p->d_pei);
   DevBuf* bufs[] = {&p->tb_state, &p->tb_aux, &p->tb_aux2, &p->scratch, &p->own_scores, &p->h_a, &p->h_b,
                     &p->h_aoff, &p->h_boff, &p->h_scores, &p->h_tb, &p->h_tblen, &p->h_coords};
   for (DevBuf* b : bufs) b->release();
@@ -257,7 +266,7 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
   if (!d || !out) return DP_E_INVALID;
   *out = nullptr;
   if (d->struct_size != sizeof(dp_desc)) return DP_E_INVALID;
-  if (d->kind < DP_EDIT || d->kind > DP_DIAG_LCS) return DP_E_INVALID;
+  if (d->kind < DP_EDIT || d->kind > DP_PROFILE_FORWARD) return DP_E_INVALID;
   if (d->max_len_a < 0 || d->max_len_b < 0) return DP_E_INVALID;
   dp_plan* p = new (std::nothrow) dp_plan();
   if (!p) return DP_E_NOMEM;
@@ -322,6 +331,21 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       p->hairpin = d->min_hairpin;
       e = upload(&p->d_pair, d->pair_mask, 16);
       break;
+    case DP_PROFILE_FORWARD:
+      p->L = d->n_positions;
+      p->K = d->alphabet_size;
+      if (p->L < 1 || p->K < 1 || !d->ptrans || !d->pemit_m || !d->pemit_i) { st = DP_E_INVALID; break; }
+      if (p->K > 32) { st = DP_E_UNSUPPORTED; break; }
+      if (p->want_tb) { st = DP_E_UNSUPPORTED; break; }
+      if (smem_limit > 0 && dpk::phmm_smem_bytes(p->L, p->K, d->max_len_a) > (size_t)smem_limit) {
+        st = DP_E_TOO_LARGE;
+        break;
+      }
+      p->S = p->L;
+      e = upload(&p->d_ptr, d->ptrans, (size_t)(p->L + 1) * 9);
+      if (e == cudaSuccess) e = upload(&p->d_pem, d->pemit_m, (size_t)(p->L + 1) * p->K);
+      if (e == cudaSuccess) e = upload(&p->d_pei, d->pemit_i, (size_t)(p->L + 1) * p->K);
+      break;
     case DP_HMM_FORWARD:
     case DP_HMM_VITERBI:
       p->S = d->n_states;
@@ -367,7 +391,7 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
     // The kernels implement the derived schedule; a user schedule that is valid
     // but differs would need another kernel (conditional schedules, §4.7: NEXT).
     // Coefficients of a dimension of extent 1 do not change the partitions.
-    static const int32_t expect[6][2] = {{1, 1}, {1, 1}, {-1, 1}, {0, 1}, {0, 1}, {1, 1}};
+    static const int32_t expect[8][2] = {{1, 1}, {1, 1}, {-1, 1}, {0, 1}, {0, 1}, {1, 1}, {0, 0}, {1, 1}};
     for (int i = 0; i < 2; ++i)
       if (p->ext[i] > 1 && p->coeff[i] != expect[d->kind][i]) st = DP_E_UNSUPPORTED;
   }
@@ -516,6 +540,14 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       }
       break;
     }
+    case DP_PROFILE_FORWARD: {
+      dpk::PhmmArgs P{};
+      P.n = n; P.x_cat = a_cat; P.x_off = a_off; P.max_len = max_len_a; P.L = p->L; P.K = p->K;
+      P.trans = p->d_ptr; P.emit_m = p->d_pem; P.emit_i = p->d_pei;
+      P.ll_out = static_cast<float*>(scores_out);
+      e = dpk::phmm_forward(P, s, &p->launches);
+      break;
+    }
     case DP_HMM_FORWARD:
     case DP_HMM_VITERBI: {
       dpk::HmmArgs H{};
@@ -598,7 +630,7 @@ dp_status dp_solve(dp_plan_t p, const uint8_t* a, int64_t len_a, const uint8_t* 
 dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, int64_t stride, int32_t* out_len,
                        int32_t* coords, void* stream) {
   if (!p) return DP_E_INVALID;
-  if (p->kind == DP_HMM_FORWARD) return DP_E_UNSUPPORTED;
+  if (p->kind == DP_HMM_FORWARD || p->kind == DP_PROFILE_FORWARD) return DP_E_UNSUPPORTED;
   if (!p->want_tb || p->last_n < 0) return DP_E_NO_TRACEBACK;
   if (first < 0 || count < 0 || first + count > p->last_n || stride < 0) return DP_E_INVALID;
   if (count > 0 && (!out || !out_len)) return DP_E_INVALID;

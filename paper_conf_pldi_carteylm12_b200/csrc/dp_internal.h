@@ -148,4 +148,20 @@ cudaError_t hmm_viterbi(const HmmArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t hmm_viterbi_traceback(const HmmArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                                   int32_t* out_len, cudaStream_t s, int64_t* launches);
 
+// ---------------------------------------------------------------- profile HMM (phmm.cu)
+struct PhmmArgs {
+  int64_t n;
+  const uint8_t* x_cat;
+  const int64_t* x_off;
+  int64_t max_len;
+  int L, K;
+  const float* trans;    // device [(L+1) x 9]: from (M_j, I_j, D_j) to (M_{j+1}, I_j, D_{j+1})
+  const float* emit_m;   // device [(L+1) x K] (row 0 unused)
+  const float* emit_i;   // device [(L+1) x K]
+  float* ll_out;         // n natural-log likelihoods
+  int rows_tab;          // set by the launcher
+};
+size_t phmm_smem_bytes(int L, int K, int64_t max_len);
+cudaError_t phmm_forward(const PhmmArgs& a, cudaStream_t s, int64_t* launches);
+
 }  // namespace dpk

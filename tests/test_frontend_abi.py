@@ -30,7 +30,7 @@ def test_exports_match_header(dp):
     L = dp.lib()
     for name in declared:
         assert hasattr(L, name), name
-    assert L.dp_abi_version() == 3
+    assert L.dp_abi_version() == 4
     for code in range(8):
         assert L.dp_status_string(code)
 
@@ -195,3 +195,19 @@ def test_conditional_matches_bruteforce(dp, seed):
         a = dp.schedule_derive(tuple(ext), deps, coeff_bound=B)["a"]
         assert a in got
         assert got[dp.schedule_select(got, tuple(ext))] == a
+
+
+def test_profile_schedule_depends_on_state_order():
+    """"the ordering of the model elements may be important ... different
+    orderings may permit or restrict the available schedules". A profile HMM's silent deletes read
+    the same index: with the generic `transitionsto` reading ("t.start varies over any state",
+    L466-L472) that is a ranged family over all states at offset 0 in i, cyclic -> no schedule;
+    with the states in position-major order the families are uniform, (-1,-1), (0,-1), (-1,0),
+    and the schedule is the anti-diagonal (1,1)."""
+    import paper_conf_pldi_carteylm12_b200 as dp
+    S = 3 * 10 + 3
+    with pytest.raises(dp.DPError) as e:
+        dp.schedule_derive((S, 50), [((0, -1), 0, -(S - 1), S - 1), ((0, 0), 0, -(S - 1), S - 1)])
+    assert e.value.code == 2
+    r = dp.schedule_derive((11, 50), [((-1, -1), None, 0, 0), ((0, -1), None, 0, 0), ((-1, 0), None, 0, 0)])
+    assert r["a"] == (1, 1) and r["window"] == 2

@@ -643,3 +643,45 @@ def test_diag_plan_schedules(dp):
     with pytest.raises(dp.DPError) as e:
         dp.Plan(dp.DIAG_LCS, 100, 50, want_traceback=True)
     assert e.value.code == 3
+
+
+# ----------------------------------------------------------------------------- profile HMM (NEXT 3)
+@pytest.mark.parametrize("L,maxT", [(1, 12), (7, 40), (100, 160), (256, 300), (300, 420), (700, 800)])
+def test_profile_forward_random(dp, orc, L, maxT, capsys):
+    """Profile-HMM forward: random profiles (one strip, several strips of 256 rows, ragged last
+    strip), sequences sampled from the model plus random ones, empty and length-1 sequences;
+    log P within relative 1e-5 of the oracle's generic silent-state forward (fp64)."""
+    g = np.random.default_rng(900 + L)
+    K = 20
+    tr, eM, eI = dpgen.profile_hmm_params(g, L, K)
+    tr32, eM32, eI32 = (v.astype(np.float32) for v in (tr, eM, eI))
+    seqs = dpgen.sample_profile(g, tr, eM, eI, 24, max_len=maxT)
+    seqs += [g.integers(0, K, size=int(g.integers(0, maxT + 1))).astype(np.uint8) for _ in range(6)]
+    seqs += [np.zeros(0, np.uint8), np.zeros(1, np.uint8)]
+    cat, off = dpgen.pack(seqs)
+    ml = max(len(s) for s in seqs)
+    with dp.Plan(dp.PROFILE_FORWARD, ml, trans=tr32, emit_m=eM32, emit_i=eI32) as p:
+        assert p.schedule()["a"] == (1, 1)
+        ll = host(p.solve_batch(cuda(cat), cuda(off), max_len_a=ml))
+    want = orc.profile_forward_batch(cat, off, L, tr32.astype(np.float64), eM32.astype(np.float64),
+                                     eI32.astype(np.float64), threads=THREADS)
+    fin = np.isfinite(want)
+    assert (np.isfinite(ll) == fin).all()
+    dl, rel = forward_errors(ll[fin], want[fin], f"profile L={L}", capsys)
+    assert rel.max() <= 1e-5
+
+
+def test_profile_workload_sampled(dp, orc, capsys):
+    """The bench workload (L = 256, 13,355 sequences sampled from the profile) at full size in the
+    bench's launch; a seeded sample against the oracle."""
+    d = dpgen.profile_hmm_workload()
+    cat, off = d["cat"], d["off"]
+    ml = int(np.diff(off).max())
+    with dp.Plan(dp.PROFILE_FORWARD, ml, **d["model"]) as p:
+        ll = host(p.solve_batch(cuda(cat), cuda(off), max_len_a=ml))
+    ids = np.sort(np.random.default_rng(901).choice(len(off) - 1, 48, replace=False))
+    sub_cat, sub_off = dpgen.pack([cat[off[q]:off[q + 1]] for q in ids])
+    want = orc.profile_forward_batch(sub_cat, sub_off, d["L"], **d["model64"], threads=THREADS)
+    dl, rel = forward_errors(ll[ids], want, "profile workload (L=256)", capsys)
+    assert rel.max() <= 1e-5
+    assert np.isfinite(ll).all()
