@@ -348,6 +348,7 @@ constexpr int kTbUnroll = TB5_UNROLL;   // re-run steps unrolled
 #define TB5_MINB 4                       // CTAs per SM (register cap; 4 / 5 / 6 with no unroll: 1.049 / 1.059 / 1.099 ms)
 #endif
 constexpr int kCW = kGL * kSlab;         // code words per group: [c - 1][m]
+constexpr int kCWp = kCW + 4;            // group stride: 4 banks apart, so the 8 groups' code stores hit 32 banks
 constexpr int kTS = 36;                  // top-row keys per group, c = 0..32
 constexpr int kBS = 40;                  // staged b residues per half (columns D-3 .. D+36)
 constexpr int kDeadCode = 31;            // residue code whose sigma row/column is kDead4 (alphabets < 32)
@@ -367,7 +368,7 @@ struct TbState {      // one problem in one half of a group (shared memory; writ
   int i, j, n;        // walk: current cell, ops written
   int ei, ej;         // end cell
 };
-constexpr int kGroupBytes = 4 * kCW + 4 * kTS + 2 * kBS + 2 * kBlk + 2 * (int)sizeof(TbState);
+constexpr int kGroupBytes = 4 * kCWp + 4 * kTS + 2 * kBS + 2 * kBlk + 2 * (int)sizeof(TbState);
 constexpr int kTbWarpBytes = kGroups * kGroupBytes;
 
 __device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
@@ -404,11 +405,11 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
   }
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, gq = lane / kGL, m = lane % kGL;
   uint8_t* wb = tsm + 2048 + warp * kTbWarpBytes;
-  uint32_t* Cs = reinterpret_cast<uint32_t*>(wb) + gq * kCW;
-  uint32_t* Ts = reinterpret_cast<uint32_t*>(wb + kGroups * 4 * kCW) + gq * kTS;
-  uint8_t* bS = wb + kGroups * 4 * (kCW + kTS) + gq * 2 * kBS;                  // [2][kBS] staged b residues
-  uint8_t* aS = wb + kGroups * (4 * (kCW + kTS) + 2 * kBS) + gq * 2 * kBlk;  // [2][kBlk] staged a residues
-  TbState* St = reinterpret_cast<TbState*>(wb + kGroups * (4 * (kCW + kTS) + 2 * kBS + 2 * kBlk)) + 2 * gq;
+  uint32_t* Cs = reinterpret_cast<uint32_t*>(wb) + gq * kCWp;
+  uint32_t* Ts = reinterpret_cast<uint32_t*>(wb + kGroups * 4 * kCWp) + gq * kTS;
+  uint8_t* bS = wb + kGroups * 4 * (kCWp + kTS) + gq * 2 * kBS;                  // [2][kBS] staged b residues
+  uint8_t* aS = wb + kGroups * (4 * (kCWp + kTS) + 2 * kBS) + gq * 2 * kBlk;  // [2][kBlk] staged a residues
+  TbState* St = reinterpret_cast<TbState*>(wb + kGroups * (4 * (kCWp + kTS) + 2 * kBS + 2 * kBlk)) + 2 * gq;
   const uint32_t sig32 = (uint32_t)__cvta_generic_to_shared(sig_s);
   const uint32_t cs32 = (uint32_t)__cvta_generic_to_shared(Cs);
   const uint32_t ts32 = (uint32_t)__cvta_generic_to_shared(Ts);

@@ -685,3 +685,19 @@ def test_profile_workload_sampled(dp, orc, capsys):
     dl, rel = forward_errors(ll[ids], want, "profile workload (L=256)", capsys)
     assert rel.max() <= 1e-5
     assert np.isfinite(ll).all()
+
+
+@pytest.mark.parametrize("count", [5, 120, 600])
+def test_nussinov_small_kernel(dp, orc, count):
+    """k_nuss_small (n <= 128; one CTA per problem, traceback decisions in shared memory): ragged
+    lengths 0..128, both hairpins, one CTA of 1024 threads per problem (few problems) and 256-thread
+    CTAs (many); scores and canonical dot-brackets bit-exact."""
+    g = np.random.default_rng(160 + count)
+    for h, pm in ((3, dpgen.rna_pair_mask()), (0, dpgen.rna_pair_mask(gu=False))):
+        seqs, _ = rand_batch(g, count, 0, 128, 4)
+        seqs[0] = g.integers(0, 4, size=128).astype(np.uint8)
+        r = run_nuss(dp, seqs, h=h, pm=pm)
+        for q, x in enumerate(seqs):
+            if count > 120 and q % 7:
+                continue
+            assert (r["scores"][q], r["db"][q]) == orc.nussinov_traceback(x, pm, h), (q, len(x))
