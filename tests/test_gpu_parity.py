@@ -688,10 +688,9 @@ def test_profile_workload_sampled(dp, orc, capsys):
 
 
 @pytest.mark.parametrize("count", [5, 120, 600])
-def test_nussinov_small_kernel(dp, orc, count):
-    """k_nuss_small (n <= 128; one CTA per problem, traceback decisions in shared memory): ragged
-    lengths 0..128, both hairpins, one CTA of 1024 threads per problem (few problems) and 256-thread
-    CTAs (many); scores and canonical dot-brackets bit-exact."""
+def test_nussinov_short_batches(dp, orc, count):
+    """Short sequences (lengths 0..128, the cell-level and tiled paths' boundary region), a few and
+    many problems per batch, both hairpins; scores and canonical dot-brackets bit-exact."""
     g = np.random.default_rng(160 + count)
     for h, pm in ((3, dpgen.rna_pair_mask()), (0, dpgen.rna_pair_mask(gu=False))):
         seqs, _ = rand_batch(g, count, 0, 128, 4)
