@@ -472,6 +472,13 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
                 a1.record(stream)
             torch.cuda.synchronize(dev)
             alone[nm] = a0.elapsed_time(a1) / reps
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            a0.record(stream)
+            tb_plan.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
+            a1.record(stream)
+        torch.cuda.synchronize(dev)
+        alone["k_viterbi_tb"] = a0.elapsed_time(a1)
 
     fixed = None
     if W["kind"] == "diag":   # §4.7 evidence: the same batch with each candidate forced for every problem

@@ -156,9 +156,6 @@ __global__ void __launch_bounds__(kHW * 32) k_forward(HmmArgs H) {
   }
 }
 
-#ifndef VIT_TB_PF
-#define VIT_TB_PF 24  // Viterbi traceback: back-pointer rows prefetched ahead (24 / 64 / 128: same)
-#endif
 constexpr int kNegKey = -(1 << 30);
 constexpr int kRenorm = 32;
 
@@ -273,27 +270,67 @@ __global__ void __launch_bounds__(kHW * 32) k_viterbi(HmmArgs H) {
   }
 }
 
-__global__ void k_viterbi_tb(HmmArgs H, int64_t first, int64_t count, uint8_t* out, int64_t stride,
-                             int32_t* out_len) {
-  const int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (q >= count) return;
-  const int64_t p = first + q;
-  const int T = (int)(H.x_off[p + 1] - H.x_off[p]);
-  if (T > stride) { out_len[q] = -1; return; }
-  const uint8_t* bp = H.bp + (p * H.max_len) * kMaxS;
-  uint8_t* o = out + q * stride;
-  int s = H.final_state[p];
-  // the walk is one dependent load per step; the rows it will read are known in advance, so
-  // pull them towards L2 kPf steps ahead (the back-pointers come straight from DRAM otherwise)
-  constexpr int kPf = VIT_TB_PF;
-  for (int i = T - 1; i >= 1 && i >= T - kPf; --i)
-    asm volatile("prefetch.global.L2 [%0];" ::"l"(bp + (int64_t)(i - 1) * kMaxS));
-  for (int i = T; i >= 1; --i) {
-    o[i - 1] = (uint8_t)s;
-    if (i - 1 - kPf >= 1) asm volatile("prefetch.global.L2 [%0];" ::"l"(bp + (int64_t)(i - 2 - kPf) * kMaxS));
-    if (i > 1) s = bp[(int64_t)(i - 1) * kMaxS + s];
+// Viterbi traceback: one warp per sequence. The walk s_{i-1} = bp[i-1][s_i] is one dependent load
+// per step; the warp stages the back-pointer rows it will need 32 at a time (row i-1 by lane
+// T - i - 32c, one coalesced 2 KB read per chunk, the next chunk's loads in flight during the
+// walk) in shared memory, lane 0 walks the 32 steps there, and the warp writes the 32 states out
+// with one coalesced store.
+constexpr int kTbW = 4;  // warps per CTA
+
+__global__ void __launch_bounds__(kTbW * 32) k_viterbi_tb(HmmArgs H, int64_t first, int64_t count, uint8_t* out,
+                                                           int64_t stride, int32_t* out_len) {
+  __shared__ __align__(16) uint8_t rows[kTbW][2][32][kMaxS];
+  __shared__ uint8_t ob[kTbW][32];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int64_t q = (int64_t)blockIdx.x * kTbW + warp; q < count; q += (int64_t)gridDim.x * kTbW) {
+    const int64_t p = first + q;
+    const int T = (int)(H.x_off[p + 1] - H.x_off[p]);
+    if (T > stride) {
+      if (lane == 0) out_len[q] = -1;
+      continue;
+    }
+    if (T == 0) {
+      if (lane == 0) out_len[q] = 0;
+      continue;
+    }
+    const uint8_t* bp = H.bp + (p * H.max_len) * kMaxS;
+    uint8_t* o = out + q * stride;
+    int s = H.final_state[p];
+    const int nch = (T + 31) / 32;
+    // chunk c: lane t holds row r = T - 1 - 32 c - t (used at position i = r + 1), valid for r >= 1
+    auto load = [&](int c, uint4* v) {
+      const int r = T - 1 - 32 * c - lane;
+      const uint4* src = reinterpret_cast<const uint4*>(bp + (int64_t)(r >= 1 ? r : 1) * kMaxS);
+#pragma unroll
+      for (int w = 0; w < kMaxS / 16; ++w) v[w] = r >= 1 ? __ldcs(src + w) : make_uint4(0, 0, 0, 0);
+    };
+    auto stash = [&](int buf, const uint4* v) {
+      uint4* dst = reinterpret_cast<uint4*>(rows[warp][buf][lane]);
+#pragma unroll
+      for (int w = 0; w < kMaxS / 16; ++w) dst[w] = v[w];
+    };
+    uint4 v[kMaxS / 16];
+    load(0, v);
+    stash(0, v);
+    for (int c = 0; c < nch; ++c) {
+      if (c + 1 < nch) load(c + 1, v);   // in flight during the walk
+      __syncwarp();
+      if (lane == 0) {
+        const uint8_t* R = &rows[warp][c & 1][0][0];
+        for (int t = 0; t < 32; ++t) {
+          const int i = T - 32 * c - t;   // position
+          if (i < 1) break;
+          ob[warp][t] = (uint8_t)s;
+          if (i >= 2) s = R[t * kMaxS + s];
+        }
+      }
+      __syncwarp();
+      const int i = T - 32 * c - lane;
+      if (i >= 1) o[i - 1] = ob[warp][lane];
+      if (c + 1 < nch) stash((c + 1) & 1, v);
+    }
+    if (lane == 0) out_len[q] = T;
   }
-  out_len[q] = T;
 }
 
 int sms_of_current() {
@@ -358,8 +395,9 @@ cudaError_t hmm_viterbi(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
 cudaError_t hmm_viterbi_traceback(const HmmArgs& H, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                                   int32_t* out_len, cudaStream_t s, int64_t* launches) {
   if (count == 0) return cudaSuccess;
+  const int64_t grid = std::min<int64_t>((count + kTbW - 1) / kTbW, (int64_t)sms_of_current() * 12);
   ++*launches;
-  k_viterbi_tb<<<(unsigned)((count + 127) / 128), 128, 0, s>>>(H, first, count, out, stride, out_len);
+  k_viterbi_tb<<<(unsigned)grid, kTbW * 32, 0, s>>>(H, first, count, out, stride, out_len);
   return cudaGetLastError();
 }
 
