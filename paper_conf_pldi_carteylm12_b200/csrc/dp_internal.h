@@ -116,6 +116,8 @@ struct NussArgs {
   unsigned long long* round_ns;  // optional: %globaltimer at each tile-diagonal round (grid sweep)
   unsigned long long* dbg = nullptr;  // DP_NUSS_TIMING: batch-kernel phase cycles (8 counters)
   int tbw = 0;                        // grid traceback window (8/16/32; DP_NUSS_TBW), 0 = default
+  int* queue = nullptr;               // batch work queue counter (set by the launcher)
+  const int* perm = nullptr;          // problems in decreasing length (set by the launcher)
 };
 int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device);
 bool nuss_tiled_supported(int64_t max_len);

@@ -20,11 +20,10 @@
 // reads) and L[k][c] (row-major int16; B operand).
 //
 // Two drivers share the tile routines:
-//   k_nuss_tiled_cta   one problem per CTA (batches), C tiles in shared memory,
-//                      __syncthreads between phases;
-//   k_nuss_tiled_grid  one large problem on the whole grid (cooperative launch):
-//                      phase A split-K over every warp of the grid with
-//                      atomicMax into global C, grid.sync between phases.
+//   k_nuss_batch  one warp per problem (batches), problems from a length-sorted work queue;
+//   k_nuss_grid2  one large problem on the whole grid (cooperative launch): phase A split-K
+//                 over the grid's warps with atomicMax into global C, one grid.sync per
+//                 tile-diagonal.
 // The canonical traceback (Durbin order, smallest k) runs right after the fill
 // with the split search spread over a warp.
 #include <algorithm>
@@ -59,9 +58,6 @@ constexpr int kWaveUnroll = NUSS_WAVE_UNROLL;    // in-tile wavefront steps
 #define NUSS_TBK_B 1
 #endif
 constexpr int kTileWords = T * T;      // int16 per tile record half
-constexpr int kRec = 2 * kTileWords;   // int16 per tile record (UT + L)
-constexpr int kCtaWarps = 2;   // batch driver: eight CTAs (eight sequences) per SM
-constexpr int kCtaPerSm = 8;
 #ifndef NUSS_GRID_WARPS
 #define NUSS_GRID_WARPS 8   // 8 measured best for config 4 (16: 10.6 ms, 12: 9.7, 8: 8.75, 4: 9.3)
 #endif
@@ -73,44 +69,11 @@ __host__ __device__ __forceinline__ int64_t tile_id(int I, int J, int nt) {
 }
 __host__ __device__ __forceinline__ int64_t tiles_of(int nt) { return (int64_t)nt * (nt + 1) / 2; }
 
-struct Tab {
-  int16_t* base;  // tile records
-  int nt;
-  __device__ __forceinline__ int16_t* UT(int I, int J) const { return base + tile_id(I, J, nt) * kRec; }
-  __device__ __forceinline__ int16_t* L(int I, int J) const { return base + tile_id(I, J, nt) * kRec + kTileWords; }
-  // gamma(i, j) for 0 <= i, j < 32 nt (0 when j - i < 1)
-  __device__ __forceinline__ int gamma(int i, int j) const {
-    if (j - i < 1) return 0;
-    return UT(i / T, j / T)[(j % T) * T + (i % T)];
-  }
-};
-
 __device__ __forceinline__ uint32_t dup16(uint32_t w, int hi) {
   uint32_t r;
   const uint32_t sel = hi ? 0x3232u : 0x1010u;
   asm("prmt.b32 %0, %1, %1, %2;" : "=r"(r) : "r"(w), "r"(sel));
   return r;
-}
-
-// Stage A = UT(I,K) (duplicated halves, [k][r]) and B = L(K,J) ([k][c]) in this warp's buffers.
-// All global loads are issued before any shared-memory store (generic pointers could
-// alias, so interleaving them would serialise twelve L2 round trips).
-__device__ __forceinline__ void stage(const int16_t* __restrict__ ut, const int16_t* __restrict__ l,
-                                      uint32_t* __restrict__ As, uint16_t* __restrict__ Bs, int lane) {
-  uint2 wa[8];
-  uint4 wb[4];
-#pragma unroll
-  for (int t = 0; t < 8; ++t) wa[t] = __ldcg(reinterpret_cast<const uint2*>(ut + (lane + 32 * t) * 4));
-#pragma unroll
-  for (int t = 0; t < 4; ++t) wb[t] = __ldcg(reinterpret_cast<const uint4*>(l + (lane + 32 * t) * 8));
-#pragma unroll
-  for (int t = 0; t < 8; ++t) {
-    const int chunk = lane + 32 * t;  // 4-row chunk: k = chunk / 8, rows 4 (chunk % 8) ..
-    *reinterpret_cast<uint4*>(As + chunk * 4) =
-        make_uint4(dup16(wa[t].x, 0), dup16(wa[t].x, 1), dup16(wa[t].y, 0), dup16(wa[t].y, 1));
-  }
-#pragma unroll
-  for (int t = 0; t < 4; ++t) *reinterpret_cast<uint4*>(Bs + (lane + 32 * t) * 8) = wb[t];
 }
 
 // acc[4 rows][4 pairs] = max(acc, A (x) B) over the 32 k of one staged K tile.
@@ -127,32 +90,6 @@ __device__ __forceinline__ void micro(const uint32_t* As, const uint16_t* Bs, ui
 #pragma unroll
       for (int q = 0; q < 4; ++q) acc[r * 4 + q] = __viaddmax_s16x2(av[r], bv[q], acc[r * 4 + q]);
   }
-}
-
-// Phase A for one (tile, K range) work unit; result max-merged into C (int32 [32][32]).
-template <bool SHARED_C>
-__device__ void product_unit(const Tab& tab, int I, int J, int K0, int K1, int* C, uint32_t* As, uint16_t* Bs,
-                             int lane) {
-  uint32_t acc[16];
-#pragma unroll
-  for (int q = 0; q < 16; ++q) acc[q] = 0;  // gamma >= 0, so 0 is a neutral start
-  for (int K = K0; K < K1; ++K) {
-    __syncwarp();
-    stage(tab.UT(I, K), tab.L(K, J), As, Bs, lane);
-    __syncwarp();
-    micro(As, Bs, acc, lane);
-  }
-  const int ty = lane >> 2, tx = lane & 3;
-#pragma unroll
-  for (int r = 0; r < 4; ++r)
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const uint32_t v = acc[r * 4 + q];
-      int* c = C + (4 * ty + r) * T + 8 * tx + 2 * q;
-      const int lo = (int)(int16_t)(v & 0xffffu), hi = (int)(int16_t)(v >> 16);
-      if (SHARED_C) { atomicMax(c, lo); atomicMax(c + 1, hi); }
-      else { atomicMax(c, lo); atomicMax(c + 1, hi); }
-    }
 }
 
 constexpr int kAS = 72;                  // int16 row stride of the in-tile operand rows (64 entries + 8 pad)
@@ -296,158 +233,6 @@ __device__ __forceinline__ void wavefront(InTileBuf& B, bool diag, int left, int
   }
 }
 
-// Phase B: finalise tile (I,J) from C (max of the middle products), write its UT/L records.
-// One cell per lane (lane = row r) per local anti-diagonal; the neighbours come from the
-// lane's own previous cell (left) and lane r+1's (below, and the pair's inner cell one step
-// later); the in-tile split points are the uniform-length AS x BC reduction above.
-__device__ void in_tile(const Tab& tab, int I, int J, const int* C, bool has_c, InTileBuf& B, const uint8_t* x,
-                        const uint8_t* pm, int n, int h, int lane) {
-  const unsigned full = 0xffffffffu;
-  const bool diag = I == J;
-  const int i0 = I * T, j0 = J * T, r = lane;
-  int16_t* ut = tab.UT(I, J);
-  int16_t* l = tab.L(I, J);
-  // ---- staging (all global loads before the shared stores of each part)
-  {
-    int16_t v[T];
-    if (!diag) {
-      const int16_t* utii = tab.UT(I, I);
-#pragma unroll
-      for (int p = 0; p < T; ++p) v[p] = utii[p * T + r];  // U(I,I)[r][p] = gamma(i0+r, i0+p)
-    }
-    uint4* row = reinterpret_cast<uint4*>(B.as + r * kAS);
-#pragma unroll
-    for (int w = 0; w < kAS / 8; ++w) {
-      uint32_t q[4];
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int p0 = 8 * w + 2 * e;
-        const int lo = (!diag && p0 < T && p0 > r) ? v[p0 < T ? p0 : 0] : kNeg;
-        const int hi = (!diag && p0 + 1 < T && p0 + 1 > r) ? v[p0 + 1 < T ? p0 + 1 : 0] : kNeg;
-        q[e] = pk16(lo, hi);
-      }
-      row[w] = make_uint4(q[0], q[1], q[2], q[3]);
-    }
-  }
-  {
-    const int c = lane;
-    int16_t v[T];
-    if (!diag) {
-      const int16_t* ljj = tab.L(J, J);
-#pragma unroll
-      for (int k = 0; k < T; ++k) v[k] = ljj[k * T + c];  // L(J,J)[k][c] = gamma(j0+k+1, j0+c)
-    }
-    const int below = diag ? 0 : (int)tab.UT(I + 1, J)[c * T + 0];  // X[32][c] = gamma(i0+32, j0+c)
-    uint4* col = reinterpret_cast<uint4*>(B.bc + c * kAS);
-#pragma unroll
-    for (int w = 0; w < kAS / 8; ++w) {
-      uint32_t q[4];
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int p0 = 8 * w + 2 * e;
-        auto val = [&](int p) -> int {
-          if (p == T - 1) return below;
-          if (p >= T && p < 2 * T) return diag ? 0 : (int)v[p - T < T && p >= T ? p - T : 0];
-          return 0;
-        };
-        q[e] = pk16(val(p0), val(p0 + 1));
-      }
-      col[w] = make_uint4(q[0], q[1], q[2], q[3]);
-    }
-    int cv[T];
-#pragma unroll
-    for (int rr = 0; rr < T; ++rr) cv[rr] = has_c ? __ldcg(C + rr * T + c) : 0;
-#pragma unroll
-    for (int rr = 0; rr < T; ++rr) B.cc[rr * kCC + c] = (int16_t)cv[rr];
-  }
-  const int left = diag ? 0 : (int)tab.UT(I, J - 1)[(T - 1) * T + r];  // gamma(i0+r, j0-1)
-  const int corner = (!diag && I + 1 <= J - 1) ? (int)tab.UT(I + 1, J - 1)[(T - 1) * T + 0] : 0;
-  const uint32_t pairbits = pair_bits(x, pm, n, i0, j0, h, lane);
-  __syncwarp();
-  wavefront(B, diag, left, corner, pairbits, lane);
-  // ---- records: UT[c][r] = X[r][c], L[k][c] = X[k+1][c] (k < 31), L[31][c] = X[32][c]
-  {
-    const uint4* xr = reinterpret_cast<const uint4*>(B.as + r * kAS + T);
-    uint4 w[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      w[q] = xr[q];
-      if (diag) {  // entries with c <= r are gamma(i, j <= i) = 0 (held as kNeg)
-        w[q].x = __vmaxs2(w[q].x, 0u); w[q].y = __vmaxs2(w[q].y, 0u);
-        w[q].z = __vmaxs2(w[q].z, 0u); w[q].w = __vmaxs2(w[q].w, 0u);
-      }
-    }
-    const uint32_t ww[16] = {w[0].x, w[0].y, w[0].z, w[0].w, w[1].x, w[1].y, w[1].z, w[1].w,
-                             w[2].x, w[2].y, w[2].z, w[2].w, w[3].x, w[3].y, w[3].z, w[3].w};
-#pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      ut[(2 * q) * T + r] = (int16_t)(ww[q] & 0xffffu);
-      ut[(2 * q + 1) * T + r] = (int16_t)(ww[q] >> 16);
-    }
-    if (r >= 1) {
-      uint4* lr = reinterpret_cast<uint4*>(l + (r - 1) * T);
-#pragma unroll
-      for (int q = 0; q < 4; ++q) lr[q] = w[q];
-    }
-    l[(T - 1) * T + lane] = B.bc[lane * kAS + (T - 1)];
-  }
-}
-
-// Canonical traceback (DESIGN.md R-TB-NUSS: Durbin order, smallest split k) by one
-// warp, right after the fill while the table is L2-resident. A warp follows an
-// interval through its unpaired / pair steps and pushes the right part of every
-// split on a stack in global memory. One step costs one round trip: lanes 0-3 load
-// gamma(i,j), gamma(i+1,j), gamma(i,j-1), gamma(i+1,j-1) while all lanes load the
-// first 32 split candidates.
-template <class TabT>
-__device__ void warp_traceback(const TabT& tab, const uint8_t* x, const uint8_t* pm, int n, int h, uint8_t* db,
-                               int2* stk, int lane) {
-  for (int k = lane; k < n; k += 32) db[k] = '.';
-  if (n <= 1) return;
-  const unsigned full = 0xffffffffu;
-  int sp = 1;
-  if (lane == 0) stk[0] = make_int2(0, n - 1);
-  __syncwarp();
-  int guard = 4 * n + 8;
-  while (sp > 0 && --guard > 0) {
-    const int2 iv = stk[sp - 1];
-    --sp;
-    int i = iv.x, j = iv.y;
-    __syncwarp();
-    while (j - i >= 1 && --guard > 0) {
-      int a = 0;
-      if (lane == 0) a = tab.gamma(i, j);
-      else if (lane == 1) a = tab.gamma(i + 1, j);
-      else if (lane == 2) a = tab.gamma(i, j - 1);
-      else if (lane == 3) a = tab.gamma(i + 1, j - 1);
-      const int k = i + 1 + lane;
-      const int sk = (k < j) ? tab.gamma(i, k) + tab.gamma(k + 1, j) : -1;
-      const int v = __shfl_sync(full, a, 0), g1 = __shfl_sync(full, a, 1);
-      const int g2 = __shfl_sync(full, a, 2), g3 = __shfl_sync(full, a, 3);
-      if (v == g1) { i += 1; continue; }
-      if (v == g2) { j -= 1; continue; }
-      if (pairable(x, pm, n, i, j, h) && v == g3 + 1) {
-        if (lane == 0) { db[i] = '('; db[j] = ')'; }
-        i += 1; j -= 1;
-        continue;
-      }
-      int kk = -1;
-      unsigned m = __ballot_sync(full, sk == v);
-      if (m) kk = i + __ffs(m);
-      for (int k0 = i + 33; kk < 0 && k0 < j; k0 += 32) {
-        const int kq = k0 + lane;
-        m = __ballot_sync(full, kq < j && v == tab.gamma(i, kq) + tab.gamma(kq + 1, j));
-        if (m) kk = k0 + __ffs(m) - 1;
-      }
-      if (kk < 0) break;  // inconsistent table: cannot happen
-      if (lane == 0) stk[sp] = make_int2(kk + 1, j);  // right part later, left part now
-      ++sp;
-      __syncwarp();
-      j = kk;
-    }
-  }
-}
-
 // The same canonical traceback with the table in global memory (far from L2) and fewer
 // round trips: an 8x8 window of gamma (rows i..i+7, columns j-7..j) is fetched in one round
 // trip into shared memory and the unpaired / pair steps run out of it (a step moves i up or
@@ -547,82 +332,6 @@ struct GridQueue {
   int cap;
 };
 __host__ __device__ __forceinline__ int grid_queue_cap(int64_t max_len) { return (int)max_len + 8192; }
-
-// ------------------------------------------------------------------ batch driver
-__global__ void __launch_bounds__(kCtaWarps * 32, kCtaPerSm) k_nuss_tiled_cta(NussArgs A, int64_t slot_elems) {
-  extern __shared__ __align__(16) uint8_t smem[];
-  __shared__ uint8_t pm[16];
-  __shared__ uint8_t xs[4096];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
-  uint8_t* wbuf = smem;                                                      // per-warp scratch
-  const size_t wbytes = sizeof(InTileBuf) > (T * T * 4 + T * T * 2) ? sizeof(InTileBuf) : (T * T * 4 + T * T * 2);
-  uint8_t* mine = wbuf + warp * ((wbytes + 15) & ~size_t(15));
-  uint32_t* As = reinterpret_cast<uint32_t*>(mine);
-  uint16_t* Bs = reinterpret_cast<uint16_t*>(mine + T * T * 4);
-  InTileBuf& IB = *reinterpret_cast<InTileBuf*>(mine);
-  Tab tab;
-  tab.base = reinterpret_cast<int16_t*>(A.scratch) + (int64_t)blockIdx.x * slot_elems;
-  // per-slot C tiles (global, L2 atomics) after the tables, then the traceback stacks
-  int* Cs = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * slot_elems) +
-            (int64_t)blockIdx.x * kCtaWarps * T * T;
-  int* stack = reinterpret_cast<int*>(reinterpret_cast<int16_t*>(A.scratch) + (int64_t)gridDim.x * slot_elems) +
-               (int64_t)gridDim.x * kCtaWarps * T * T + (int64_t)blockIdx.x * (4 * A.max_len + 8);
-  PhaseClock clk;
-  clk.dbg = A.dbg;
-  clk.start();
-  for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
-    const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
-    __syncthreads();
-    for (int q = threadIdx.x; q < n; q += blockDim.x) xs[q] = A.x_cat[A.x_off[p] + q];
-    const int nt = (n + T - 1) / T;
-    tab.nt = nt;
-    __syncthreads();
-    clk.lap(0);
-    for (int D = 0; D < nt; ++D) {
-      const int nT = nt - D;  // tiles on this diagonal (<= nt <= 128 for n <= 4096)
-      // phase A: work units (tile, K chunk); C per tile in shared memory (tiles > 16 processed in groups)
-      for (int g0 = 0; g0 < nT; g0 += kCtaWarps) {
-        const int gT = min(kCtaWarps, nT - g0);
-        if (D >= 2) {
-          for (int q = threadIdx.x; q < gT * T * T; q += blockDim.x) Cs[q] = 0;
-          __syncthreads();
-          clk.lap(1);
-          const int ksteps = D - 1;
-          const int chunks = max(1, min(ksteps, kCtaWarps / gT));
-          const int units = gT * chunks;
-          for (int u = warp; u < units; u += kCtaWarps) {
-            const int t = u / chunks, ch = u % chunks;
-            const int I = g0 + t, J = I + D;
-            const int K0 = I + 1 + (ksteps * ch) / chunks, K1 = I + 1 + (ksteps * (ch + 1)) / chunks;
-            product_unit<false>(tab, I, J, K0, K1, Cs + t * T * T, As, Bs, lane);
-          }
-          clk.lap(2);
-          __syncthreads();
-          clk.lap(3);
-        }
-        // phase B: one warp per tile
-        if (warp < gT) {
-          const int I = g0 + warp, J = I + D;
-          in_tile(tab, I, J, Cs + warp * T * T, D >= 2, IB, xs, pm, n, A.hairpin, lane);
-        }
-        clk.lap(4);
-        __syncthreads();
-        clk.lap(5);
-      }
-    }
-    if (threadIdx.x == 0) {
-      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
-      if (A.db) A.db_len[p] = n;
-    }
-    // warp 0 traces back while the other warps move on to the next problem's staging
-    // barrier (the second CTA on the SM keeps the SM busy meanwhile)
-    if (A.db && warp == 0)
-      warp_traceback(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack), lane);
-    clk.lap(6);
-  }
-  clk.flush(lane);
-}
 
 // ------------------------------------------------------------------ batch driver (one warp per problem)
 // k_nuss_batch: every warp owns one problem at a time (no CTA barriers; 1-warp CTAs, as many
@@ -822,7 +531,12 @@ __global__ void __launch_bounds__(32, 16) k_nuss_batch(NussArgs A, int64_t slot_
   PhaseClock clk;
   clk.dbg = A.dbg;
   clk.start();
-  for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
+  for (;;) {
+    int idx = 0;
+    if (lane == 0) idx = atomicAdd(A.queue, 1);   // the next problem, longest first
+    idx = __shfl_sync(0xffffffffu, idx, 0);
+    if (idx >= A.n) break;
+    const int64_t p = A.perm[idx];
     const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
     __syncwarp();
     for (int q = lane; q < n; q += 32) xs[q] = A.x_cat[A.x_off[p] + q];
@@ -1023,97 +737,6 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   }
 }
 
-// ------------------------------------------------------------------ grid driver (one large problem)
-__global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_tiled_grid(NussArgs A, int64_t p) {
-  cg::grid_group grid = cg::this_grid();
-  extern __shared__ __align__(16) uint8_t smem[];
-  __shared__ uint8_t pm[16];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
-  __syncthreads();
-  const size_t wbytes = sizeof(InTileBuf) > (T * T * 4 + T * T * 2) ? sizeof(InTileBuf) : (T * T * 4 + T * T * 2);
-  uint8_t* mine = smem + warp * ((wbytes + 15) & ~size_t(15));
-  uint32_t* As = reinterpret_cast<uint32_t*>(mine);
-  uint16_t* Bs = reinterpret_cast<uint16_t*>(mine + T * T * 4);
-  InTileBuf& IB = *reinterpret_cast<InTileBuf*>(mine);
-  const uint8_t* x = A.x_cat + A.x_off[p];
-  const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
-  const int nt = (n + T - 1) / T;
-  Tab tab;
-  tab.base = reinterpret_cast<int16_t*>(A.scratch);
-  tab.nt = nt;
-  int* Cg = reinterpret_cast<int*>(tab.base + tiles_of(nt) * kRec);  // 2 x nt x 1024 int32
-  int* stack = Cg + 2 * (int64_t)nt * T * T;
-  const int64_t gw = (int64_t)blockIdx.x * kGridWarps + warp;
-  // C buffers start at zero
-  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T;
-       q += (int64_t)gridDim.x * blockDim.x)
-    Cg[q] = 0;
-  grid.sync();
-  // Round D: phase B of tile-diagonal D (the warp of tile t first adds the two boundary
-  // K-steps K = I+1 and K = J-1, whose operands lie on diagonal D-1) overlapped with the
-  // interior K-steps I+2 <= K <= J-2 of diagonal D+1 (operands on diagonals <= D-1) on
-  // the other warps: one grid-wide barrier per tile-diagonal instead of two.
-  for (int D = 0; D < nt; ++D) {
-    if (A.round_ns && gw == 0 && lane == 0) {
-      unsigned long long t;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-      A.round_ns[D] = t;
-    }
-    const int nT = nt - D;
-    int* C = Cg + (int64_t)(D & 1) * nt * T * T;        // diagonal D (interior products already in)
-    int* Cn = Cg + (int64_t)((D + 1) & 1) * nt * T * T; // diagonal D+1
-    // Phase B runs on the first warp of each SM sub-partition group (warp % 4 == 0, i.e.
-    // SMSP 0), tiles spread over the SMs, so a latency-bound in-tile wavefront never
-    // shares its issue slots with another phase-B warp or with the phase-A warps, which
-    // run on the other three sub-partitions.
-    if ((warp & 3) == 0) {
-      for (int64_t tt = blockIdx.x + (int64_t)gridDim.x * (warp >> 2); tt < nT; tt += (int64_t)gridDim.x * (kGridWarps / 4)) {
-        const int t = (int)tt, I = t, J = t + D;
-        int* Ct = C + (int64_t)t * T * T;
-        if (D >= 2) {
-          product_unit<false>(tab, I, J, I + 1, I + 2, Ct, As, Bs, lane);
-          if (D >= 3) product_unit<false>(tab, I, J, J - 1, J, Ct, As, Bs, lane);
-          __threadfence();
-          __syncwarp();
-        }
-        in_tile(tab, I, J, Ct, D >= 2, IB, x, pm, n, A.hairpin, lane);
-        // this C slot is reused by diagonal D+2: clear it (in_tile has read it)
-        for (int q = lane; q < T * T; q += 32) Ct[q] = 0;
-      }
-    } else if (D + 1 < nt && D >= 3) {
-      // interior K-steps of diagonal D+1: tiles t' (I = t', J = t' + D + 1), K in [I+2, J-2]
-      const int nT1 = nt - (D + 1), ks = D - 2;
-      const int64_t total = (int64_t)nT1 * ks;
-      const int64_t nwA = (int64_t)gridDim.x * (kGridWarps - kGridWarps / 4);
-      const int64_t wA = (int64_t)blockIdx.x * (kGridWarps - kGridWarps / 4) + (warp - (warp >> 2) - 1);
-      const int64_t per = (total + nwA - 1) / nwA;
-      const int64_t b0 = wA * per, b1 = min(total, b0 + per);
-      int64_t it = b0;
-      while (it < b1) {
-        const int t = (int)(it / ks), kk = (int)(it % ks);
-        const int64_t e = min(b1, (int64_t)(t + 1) * ks);
-        const int I = t, J = t + D + 1;
-        product_unit<false>(tab, I, J, I + 2 + kk, I + 2 + kk + (int)(e - it), Cn + (int64_t)t * T * T, As, Bs, lane);
-        it = e;
-      }
-    }
-    grid.sync();
-  }
-  if (gw == 0) {
-    if (lane == 0) {
-      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
-      if (A.db) A.db_len[p] = n;
-    }
-    if (A.db) warp_traceback(tab, x, pm, n, A.hairpin, A.db + p * A.db_stride, reinterpret_cast<int2*>(stack), lane);
-  }
-}
-
-size_t warp_bytes() {
-  const size_t w = sizeof(InTileBuf) > (T * T * 4 + T * T * 2) ? sizeof(InTileBuf) : (T * T * 4 + T * T * 2);
-  return (w + 15) & ~size_t(15);
-}
-
 int num_sms_t(int device) {
   int v = 0;
   cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device);
@@ -1134,7 +757,43 @@ int batch_ctas_per_sm(int64_t max_len) {
   return per_sm > 0 ? per_sm : 1;
 }
 
-bool use_v1() { return getenv("DP_NUSS_V1") != nullptr; }
+// ------------------------------------------------------------------ cost-sorted work queue (A7)
+// the batch warps take problems from an atomic counter in
+// decreasing length (cost ~ n^3), so the last problems handed out are the cheapest and the
+// warps finish together. The order is a device counting sort by length: histogram, a descending
+// exclusive scan (one CTA), a scatter (ties in any order: outputs are written by problem id).
+__global__ void k_len_hist(const int64_t* off, int64_t n, int* hist, int64_t max_len) {
+  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&hist[min(off[p + 1] - off[p], max_len)], 1);
+}
+
+__global__ void k_len_scan(int* hist, int64_t max_len) {  // one CTA: hist[l] <- sum of hist[l' > l]
+  __shared__ int part[1024];
+  const int nb = (int)max_len + 1, t = threadIdx.x;
+  const int per = (nb + 1023) / 1024;
+  // thread t owns lengths (in descending order) d in [t per, (t+1) per), d = max_len - l
+  int sum = 0;
+  for (int d = t * per; d < min(nb, (t + 1) * per); ++d) sum += hist[(int)max_len - d];
+  part[t] = sum;
+  __syncthreads();
+  for (int o = 1; o < 1024; o <<= 1) {
+    const int v = t >= o ? part[t - o] : 0;
+    __syncthreads();
+    part[t] += v;
+    __syncthreads();
+  }
+  int run = t > 0 ? part[t - 1] : 0;
+  for (int d = t * per; d < min(nb, (t + 1) * per); ++d) {
+    const int l = (int)max_len - d, c = hist[l];
+    hist[l] = run;
+    run += c;
+  }
+}
+
+__global__ void k_len_scatter(const int64_t* off, int64_t n, int* hist, int* perm, int64_t max_len) {
+  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x)
+    perm[atomicAdd(&hist[min(off[p + 1] - off[p], max_len)], 1)] = (int)p;
+}
 
 }  // namespace
 
@@ -1142,18 +801,12 @@ bool nuss_tiled_supported(int64_t max_len) { return max_len <= 65536; }
 
 int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
   const int nt = (int)((max_len + T - 1) / T);
-  const int64_t stack_bytes = (4 * max_len + 8) * 4;
-  if (n == 1 && max_len > kGridMin) {
-    if (use_v1()) return tiles_of(nt) * kRec * 2 + 2 * (int64_t)nt * T * T * 4 + stack_bytes + 256;
+  if (n == 1 && max_len > kGridMin)
     return (tiles_of(nt) * kRecW + (int64_t)nt * kDiagW + 2 * (int64_t)nt * T * T) * 4 +
            (4 + 3 * (int64_t)grid_queue_cap(max_len) + 2) * 4 + 256;
-  }
-  if (use_v1()) {
-    const int64_t grid = std::min<int64_t>(n, kCtaPerSm * (int64_t)num_sms_t(device));
-    return grid * (tiles_of(nt) * kRec * 2 + (int64_t)kCtaWarps * T * T * 4 + stack_bytes) + 256;
-  }
   const int64_t grid = std::min<int64_t>(n, (int64_t)batch_ctas_per_sm(max_len) * num_sms_t(device));
-  return grid * batch_slot_words(max_len) * 4 + 256;
+  // + the work queue: counter, length histogram, permutation
+  return grid * batch_slot_words(max_len) * 4 + 256 + 16 + (max_len + 1) * 4 + n * 4 + 256;
 }
 
 cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
@@ -1161,8 +814,7 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
   int dev = 0;
   cudaGetDevice(&dev);
   const int sms = num_sms_t(dev);
-  const int nt = (int)((A.max_len + T - 1) / T);
-  if (A.n == 1 && A.max_len > kGridMin && !use_v1()) {
+  if (A.n == 1 && A.max_len > kGridMin) {
     const size_t smem = kGridWarps * kBatchBuf;
     cudaError_t e = cudaFuncSetAttribute(k_nuss_grid2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -1176,35 +828,25 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
     ++*launches;
     return cudaLaunchCooperativeKernel((void*)k_nuss_grid2, sms, kGridWarps * 32, args, smem, s);
   }
-  if (A.n == 1 && A.max_len > kGridMin) {
-    const size_t smem = kGridWarps * warp_bytes();
-    cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_grid, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    int per_sm = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_nuss_tiled_grid, kGridWarps * 32, smem);
-    if (e != cudaSuccess) return e;
-    if (per_sm < 1) return cudaErrorInvalidConfiguration;
-    NussArgs a2 = A;
-    int64_t p = 0;
-    void* args[2] = {&a2, &p};
-    ++*launches;
-    return cudaLaunchCooperativeKernel((void*)k_nuss_tiled_grid, sms, kGridWarps * 32, args, smem, s);
-  }
   if (A.max_len > 4096) return cudaErrorInvalidValue;  // batch path keeps the sequence in shared memory
-  if (!use_v1()) {
-    int per_sm = batch_ctas_per_sm(A.max_len);
-    if (getenv("DP_NUSS_BATCH_PER_SM")) per_sm = std::max(1, std::min(per_sm, atoi(getenv("DP_NUSS_BATCH_PER_SM"))));  // diagnostic
-    const int64_t grid = std::min<int64_t>(A.n, (int64_t)per_sm * sms);
-    ++*launches;
-    k_nuss_batch<<<(unsigned)grid, 32, batch_warp_bytes(A.max_len), s>>>(A, batch_slot_words(A.max_len));
-    return cudaGetLastError();
-  }
-  const size_t smem = kCtaWarps * warp_bytes();
-  cudaError_t e = cudaFuncSetAttribute(k_nuss_tiled_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const int per_sm = batch_ctas_per_sm(A.max_len);
+  const int64_t grid = std::min<int64_t>(A.n, (int64_t)per_sm * sms);
+  const int64_t slot_words = batch_slot_words(A.max_len);
+  // work queue after the slots: [counter, pad][hist: max_len + 1][perm: n]
+  NussArgs a2 = A;
+  int* q = reinterpret_cast<int*>(reinterpret_cast<uint8_t*>(A.scratch) + ((grid * slot_words * 4 + 255) & ~int64_t(255)));
+  a2.queue = q;
+  int* hist = q + 4;
+  int* perm = hist + ((A.max_len + 1 + 3) & ~int64_t(3));
+  a2.perm = perm;
+  cudaError_t e = cudaMemsetAsync(q, 0, (size_t)(4 + A.max_len + 1) * 4, s);
   if (e != cudaSuccess) return e;
-  const int64_t grid = std::min<int64_t>(A.n, kCtaPerSm * (int64_t)sms);
-  ++*launches;
-  k_nuss_tiled_cta<<<(unsigned)grid, kCtaWarps * 32, smem, s>>>(A, tiles_of(nt) * kRec);
+  const unsigned gs = (unsigned)std::min<int64_t>((A.n + 255) / 256, (int64_t)sms * 8);
+  k_len_hist<<<gs, 256, 0, s>>>(A.x_off, A.n, hist, A.max_len);
+  k_len_scan<<<1, 1024, 0, s>>>(hist, A.max_len);
+  k_len_scatter<<<gs, 256, 0, s>>>(A.x_off, A.n, hist, perm, A.max_len);
+  *launches += 4;
+  k_nuss_batch<<<(unsigned)grid, 32, batch_warp_bytes(A.max_len), s>>>(a2, slot_words);
   return cudaGetLastError();
 }
 
