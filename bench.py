@@ -377,7 +377,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
             final["tl"] = gat("tl", tb_len)
 
     def step(timed):
-        with torch.cuda.stream(stream):
+        with torch.cuda.stream(stream), torch.cuda.nvtx.range(f"step {name}"):
             marks = [ev()] if timed else None
             if side is not None:
                 # HMM: the forward (tensor cores) and Viterbi (ALU) are independent passes over the
@@ -410,7 +410,8 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
                 for q in range(len(phase_names)):
                     ev_phase[q].append(pairs[q])
             if sharded:
-                gather()
+                with torch.cuda.nvtx.range("gather (NCCL all-gather, input order)"):
+                    gather()
 
     for _ in range(warmup):
         step(False)

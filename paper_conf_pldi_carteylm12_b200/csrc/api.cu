@@ -9,6 +9,7 @@
 #include <utility>
 #include <vector>
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "dp.h"
 #include "dp_internal.h"
@@ -32,6 +33,13 @@ struct DevBuf {
     ptr = nullptr;
     bytes = 0;
   }
+};
+
+// NVTX range around an ABI call (header-only NVTX v3: a no-op unless a profiler attaches), so
+// nsight timelines show plan / solve / traceback / host-pipeline phases (SURVEY §5 tracing).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
 };
 
 // Makes the plan's device current for the lifetime of a call and restores the caller's on every
@@ -263,6 +271,7 @@ void dp_plan_destroy(dp_plan_t p) {
 }
 
 dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
+  NvtxRange nvtx("dp_plan_create");
   if (!d || !out) return DP_E_INVALID;
   *out = nullptr;
   if (d->struct_size != sizeof(dp_desc)) return DP_E_INVALID;
@@ -419,6 +428,7 @@ int64_t dp_plan_launch_count(dp_plan_t p) { return p ? p->launches : -1; }
 dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int64_t* a_off, const uint8_t* b_cat,
                          const int64_t* b_off, int64_t max_len_a, int64_t max_len_b, void* scores_out,
                          void* stream) {
+  NvtxRange nvtx("dp_solve_batch");
   if (!p || n < 0) return DP_E_INVALID;
   if (n > 0 && (!a_off || !scores_out)) return DP_E_INVALID;
   const bool align =
@@ -629,6 +639,7 @@ dp_status dp_solve(dp_plan_t p, const uint8_t* a, int64_t len_a, const uint8_t* 
 
 dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, int64_t stride, int32_t* out_len,
                        int32_t* coords, void* stream) {
+  NvtxRange nvtx("dp_traceback");
   if (!p) return DP_E_INVALID;
   if (p->kind == DP_HMM_FORWARD || p->kind == DP_PROFILE_FORWARD) return DP_E_UNSUPPORTED;
   if (!p->want_tb || p->last_n < 0) return DP_E_NO_TRACEBACK;
@@ -709,6 +720,7 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
 dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int64_t* a_off,
                               const uint8_t* b_cat, const int64_t* b_off, void* scores_out, uint8_t* tb_out,
                               int64_t tb_stride, int32_t* tb_len, int32_t* tb_coords, void* stream) {
+  NvtxRange nvtx("dp_solve_batch_host");
   if (!p || n < 0 || (n > 0 && (!a_off || !a_cat || !scores_out))) return DP_E_INVALID;
   const bool align =
       p->kind == DP_EDIT || p->kind == DP_SW_LINEAR || p->kind == DP_SW_AFFINE || p->kind == DP_DIAG_LCS;

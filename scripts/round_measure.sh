@@ -1,25 +1,43 @@
-# Full measurement pass (run under gpurun): tests, bench lines for every config,
-# launch lists and ncu captures of the dominant kernels. Outputs in gpurun_out/.
-set -x
+#!/bin/bash
+# Round-2 measurement pass (run under gpurun; outputs in gpurun_out/, copied to profiles/ by
+# scripts/collect_profiles.sh r02): GPU tests, the default bench line (every config), the
+# reference arm, ncu launch lists and one --set full capture per dominant kernel, the traffic
+# table, compute-sanitizer logs, the micro-benchmarks.
+cd "$GRAFT_REPO_ROOT" || exit 1
+mkdir -p gpurun_out/san
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > gpurun_out/gpu_info.txt
-python -m pytest tests -m gpu -q 2>&1 | tail -3 > gpurun_out/gpu_tests.log
-python bench.py 2>gpurun_out/bench_sw.err | tail -1 > gpurun_out/bench_sw.json
-python bench.py --impl reference --steps 3 --warmup 1 2>/dev/null | tail -1 > gpurun_out/bench_ref.json
-python bench.py --config swa --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_swa.json
-python bench.py --config hmm --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_hmm.json
-python bench.py --config nuss1 --warmup 5 2>/dev/null | tail -1 > gpurun_out/bench_nuss1.json
-python bench.py --config nuss4 --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_nuss4.json
-python bench.py --config nuss5 --steps 2 --warmup 3 2>gpurun_out/bench_nuss5.err | tail -1 > gpurun_out/bench_nuss5.json
-python bench.py --config diag --warmup 3 2>/dev/null | tail -1 > gpurun_out/bench_diag.json
-ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_sw.csv python bench.py --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
-ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_hmm.csv python bench.py --config hmm --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
-ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_nuss4.csv python bench.py --config nuss4 --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
-ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_nuss5.csv env DP_NUSS5_N=50000 python bench.py --config nuss5 --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
-ncu --metrics gpu__time_duration.sum --clock-control none -c 12 --csv --log-file gpurun_out/launches_diag.csv python bench.py --config diag --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_sw16" -c 2 -o gpurun_out/ncu_sw python bench.py --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_forward_tc|k_viterbi" -c 3 -o gpurun_out/ncu_hmm python bench.py --config hmm --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_nuss" -c 1 -o gpurun_out/ncu_nuss4 python bench.py --config nuss4 --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_nuss" -c 1 -o gpurun_out/ncu_nuss5 env DP_NUSS5_N=50000 python bench.py --config nuss5 --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_diag|k_align_affine" -c 2 -o gpurun_out/ncu_diag python bench.py --config diag --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_align_affine" -c 2 -o gpurun_out/ncu_swa python bench.py --config swa --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
+timeout 1500 python -m pytest tests -m gpu -q -rA 2>&1 | grep -vE "^PASSED" | tail -60 > gpurun_out/gpu_tests.log
+timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err
+timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_ref.json 2>/dev/null
+for c in sw hmm nuss1 nuss4 swa diag phmm; do
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv --log-file gpurun_out/launches_$c.csv \
+    python bench.py --config $c --only --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
+done
+DP_NUSS5_N=50000 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv \
+  --log-file gpurun_out/launches_nuss5.csv python bench.py --config nuss5 --only --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
+full() {  # full() TAG REGEX COUNT [env...]
+  local tag=$1 rx=$2 cnt=$3; shift 3
+  env "$@" timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$rx" -c $cnt -o gpurun_out/ncu_$tag \
+    python bench.py --config $tag --only --steps 1 --warmup 0 --no-cpu > /dev/null 2>&1
+}
+full sw "k_sw16" 2
+full hmm "k_forward_tc|k_viterbi" 3
+full nuss1 "k_nuss" 1
+full nuss4 "k_nuss" 1
+full nuss5 "k_nuss_batch" 1 DP_NUSS5_N=50000
+full swa "k_align_affine" 2
+full diag "k_diag" 1
+full phmm "k_phmm" 1
+python scripts/ncu_traffic.py gpurun_out/traffic.json \
+  k_sw16=gpurun_out/ncu_sw.ncu-rep k_sw16_tb5=gpurun_out/ncu_sw.ncu-rep \
+  k_forward_tc=gpurun_out/ncu_hmm.ncu-rep k_viterbi=gpurun_out/ncu_hmm.ncu-rep \
+  k_nuss_batch=gpurun_out/ncu_nuss5.ncu-rep:20:"50k-problem capture of config 5 x 20" \
+  k_nuss_grid2=gpurun_out/ncu_nuss4.ncu-rep k_align_affine=gpurun_out/ncu_swa.ncu-rep \
+  k_diag=gpurun_out/ncu_diag.ncu-rep k_phmm_forward=gpurun_out/ncu_phmm.ncu-rep > gpurun_out/traffic.log 2>&1
+for t in memcheck racecheck synccheck; do
+  for w in align nuss hmm; do
+    timeout 900 compute-sanitizer --tool $t --print-limit 20 python scripts/sanitize_small.py $w > gpurun_out/san/${t}_$w.log 2>&1
+  done
+done
+(cd ubench && timeout 300 ./ubench > ../gpurun_out/ubench.jsonl 2>&1)
 ls -la gpurun_out

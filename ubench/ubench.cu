@@ -33,8 +33,10 @@ __global__ void __launch_bounds__(1024, 1) k_alu(const int* in, int* out, long l
       if (OP == 1) a[q] = (int)__viaddmax_s16x2((unsigned)a[q], (unsigned)b, (unsigned)c);
       if (OP == 2) a[q] = __vimax3_s32(a[q], b, c);
       if (OP == 3) a[q] = (int)__vimax3_s16x2_relu((unsigned)a[q], (unsigned)b, (unsigned)c);
-      if (OP == 4) a[q] = max(a[q], b);
-      if (OP == 5) a[q] = a[q] + b;
+      // plain IMNMX / IADD chains in volatile asm: a C++ max(a, b) or a + b chain is folded by
+      // the compiler (round 1's rows of 7.9 / 10.9 warp-instructions per clock were such folds)
+      if (OP == 4) asm volatile("max.s32 %0, %0, %1;" : "+r"(a[q]) : "r"(b + q));
+      if (OP == 5) asm volatile("add.s32 %0, %0, %1;" : "+r"(a[q]) : "r"(b));
       if (OP == 6) a[q] = __viaddmax_s32_relu(a[q], b, c);
       if (OP == 7) a[q] = (int)__viaddmax_s16x2_relu((unsigned)a[q], (unsigned)b, (unsigned)c);
     }
