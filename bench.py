@@ -824,10 +824,18 @@ def main():
             print(json.dumps(res), flush=True)
         return
     import torch
+    # DP_BENCH_BACKEND=gloo (tests only): several ranks on fewer GPUs, to exercise the N > 1 shard /
+    # gather path where only one GPU is available; the product path is NCCL, one rank per GPU
+    backend = os.environ.get("DP_BENCH_BACKEND", "nccl")
+    if backend != "nccl":
+        local_rank = local_rank % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local_rank)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            dist.init_process_group(backend)
     head = run_config(args.config, args, rank, world, local_rank, args.steps, args.warmup, True)
     res = {"metric": METRIC, "value": head.pop("value"), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": head.pop("ms_per_step"), "higher_is_better": True,
