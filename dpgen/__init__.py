@@ -6,7 +6,7 @@ fixed scoring tables the workloads name, so both sides of every parity check
 see byte-identical problem definitions (task ③: "only the seeded input
 generators serve both, from a module of their own").
 
-Workload recipe (SURVEY.md §8(d) D1–D5):
+Workload recipe (SURVEY.md §8(d) D1–D5; DESIGN.md §2 "Inputs"):
   * master seed 20120611 + config index, numpy PCG64;
   * RNA  : bases i.i.d. uniform over ACGU (codes 0..3);
   * protein: residues i.i.d. uniform over the 20 standard amino acids (codes 0..19

@@ -11,7 +11,7 @@
 //   * thread 0 issues 8 tcgen05.mma.kind::f16 (M=128, K=16) into the fp32 TMEM
 //     accumulator: alpha_hi x [A_hi | A_lo] (N=128) and alpha_lo x A_hi (N=64),
 //     where x = x_hi + x_lo is a two-term bf16 split (the dropped lo x lo term is
-//     ~2^-16 of a 2^-8 term: ~1e-7 relative per step);
+//     ~2^-16 of a 2^-8 term: ~1e-7 relative per step, DESIGN.md §2 "HMM precision");
 //     columns 64..127 hold alpha_hi A_lo and are added in the epilogue;
 //   * tcgen05.commit arrives on an mbarrier; every thread reads its 16 (+16)
 //     columns with tcgen05.ld, multiplies by e_s(x_i), scales by 1/R_{i-1} (the
