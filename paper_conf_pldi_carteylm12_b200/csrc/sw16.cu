@@ -108,8 +108,11 @@ __device__ __forceinline__ void sw_step(FwdState& S, uint32_t rec, int j, int lb
   const uint32_t fa = __shfl_up_sync(0xffffffffu, S.G[kRows - 1], 1);
   uint32_t Gu;
   if (MULTI) {
-    const uint32_t bw = lds_u32_v(rec + 4);
-    Gu = lane0 ? ((from_bnd && live) ? bw : NEG_G2) : fa;
+    // only lane 0 reads the boundary word (any other lane's read would race with lane 31 rewriting
+    // that column's word a few steps later)
+    uint32_t bw = NEG_G2;
+    if (lane0 && from_bnd && live) bw = lds_u32_v(rec + 4);
+    Gu = lane0 ? bw : fa;
   } else {
     Gu = lane0 ? NEG_G2 : fa;
   }
@@ -264,9 +267,13 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
       // steady range: lane 31 at j >= 1 and lane 0 at j <= lbm - 1
       const int s0 = min(max(kb, 31), ke), s1 = max(s0, min(ke, lbm - 1));
       int k = kb;
-      for (; k < s0; ++k)
+      for (; k < s0; ++k) {
         sw_step<TB, true, MULTI>(S, rec0 + kRec * k, k - lane + 1, lbm, lane0, odd, spill31, from_bnd, NEG_G2,
                                  laneA, laneB, rowck + (k - lane));
+        // lane 0 reads column j's boundary word at step j - 1, lane 31 rewrites it at step j + 30: a
+        // __syncwarp at least every 31 steps orders the two (MULTI: more than one strip of rows)
+        if (MULTI) __syncwarp();
+      }
       for (; k + U <= s1; k += U) {
         const uint32_t rec = rec0 + kRec * k;
         uint32_t* rk = rowck + (k - lane);
@@ -276,9 +283,11 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
                                     laneA, laneB, rk + u);
         if (MULTI) __syncwarp();
       }
-      for (; k < s1; ++k)
+      for (; k < s1; ++k) {
         sw_step<TB, false, MULTI>(S, rec0 + kRec * k, k - lane + 1, lbm, lane0, odd, spill31, from_bnd, NEG_G2,
                                   laneA, laneB, rowck + (k - lane));
+        if (MULTI) __syncwarp();
+      }
       for (; k < ke; ++k) {
         sw_step<TB, true, MULTI>(S, rec0 + kRec * k, k - lane + 1, lbm, lane0, odd, spill31, from_bnd, NEG_G2,
                                  laneA, laneB, rowck + (k - lane));
@@ -432,7 +441,9 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
     // A) idle halves take their next problem; a problem with score 0 finishes at once
 #pragma unroll
     for (int hf = 0; hf < 2; ++hf) {
-      if (St[hf].mode != kIdle) continue;
+      const bool idle = St[hf].mode == kIdle;
+      __syncwarp(gmask);  // every lane of the group has read the mode before lane 0 rewrites the state
+      if (!idle) continue;
       int64_t q = 0;
       if (m == 0) q = atomicAdd(reinterpret_cast<unsigned long long*>(A.tb_ctr) + hf, 1ull);
       q = __shfl_sync(gmask, q, lane & ~(kGL - 1));
@@ -699,6 +710,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         }
       }
     }
+    __syncwarp();  // phase G's state updates (lane 0 of a group) before the walkers (lanes 0, 1) read them
     clk.lap(4);
     // H) walking halves: lane m == half walks its problem through the block's codes
     if (m < 2) {
