@@ -12,7 +12,7 @@ config (1, 3, 4, 5) and the §8(f) NEXT workloads, each with its own value,
 step time, roofline, e2e and cpu_baseline.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                  [--config sw|swa|nuss1|hmm|nuss4|nuss5|diag|phmm] [--only]
+                  [--config sw|swa|swshort|nuss1|hmm|nuss4|nuss5|diag|phmm] [--only]
                   [--scaling strong|weak]
 
 Multi-GPU (the paper's `map`, L194–L195, one problem per
@@ -49,9 +49,9 @@ MEASURED_UBENCH = {  # profiles/ubench_r01.jsonl, lane-ops per SM clock on B200 
     "viaddmnmx_s32": 64.0, "viaddmnmx_s16x2": 128.0, "ffma": 128.0, "lds_bytes": 128.0,
 }
 SMS = 148
-ALL_CONFIGS = ["sw", "nuss1", "hmm", "nuss4", "nuss5", "swa", "diag", "phmm"]
+ALL_CONFIGS = ["sw", "nuss1", "hmm", "nuss4", "nuss5", "swa", "swshort", "diag", "phmm"]
 # configs in the `configs` block at N > 1: the batched ones (the others are single tables: replicas only)
-SHARDED = {"sw", "hmm", "nuss5", "swa", "diag", "phmm"}
+SHARDED = {"sw", "hmm", "nuss5", "swa", "swshort", "diag", "phmm"}
 
 
 def peaks():
@@ -254,6 +254,21 @@ def workload(name, rank=0, world=1, scaling="strong"):
                 "cells_local": int((lens * (lens - 1) // 2).sum()),
                 "inner_local": int((lens * (lens - 1) * (lens - 2) // 6).sum()), "tb_stride": 512,
                 "workload": "BASELINE config 5: 1M RNAs of length U[128,512], Nussinov batch, with tracebacks"}
+    if name == "swshort":
+        n = 1_000_000
+        a_cat, a_off, b_cat, b_off = dpgen.short_protein_pairs(n)
+        ids = shard_ids(name, n, None, rank, world, scaling)
+        la, lb = np.diff(a_off), np.diff(b_off)
+        if world > 1:
+            a_cat, a_off2 = subset(a_cat, a_off, ids)
+            b_cat, b_off2 = subset(b_cat, b_off, ids)
+            a_off, b_off = a_off2, b_off2
+        cells_local = int((np.diff(a_off) * np.diff(b_off)).sum())
+        return {"kind": "swshort", "n_total": n, "ids": ids, "a_cat": a_cat, "a_off": a_off, "b_cat": b_cat,
+                "b_off": b_off, "max_la": 64, "max_lb": 64, "cells_total": int((la * lb).sum()),
+                "cells_local": cells_local, "ops_local": 3 * cells_local, "tb_stride": 129,
+                "workload": "SURVEY 8(f) NEXT 1 (hybrid, short side): 1M protein pairs, |a| and |b| uniform in "
+                            "[8, 64], Smith-Waterman, BLOSUM62, linear gap 4, with tracebacks (inter-task kernel)"}
     if name == "diag":
         n = 20_000
         a_cat, a_off, b_cat, b_off = dpgen.diag_pairs(n)
@@ -301,7 +316,7 @@ def workload(name, rank=0, world=1, scaling="strong"):
 
 # ----------------------------------------------------------------------------- our arm
 def make_plans(dp, W):
-    if W["kind"] == "sw":
+    if W["kind"] in ("sw", "swshort"):
         return [dp.Plan(dp.SW_LINEAR, W["max_la"], W["max_lb"], sigma=dpgen.blosum62(), gap=dpgen.SW_GAP,
                         want_traceback=True)]
     if W["kind"] == "swa":
@@ -322,6 +337,7 @@ def make_plans(dp, W):
 
 PHASES = {
     "sw": ["k_sw16 (partition sweep)", "k_sw16_tb5 (traceback)"],
+    "swshort": ["k_sw_inter (length sort + inter-task sweep)", "k_sw_inter_tb (traceback)"],
     "swa": ["k_align_affine (partition sweep)", "k_align_affine_tb (traceback)"],
     "nuss": ["k_nuss (fill + in-kernel traceback)", "dp_traceback (copy)"],
     "diag": ["k_diag (conditional schedule)"],
@@ -353,7 +369,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
     stride = W["tb_stride"] or 0
     tb_out = torch.empty((n, stride), dtype=torch.uint8, device=dev)
     tb_len = torch.empty(n, dtype=torch.int32, device=dev)
-    tb_co = torch.empty((n, 4), dtype=torch.int32, device=dev) if W["kind"] in ("sw", "swa") else None
+    tb_co = torch.empty((n, 4), dtype=torch.int32, device=dev) if W["kind"] in ("sw", "swa", "swshort") else None
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     sharded = world > 1 and name in SHARDED and args.scaling == "strong"
     gat = Gatherer(W["ids"], W["n_total"], dev) if sharded else None
@@ -482,6 +498,25 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
         alone["k_viterbi_tb"] = a0.elapsed_time(a1)
 
     fixed = None
+    intra = None
+    if W["kind"] == "swshort":   # the hybrid's evidence: the same batch on the intra-task warp kernel
+        os.environ["DP_SW_INTRA"] = "1"
+        try:
+            with make_plans(dp, W)[0] as pi:
+                def both():
+                    pi.solve_batch(*dev_in, max_len_a=W["max_la"], max_len_b=W["max_lb"], out=scores[0], stream=stream)
+                    pi.traceback_into(0, n, tb_out, stride, tb_len, tb_co, stream=stream)
+                with torch.cuda.stream(stream):
+                    both()
+                    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    f0.record(stream)
+                    for _ in range(3):
+                        both()
+                    f1.record(stream)
+                torch.cuda.synchronize(dev)
+                intra = round(f0.elapsed_time(f1) / 3, 4)
+        finally:
+            del os.environ["DP_SW_INTRA"]
     if W["kind"] == "diag":   # §4.7 evidence: the same batch with each candidate forced for every problem
         fixed = {}
         for a in dp.schedule_conditional(2, [((-1, -1), None, 0, 0)]):
@@ -508,7 +543,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
         "scaling": ("strong" if sharded else ("replicas" if world > 1 and name in ("nuss1", "nuss4") else
                                               ("weak" if world > 1 else "strong"))),
         "dtype": {"sw": "s16x2 (int16 lanes; score range plan-checked, else int32)",
-                  "swa": "int32", "nuss": "int16 table, s16x2 max-plus (score <= n/2)",
+                  "swa": "int32", "swshort": "int32", "nuss": "int16 table, s16x2 max-plus (score <= n/2)",
                   "diag": "uint16 table / int32", "hmm": "f32 (forward; bf16x3 tensor-core split) + int32 (Viterbi)",
                   "phmm": "f32 (scaled linear space, per-lane power-of-two exponents)"}[W["kind"]],
         "config": {"workload": W["workload"], "config": name, "problems": W["n_total"], "problems_per_gpu": n,
@@ -522,6 +557,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
         "gpu_launches": int(launches),
         "result_sha256": digest,
         **({"alone_ms": {k: round(v, 4) for k, v in alone.items()}} if alone else {}),
+        **({"intra_task_ms": intra, "inter_task_ms": round(ms_step, 4)} if intra else {}),
         **({"fixed_schedule_ms": fixed, "conditional_schedule_ms": round(ms_step, 4)} if fixed else {}),
         "e2e": e2e,
         "clocks": clk.summary(),
@@ -559,6 +595,12 @@ def roofline(W, name, phase_ms, alone, pk):
                 "ubench_r01 VIADDMNMX.S16x2 128 lane-ops/clk/SM x 148 SMs x sm_max_mhz (3 max-plus ops per cell)",
                 units=W["cells_local"] / 6.5536e9)
         r["frac_vs_int32_peak"] = round(ops / (phase_ms[0] * 1e-3) / peak32, 4)
+        r["traceback_ms"] = round(phase_ms[1], 4)
+        return r
+    if W["kind"] == "swshort":
+        r = alu("k_sw_inter", W["ops_local"], phase_ms[0], peak32,
+                "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (3 max-plus ops per cell; "
+                "kernel time includes the 3 small length-sort launches)")
         r["traceback_ms"] = round(phase_ms[1], 4)
         return r
     if W["kind"] == "swa":
@@ -623,7 +665,7 @@ def e2e_host(W, plans, dev, stream, world, steps):
         sc = pin(np.empty(n, np.float32 if (fwd_like and k == 0) else np.int32))
         tb = pin(np.empty((n, stride), np.uint8)) if p.want_traceback else None
         tl = pin(np.empty(n, np.int32)) if p.want_traceback else None
-        tc = pin(np.empty((n, 4), np.int32)) if (p.want_traceback and W["kind"] in ("sw", "swa")) else None
+        tc = pin(np.empty((n, 4), np.int32)) if (p.want_traceback and W["kind"] in ("sw", "swa", "swshort")) else None
         outs.append((sc, tb, tl, tc))
     h2d = (a_cat.nbytes + a_off.nbytes + (b_cat.nbytes + b_off.nbytes if b_cat is not None else 0)) * len(plans)
     d2h = sum(o[0].nbytes + (o[1].nbytes + o[2].nbytes if o[1] is not None else 0) +
@@ -699,6 +741,16 @@ def oracle_sample(config, W):
         oracle.sw_traceback_batch(a_cat, a_off, b_cat, b_off, sig, dpgen.SW_GAP, 513, threads=cores)
         dt = time.perf_counter() - t
         return k * 65536 / dt, f"first {k} pairs of config 2 (scores + canonical tracebacks)", cores
+    if config == "swshort":
+        k = 60000
+        a_cat, a_off, b_cat, b_off = dpgen.short_protein_pairs(k)
+        sig = dpgen.blosum62()
+        t = time.perf_counter()
+        oracle.sw_batch(a_cat, a_off, b_cat, b_off, sig, dpgen.SW_GAP, threads=cores)
+        oracle.sw_traceback_batch(a_cat, a_off, b_cat, b_off, sig, dpgen.SW_GAP, 129, threads=cores)
+        dt = time.perf_counter() - t
+        return int((np.diff(a_off) * np.diff(b_off)).sum()) / dt, \
+            f"first {k} pairs of the short-pair workload (scores + canonical tracebacks)", cores
     if config == "swa":
         k = 1500
         a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(k)
@@ -791,7 +843,7 @@ def run_reference(args, rank, world):
     }
 
 
-DEFAULT_STEPS = {"sw": 60, "swa": 20, "hmm": 30, "nuss1": 200, "nuss4": 15, "nuss5": 2, "diag": 25, "phmm": 20}
+DEFAULT_STEPS = {"sw": 60, "swa": 20, "swshort": 30, "hmm": 30, "nuss1": 200, "nuss4": 15, "nuss5": 2, "diag": 25, "phmm": 20}
 
 
 def main():

@@ -156,6 +156,24 @@ def diag_pairs(n_pairs: int = 20_000, lo: int = 32, hi: int = 4096, first: int =
     return a.copy(), ao, b.copy(), bo
 
 
+def short_protein_pairs(n_pairs: int = 1_000_000, lo: int = 8, hi: int = 64, first: int = 0):
+    """Short-pair batch for the inter-task kernel (SURVEY §8(f) NEXT 1, the hybrid's short side;
+    PAPER.md §6.1): protein pairs whose lengths |a|, |b| are i.i.d. uniform integers in
+    [lo, hi], residues i.i.d. uniform over the 20 standard amino acids; seed 20120611+11.
+    Returns (a_cat, a_off, b_cat, b_off); `first` skips that many pairs of the stream."""
+    g = rng(11)
+    total = first + n_pairs
+    la = g.integers(lo, hi + 1, total, dtype=np.int64)
+    lb = g.integers(lo, hi + 1, total, dtype=np.int64)
+    a = g.integers(0, 20, int(la.sum()), dtype=np.uint8)
+    b = g.integers(0, 20, int(lb.sum()), dtype=np.uint8)
+    ao = np.concatenate([[0], np.cumsum(la)]).astype(np.int64)
+    bo = np.concatenate([[0], np.cumsum(lb)]).astype(np.int64)
+    a, b = a[ao[first]:], b[bo[first]:]
+    ao, bo = ao[first:] - ao[first], bo[first:] - bo[first]
+    return a.copy(), ao, b.copy(), bo
+
+
 def hmm_params(g: np.random.Generator, S: int = HMM_STATES, K: int = 4):
     """Rows of pi (1xS), A (SxS), E (SxK) ~ Dirichlet(1), float64."""
     pi = g.dirichlet(np.ones(S))

@@ -76,6 +76,7 @@ struct dp_plan {
   int8_t* d_sigma = nullptr;
   std::vector<int8_t> h_sigma;
   bool packed16 = false;  // SW on the s16x2 two-problems-per-warp kernels
+  bool inter = false;     // SW on the inter-task kernel (one pair per thread; short pairs)
   uint8_t* d_pair = nullptr;
   float *d_pi = nullptr, *d_A = nullptr, *d_E = nullptr;
   int32_t *d_lpi = nullptr, *d_lA = nullptr, *d_lE = nullptr;
@@ -107,7 +108,7 @@ struct dp_plan {
   // diagnostics (environment, read once at dp_plan_create; tests and experiments only)
   struct {
     bool force_int32 = false, nuss_cell = false, hmm_timing = false, nuss_timing = false, sw_timing = false;
-    bool nuss_rounds = false, diag_generic = false;
+    bool nuss_rounds = false, diag_generic = false, sw_intra = false;
     int64_t nuss_tiled_min = 32;
     int nuss_tbw = 0, diag_force = -1, host_chunks = 4;
   } env;
@@ -124,6 +125,7 @@ void read_env(dp_plan* p) {
   p->env.sw_timing = on("DP_SW_TIMING");
   p->env.nuss_rounds = on("DP_NUSS_ROUNDS");
   p->env.diag_generic = on("DP_DIAG_GENERIC");
+  p->env.sw_intra = on("DP_SW_INTRA");
   if (on("DP_NUSS_TILED_MIN")) p->env.nuss_tiled_min = atoll(getenv("DP_NUSS_TILED_MIN"));
   if (on("DP_NUSS_TBW")) p->env.nuss_tbw = atoi(getenv("DP_NUSS_TBW"));
   if (on("DP_DIAG_FORCE")) p->env.diag_force = atoi(getenv("DP_DIAG_FORCE"));
@@ -306,10 +308,13 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) { st = DP_E_TOO_LARGE; break; }
       e = upload(&p->d_sigma, d->sigma, (size_t)p->asz * p->asz);
       p->h_sigma.assign(d->sigma, d->sigma + (size_t)p->asz * p->asz);
-      p->packed16 = dpk::sw16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap, d->want_traceback != 0) &&
+      // hybrid dispatch (§6.1): short pairs one per thread (inter-task), longer ones on the
+      // warp kernels (intra-task); DP_SW_INTRA=1 keeps short pairs on the warp kernels (comparison)
+      p->inter = dpk::sw_inter_eligible(d->max_len_a, d->max_len_b, p->asz, p->gap) && !p->env.sw_intra;
+      p->packed16 = !p->inter && dpk::sw16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap, d->want_traceback != 0) &&
                     !p->env.force_int32 &&
                     (smem_limit <= 0 || dpk::sw16_smem_bytes(p->asz, d->max_len_a, d->max_len_b) <= (size_t)smem_limit);
-      if (!p->packed16 && smem_limit > 0 &&
+      if (!p->inter && !p->packed16 && smem_limit > 0 &&
           dpk::align_smem_bytes(p->asz, true, d->max_len_a, d->max_len_b) > (size_t)smem_limit)
         st = DP_E_TOO_LARGE;
       break;
@@ -456,6 +461,25 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       break;
     }
     case DP_SW_LINEAR:
+      if (p->inter) {
+        dpk::AlignArgs A{};
+        A.n = n; A.a_cat = a_cat; A.b_cat = b_cat; A.a_off = a_off; A.b_off = b_off;
+        A.max_la = max_len_a; A.max_lb = max_len_b;
+        A.sigma = p->d_sigma; A.asz = p->asz; A.gap = p->gap; A.local = true;
+        A.scores = static_cast<int32_t*>(scores_out);
+        if (p->want_tb) {
+          A.dir_stride = dpk::sw_inter_dir_words(p->max_la);
+          e = p->tb_state.ensure((size_t)(n * A.dir_stride * 4 + 16));
+          if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 2 * 4 + 16));
+          if (e != cudaSuccess) break;
+          A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
+          A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
+          p->last_scores = A.scores;
+        }
+        e = p->scratch.ensure(dpk::sw_inter_work_bytes(n));
+        if (e == cudaSuccess) e = dpk::sw_inter_solve(A, p->scratch.ptr, s, &p->launches);
+        break;
+      }
       if (p->packed16) {
         dpk::Sw16Args A{};
         e = sw16_args(p, n, a_cat, a_off, b_cat, b_off, max_len_a, max_len_b, static_cast<int32_t*>(scores_out), &A);
@@ -650,6 +674,18 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
   cudaError_t e = cudaSuccess;
   switch (p->kind) {
     case DP_SW_LINEAR:
+      if (p->inter) {
+        if (stride < p->last_max_la + p->last_max_lb) return DP_E_TOO_LARGE;
+        dpk::AlignArgs A{};
+        A.n = p->last_n; A.a_cat = p->last_a; A.b_cat = p->last_b; A.a_off = p->last_aoff; A.b_off = p->last_boff;
+        A.scores = p->last_scores;
+        A.sigma = p->d_sigma; A.asz = p->asz; A.gap = p->gap;
+        A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
+        A.dir_stride = dpk::sw_inter_dir_words(p->max_la);
+        A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
+        e = dpk::sw_inter_traceback(A, p->scratch.ptr, first, count, out, stride, out_len, coords, s, &p->launches);
+        break;
+      }
       if (p->packed16) {
         if (stride < p->last_max_la + p->last_max_lb) return DP_E_TOO_LARGE;
         dpk::Sw16Args A{};

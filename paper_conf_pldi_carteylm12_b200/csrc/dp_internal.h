@@ -55,6 +55,15 @@ cudaError_t align_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t align_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                             int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
 
+// ---------------------------------------------------------------- inter-task SW (sw_inter.cu): one pair per thread
+bool sw_inter_eligible(int64_t max_la, int64_t max_lb, int asz, int gap);  // max(|a|, |b|) <= 64, gap >= 1
+int64_t sw_inter_dir_words(int64_t max_la);                                  // code words per problem (16 B per row)
+size_t sw_inter_work_bytes(int64_t n);                                       // sort workspace (histogram + order)
+cudaError_t sw_inter_solve(const AlignArgs& a, void* work, cudaStream_t s, int64_t* launches);
+cudaError_t sw_inter_traceback(const AlignArgs& a, const void* work, int64_t first, int64_t count, uint8_t* out,
+                               int64_t stride,
+                               int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
+
 // ---------------------------------------------------------------- packed SW (two problems per warp)
 struct Sw16Args {
   int64_t n;

@@ -35,6 +35,13 @@ def main(which):
             b4 = [x % 4 for x in b]
             (ac, ao), (bc, bo) = dpgen.pack(a4), dpgen.pack(b4)
             p.solve_batch(cu(ac), cu(ao), cu(bc), cu(bo), max_len_a=la, max_len_b=lb)
+    if which in ("all", "inter"):   # short pairs: the inter-task kernel (one pair per thread)
+        a = [g.integers(0, 20, int(l)).astype(np.uint8) for l in g.integers(0, 65, 300)]
+        b = [g.integers(0, 20, int(l)).astype(np.uint8) for l in g.integers(0, 65, 300)]
+        (ac, ao), (bc, bo) = dpgen.pack(a), dpgen.pack(b)
+        with dp.Plan(dp.SW_LINEAR, 64, 64, sigma=sig, gap=4, want_traceback=True) as p:
+            p.solve_batch(cu(ac), cu(ao), cu(bc), cu(bo), max_len_a=64, max_len_b=64)
+            p.traceback(0, len(a), 129)
     if which in ("all", "nuss"):
         seqs = [g.integers(0, 4, int(l)).astype(np.uint8) for l in (1, 20, 33, 64, 100, 130, 200)]
         c, o = dpgen.pack(seqs)

@@ -128,6 +128,77 @@ def test_sw_s16_guard_crosses_to_int32(dp, orc):
     assert r2["scores"][0] == 127 * 300 == orc.sw(a2[0], a2[0], sig2, 5)[0] > 32767
 
 
+def _sw_check_all(orc, r, a, b, sig, gap):
+    for q in range(len(a)):
+        sc, _, _ = orc.sw(a[q], b[q], sig, gap)
+        ops, co = orc.sw_traceback(a[q], b[q], sig, gap)
+        assert r["scores"][q] == sc and r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+
+
+def test_sw_inter_short_pairs(dp, orc):
+    """SURVEY §8(f) NEXT 1 (inter-task, one pair per thread): a batch whose
+    pairs all have max(|a|, |b|) <= 64 runs k_sw_inter. Lengths 0..64 cover every column bucket,
+    empty sides, the 64-column maximum and ragged warps (3001 pairs: a partial last warp)."""
+    g = np.random.default_rng(120)
+    sig = dpgen.blosum62()
+    n = 3001
+    a, _ = rand_batch(g, n, 0, 64, 20)
+    b, _ = rand_batch(g, n, 0, 64, 20)
+    a[0], b[0] = a[0][:0], b[0][:5]          # empty a
+    a[1], b[1] = a[1][:64], b[1][:0]         # empty b
+    r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24)
+    _sw_check_all(orc, r, a, b, sig, 4)
+
+
+def test_sw_inter_ties_and_gap_one(dp, orc):
+    """Low-entropy alphabet (frequent ties: end-cell and direction tie-breaks), gap 1 (the
+    smallest gap the inter-task kernel's sentinel-column argument allows), self-alignments."""
+    g = np.random.default_rng(121)
+    sig = dpgen.blosum62()
+    a, _ = rand_batch(g, 500, 1, 64, 3)
+    b, _ = rand_batch(g, 500, 1, 64, 3)
+    b[:40] = [x.copy() for x in a[:40]]
+    for gap in (1, 4):
+        r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=gap, asz=24)
+        _sw_check_all(orc, r, a, b, sig, gap)
+
+
+def test_sw_inter_matches_intra(dp, orc, monkeypatch):
+    """The hybrid's two kernels agree on the same short batch: the inter-task path (default) and
+    the intra-task warp kernel (DP_SW_INTRA=1) give identical scores, ops and coordinates, and
+    launch different kernels (launch counts differ)."""
+    g = np.random.default_rng(122)
+    sig = dpgen.blosum62()
+    a, _ = rand_batch(g, 700, 1, 64, 20)
+    b, _ = rand_batch(g, 700, 1, 64, 20)
+    r1 = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24)
+    monkeypatch.setenv("DP_SW_INTRA", "1")
+    r2 = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24)
+    assert (r1["scores"] == r2["scores"]).all()
+    assert r1["ops"] == r2["ops"] and (r1["coords"] == r2["coords"]).all()
+    for q in range(0, 700, 7):
+        assert r1["scores"][q] == orc.sw(a[q], b[q], sig, 4)[0]
+
+
+def test_sw_inter_score_only_and_host_path(dp, orc):
+    """Score-only plan (no code retention) and the host entry point (chunked H2D / solve /
+    traceback / D2H) on a short batch larger than one host chunk."""
+    g = np.random.default_rng(123)
+    sig = dpgen.blosum62()
+    n = 40000
+    a, (a_cat, a_off) = rand_batch(g, n, 0, 64, 20)
+    b, (b_cat, b_off) = rand_batch(g, n, 0, 64, 20)
+    r = run_align(dp, dp.SW_LINEAR, a, b, sigma=sig, gap=4, asz=24, tb=False)
+    want = orc.sw_batch(a_cat, a_off, b_cat, b_off, sig, 4, threads=THREADS)
+    assert (r["scores"] == want).all()
+    with dp.Plan(dp.SW_LINEAR, 64, 64, sigma=sig, gap=4, want_traceback=True) as p:
+        sc, tb, tl, co = p.solve_batch_host(a_cat, a_off, b_cat, b_off, tb_stride=129)
+    assert (sc == want).all()
+    for q in range(0, n, 97):
+        ops, c = orc.sw_traceback(a[q], b[q], sig, 4)
+        assert bytes(tb[q, :tl[q]]).decode() == ops and tuple(co[q]) == c, q
+
+
 def test_sw_packed_odd_batch_and_ties(dp, orc):
     """Odd batch (last warp half empty), mismatched pair lengths in one warp, and
     a low-entropy alphabet that makes ties frequent (end cell / traceback tie-breaks)."""
