@@ -612,7 +612,7 @@ def roofline(W, name, phase_ms, alone, pk):
     if W["kind"] == "nuss":
         if name == "nuss1":  # one problem, one SM: latency-bound; the fraction is of ONE SM's peak (§8(d) D1)
             one_sm = MEASURED_UBENCH["viaddmnmx_s16x2"] * clock_hz
-            r = alu("k_nuss_cta", W["inner_local"], phase_ms[0], one_sm,
+            r = alu("k_nuss_small", W["inner_local"], phase_ms[0], one_sm,
                     "ubench_r01 VIADDMNMX.S16x2 128 lane-ops/clk x ONE SM x sm_max_mhz (one split evaluation = one "
                     "max-plus); latency-bound: 64 dependent partitions")
             r["bound"] = "latency"

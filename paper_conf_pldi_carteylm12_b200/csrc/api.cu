@@ -540,6 +540,13 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       // cell-level CTA kernel (table in shared memory) for short sequences, tiled
       // max-plus kernels above (SURVEY §8(a) A6b'); DP_NUSS_CELL=1 forces the cell level
       // (config 1, n = 64: tiled 0.097 ms per step vs 0.109 cell-level)
+      // latency regime (config 1: a few problems of <= 128 nt): one CTA per problem, table and
+      // traceback in shared memory, one barrier per partition (DP_NUSS_CELL / DP_NUSS_TILED_MIN: the
+      // other paths, for comparison)
+      if (dpk::nuss_small_supported(A.max_len, n, p->device) && !p->env.nuss_cell && p->env.nuss_tiled_min == 32) {
+        e = dpk::nuss_small_solve(A, s, &p->launches);
+        break;
+      }
       const bool tiled = A.max_len > p->env.nuss_tiled_min && !p->env.nuss_cell && (n == 1 || A.max_len <= 4096);
       A.scratch_bytes = tiled ? dpk::nuss_tiled_scratch_bytes(A.max_len, n, p->device)
                               : dpk::nuss_scratch_bytes(A.max_len, n, p->device);

@@ -133,6 +133,9 @@ bool nuss_tiled_supported(int64_t max_len);
 int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device);
 cudaError_t nuss_tiled_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t nuss_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
+// one CTA per problem, table + traceback in shared memory (latency regime: max_len <= 128, few problems)
+bool nuss_small_supported(int64_t max_len, int64_t n, int device);
+cudaError_t nuss_small_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
 // copy rows [first, first+count) of the dot-bracket scratch (row stride ds) and their lengths
 cudaError_t nuss_copy_db(const uint8_t* db, int64_t ds, const int32_t* lens, int64_t first, int64_t count,
                          uint8_t* out, int64_t stride, int32_t* out_len, cudaStream_t s, int64_t* launches);

@@ -182,6 +182,143 @@ __global__ void __launch_bounds__(kNussThreads) k_nuss_cta(NussArgs A, int64_t s
   }
 }
 
+// ------------------------------------------------------------------ short problems, latency-bound
+// k_nuss_small (one 64-nt RNA is 63 dependent partitions, a latency problem):
+// one small CTA per problem, the whole table in shared memory, one barrier per partition (Fig.8's
+// `sync`, L251–L253), thread r owning the cells of rows r, r + 64; the traceback from the same
+// shared table. Measured (config 1, clock64): ~600 cycles per partition, set by each cell's
+// serial chain of dependent shared-memory round trips (the loop and barrier alone: 28 cycles),
+// 13k cycles of traceback. Both copies are full squares
+// of row stride W (W / 8 odd: rows 8 lanes apart fall on distinct bank quads):
+//   U[i][k] = gamma(i, k) (k >= i), L[j][k] = gamma(k+1, j) (k < j), L[j][j] = 0,
+// every other entry (and every entry not yet computed) kNeg. Then for a cell of partition d
+//   max_{i <= k <= j} U[i][k] + L[j][k] = max(gamma(i+1, j), gamma(i, j-1), split terms)
+// (k = i: the "i unpaired" term; k = j-1: "j unpaired"; k = j and k < i: kNeg), so a cell is one
+// s16x2 max-plus reduction over the aligned 8-wide chunks covering [i, j] plus the pair term.
+// Entries read but written in the same partition (U[i][j], L[j][i-1]) are this cell's own and
+// pair with kNeg; they are written after the cell's reduction.
+constexpr int kSmallMaxN = 128;
+constexpr int kSmallThreads = 64;  // n <= 64: one cell per thread per partition (32 / 64 / 128 threads:
+                                   // 45.1k / 41.5k / 41.5k cycles of fill for config 1)
+constexpr int16_t kSNeg = -16000;
+
+__host__ __device__ __forceinline__ int small_w(int64_t max_len) { return 8 * ((int)((max_len + 7) / 8) | 1); }
+size_t small_smem_bytes(int64_t max_len) {
+  const int w = small_w(max_len);
+  return (size_t)2 * max_len * w * 2 + 128 + 16 + 128 + (size_t)(4 * max_len + 8) * 4;
+}
+
+__global__ void __launch_bounds__(kSmallThreads) k_nuss_small(NussArgs A) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int W = small_w(A.max_len);
+  int16_t* U = reinterpret_cast<int16_t*>(smem);
+  int16_t* L = U + A.max_len * W;
+  uint8_t* xs = reinterpret_cast<uint8_t*>(L + A.max_len * W);
+  uint8_t* pm = xs + 128;
+  uint8_t* prow = pm + 16;
+  int* stack = reinterpret_cast<int*>(prow + 128);
+  const int tid = threadIdx.x, lane = tid & 31;
+  if (tid < 16) pm[tid] = A.pair_mask[tid];
+  const uint32_t NEG2 = (uint32_t)(uint16_t)kSNeg * 0x10001u;
+  for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
+    const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+    __syncthreads();
+    for (int q = tid; q < n; q += blockDim.x) xs[q] = A.x_cat[A.x_off[p] + q];
+    for (int r = tid >> 5; r < n; r += kSmallThreads / 32) {  // a warp per row, two entries per word
+      uint32_t* ur = reinterpret_cast<uint32_t*>(U + r * W);
+      uint32_t* lr = reinterpret_cast<uint32_t*>(L + r * W);
+      for (int c = 2 * lane; c < W; c += 64) {
+        ur[c >> 1] = (c == r ? 0u : (NEG2 & 0xffffu)) | (c + 1 == r ? 0u : (NEG2 & 0xffff0000u));  // gamma(i,i) = 0
+        const bool z0 = c == r || c + 1 == r, z1 = c + 1 == r || c + 2 == r;  // L[j][j-1] = L[j][j] = 0
+        lr[c >> 1] = (z0 ? 0u : (NEG2 & 0xffffu)) | (z1 ? 0u : (NEG2 & 0xffff0000u));
+      }
+    }
+    __syncthreads();
+    for (int i = tid; i < n; i += kSmallThreads) {  // prow[i] bit y: x_i may pair with base y; then x_i itself
+      const int xi = xs[i];
+      prow[i] = (uint8_t)(pm[xi * 4] | pm[xi * 4 + 1] << 1 | pm[xi * 4 + 2] << 2 | pm[xi * 4 + 3] << 3);
+    }
+    __syncthreads();
+    for (int d = 1; d < n; ++d) {
+      // lane owns rows lane, lane + 32, ...: the cell (i, i + d) of each live row
+#pragma unroll 1
+      for (int i = tid; i + d < n; i += kSmallThreads) {  // (a small loop body: the loop stays in the
+        const int j = i + d;                    // instruction cache)
+        {
+          const int xj = xs[j];                                   // issued early: the pair test needs it
+          const int inner = d >= 2 ? (int)U[(i + 1) * W + j - 1] : 0;  // gamma(i+1, j-1)
+          const uint4* ur = reinterpret_cast<const uint4*>(U + i * W);
+          const uint4* lr = reinterpret_cast<const uint4*>(L + j * W);
+          uint32_t acc0 = 0, acc1 = 0;  // gamma >= 0 and the k = i term is >= 0: 0 is neutral
+#pragma unroll 1
+          for (int c = i >> 3; c <= (j >> 3); ++c) {
+            const uint4 a = ur[c], b = lr[c];
+            acc0 = __viaddmax_s16x2(a.x, b.x, acc0);
+            acc1 = __viaddmax_s16x2(a.y, b.y, acc1);
+            acc0 = __viaddmax_s16x2(a.z, b.z, acc0);
+            acc1 = __viaddmax_s16x2(a.w, b.w, acc1);
+          }
+          const uint32_t acc = __vmaxs2(acc0, acc1);
+          int v = max((int)(int16_t)(acc & 0xffffu), (int)(int16_t)(acc >> 16));
+          if (((prow[i] >> xj) & 1u) && d - 1 >= A.hairpin) v = max(v, inner + 1);
+          U[i * W + j] = (int16_t)v;
+          if (i >= 1) L[j * W + i - 1] = (int16_t)v;
+        }
+      }
+      if (kSmallThreads == 32) __syncwarp();
+      else __syncthreads();
+    }
+    if (tid == 0) A.scores[p] = n <= 1 ? 0 : (int)U[n - 1];
+    if (A.db && tid < 32) {  // canonical traceback (R-TB-NUSS), one warp, stack in shared memory
+      uint8_t* db = A.db + p * A.db_stride;
+      for (int k = lane; k < n; k += 32) db[k] = '.';
+      int sp = 0;
+      if (n > 1) {
+        if (lane == 0) { stack[0] = 0; stack[1] = n - 1; }
+        sp = 2;
+      }
+      auto gam = [&](int i, int j) -> int { return j - i < 1 ? 0 : (int)U[i * W + j]; };
+      int guard = 4 * n + 8;
+      while (sp > 0 && --guard > 0) {
+        __syncwarp();
+        const int j = stack[sp - 1], i = stack[sp - 2];
+        sp -= 2;
+        __syncwarp();
+        if (j - i < 1) continue;
+        // the four table reads of a step issued together (j - i >= 1)
+        const int v = U[i * W + j], g1 = gam(i + 1, j), g2 = gam(i, j - 1), g3 = gam(i + 1, j - 1);
+        const bool pr = pm[xs[i] * 4 + xs[j]] && j - i - 1 >= A.hairpin;
+        int ni0 = -1, nj0 = 0, ni1 = -1, nj1 = 0;
+        if (v == g1) { ni0 = i + 1; nj0 = j; }
+        else if (v == g2) { ni0 = i; nj0 = j - 1; }
+        else if (pr && v == g3 + 1) {
+          if (lane == 0) { db[i] = '('; db[j] = ')'; }
+          ni0 = i + 1; nj0 = j - 1;
+        } else {
+          for (int k0 = i + 1; k0 < j; k0 += 32) {  // smallest split k
+            const int k = k0 + lane;
+            const unsigned hit = __ballot_sync(0xffffffffu, k < j && v == (int)U[i * W + k] + (int)L[j * W + k]);
+            if (hit) {
+              const int kk = k0 + __ffs(hit) - 1;
+              ni0 = kk + 1; nj0 = j; ni1 = i; nj1 = kk;
+              break;
+            }
+          }
+        }
+        if (ni0 >= 0) {
+          if (lane == 0) { stack[sp] = ni0; stack[sp + 1] = nj0; }
+          sp += 2;
+        }
+        if (ni1 >= 0) {
+          if (lane == 0) { stack[sp] = ni1; stack[sp + 1] = nj1; }
+          sp += 2;
+        }
+      }
+      if (lane == 0) A.db_len[p] = n;
+    }
+  }
+}
+
 // One problem over the whole grid: partitions separated by grid-wide barriers
 // (cooperative launch), the table in global memory (L2-resident).
 __global__ void __launch_bounds__(kNussThreads) k_nuss_grid(NussArgs A, int64_t p) {
@@ -247,6 +384,22 @@ int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device) {
   if (n == 1) return table_elems(max_len) * 2 + stack_bytes + 256;
   const int64_t grid = std::min<int64_t>(n, (int64_t)num_sms(device) * 2);
   return grid * (table_elems(max_len) * 2 + stack_bytes) + 256;
+}
+
+bool nuss_small_supported(int64_t max_len, int64_t n, int device) {
+  return max_len <= kSmallMaxN && n <= (int64_t)num_sms(device) * 4;
+}
+
+cudaError_t nuss_small_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
+  if (A.n == 0) return cudaSuccess;
+  const size_t smem = small_smem_bytes(std::max<int64_t>(A.max_len, 1));
+  cudaError_t e = cudaFuncSetAttribute(k_nuss_small, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  ++*launches;
+  NussArgs a2 = A;
+  a2.max_len = std::max<int64_t>(A.max_len, 1);
+  k_nuss_small<<<(unsigned)A.n, kSmallThreads, smem, s>>>(a2);
+  return cudaGetLastError();
 }
 
 cudaError_t nuss_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {

@@ -11,9 +11,10 @@ import paper_conf_pldi_carteylm12_b200 as dp
 x = dpgen.config1_rna64()
 cat, off = dpgen.pack([x])
 c, o = torch.from_numpy(cat).cuda(), torch.from_numpy(off).cuda()
-for env in ({}, {"DP_NUSS_CELL": "1"}):
+for env in ({}, {"DP_NUSS_CELL": "1"}, {"DP_NUSS_TILED_MIN": "31"}):
     for tb in (False, True):
         os.environ.pop("DP_NUSS_CELL", None)
+        os.environ.pop("DP_NUSS_TILED_MIN", None)
         os.environ.update(env)
         with dp.Plan(dp.NUSSINOV, 64, pair_mask=dpgen.rna_pair_mask(), min_hairpin=3, want_traceback=tb) as p:
             out = torch.empty(1, dtype=torch.int32, device="cuda")

@@ -349,6 +349,23 @@ def test_nussinov_random_smem(dp, orc, h):
         assert r["db"][q] == db, q
 
 
+@pytest.mark.parametrize("h", [0, 1, 3])
+def test_nussinov_small_kernel_edges(dp, orc, h):
+    """k_nuss_small (one CTA per problem, table in shared memory; a few problems of <= 128 nt):
+    lengths at the 8-wide chunk edges and the 128 maximum, empty and 1-nt problems, hairpins 0
+    (the d = 1 pair term), 1 and 3, poly-A (score 0) and a fully pairing hairpin."""
+    g = np.random.default_rng(170 + h)
+    lens = [0, 1, 2, 3, 4, 5, 7, 8, 9, 15, 16, 17, 63, 64, 65, 100, 127, 128]
+    seqs = [g.integers(0, 4, size=l).astype(np.uint8) for l in lens]
+    seqs += [dpgen.encode("A" * 90, dpgen.RNA), dpgen.encode("GGGGGGGGAAAACCCCCCCC", dpgen.RNA)]
+    pm = dpgen.rna_pair_mask(gu=(h != 0))
+    r = run_nuss(dp, seqs, h=h, pm=pm)
+    for q, x in enumerate(seqs):
+        assert (r["scores"][q], r["db"][q]) == orc.nussinov_traceback(x, pm, h), (q, len(x))
+    r1 = run_nuss(dp, [seqs[-4]], h=h, pm=pm)  # a single problem (config 1's launch)
+    assert (r1["scores"][0], r1["db"][0]) == orc.nussinov_traceback(seqs[-4], pm, h)
+
+
 def test_nussinov_cell_level_path(dp, orc, monkeypatch):
     """The cell-level CTA kernels (shared-memory table; L2 table above 340) on the same cases."""
     monkeypatch.setenv("DP_NUSS_CELL", "1")
