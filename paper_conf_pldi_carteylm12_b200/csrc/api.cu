@@ -111,6 +111,8 @@ struct dp_plan {
     bool nuss_rounds = false, diag_generic = false, sw_intra = false;
     int64_t nuss_tiled_min = 32;
     int nuss_tbw = 0, diag_force = -1, host_chunks = 4;
+    bool hmm_simt = false;
+    int hmm_ns = 0, hmm_tc_smem_kb = -1;
   } env;
 };
 
@@ -129,6 +131,9 @@ void read_env(dp_plan* p) {
   if (on("DP_NUSS_TILED_MIN")) p->env.nuss_tiled_min = atoll(getenv("DP_NUSS_TILED_MIN"));
   if (on("DP_NUSS_TBW")) p->env.nuss_tbw = atoi(getenv("DP_NUSS_TBW"));
   if (on("DP_DIAG_FORCE")) p->env.diag_force = atoi(getenv("DP_DIAG_FORCE"));
+  p->env.hmm_simt = on("DP_HMM_SIMT");
+  if (on("DP_HMM_NS")) p->env.hmm_ns = atoi(getenv("DP_HMM_NS"));
+  if (on("DP_HMM_TC_SMEM_KB")) p->env.hmm_tc_smem_kb = atoi(getenv("DP_HMM_TC_SMEM_KB"));
   if (on("DP_HOST_CHUNKS")) p->env.host_chunks = std::max(1, std::min(dp_plan::kMaxChunks, atoi(getenv("DP_HOST_CHUNKS"))));
 }
 
@@ -592,6 +597,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
     case DP_HMM_FORWARD:
     case DP_HMM_VITERBI: {
       dpk::HmmArgs H{};
+      H.ns_override = p->env.hmm_ns;
       H.n = n; H.x_cat = a_cat; H.x_off = a_off; H.max_len = max_len_a; H.S = p->S; H.K = p->K;
       if (p->kind == DP_HMM_FORWARD) {
         H.pi = p->d_pi; H.A = p->d_A; H.E = p->d_E;
@@ -599,7 +605,8 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         // the [batch x S] x [S x S] step on tcgen05 (SIMT fallback kernel via DP_HMM_SIMT=1)
         unsigned long long* dbg = nullptr;
         if (p->env.hmm_timing) cudaMalloc(&dbg, 8 * 4 * 66), cudaMemset(dbg, 0, 8 * 4 * 66), H.dbg = dbg;
-        e = dpk::hmm_forward_tc_supported(p->S) ? dpk::hmm_forward_tc(H, s, &p->launches)
+        H.tc_smem_kb = p->env.hmm_tc_smem_kb;
+        e = (dpk::hmm_forward_tc_supported(p->S) && !p->env.hmm_simt) ? dpk::hmm_forward_tc(H, s, &p->launches)
                                                  : dpk::hmm_forward(H, s, &p->launches);
         if (dbg) {  // diagnostic: CTA 0 step phases (ns): MMA issue, wait for MMA, epilogue, barrier
           unsigned long long h[4 * 66];

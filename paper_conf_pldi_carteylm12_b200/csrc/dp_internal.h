@@ -154,6 +154,8 @@ struct HmmArgs {
   uint8_t* bp;                      // Viterbi back-pointers (n x max_len x 64) or nullptr
   int32_t* final_state;             // n
   unsigned long long* dbg = nullptr;  // diagnostic step timestamps (DP_HMM_TIMING), else nullptr
+  int ns_override = 0;                // diagnostic: sequences per warp of the SIMT kernels (DP_HMM_NS)
+  int tc_smem_kb = -1;                // shared memory the tcgen05 forward reserves per CTA (-1: default)
 };
 cudaError_t hmm_forward(const HmmArgs& a, cudaStream_t s, int64_t* launches);
 bool hmm_forward_tc_supported(int S);

@@ -346,7 +346,7 @@ void* fwd_ptr(bool viterbi) { return viterbi ? (void*)k_viterbi<NS> : (void*)k_f
 // Sequences per warp: minimise (waves of resident warps) x (NS + latency term): the per-warp
 // time grows with NS plus (forward) a latency term that NS independent sequences share;
 // ties go to the smaller NS.
-int pick_ns(int64_t n, bool viterbi, void** kern) {
+int pick_ns(int64_t n, bool viterbi, void** kern, int ns_override) {
   void* ks[8] = {fwd_ptr<1>(viterbi), fwd_ptr<2>(viterbi), fwd_ptr<3>(viterbi), fwd_ptr<4>(viterbi),
                  fwd_ptr<5>(viterbi), fwd_ptr<6>(viterbi), fwd_ptr<7>(viterbi), fwd_ptr<8>(viterbi)};
   const int sms = sms_of_current();
@@ -363,7 +363,7 @@ int pick_ns(int64_t n, bool viterbi, void** kern) {
     const int64_t cost = ((warps + wave - 1) / wave) * (ns + (viterbi ? 0 : 2));
     if (cost < best_cost) { best_cost = cost; best = ns; }
   }
-  if (getenv("DP_HMM_NS")) best = std::max(1, std::min(8, atoi(getenv("DP_HMM_NS"))));  // diagnostic
+  if (ns_override > 0) best = std::max(1, std::min(8, ns_override));  // diagnostic (DP_HMM_NS)
   *kern = ks[best - 1];
   return best;
 }
@@ -373,7 +373,7 @@ int pick_ns(int64_t n, bool viterbi, void** kern) {
 cudaError_t hmm_forward(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
   if (H.n == 0) return cudaSuccess;
   void* kern = nullptr;
-  const int ns = pick_ns(H.n, false, &kern);
+  const int ns = pick_ns(H.n, false, &kern, H.ns_override);
   const int64_t warps = (H.n + ns - 1) / ns;
   HmmArgs h2 = H;
   void* args[1] = {&h2};
@@ -384,7 +384,7 @@ cudaError_t hmm_forward(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
 cudaError_t hmm_viterbi(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
   if (H.n == 0) return cudaSuccess;
   void* kern = nullptr;
-  const int ns = pick_ns(H.n, true, &kern);
+  const int ns = pick_ns(H.n, true, &kern, H.ns_override);
   const int64_t warps = (H.n + ns - 1) / ns;
   HmmArgs h2 = H;
   void* args[1] = {&h2};

@@ -1,27 +1,28 @@
 // HMM forward on the 5th-generation tensor cores (tcgen05 + TMEM): the one
 // step of the hot path that really is a dense GEMM (BASELINE north_star;
 // SURVEY.md §8(a) A6c). Schedule S(s,i) = i (§5.2): the
-// partition i of 128 sequences is one [128 x 64] x [64 x 64] product
+// partition i of a group of 128 sequences is one [128 x 64] x [64 x 64] product
 //     D[b][s] = sum_p alpha_{i-1}[b][p] * t_{p,s}
 // followed by the emission / normalisation epilogue of Fig.11a (L472–L474).
 //
-// One CTA = 128 sequences (the MMA's M), 16 warps: warp w reads TMEM lane
-// quarter w % 4 (sequences 32 (w % 4) ..) and handles states 16 (w / 4) .. + 15.
-// Per step:
-//   * thread 0 issues 8 tcgen05.mma.kind::f16 (M=128, K=16) into the fp32 TMEM
-//     accumulator: alpha_hi x [A_hi | A_lo] (N=128) and alpha_lo x A_hi (N=64),
+// Warp-specialised CTA of kNG = 4 groups of 128 sequences (the MMA's M):
+//   * the MMA warp (one elected lane) issues, per step and group, 12
+//     tcgen05.mma.kind::f16 (M=128, N=64, K=16) into that group's fp32 TMEM
+//     accumulator (64 columns): alpha_hi x A_hi + alpha_hi x A_lo + alpha_lo x A_hi,
 //     where x = x_hi + x_lo is a two-term bf16 split (the dropped lo x lo term is
 //     ~2^-16 of a 2^-8 term: ~1e-7 relative per step, DESIGN.md §2 "HMM precision");
-//     columns 64..127 hold alpha_hi A_lo and are added in the epilogue;
-//   * tcgen05.commit arrives on an mbarrier; every thread reads its 16 (+16)
-//     columns with tcgen05.ld, multiplies by e_s(x_i), scales by 1/R_{i-1} (the
-//     previous step's row sum: lagged scaling keeps the row reduction off the
-//     critical path, log P = sum_i log R_i), splits into bf16 hi/lo and stores
-//     the next A operand in the canonical K-major no-swizzle UMMA layout
-//     (8x16-byte core matrices).
-// Operands live in shared memory (alpha hi/lo 2 x 16 KB, transitions 16 KB);
-// the accumulator lives in TMEM (128 columns). DP_HMM_TIMING=1 prints per-phase
-// step times of CTA 0 (diagnostic).
+//     a tcgen05.commit arrives on the group's `full` mbarrier;
+//   * four epilogue warps per group (warp w reads TMEM lane quarter w % 4), ONE
+//     SEQUENCE PER THREAD over all 64 states: tcgen05.ld of the row, times e_s(x_i),
+//     scaled by 1/R_{i-1} (the previous step's row sum, thread-local: lagged
+//     scaling, log P = sum_i log R_i), split into bf16 hi/lo and stored as the
+//     next A operand in the canonical K-major no-swizzle UMMA layout (8x16-byte
+//     core matrices); then all 128 threads arrive on the group's `empty` mbarrier.
+// The groups' chains are independent, so the tensor pipe works on one group while
+// the epilogue warps of the others run; no CTA-wide barrier inside the step loop
+// (the row sum needs no cross-warp reduction when a thread owns a whole row).
+// Operands live in shared memory (alpha hi/lo 2 x 16 KB per group, transitions
+// hi/lo 16 KB); the accumulators in TMEM (4 x 64 columns).
 #include <algorithm>
 #include <cstdint>
 #include <cstdlib>
@@ -37,7 +38,7 @@ constexpr int kM = 128;       // sequences per CTA (UMMA M)
 constexpr int kS = 64;        // states (UMMA N and K)
 constexpr int kCore = 128;    // bytes per 8x(16 B) core matrix
 constexpr int kN2 = 2 * kS;    // N of the alpha_hi x [A_hi | A_lo] product
-constexpr int kTmemCols = kN2;
+constexpr int kTmemCols = kS;   // per group: the three products accumulate into the same 64 columns
 
 // K-major no-swizzle operand: core matrix (row group rg, k chunk kc) at
 // (kc * row_groups + rg) * 128 bytes, rows of a core matrix 16 bytes apart.
@@ -93,17 +94,24 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]) \
       : "r"(taddr))
 
-constexpr int kThreads = 512;  // 16 warps: warp w serves TMEM lane quarter w % 4 and states 16 (w / 4) ..
+constexpr int kNG = 4;                     // sequence groups per CTA
+constexpr int kEpiWarps = 4 * kNG;         // epilogue warps (4 per group: the TMEM lane quarters)
+constexpr int kThreads = 32 * (kEpiWarps + 1);  // + the MMA warp
 
 struct TcSmem {
-  alignas(128) uint8_t a_hi[kM * kS * 2];   // alpha (A operand), K-major core matrices
-  alignas(128) uint8_t a_lo[kM * kS * 2];
+  alignas(128) uint8_t a_hi[kNG][kM * kS * 2];   // alpha (A operand), K-major core matrices, per group
+  alignas(128) uint8_t a_lo[kNG][kM * kS * 2];
   alignas(128) uint8_t b_cat[kN2 * kS * 2];  // transitions (B operand): row n = s (A_hi) or 64 + s (A_lo), k = p
-  alignas(16) float E[16][kS + 4];          // emission rows, padded against bank conflicts
-  float psum[2][4][kM];                     // per-step partial row sums (double-buffered by step parity)
-  uint64_t bar;
+  alignas(16) float E[16][kS + 4];          // emission rows
+  uint64_t full[kNG];                       // MMA -> epilogue: the group's accumulator is ready
+  uint64_t empty[kNG];                      // epilogue -> MMA: the group's next operand is stored
   uint32_t tmem_base;
+  int tmax;
 };
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
 
 // Two bf16x2 words (hi, lo) with a + b = (hi.x + lo.x, hi.y + lo.y) to ~2^-16.
 __device__ __forceinline__ void split2(float a, float b, uint32_t& hi, uint32_t& lo) {
@@ -116,18 +124,12 @@ __device__ __forceinline__ void split2(float a, float b, uint32_t& hi, uint32_t&
 
 // Per step, with lagged scaling: alpha^_i = ((alpha^_{i-1} A) o e(x_i)) / R_{i-1},
 // R_i = sum_s alpha^_i(s); then P(x) = prod_{i<=T} R_i and log P = sum log R_i. Dividing by the
-// previous step's sum (known before the MMA finishes) keeps R_i within the emission range
-// because A is row-stochastic, and takes the row reduction off the critical path.
+// previous step's sum keeps R_i within the emission range because A is row-stochastic.
 __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
   extern __shared__ __align__(1024) uint8_t tc_raw[];
   TcSmem& sm = *reinterpret_cast<TcSmem*>(tc_raw);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int lq = warp & 3, cg = warp >> 2;  // TMEM lane quarter, state group
-  const int b = 32 * lq + lane;             // this thread's sequence (row) in the CTA
-  const int s0 = 16 * cg;                   // this thread's 16 states
   const int S = H.S, K = H.K;
-  const int64_t p = (int64_t)blockIdx.x * kM + b;
-  const bool live = p < H.n;
 
   // transitions: B[s][p] = t_{p,s} (K = p contiguous), split into bf16 hi/lo
   for (int q = tid; q < kS * kS; q += kThreads) {
@@ -143,164 +145,170 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
     sm.E[c][s] = (c < K && s < S) ? H.E[s * K + c] : 0.f;
   }
   if (tid == 0) {
-    mbar_init(&sm.bar, 1);
+    for (int g = 0; g < kNG; ++g) {
+      mbar_init(&sm.full[g], 1);
+      mbar_init(&sm.empty[g], 128);
+    }
+    sm.tmax = 0;
     asm volatile("fence.mbarrier_init.release.cluster;");
   }
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&sm.tmem_base)),
-                 "n"(kTmemCols));
+                 "n"(kNG * kTmemCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
+  // epilogue threads: group g, row b (TMEM lane 32 lq + lane)
+  const bool epi = warp < kEpiWarps;
+  const int g = epi ? warp >> 2 : 0, lq = warp & 3, b = 32 * lq + lane;
+  const int64_t p = ((int64_t)blockIdx.x * kNG + g) * kM + b;
+  const bool live = epi && p < H.n;
   const uint8_t* x = live ? H.x_cat + H.x_off[p] : nullptr;
   const int T = live ? (int)(H.x_off[p + 1] - H.x_off[p]) : 0;
-  __shared__ int tmax_s;
-  if (tid == 0) tmax_s = 0;
-  asm volatile("fence.proxy.async.shared::cta;");
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
   const uint32_t tmem = sm.tmem_base;
-  if (cg == 0) atomicMax(&tmax_s, T);
-
-  const uint32_t a_hi = smem_u32(sm.a_hi), a_lo = smem_u32(sm.a_lo);
-  // descriptors: K chunk pairs 32 bytes... (2 core matrices of 8 k) apart by 2 x LBO
-  const uint64_t dA_hi = make_desc(a_hi, (kM / 8) * kCore, kCore), dA_lo = make_desc(a_lo, (kM / 8) * kCore, kCore);
-  const uint64_t dB = make_desc(smem_u32(sm.b_cat), (kN2 / 8) * kCore, kCore);
-  const uint32_t taddr = tmem + ((uint32_t)(lq * 32) << 16) + (uint32_t)s0;
-  // store 16 values of alpha^ as the A operand (k = s0 .. s0 + 15: two k chunks of 8)
-  auto store_operand = [&](const float* v) {
-    uint32_t hw[8], lw[8];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) split2(v[2 * q], v[2 * q + 1], hw[q], lw[q]);
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const uint32_t off = op_offset(b, s0 + 8 * h, kM / 8);
-      *reinterpret_cast<uint4*>(sm.a_hi + off) = make_uint4(hw[4 * h], hw[4 * h + 1], hw[4 * h + 2], hw[4 * h + 3]);
-      *reinterpret_cast<uint4*>(sm.a_lo + off) = make_uint4(lw[4 * h], lw[4 * h + 1], lw[4 * h + 2], lw[4 * h + 3]);
-    }
-  };
-  // i = 1: alpha^_1(s) = pi_s e_s(x_1) (no scaling)
-  {
-    const int c = T > 0 ? x[0] : 0;
-    float v[16], tot = 0.f;
-#pragma unroll
-    for (int q = 0; q < 16; ++q) {
-      const int s = s0 + q;
-      v[q] = (s < S && T > 0) ? H.pi[s] * sm.E[c][s] : 0.f;
-      tot += v[q];
-    }
-    store_operand(v);
-    sm.psum[1][cg][b] = tot;
-  }
-  asm volatile("fence.proxy.async.shared::cta;");
-  asm volatile("tcgen05.fence::before_thread_sync;");
+  if (T > 0) atomicMax(&sm.tmax, T);
   __syncthreads();
-  const int Tmax = tmax_s;
-  double prod = 1.0;  // prod of R_i, renormalised: P = prod * 2^pexp
-  int pexp = 0;
-  uint32_t parity = 0;
-  uint4 xs = make_uint4(0, 0, 0, 0);
-  auto stamp = [&](int i, int k) {
-    if (H.dbg && blockIdx.x == 0 && tid == 0 && i < 66) {
-      unsigned long long t;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-      H.dbg[4 * i + k] = t;
-    }
-  };
-  for (int i = 2; i <= Tmax; ++i) {
-    stamp(i, 0);
-    if (tid == 0) {
-      asm volatile("tcgen05.fence::after_thread_sync;");
-      // D[:, 0:64] = a_hi*A_hi + a_lo*A_hi, D[:, 64:128] = a_hi*A_lo; K = 64 in 4 steps of 16.
+  const int Tmax = sm.tmax;
+
+  if (!epi) {  // ------------------------------------------------------------ the MMA warp
+    if (lane == 0) {
+      const uint64_t dB = make_desc(smem_u32(sm.b_cat), (kN2 / 8) * kCore, kCore);
+      // A_lo: rows n = 64 .. 127 of the B buffer (8 row groups further on)
+      const uint64_t dB_lo = make_desc(smem_u32(sm.b_cat) + (kS / 8) * kCore, (kN2 / 8) * kCore, kCore);
+      // D_g = a_hi*A_hi + a_hi*A_lo + a_lo*A_hi: three N = 64 products into the same 64 columns;
+      // K = 64 in 4 steps of 16.
       // Descriptor address fields count 16-byte units: a K step of 16 is two core matrices.
+      for (int i = 2; i <= Tmax; ++i) {
+        for (int q = 0; q < kNG; ++q) {
+          mbar_wait(&sm.empty[q], (uint32_t)(i - 2) & 1u);
+          asm volatile("tcgen05.fence::after_thread_sync;");
+          const uint64_t dA_hi = make_desc(smem_u32(sm.a_hi[q]), (kM / 8) * kCore, kCore);
+          const uint64_t dA_lo = make_desc(smem_u32(sm.a_lo[q]), (kM / 8) * kCore, kCore);
+          const uint32_t td = tmem + (uint32_t)(q * kTmemCols);
 #pragma unroll
-      for (int kk = 0; kk < kS / 16; ++kk)
-        mma_bf16<kN2>(tmem, dA_hi + (uint64_t)(2 * kk * (kM / 8) * kCore >> 4),
-                      dB + (uint64_t)(2 * kk * (kN2 / 8) * kCore >> 4), kk > 0);
-#pragma unroll
-      for (int kk = 0; kk < kS / 16; ++kk)
-        mma_bf16<kS>(tmem, dA_lo + (uint64_t)(2 * kk * (kM / 8) * kCore >> 4),
-                     dB + (uint64_t)(2 * kk * (kN2 / 8) * kCore >> 4), 1);
-      asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-          smem_u32(&sm.bar)));
-    }
-    stamp(i, 1);
-    // while the MMAs run: R_{i-1}, the scale, the symbol and its emission row
-    const float* ps = &sm.psum[(i - 1) & 1][0][0];
-    const float R = (ps[b] + ps[kM + b]) + (ps[2 * kM + b] + ps[3 * kM + b]);
-    const float inv = R > 0.f ? 1.f / R : 0.f;
-    if (i - 1 <= T) {
-      prod *= (double)R;
-      if ((i & 15) == 0) {  // keep the product normal: P = prod * 2^pexp
-        int e2;
-        prod = frexp(prod, &e2);
-        pexp += e2;
+          for (int kk = 0; kk < kS / 16; ++kk) {
+            const uint64_t ka = (uint64_t)(2 * kk * (kM / 8) * kCore >> 4);
+            const uint64_t kb = (uint64_t)(2 * kk * (kN2 / 8) * kCore >> 4);
+            mma_bf16<kS>(td, dA_hi + ka, dB + kb, kk > 0);  // a_hi x A_hi
+            mma_bf16<kS>(td, dA_hi + ka, dB_lo + kb, 1);    // a_hi x A_lo
+            mma_bf16<kS>(td, dA_lo + ka, dB + kb, 1);       // a_lo x A_hi
+          }
+          asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+              smem_u32(&sm.full[q])));
+        }
       }
     }
-    if (((i - 2) & 15) == 0 && i - 1 < T) {
-      uint8_t tmp[16];
+  } else {  // -------------------------------------------------------------- epilogue warps
+    uint8_t* ahi = sm.a_hi[g];
+    uint8_t* alo = sm.a_lo[g];
+    // 16 values of alpha^ (states k0 .. k0 + 15) as the group's A operand: two k chunks of 8
+    auto store16 = [&](int k0, const float* v) {
+      uint32_t hw[8], lw[8];
 #pragma unroll
-      for (int q = 0; q < 16; ++q) tmp[q] = (i - 1 + q < T) ? x[i - 1 + q] : 0;
-      xs = *reinterpret_cast<uint4*>(tmp);
-    }
-    const int sh = (i - 2) & 15;
-    const uint32_t word = sh < 4 ? xs.x : sh < 8 ? xs.y : sh < 12 ? xs.z : xs.w;
-    const int c = (word >> (8 * (sh & 3))) & 0xff;
-    const float4* er = reinterpret_cast<const float4*>(&sm.E[c][s0]);
-    const float4 e0 = er[0], e1 = er[1], e2 = er[2], e3 = er[3];
-    mbar_wait(&sm.bar, parity);
-    stamp(i, 2);
-    parity ^= 1;
-    asm volatile("tcgen05.fence::after_thread_sync;");
-    uint32_t r[16], r2[16];
-    TMEM_LD16(taddr, r);
-    TMEM_LD16(taddr + kS, r2);
-    asm volatile("tcgen05.wait::ld.sync.aligned;");
-    if (i <= T) {
-      const float ev[16] = {e0.x, e0.y, e0.z, e0.w, e1.x, e1.y, e1.z, e1.w,
-                            e2.x, e2.y, e2.z, e2.w, e3.x, e3.y, e3.z, e3.w};
-      float v[16], tot = 0.f;
+      for (int q = 0; q < 8; ++q) split2(v[2 * q], v[2 * q + 1], hw[q], lw[q]);
 #pragma unroll
-      for (int q = 0; q < 16; ++q) {
-        v[q] = (__uint_as_float(r[q]) + __uint_as_float(r2[q])) * ev[q] * inv;
-        tot += v[q];
+      for (int h = 0; h < 2; ++h) {
+        const uint32_t off = op_offset(b, k0 + 8 * h, kM / 8);
+        *reinterpret_cast<uint4*>(ahi + off) = make_uint4(hw[4 * h], hw[4 * h + 1], hw[4 * h + 2], hw[4 * h + 3]);
+        *reinterpret_cast<uint4*>(alo + off) = make_uint4(lw[4 * h], lw[4 * h + 1], lw[4 * h + 2], lw[4 * h + 3]);
       }
-      store_operand(v);
-      sm.psum[i & 1][cg][b] = tot;
+    };
+    double prod = 1.0;  // prod of R_i, renormalised: P = prod * 2^pexp
+    int pexp = 0;
+    float R = 0.f;      // this row's sum of the previous step
+    // i = 1: alpha^_1(s) = pi_s e_s(x_1) (no scaling)
+    {
+      const int c = T > 0 ? x[0] : 0;
+#pragma unroll
+      for (int k0 = 0; k0 < kS; k0 += 16) {
+        float v[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+          const int s = k0 + q;
+          v[q] = (s < S && T > 0) ? H.pi[s] * sm.E[c][s] : 0.f;
+          R += v[q];
+        }
+        store16(k0, v);
+      }
     }
-    stamp(i, 3);
     asm volatile("fence.proxy.async.shared::cta;");
-    asm volatile("tcgen05.fence::before_thread_sync;");
-    __syncthreads();
-  }
-  if (cg == 0 && Tmax >= 1 && Tmax <= T) {  // R_T of the sequences that run to the end
-    const float* ps = &sm.psum[Tmax & 1][0][0];
-    const float R = (ps[b] + ps[kM + b]) + (ps[2 * kM + b] + ps[3 * kM + b]);
-    prod *= (double)R;
+    mbar_arrive(&sm.empty[g]);
+    uint4 xs = make_uint4(0, 0, 0, 0);
+    const uint32_t taddr = tmem + ((uint32_t)(lq * 32) << 16) + (uint32_t)(g * kTmemCols);
+    for (int i = 2; i <= Tmax; ++i) {
+      const float inv = R > 0.f ? 1.f / R : 0.f;
+      if (i - 1 <= T) {
+        prod *= (double)R;
+        if ((i & 15) == 0) {  // keep the product normal: P = prod * 2^pexp
+          int e2;
+          prod = frexp(prod, &e2);
+          pexp += e2;
+        }
+      }
+      if (((i - 2) & 15) == 0 && i - 1 < T) {
+        uint8_t tmp[16];
+#pragma unroll
+        for (int u = 0; u < 16; ++u) tmp[u] = (i - 1 + u < T) ? x[i - 1 + u] : 0;
+        xs = *reinterpret_cast<uint4*>(tmp);
+      }
+      const int sh = (i - 2) & 15;
+      const uint32_t word = sh < 4 ? xs.x : sh < 8 ? xs.y : sh < 12 ? xs.z : xs.w;
+      const float* er = &sm.E[(word >> (8 * (sh & 3))) & 0xff][0];
+      mbar_wait(&sm.full[g], (uint32_t)(i - 2) & 1u);
+      asm volatile("tcgen05.fence::after_thread_sync;");
+      float tot = 0.f;
+      uint32_t r[kS];  // the row: 64 accumulators, four loads and one wait
+      TMEM_LD16(taddr, r);
+      TMEM_LD16(taddr + 16, (r + 16));
+      TMEM_LD16(taddr + 32, (r + 32));
+      TMEM_LD16(taddr + 48, (r + 48));
+      asm volatile("tcgen05.wait::ld.sync.aligned;");
+#pragma unroll
+      for (int k0 = 0; k0 < kS; k0 += 16) {
+        const float4* e4 = reinterpret_cast<const float4*>(er + k0);
+        const float4 e0 = e4[0], e1 = e4[1], e2 = e4[2], e3 = e4[3];
+        const float ev[16] = {e0.x, e0.y, e0.z, e0.w, e1.x, e1.y, e1.z, e1.w,
+                              e2.x, e2.y, e2.z, e2.w, e3.x, e3.y, e3.z, e3.w};
+        float v[16];
+#pragma unroll
+        for (int u = 0; u < 16; ++u) {
+          v[u] = __uint_as_float(r[k0 + u]) * (ev[u] * inv);
+          tot += v[u];
+        }
+        if (i <= T) store16(k0, v);
+      }
+      if (i <= T) R = tot;
+      asm volatile("fence.proxy.async.shared::cta;");
+      asm volatile("tcgen05.fence::before_thread_sync;");
+      mbar_arrive(&sm.empty[g]);
+    }
+    if (Tmax >= 1 && Tmax <= T) prod *= (double)R;  // R_T of the sequences that run to the end
+    if (live) H.ll_out[p] = T == 0 ? 0.f : (float)(log(prod) + (double)pexp * 0.69314718055994530942);
   }
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   if (warp == 0) {
     asm volatile("tcgen05.fence::after_thread_sync;");
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kTmemCols));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kNG * kTmemCols));
   }
-  if (live && cg == 0) H.ll_out[p] = T == 0 ? 0.f : (float)(log(prod) + (double)pexp * 0.69314718055994530942);
 }
 
 }  // namespace
 
-bool hmm_forward_tc_supported(int S) { return S <= kS && getenv("DP_HMM_SIMT") == nullptr; }
+bool hmm_forward_tc_supported(int S) { return S <= kS; }
 
 cudaError_t hmm_forward_tc(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
   if (H.n == 0) return cudaSuccess;
-  // The step is a latency chain (MMA -> epilogue -> MMA): reserving the SM's shared memory keeps
-  // other kernels' CTAs (e.g. a concurrent Viterbi) off the SMs running it. DP_HMM_TC_SHARE=1: no.
+  // The step is a latency chain (MMA -> epilogue -> MMA); the shared memory a CTA reserves decides
+  // how many of a concurrent kernel's CTAs (Viterbi) may share its SM (tc_smem_kb).
   const size_t need = sizeof(TcSmem) + 1024;
-  const size_t smem = getenv("DP_HMM_TC_SHARE") ? need : std::max(need, (size_t)200 * 1024);
+  const size_t smem = std::max(need, (size_t)(H.tc_smem_kb >= 0 ? H.tc_smem_kb : 200) * 1024);
   cudaError_t e = cudaFuncSetAttribute(k_forward_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   ++*launches;
-  k_forward_tc<<<(unsigned)((H.n + kM - 1) / kM), kThreads, smem, s>>>(H);
+  k_forward_tc<<<(unsigned)((H.n + kNG * kM - 1) / (kNG * kM)), kThreads, smem, s>>>(H);
   return cudaGetLastError();
 }
 
