@@ -5,7 +5,7 @@
 //     D[b][s] = sum_p alpha_{i-1}[b][p] * t_{p,s}
 // followed by the emission / normalisation epilogue of Fig.11a (L472–L474).
 //
-// Warp-specialised CTA of kNG = 4 groups of 128 sequences (the MMA's M):
+// Warp-specialised CTA of kNG groups of 128 sequences (the MMA's M):
 //   * the MMA warp (one elected lane) issues, per step and group, 12
 //     tcgen05.mma.kind::f16 (M=128, N=64, K=16) into that group's fp32 TMEM
 //     accumulator (64 columns): alpha_hi x A_hi + alpha_hi x A_lo + alpha_lo x A_hi,
@@ -38,7 +38,6 @@ constexpr int kM = 128;       // sequences per CTA (UMMA M)
 constexpr int kS = 64;        // states (UMMA N and K)
 constexpr int kCore = 128;    // bytes per 8x(16 B) core matrix
 constexpr int kN2 = 2 * kS;    // N of the alpha_hi x [A_hi | A_lo] product
-constexpr int kTmemCols = kS;   // per group: the three products accumulate into the same 64 columns
 
 // K-major no-swizzle operand: core matrix (row group rg, k chunk kc) at
 // (kc * row_groups + rg) * 128 bytes, rows of a core matrix 16 bytes apart.
@@ -70,6 +69,18 @@ __device__ __forceinline__ void mma_bf16(uint32_t tmem_d, uint64_t adesc, uint64
       : "r"(tmem_d), "l"(adesc), "l"(bdesc), "n"(idesc<N>()), "r"(accumulate));
 }
 
+// A from TMEM (the ".kind::f16 [d], [a], b_desc" form): A's rows in TMEM lanes, its K values
+// packed two bf16 per 32-bit column (K-major), B from shared memory.
+template <int N>
+__device__ __forceinline__ void mma_bf16_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}\n"
+      :
+      : "r"(tmem_d), "r"(tmem_a), "l"(bdesc), "n"(idesc<N>()), "r"(accumulate));
+}
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
 }
@@ -94,13 +105,21 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]) \
       : "r"(taddr))
 
-constexpr int kNG = 4;                     // sequence groups per CTA
+#ifndef HMM_TC_GROUPS
+#define HMM_TC_GROUPS 1   // 1 / 2 / 4 groups: forward alone 1.07 / 1.26 / 2.17 ms, config-3 step 3.61 / 3.66 / 3.62 ms
+#endif
+constexpr int kNG = HMM_TC_GROUPS;         // sequence groups per CTA
 constexpr int kEpiWarps = 4 * kNG;         // epilogue warps (4 per group: the TMEM lane quarters)
 constexpr int kThreads = 32 * (kEpiWarps + 1);  // + the MMA warp
+// TMEM columns per group: the fp32 accumulator (64), then alpha_hi and alpha_lo as the next A
+// operand (64 bf16 = 32 columns each)
+constexpr int kColsAcc = 0, kColsAHi = kS, kColsALo = kS + kS / 2, kColsGroup = 2 * kS;
+
+#define TMEM_ST8(taddr, w)                                                                      \
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr), \
+               "r"(w[0]), "r"(w[1]), "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7]) : "memory")
 
 struct TcSmem {
-  alignas(128) uint8_t a_hi[kNG][kM * kS * 2];   // alpha (A operand), K-major core matrices, per group
-  alignas(128) uint8_t a_lo[kNG][kM * kS * 2];
   alignas(128) uint8_t b_cat[kN2 * kS * 2];  // transitions (B operand): row n = s (A_hi) or 64 + s (A_lo), k = p
   alignas(16) float E[16][kS + 4];          // emission rows
   uint64_t full[kNG];                       // MMA -> epilogue: the group's accumulator is ready
@@ -154,7 +173,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
   }
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&sm.tmem_base)),
-                 "n"(kNG * kTmemCols));
+                 "n"(kNG * kColsGroup));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   // epilogue threads: group g, row b (TMEM lane 32 lq + lane)
@@ -164,6 +183,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
   const bool live = epi && p < H.n;
   const uint8_t* x = live ? H.x_cat + H.x_off[p] : nullptr;
   const int T = live ? (int)(H.x_off[p + 1] - H.x_off[p]) : 0;
+  asm volatile("fence.proxy.async.shared::cta;");  // B (generic stores) -> the MMAs (async proxy)
   asm volatile("tcgen05.fence::before_thread_sync;");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;");
@@ -184,16 +204,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
         for (int q = 0; q < kNG; ++q) {
           mbar_wait(&sm.empty[q], (uint32_t)(i - 2) & 1u);
           asm volatile("tcgen05.fence::after_thread_sync;");
-          const uint64_t dA_hi = make_desc(smem_u32(sm.a_hi[q]), (kM / 8) * kCore, kCore);
-          const uint64_t dA_lo = make_desc(smem_u32(sm.a_lo[q]), (kM / 8) * kCore, kCore);
-          const uint32_t td = tmem + (uint32_t)(q * kTmemCols);
+          const uint32_t td = tmem + (uint32_t)(q * kColsGroup + kColsAcc);
+          const uint32_t ta_hi = tmem + (uint32_t)(q * kColsGroup + kColsAHi);
+          const uint32_t ta_lo = tmem + (uint32_t)(q * kColsGroup + kColsALo);
 #pragma unroll
-          for (int kk = 0; kk < kS / 16; ++kk) {
-            const uint64_t ka = (uint64_t)(2 * kk * (kM / 8) * kCore >> 4);
+          for (int kk = 0; kk < kS / 16; ++kk) {  // a K step of 16 bf16: 8 TMEM columns of A
             const uint64_t kb = (uint64_t)(2 * kk * (kN2 / 8) * kCore >> 4);
-            mma_bf16<kS>(td, dA_hi + ka, dB + kb, kk > 0);  // a_hi x A_hi
-            mma_bf16<kS>(td, dA_hi + ka, dB_lo + kb, 1);    // a_hi x A_lo
-            mma_bf16<kS>(td, dA_lo + ka, dB + kb, 1);       // a_lo x A_hi
+            mma_bf16_ts<kS>(td, ta_hi + 8 * kk, dB + kb, kk > 0);  // a_hi x A_hi
+            mma_bf16_ts<kS>(td, ta_hi + 8 * kk, dB_lo + kb, 1);    // a_hi x A_lo
+            mma_bf16_ts<kS>(td, ta_lo + 8 * kk, dB + kb, 1);       // a_lo x A_hi
           }
           asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
               smem_u32(&sm.full[q])));
@@ -201,19 +220,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
       }
     }
   } else {  // -------------------------------------------------------------- epilogue warps
-    uint8_t* ahi = sm.a_hi[g];
-    uint8_t* alo = sm.a_lo[g];
-    // 16 values of alpha^ (states k0 .. k0 + 15) as the group's A operand: two k chunks of 8
+    const uint32_t trow = tmem + ((uint32_t)(lq * 32) << 16) + (uint32_t)(g * kColsGroup);
+    // 16 values of alpha^ (states k0 .. k0 + 15) into this row of the group's TMEM A operand
     auto store16 = [&](int k0, const float* v) {
       uint32_t hw[8], lw[8];
 #pragma unroll
       for (int q = 0; q < 8; ++q) split2(v[2 * q], v[2 * q + 1], hw[q], lw[q]);
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const uint32_t off = op_offset(b, k0 + 8 * h, kM / 8);
-        *reinterpret_cast<uint4*>(ahi + off) = make_uint4(hw[4 * h], hw[4 * h + 1], hw[4 * h + 2], hw[4 * h + 3]);
-        *reinterpret_cast<uint4*>(alo + off) = make_uint4(lw[4 * h], lw[4 * h + 1], lw[4 * h + 2], lw[4 * h + 3]);
-      }
+      TMEM_ST8(trow + kColsAHi + k0 / 2, hw);
+      TMEM_ST8(trow + kColsALo + k0 / 2, lw);
     };
     double prod = 1.0;  // prod of R_i, renormalised: P = prod * 2^pexp
     int pexp = 0;
@@ -233,10 +247,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
         store16(k0, v);
       }
     }
-    asm volatile("fence.proxy.async.shared::cta;");
+    asm volatile("tcgen05.wait::st.sync.aligned;");
+    asm volatile("tcgen05.fence::before_thread_sync;");
     mbar_arrive(&sm.empty[g]);
     uint4 xs = make_uint4(0, 0, 0, 0);
-    const uint32_t taddr = tmem + ((uint32_t)(lq * 32) << 16) + (uint32_t)(g * kTmemCols);
+    const uint32_t taddr = trow + kColsAcc;
     for (int i = 2; i <= Tmax; ++i) {
       const float inv = R > 0.f ? 1.f / R : 0.f;
       if (i - 1 <= T) {
@@ -277,10 +292,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
           v[u] = __uint_as_float(r[k0 + u]) * (ev[u] * inv);
           tot += v[u];
         }
-        if (i <= T) store16(k0, v);
+        if (i > T) {  // a finished row keeps its operand (.sync.aligned stores: warp-uniform calls)
+#pragma unroll
+          for (int u = 0; u < 16; ++u) v[u] = 0.f;
+        }
+        store16(k0, v);
       }
       if (i <= T) R = tot;
-      asm volatile("fence.proxy.async.shared::cta;");
+      asm volatile("tcgen05.wait::st.sync.aligned;");
       asm volatile("tcgen05.fence::before_thread_sync;");
       mbar_arrive(&sm.empty[g]);
     }
@@ -291,7 +310,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
   __syncthreads();
   if (warp == 0) {
     asm volatile("tcgen05.fence::after_thread_sync;");
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kNG * kTmemCols));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kNG * kColsGroup));
   }
 }
 
@@ -304,7 +323,7 @@ cudaError_t hmm_forward_tc(const HmmArgs& H, cudaStream_t s, int64_t* launches) 
   // The step is a latency chain (MMA -> epilogue -> MMA); the shared memory a CTA reserves decides
   // how many of a concurrent kernel's CTAs (Viterbi) may share its SM (tc_smem_kb).
   const size_t need = sizeof(TcSmem) + 1024;
-  const size_t smem = std::max(need, (size_t)(H.tc_smem_kb >= 0 ? H.tc_smem_kb : 200) * 1024);
+  const size_t smem = std::max(need, (size_t)(H.tc_smem_kb >= 0 ? H.tc_smem_kb : 0) * 1024);
   cudaError_t e = cudaFuncSetAttribute(k_forward_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   ++*launches;
