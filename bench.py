@@ -12,7 +12,7 @@ config (1, 3, 4, 5) and the §8(f) NEXT workloads, each with its own value,
 step time, roofline, e2e and cpu_baseline.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                  [--config sw|swa|swshort|nuss1|hmm|nuss4|nuss5|diag|phmm] [--only]
+                  [--config sw|swa|swshort|nuss1|hmm|nuss4|nuss5|nussmid|diag|phmm] [--only]
                   [--scaling strong|weak]
 
 Multi-GPU (the paper's `map`, L194–L195, one problem per
@@ -49,7 +49,7 @@ MEASURED_UBENCH = {  # profiles/ubench_r01.jsonl, lane-ops per SM clock on B200 
     "viaddmnmx_s32": 64.0, "viaddmnmx_s16x2": 128.0, "ffma": 128.0, "lds_bytes": 128.0,
 }
 SMS = 148
-ALL_CONFIGS = ["sw", "nuss1", "hmm", "nuss4", "nuss5", "swa", "swshort", "diag", "phmm"]
+ALL_CONFIGS = ["sw", "nuss1", "hmm", "nuss4", "nuss5", "swa", "swshort", "nussmid", "diag", "phmm"]
 # configs in the `configs` block at N > 1: the batched ones (the others are single tables: replicas only)
 SHARDED = {"sw", "hmm", "nuss5", "swa", "swshort", "diag", "phmm"}
 
@@ -240,6 +240,15 @@ def workload(name, rank=0, world=1, scaling="strong"):
                 "workload": ("BASELINE config 1: one 64-nt RNA, Nussinov (h=3, WC+GU), with traceback" if name == "nuss1"
                              else "BASELINE config 4: one 8192-nt RNA, Nussinov grid-wide hyperplane sweep, "
                                   "with traceback")}
+    if name == "nussmid":
+        cat, off = dpgen.mid_rna_batch()
+        lens = np.diff(off)
+        return {"kind": "nuss", "config": name, "n_total": len(lens), "ids": np.arange(len(lens), dtype=np.int64),
+                "a_cat": cat, "a_off": off, "max_la": int(lens.max()),
+                "cells_total": int((lens * (lens - 1) // 2).sum()), "cells_local": int((lens * (lens - 1) // 2).sum()),
+                "inner_local": int((lens * (lens - 1) * (lens - 2) // 6).sum()), "tb_stride": int(lens.max()),
+                "workload": "SURVEY 8(f) NEXT 4: 16 RNAs of length U[482,1024], Nussinov with tracebacks, one "
+                            "thread-block cluster per problem (table in distributed shared memory)"}
     if name == "nuss5":
         nseq = int(os.environ.get("DP_NUSS5_N", 1_000_000))
         cat, off = dpgen.config5_rna_batch(nseq)
@@ -503,6 +512,22 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
 
     fixed = None
     intra = None
+    nocl = None
+    if name == "nussmid":   # NEXT 4 evidence: the same batch on the warp-per-problem batch kernel
+        os.environ["DP_NUSS_NO_CLUSTER"] = "1"
+        try:
+            with make_plans(dp, W)[0] as pb:
+                with torch.cuda.stream(stream):
+                    pb.solve_batch(*dev_in, max_len_a=W["max_la"], out=scores[0], stream=stream)
+                    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    f0.record(stream)
+                    for _ in range(3):
+                        pb.solve_batch(*dev_in, max_len_a=W["max_la"], out=scores[0], stream=stream)
+                    f1.record(stream)
+                torch.cuda.synchronize(dev)
+                nocl = round(f0.elapsed_time(f1) / 3, 4)
+        finally:
+            del os.environ["DP_NUSS_NO_CLUSTER"]
     if W["kind"] == "swshort":   # the hybrid's evidence: the same batch on the intra-task warp kernel
         os.environ["DP_SW_INTRA"] = "1"
         try:
@@ -561,6 +586,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
         "gpu_launches": int(launches),
         "result_sha256": digest,
         **({"alone_ms": {k: round(v, 4) for k, v in alone.items()}} if alone else {}),
+        **({"batch_kernel_ms": nocl, "cluster_kernel_ms": round(phase_ms[0], 4)} if nocl else {}),
         **({"intra_task_ms": intra, "inter_task_ms": round(ms_step, 4)} if intra else {}),
         **({"fixed_schedule_ms": fixed, "conditional_schedule_ms": round(ms_step, 4)} if fixed else {}),
         "e2e": e2e,
@@ -621,7 +647,7 @@ def roofline(W, name, phase_ms, alone, pk):
                     "max-plus); latency-bound: 64 dependent partitions")
             r["bound"] = "latency"
             return r
-        kname = "k_nuss_grid2" if name == "nuss4" else "k_nuss_batch"
+        kname = {"nuss4": "k_nuss_grid2", "nussmid": "k_nuss_cluster"}.get(name, "k_nuss_batch")
         return alu(kname, W["inner_local"], phase_ms[0], peak16,
                    "ubench_r01 VIADDMNMX.S16x2 x 148 SMs x sm_max_mhz (one split evaluation = one max-plus)")
     if W["kind"] == "phmm":
@@ -793,6 +819,15 @@ def oracle_sample(config, W):
         dt8 = dt * ev(8192) / ev(2048)
         return 8192 * 8191 / 2 / dt8, (f"first 2048 nt of config 4 (score + traceback, 1 core) in {dt:.1f} s, "
                                        f"extrapolated by split evaluations to n = 8192 ({dt8:.0f} s)"), 1
+    if config == "nussmid":
+        cat, off = dpgen.mid_rna_batch()
+        k = 3
+        t = time.perf_counter()
+        for q in range(k):
+            oracle.nussinov_traceback(cat[off[q]:off[q + 1]], dpgen.rna_pair_mask(), 3)
+        dt = time.perf_counter() - t
+        lens = np.diff(off)[:k]
+        return int((lens * (lens - 1) // 2).sum()) / dt, f"first {k} problems of the nussmid batch (score + traceback, 1 core)", 1
     if config == "nuss5":
         ids = dpgen.config5_sample_ids(k=2000)
         cat, off = dpgen.config5_rna_batch(ids=ids)
@@ -849,7 +884,7 @@ def run_reference(args, rank, world):
     }
 
 
-DEFAULT_STEPS = {"sw": 60, "swa": 20, "swshort": 30, "hmm": 30, "nuss1": 200, "nuss4": 15, "nuss5": 2, "diag": 25, "phmm": 20}
+DEFAULT_STEPS = {"sw": 60, "swa": 20, "swshort": 30, "nussmid": 20, "hmm": 30, "nuss1": 200, "nuss4": 15, "nuss5": 2, "diag": 25, "phmm": 20}
 
 
 def main():

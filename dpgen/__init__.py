@@ -229,6 +229,15 @@ def config4_rna8192(n: int = 8192) -> np.ndarray:
     return random_seq(rng(5), n, 4)
 
 
+def mid_rna_batch(n_seqs: int = 16, lo: int = 482, hi: int = 1024):
+    """Mid-length Nussinov batch (n between the batch kernel's and the
+    grid kernel's regimes): n_seqs RNAs, lengths i.i.d. uniform integers in [lo, hi], bases
+    i.i.d. uniform over ACGU; seed 20120611+12. Returns (cat, off)."""
+    g = rng(12)
+    lens = g.integers(lo, hi + 1, n_seqs, dtype=np.int64)
+    return pack([random_seq(g, int(l), 4) for l in lens])
+
+
 def config5_lengths(n_seqs: int = 1_000_000, lo: int = 128, hi: int = 512) -> np.ndarray:
     return rng(6).integers(lo, hi + 1, size=n_seqs, dtype=np.int64)
 

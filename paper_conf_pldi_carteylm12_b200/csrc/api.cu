@@ -111,7 +111,7 @@ struct dp_plan {
     bool nuss_rounds = false, diag_generic = false, sw_intra = false;
     int64_t nuss_tiled_min = 32;
     int nuss_tbw = 0, diag_force = -1, host_chunks = 4;
-    bool hmm_simt = false;
+    bool hmm_simt = false, nuss_no_cluster = false;
     int hmm_ns = 0, hmm_tc_smem_kb = -1;
   } env;
 };
@@ -132,6 +132,7 @@ void read_env(dp_plan* p) {
   if (on("DP_NUSS_TBW")) p->env.nuss_tbw = atoi(getenv("DP_NUSS_TBW"));
   if (on("DP_DIAG_FORCE")) p->env.diag_force = atoi(getenv("DP_DIAG_FORCE"));
   p->env.hmm_simt = on("DP_HMM_SIMT");
+  p->env.nuss_no_cluster = on("DP_NUSS_NO_CLUSTER");
   if (on("DP_HMM_NS")) p->env.hmm_ns = atoi(getenv("DP_HMM_NS"));
   if (on("DP_HMM_TC_SMEM_KB")) p->env.hmm_tc_smem_kb = atoi(getenv("DP_HMM_TC_SMEM_KB"));
   if (on("DP_HOST_CHUNKS")) p->env.host_chunks = std::max(1, std::min(dp_plan::kMaxChunks, atoi(getenv("DP_HOST_CHUNKS"))));
@@ -550,6 +551,17 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       // other paths, for comparison)
       if (dpk::nuss_small_supported(A.max_len, n, p->device) && !p->env.nuss_cell && p->env.nuss_tiled_min == 32) {
         e = dpk::nuss_small_solve(A, s, &p->launches);
+        break;
+      }
+      // a few mid-length problems: one thread-block cluster each, the table in distributed shared
+      // memory (DP_NUSS_NO_CLUSTER: the batch / grid kernels, for comparison)
+      if (dpk::nuss_cluster_supported(A.max_len, n, p->device) && !p->env.nuss_cell && !p->env.nuss_no_cluster &&
+          p->env.nuss_tiled_min == 32) {
+        A.scratch_bytes = dpk::nuss_cluster_scratch_bytes(A.max_len, n);
+        e = p->scratch.ensure((size_t)A.scratch_bytes);
+        if (e != cudaSuccess) break;
+        A.scratch = p->scratch.ptr;
+        e = dpk::nuss_cluster_solve(A, s, &p->launches);
         break;
       }
       const bool tiled = A.max_len > p->env.nuss_tiled_min && !p->env.nuss_cell && (n == 1 || A.max_len <= 4096);

@@ -132,6 +132,10 @@ int64_t nuss_scratch_bytes(int64_t max_len, int64_t n, int device);
 bool nuss_tiled_supported(int64_t max_len);
 int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device);
 cudaError_t nuss_tiled_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
+// a few mid-length problems, one thread-block cluster each, tables in distributed shared memory
+bool nuss_cluster_supported(int64_t max_len, int64_t n, int device);
+int64_t nuss_cluster_scratch_bytes(int64_t max_len, int64_t n);
+cudaError_t nuss_cluster_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t nuss_solve(const NussArgs& a, cudaStream_t s, int64_t* launches);
 // one CTA per problem, table + traceback in shared memory (latency regime: max_len <= 128, few problems)
 bool nuss_small_supported(int64_t max_len, int64_t n, int device);

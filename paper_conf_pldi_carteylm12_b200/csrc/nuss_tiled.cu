@@ -280,8 +280,7 @@ __device__ __forceinline__ void trace_interval(const TabT& tab, const uint8_t* x
         const int kq = k0 + lane + 32 * u;
         // gamma(i, kq) along row i from the row-major L record of row i (L(I',K)[k][c] =
         // gamma(32I'+k+1, 32K+c)): 32 consecutive k are 64 contiguous bytes instead of 32 lines
-        const int gik = kq >= j ? 0 : (i >= 1 ? (int)__ldcg(tab.L((i - 1) / T, kq / T) + ((i - 1) % T) * T + kq % T)
-                                              : tab.gamma(i, kq));
+        const int gik = kq >= j ? 0 : (i >= 1 ? tab.lrow(i, kq) : tab.gamma(i, kq));
         s[u] = kq < j ? gik + tab.gamma(kq + 1, j) : -1;
       }
 #pragma unroll
@@ -362,6 +361,11 @@ struct Tab2 {
   __device__ __forceinline__ int gamma(int i, int j) const {
     if (j - i < 1) return 0;
     return g16(i / T, j / T, j % T, i % T);
+  }
+  // gamma(i, k), i >= 1, from the row-major L record of row i - 1 (32 consecutive k are 64
+  // contiguous bytes: the traceback's split search reads rows)
+  __device__ __forceinline__ int lrow(int i, int k) const {
+    return (int)__ldcg(L((i - 1) / T, k / T) + ((i - 1) % T) * T + k % T);
   }
 };
 
@@ -737,6 +741,243 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   }
 }
 
+// ------------------------------------------------------------------ cluster driver
+// k_nuss_cluster: one thread-block cluster of kcl CTAs per problem (mid-length problems, a few
+// per batch: the regime between one warp per problem and the whole grid for one problem). The
+// problem's table lives in the cluster's DISTRIBUTED SHARED MEMORY: tile (I,J) is computed by
+// and stored in CTA J mod kcl (compact records: U16[c][r] = gamma(32I+r, 32J+c), column-major,
+// and L16[k][c] = gamma(32I+k+1, 32J+c), row-major, 2 KB each; diagonal tiles add the phase-B
+// rows ASd / BCd). Tile-diagonals are separated by cluster barriers (barrier.cluster
+// arrive.release / wait.acquire: the records of diagonal D are visible cluster-wide before D+1).
+// Phase A stages U16(I,K) (remote, duplicated into both s16 halves on the way) and L16(K,J)
+// (local: same owner as (I,J)) through registers: the next K's DSMEM loads are in flight during
+// the current micro-kernel. Phase B and the micro-kernel are the batch kernel's.
+constexpr int kClTile = 2 * T * T;   // int16 per tile record: U16 + L16
+constexpr int kClDiag = 2 * T * T;   // int16 per diagonal extra: ASd + BCd
+constexpr int kClMaxCl = 16;
+
+struct ClArgs {
+  int kcl;            // CTAs per cluster
+  int warps;          // warps per CTA
+  int slots, dslots;  // record slots per CTA (tiles, diagonal extras)
+};
+
+__host__ __device__ __forceinline__ int cl_slot(int I, int J, int kcl) {  // tile (I,J) in CTA J mod kcl
+  const int o = J % kcl, m = J / kcl;
+  return m * (o + 1) + kcl * m * (m - 1) / 2 + I;
+}
+inline int cl_slots(int nt, int kcl) {  // most tiles any CTA owns
+  int mx = 0;
+  for (int o = 0; o < kcl; ++o) {
+    int c = 0;
+    for (int J = o; J < nt; J += kcl) c += J + 1;
+    mx = std::max(mx, c);
+  }
+  return mx;
+}
+
+struct ClTab {
+  int16_t* base[kClMaxCl];  // each rank's record area (generic pointers into the cluster's shared memory)
+  int kcl, slots;
+  __device__ __forceinline__ int16_t* U16(int I, int J) const {
+    return base[J % kcl] + (int64_t)cl_slot(I, J, kcl) * kClTile;
+  }
+  __device__ __forceinline__ int16_t* L16(int I, int J) const { return U16(I, J) + T * T; }
+  __device__ __forceinline__ int16_t* ASd(int I) const { return base[I % kcl] + (int64_t)slots * kClTile + (I / kcl) * kClDiag; }
+  __device__ __forceinline__ int16_t* BCd(int I) const { return ASd(I) + T * T; }
+  __device__ __forceinline__ int gamma(int i, int j) const {
+    if (j - i < 1) return 0;
+    return U16(i / T, j / T)[(j % T) * T + (i % T)];
+  }
+  __device__ __forceinline__ int lrow(int i, int k) const { return L16((i - 1) / T, k / T)[((i - 1) % T) * T + k % T]; }
+};
+
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+// Phase A over K in [K0, K1) from DSMEM: acc = max(acc, U(I,K) (x) L(K,J)).
+__device__ __forceinline__ void cl_products(const ClTab& tab, int I, int J, int K0, int K1, uint8_t* stg,
+                                            uint32_t (&acc)[16], int lane) {
+  if (K0 >= K1) return;
+  uint4 ra[4], rb[4];  // U16 (2 KB) and L16 (2 KB) of one K: 4 x 16 B per lane each
+  auto load = [&](int K) {
+    const uint4* u = reinterpret_cast<const uint4*>(tab.U16(I, K));
+    const uint4* l = reinterpret_cast<const uint4*>(tab.L16(K, J));
+#pragma unroll
+    for (int t = 0; t < 4; ++t) { ra[t] = u[lane + 32 * t]; rb[t] = l[lane + 32 * t]; }
+  };
+  load(K0);
+  uint32_t* As = reinterpret_cast<uint32_t*>(stg);
+  uint4* Bs = reinterpret_cast<uint4*>(stg + 4096);
+  for (int K = K0; K < K1; ++K) {
+    __syncwarp();
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {  // U16 word index e = lane + 32 t holds 8 int16: entries 8e .. 8e+7
+      const int e = lane + 32 * t;
+      const uint32_t w[4] = {ra[t].x, ra[t].y, ra[t].z, ra[t].w};
+      uint4* dst = reinterpret_cast<uint4*>(As + 8 * e);
+      dst[0] = make_uint4(dup16(w[0], 0), dup16(w[0], 1), dup16(w[1], 0), dup16(w[1], 1));
+      dst[1] = make_uint4(dup16(w[2], 0), dup16(w[2], 1), dup16(w[3], 0), dup16(w[3], 1));
+      Bs[e] = rb[t];
+    }
+    __syncwarp();
+    if (K + 1 < K1) load(K + 1);
+    micro(As, reinterpret_cast<const uint16_t*>(Bs), acc, lane);
+  }
+}
+
+// Phase B of tile (I,J) from C in registers, then its records (in this CTA's shared memory).
+__device__ void cl_tile_finish(const ClTab& tab, int I, int J, const uint32_t (&acc)[16], int below, int left,
+                               int corner, InTileBuf& B, const uint8_t* x, const uint8_t* pm, int n, int h, int lane) {
+  const bool diag = I == J;
+  const int r = lane;
+  __syncwarp();
+  if (!diag) {  // phase-B rows: AS[r][0..31] = ASd(I)[r][*], BC[r][32..63] = BCd(J)[r][*] (DSMEM)
+    const uint4* asd = reinterpret_cast<const uint4*>(tab.ASd(I) + r * T);
+    const uint4* bcd = reinterpret_cast<const uint4*>(tab.BCd(J) + r * T);
+    uint4* ar = reinterpret_cast<uint4*>(B.as + r * kAS);
+    uint4* br = reinterpret_cast<uint4*>(B.bc + r * kAS + T);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) { ar[q] = asd[q]; br[q] = bcd[q]; }
+  }
+  {
+    const int ty = lane >> 2, tx = lane & 3;
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr)
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        *reinterpret_cast<uint32_t*>(B.cc + (4 * ty + rr) * kCC + 8 * tx + 2 * q) = acc[rr * 4 + q];
+    const uint32_t NEG2 = pk16(kNeg, kNeg);
+    uint4* ar = reinterpret_cast<uint4*>(B.as + r * kAS);
+    uint4* bc = reinterpret_cast<uint4*>(B.bc + r * kAS);
+    const uint4 negs = make_uint4(NEG2, NEG2, NEG2, NEG2), zero = make_uint4(0, 0, 0, 0);
+#pragma unroll
+    for (int q = 4; q < 9; ++q) ar[q] = negs;
+    if (diag) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) { ar[q] = negs; bc[4 + q] = zero; }
+    }
+#pragma unroll
+    for (int q = 0; q < 3; ++q) bc[q] = zero;
+    bc[3] = make_uint4(0, 0, 0, pk16(0, below));
+    bc[8] = zero;
+  }
+  const uint32_t pairbits = pair_bits(x, pm, n, I * T, J * T, h, lane);
+  __syncwarp();
+  wavefront(B, diag, left, corner, pairbits, lane);
+  // records: U16[c][r] (column-major) and L16[k][c] (row-major; row 31 = the row below)
+  {
+    const uint4* xr = reinterpret_cast<const uint4*>(B.as + r * kAS + T);
+    uint4 w[4], raw[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      raw[q] = w[q] = xr[q];
+      if (diag) {
+        w[q].x = __vmaxs2(w[q].x, 0u); w[q].y = __vmaxs2(w[q].y, 0u);
+        w[q].z = __vmaxs2(w[q].z, 0u); w[q].w = __vmaxs2(w[q].w, 0u);
+      }
+    }
+    int16_t* u = tab.U16(I, J);
+    const uint32_t ww[16] = {w[0].x, w[0].y, w[0].z, w[0].w, w[1].x, w[1].y, w[1].z, w[1].w,
+                             w[2].x, w[2].y, w[2].z, w[2].w, w[3].x, w[3].y, w[3].z, w[3].w};
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      u[(2 * q) * T + r] = (int16_t)(ww[q] & 0xffffu);
+      u[(2 * q + 1) * T + r] = (int16_t)(ww[q] >> 16);
+    }
+    int16_t* l = tab.L16(I, J);
+    if (r >= 1) {
+      uint4* lr = reinterpret_cast<uint4*>(l + (r - 1) * T);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) lr[q] = w[q];
+    }
+    l[(T - 1) * T + lane] = B.bc[lane * kAS + (T - 1)];
+    if (diag) {
+      uint4* asd = reinterpret_cast<uint4*>(tab.ASd(I) + r * T);
+      uint4* bcd = reinterpret_cast<uint4*>(tab.BCd(I) + r * T);
+      const uint4* bcr = reinterpret_cast<const uint4*>(B.bc + r * kAS + T);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) { asd[q] = raw[q]; bcd[q] = bcr[q]; }
+    }
+  }
+  __syncwarp();
+}
+
+__global__ void k_nuss_cluster(NussArgs A, ClArgs C) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  cg::cluster_group cluster = cg::this_cluster();
+  const int rank = (int)cluster.block_rank(), kcl = C.kcl;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, W = C.warps;
+  int16_t* rec = reinterpret_cast<int16_t*>(smem);
+  uint8_t* xs = smem + ((int64_t)C.slots * kClTile + (int64_t)C.dslots * kClDiag) * 2;
+  uint8_t* pm = xs + ((A.max_len + 15) & ~int64_t(15));
+  uint8_t* wbuf = pm + 16 + warp * kBatchBuf;
+  int* win = reinterpret_cast<int*>(pm + 16 + W * kBatchBuf);
+  int2* sstk = reinterpret_cast<int2*>(win + 64);
+  if (threadIdx.x < 16) pm[threadIdx.x] = A.pair_mask[threadIdx.x];
+  ClTab tab;
+  tab.kcl = kcl;
+  tab.slots = C.slots;
+  for (int q = 0; q < kcl; ++q) tab.base[q] = cluster.map_shared_rank(rec, q);
+  InTileBuf& IB = *reinterpret_cast<InTileBuf*>(wbuf);
+  const int64_t nclusters = gridDim.x / kcl, cid = blockIdx.x / kcl;
+  int2* gstack = reinterpret_cast<int2*>(A.scratch) + cid * (2 * A.max_len + 8);
+  for (int64_t p = cid; p < A.n; p += nclusters) {
+    const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+    const int nt = (n + T - 1) / T;
+    cluster_sync_all();  // the previous problem's traceback no longer reads any rank's records
+    for (int q = threadIdx.x; q < n; q += blockDim.x) xs[q] = A.x_cat[A.x_off[p] + q];
+    __syncthreads();
+    for (int D = 0; D < nt; ++D) {
+      // this CTA's tiles of diagonal D: J = I + D with J mod kcl == rank, one warp each
+      const int I0 = ((rank - D) % kcl + kcl) % kcl;
+      for (int I = I0 + kcl * warp; I + D < nt; I += kcl * W) {
+        const int J = I + D;
+        const bool diag = D == 0;
+        const int below = diag ? 0 : tab.U16(I + 1, J)[lane * T + 0];           // X[32][c], c = lane
+        const int left = diag ? 0 : tab.U16(I, J - 1)[(T - 1) * T + lane];      // gamma(32I + r, 32J - 1)
+        const int corner = (!diag && I + 1 <= J - 1) ? tab.U16(I + 1, J - 1)[(T - 1) * T] : 0;
+        uint32_t acc[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) acc[q] = 0;
+        cl_products(tab, I, J, I + 1, J, wbuf, acc, lane);
+        cl_tile_finish(tab, I, J, acc, below, left, corner, IB, xs, pm, n, A.hairpin, lane);
+      }
+      cluster_sync_all();  // diagonal D's records visible to every rank
+    }
+    if (rank == 0 && threadIdx.x == 0) {
+      A.scores[p] = n <= 1 ? 0 : tab.gamma(0, n - 1);
+      if (A.db) A.db_len[p] = n;
+    }
+    if (A.db && rank == 0 && warp == 0)
+      warp_traceback_win<NUSS_TBW_B, NUSS_TBK_B>(tab, xs, pm, n, A.hairpin, A.db + p * A.db_stride, gstack, win, sstk,
+                                                 lane);
+  }
+  cluster_sync_all();  // no rank exits while rank 0 may still read its records
+}
+
+size_t cl_smem_bytes(int64_t max_len, int slots, int dslots, int warps) {
+  return ((size_t)slots * kClTile + (size_t)dslots * kClDiag) * 2 + ((max_len + 15) & ~int64_t(15)) + 16 +
+         (size_t)warps * kBatchBuf + 256 + 8 * kStk;
+}
+
+// the cluster configuration for problems of max_len: the smallest kcl whose per-CTA records and
+// at least two warps' buffers fit; 0 if none
+ClArgs cl_config(int64_t max_len, int smem_optin) {
+  ClArgs c{};
+  const int nt = (int)((max_len + T - 1) / T);
+  for (int kcl : {2, 4, 8, 16}) {
+    const int slots = cl_slots(nt, kcl), dslots = (nt + kcl - 1) / kcl;
+    for (int w = 4; w >= 2; --w)
+      if (cl_smem_bytes(max_len, slots, dslots, w) <= (size_t)smem_optin) {
+        c.kcl = kcl; c.warps = w; c.slots = slots; c.dslots = dslots;
+        return c;
+      }
+  }
+  return c;
+}
+
 int num_sms_t(int device) {
   int v = 0;
   cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device);
@@ -796,6 +1037,48 @@ __global__ void k_len_scatter(const int64_t* off, int64_t n, int* hist, int* per
 }
 
 }  // namespace
+
+// NEXT 4: a few mid-length problems, one cluster each (see k_nuss_cluster)
+bool nuss_cluster_supported(int64_t max_len, int64_t n, int device) {
+  if (max_len <= 128 || max_len > 1024 || n > 64) return false;
+  int optin = 0;
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+  return cl_config(max_len, optin).kcl > 0;
+}
+
+int64_t nuss_cluster_scratch_bytes(int64_t max_len, int64_t n) { return n * (2 * max_len + 8) * 8 + 256; }
+
+cudaError_t nuss_cluster_solve(const NussArgs& A, cudaStream_t s, int64_t* launches) {
+  if (A.n == 0) return cudaSuccess;
+  int dev = 0, optin = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  const ClArgs C = cl_config(A.max_len, optin);
+  if (C.kcl == 0) return cudaErrorInvalidValue;
+  const size_t smem = cl_smem_bytes(A.max_len, C.slots, C.dslots, C.warps);
+  cudaError_t e = cudaFuncSetAttribute(k_nuss_cluster, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess && C.kcl > 8) e = cudaFuncSetAttribute(k_nuss_cluster, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = C.kcl;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.blockDim = dim3(32 * C.warps, 1, 1);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cfg.gridDim = dim3(C.kcl, 1, 1);
+  int clusters = 0;
+  e = cudaOccupancyMaxActiveClusters(&clusters, k_nuss_cluster, &cfg);
+  if (e != cudaSuccess) return e;
+  if (clusters < 1) return cudaErrorInvalidConfiguration;
+  cfg.gridDim = dim3((unsigned)(std::min<int64_t>(A.n, clusters) * C.kcl), 1, 1);
+  ++*launches;
+  return cudaLaunchKernelEx(&cfg, k_nuss_cluster, A, C);
+}
 
 bool nuss_tiled_supported(int64_t max_len) { return max_len <= 65536; }
 

@@ -366,6 +366,26 @@ def test_nussinov_small_kernel_edges(dp, orc, h):
     assert (r1["scores"][0], r1["db"][0]) == orc.nussinov_traceback(seqs[-4], pm, h)
 
 
+@pytest.mark.parametrize("lens", [[129, 160, 300, 512, 33, 0, 1], [513, 700, 1000, 1024, 640]])
+def test_nussinov_cluster_path(dp, orc, lens, monkeypatch):
+    """a few mid-length problems, one thread-block cluster each with the
+    table in distributed shared memory (tile-diagonals separated by cluster barriers); lengths
+    around tile multiples, the cluster sizes' capacity edges (512 / 1024), empty and 1-nt
+    problems in the same batch. Bit-exact scores and canonical dot-brackets against the oracle
+    and against the batch kernel (DP_NUSS_NO_CLUSTER=1) on the same batch."""
+    g = np.random.default_rng(180 + len(lens))
+    seqs = [g.integers(0, 4, size=l).astype(np.uint8) for l in lens]
+    r = run_nuss(dp, seqs)
+    pm = dpgen.rna_pair_mask()
+    with concurrent.futures.ThreadPoolExecutor(THREADS) as ex:
+        want = list(ex.map(lambda x: orc.nussinov_traceback(x, pm, 3), seqs))
+    for q, x in enumerate(seqs):
+        assert (r["scores"][q], r["db"][q]) == want[q], (q, len(x))
+    monkeypatch.setenv("DP_NUSS_NO_CLUSTER", "1")
+    r2 = run_nuss(dp, seqs)
+    assert list(r2["scores"]) == list(r["scores"]) and r2["db"] == r["db"]
+
+
 def test_nussinov_cell_level_path(dp, orc, monkeypatch):
     """The cell-level CTA kernels (shared-memory table; L2 table above 340) on the same cases."""
     monkeypatch.setenv("DP_NUSS_CELL", "1")
