@@ -9,7 +9,7 @@ nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > gp
 timeout 1500 python -m pytest tests -m gpu -q -rA 2>&1 | grep -vE "^PASSED" | tail -60 > gpurun_out/gpu_tests.log
 timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err
 timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_ref.json 2>/dev/null
-for c in sw hmm nuss1 nuss4 swa diag phmm; do
+for c in sw hmm nuss1 nuss4 swa swshort nussmid diag phmm; do
   timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv --log-file gpurun_out/launches_$c.csv \
     python bench.py --config $c --only --steps 2 --warmup 1 --no-cpu > /dev/null 2>&1
 done
@@ -26,6 +26,8 @@ full nuss1 "k_nuss" 1
 full nuss4 "k_nuss" 1
 full nuss5 "k_nuss_batch" 1 DP_NUSS5_N=50000
 full swa "k_align_affine" 2
+full swshort "k_sw_inter" 2
+full nussmid "k_nuss_cluster" 1
 full diag "k_diag" 1
 full phmm "k_phmm" 1
 python scripts/ncu_traffic.py gpurun_out/traffic.json \
@@ -33,9 +35,11 @@ python scripts/ncu_traffic.py gpurun_out/traffic.json \
   k_forward_tc=gpurun_out/ncu_hmm.ncu-rep k_viterbi=gpurun_out/ncu_hmm.ncu-rep \
   k_nuss_batch=gpurun_out/ncu_nuss5.ncu-rep:20:"50k-problem capture of config 5 x 20" \
   k_nuss_grid2=gpurun_out/ncu_nuss4.ncu-rep k_align_affine=gpurun_out/ncu_swa.ncu-rep \
-  k_diag=gpurun_out/ncu_diag.ncu-rep k_phmm_forward=gpurun_out/ncu_phmm.ncu-rep > gpurun_out/traffic.log 2>&1
+  k_diag=gpurun_out/ncu_diag.ncu-rep k_phmm_forward=gpurun_out/ncu_phmm.ncu-rep \
+  k_sw_inter=gpurun_out/ncu_swshort.ncu-rep k_sw_inter_tb=gpurun_out/ncu_swshort.ncu-rep \
+  k_nuss_small=gpurun_out/ncu_nuss1.ncu-rep k_nuss_cluster=gpurun_out/ncu_nussmid.ncu-rep > gpurun_out/traffic.log 2>&1
 for t in memcheck racecheck synccheck; do
-  for w in align nuss hmm; do
+  for w in align inter nuss hmm; do
     timeout 900 compute-sanitizer --tool $t --print-limit 20 python scripts/sanitize_small.py $w > gpurun_out/san/${t}_$w.log 2>&1
   done
 done

@@ -28,8 +28,9 @@ def main(which):
         for kind, kw in ((dp.SW_LINEAR, dict(gap=4)), (dp.SW_AFFINE, dict(gap_open=11, gap_extend=1)),
                          (dp.EDIT, dict(alphabet_size=24))):
             with dp.Plan(kind, la, lb, sigma=None if kind == dp.EDIT else sig, want_traceback=True, **kw) as p:
-                p.solve_batch(cu(ac), cu(ao), cu(bc), cu(bo), max_len_a=la, max_len_b=lb)
-                p.traceback(0, len(a), la + lb + 1)
+                sc = p.solve_batch(cu(ac), cu(ao), cu(bc), cu(bo), max_len_a=la, max_len_b=lb)  # kept: the
+                p.traceback(0, len(a), la + lb + 1)                                           # traceback reads it
+                del sc
         with dp.Plan(dp.DIAG_LCS, la, lb, alphabet_size=4) as p:
             a4 = [x % 4 for x in a]
             b4 = [x % 4 for x in b]
@@ -40,9 +41,19 @@ def main(which):
         b = [g.integers(0, 20, int(l)).astype(np.uint8) for l in g.integers(0, 65, 300)]
         (ac, ao), (bc, bo) = dpgen.pack(a), dpgen.pack(b)
         with dp.Plan(dp.SW_LINEAR, 64, 64, sigma=sig, gap=4, want_traceback=True) as p:
-            p.solve_batch(cu(ac), cu(ao), cu(bc), cu(bo), max_len_a=64, max_len_b=64)
+            sc = p.solve_batch(cu(ac), cu(ao), cu(bc), cu(bo), max_len_a=64, max_len_b=64)
             p.traceback(0, len(a), 129)
+            del sc
     if which in ("all", "nuss"):
+        for lens in ((1, 20, 64, 100, 128),                        # k_nuss_small (a few problems <= 128 nt)
+                     tuple(int(l) for l in g.integers(0, 200, 70))):  # k_nuss_batch (more than 64 problems)
+            seqs = [g.integers(0, 4, int(l)).astype(np.uint8) for l in lens]
+            c, o = dpgen.pack(seqs)
+            ml = max(lens)
+            with dp.Plan(dp.NUSSINOV, ml, pair_mask=dpgen.rna_pair_mask(), min_hairpin=3, want_traceback=True) as p:
+                p.solve_batch(cu(c), cu(o), max_len_a=ml)
+                p.traceback(0, len(seqs), ml, coords=False)
+        # k_nuss_cluster (a few problems of 129..1024 nt)
         seqs = [g.integers(0, 4, int(l)).astype(np.uint8) for l in (1, 20, 33, 64, 100, 130, 200)]
         c, o = dpgen.pack(seqs)
         with dp.Plan(dp.NUSSINOV, 200, pair_mask=dpgen.rna_pair_mask(), min_hairpin=3, want_traceback=True) as p:
