@@ -561,7 +561,29 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         e = p->scratch.ensure((size_t)A.scratch_bytes);
         if (e != cudaSuccess) break;
         A.scratch = p->scratch.ptr;
+        unsigned long long* rounds = nullptr;
+        if (p->env.nuss_rounds) cudaMalloc(&rounds, 8 * 4096), cudaMemset(rounds, 0, 8 * 4096), A.round_ns = rounds;
+        unsigned long long* dbg = nullptr;
+        if (p->env.nuss_timing) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
         e = dpk::nuss_cluster_solve(A, s, &p->launches);
+        if (dbg) {  // diagnostic: cluster-kernel phase cycles summed over warps (stderr)
+          unsigned long long h[8];
+          cudaStreamSynchronize(s);
+          cudaMemcpy(h, dbg, sizeof(h), cudaMemcpyDeviceToHost);
+          fprintf(stderr, "cluster: staging %llu micro %llu setupB %llu wavefront %llu records %llu | tiles %llu ksteps %llu\n",
+                  h[0], h[1], h[2], h[3], h[4], h[5], h[6]);
+          cudaFree(dbg);
+        }
+        if (rounds) {  // diagnostic: per tile-diagonal [products, finish] durations of cluster 0 (stderr)
+          static unsigned long long h[4096];
+          cudaStreamSynchronize(s);
+          cudaMemcpy(h, rounds, sizeof(h), cudaMemcpyDeviceToHost);
+          const int nt = (int)((A.max_len + 31) / 32);
+          for (int d = 0; d + 1 < nt; ++d)
+            fprintf(stderr, "cluster round %d %.1f us (split-K products %.1f us)\n", d, (h[2 * d + 2] - h[2 * d]) * 1e-3,
+                    h[2 * d + 1] ? (h[2 * d + 1] - h[2 * d]) * 1e-3 : 0.0);
+          cudaFree(rounds);
+        }
         break;
       }
       const bool tiled = A.max_len > p->env.nuss_tiled_min && !p->env.nuss_cell && (n == 1 || A.max_len <= 4096);

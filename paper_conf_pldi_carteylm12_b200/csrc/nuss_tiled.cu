@@ -751,7 +751,9 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
 // arrive.release / wait.acquire: the records of diagonal D are visible cluster-wide before D+1).
 // Phase A stages U16(I,K) (remote, duplicated into both s16 halves on the way) and L16(K,J)
 // (local: same owner as (I,J)) through registers: the next K's DSMEM loads are in flight during
-// the current micro-kernel. Phase B and the micro-kernel are the batch kernel's.
+// the current micro-kernel. Phase B and the micro-kernel are the batch kernel's. A diagonal with
+// at most half as many tiles as the cluster has warps splits each tile's K range over the whole
+// cluster (partials merged by the tile's owner warp through DSMEM; one more cluster barrier).
 constexpr int kClTile = 2 * T * T;   // int16 per tile record: U16 + L16
 constexpr int kClDiag = 2 * T * T;   // int16 per diagonal extra: ASd + BCd
 constexpr int kClMaxCl = 16;
@@ -798,8 +800,9 @@ __device__ __forceinline__ void cluster_sync_all() {
 
 // Phase A over K in [K0, K1) from DSMEM: acc = max(acc, U(I,K) (x) L(K,J)).
 __device__ __forceinline__ void cl_products(const ClTab& tab, int I, int J, int K0, int K1, uint8_t* stg,
-                                            uint32_t (&acc)[16], int lane) {
+                                            uint32_t (&acc)[16], int lane, PhaseClock& clk) {
   if (K0 >= K1) return;
+  clk.lap(7);
   uint4 ra[4], rb[4];  // U16 (2 KB) and L16 (2 KB) of one K: 4 x 16 B per lane each
   auto load = [&](int K) {
     const uint4* u = reinterpret_cast<const uint4*>(tab.U16(I, K));
@@ -822,17 +825,22 @@ __device__ __forceinline__ void cl_products(const ClTab& tab, int I, int J, int 
       Bs[e] = rb[t];
     }
     __syncwarp();
+    clk.lap(0);  // staging (waits for this K's DSMEM loads)
     if (K + 1 < K1) load(K + 1);
     micro(As, reinterpret_cast<const uint16_t*>(Bs), acc, lane);
+    clk.lap(1);  // micro-kernel
+    clk.count(6);
   }
 }
 
 // Phase B of tile (I,J) from C in registers, then its records (in this CTA's shared memory).
 __device__ void cl_tile_finish(const ClTab& tab, int I, int J, const uint32_t (&acc)[16], int below, int left,
-                               int corner, InTileBuf& B, const uint8_t* x, const uint8_t* pm, int n, int h, int lane) {
+                               int corner, InTileBuf& B, const uint8_t* x, const uint8_t* pm, int n, int h, int lane,
+                               PhaseClock& clk) {
   const bool diag = I == J;
   const int r = lane;
   __syncwarp();
+  clk.lap(7);
   if (!diag) {  // phase-B rows: AS[r][0..31] = ASd(I)[r][*], BC[r][32..63] = BCd(J)[r][*] (DSMEM)
     const uint4* asd = reinterpret_cast<const uint4*>(tab.ASd(I) + r * T);
     const uint4* bcd = reinterpret_cast<const uint4*>(tab.BCd(J) + r * T);
@@ -865,7 +873,9 @@ __device__ void cl_tile_finish(const ClTab& tab, int I, int J, const uint32_t (&
   }
   const uint32_t pairbits = pair_bits(x, pm, n, I * T, J * T, h, lane);
   __syncwarp();
+  clk.lap(2);  // phase-B setup (DSMEM rows, C, pair bits)
   wavefront(B, diag, left, corner, pairbits, lane);
+  clk.lap(3);  // wavefront
   // records: U16[c][r] (column-major) and L16[k][c] (row-major; row 31 = the row below)
   {
     const uint4* xr = reinterpret_cast<const uint4*>(B.as + r * kAS + T);
@@ -902,6 +912,8 @@ __device__ void cl_tile_finish(const ClTab& tab, int I, int J, const uint32_t (&
     }
   }
   __syncwarp();
+  clk.lap(4);  // records
+  clk.count(5);
 }
 
 __global__ void k_nuss_cluster(NussArgs A, ClArgs C) {
@@ -921,6 +933,9 @@ __global__ void k_nuss_cluster(NussArgs A, ClArgs C) {
   tab.slots = C.slots;
   for (int q = 0; q < kcl; ++q) tab.base[q] = cluster.map_shared_rank(rec, q);
   InTileBuf& IB = *reinterpret_cast<InTileBuf*>(wbuf);
+  PhaseClock clk;  // DP_NUSS_TIMING (diagnostic): 0 staging, 1 micro, 2 phase-B setup, 3 wavefront,
+  clk.dbg = A.dbg; // 4 records, 5 tiles, 6 K-steps
+  clk.start();
   const int64_t nclusters = gridDim.x / kcl, cid = blockIdx.x / kcl;
   int2* gstack = reinterpret_cast<int2*>(A.scratch) + cid * (2 * A.max_len + 8);
   for (int64_t p = cid; p < A.n; p += nclusters) {
@@ -930,19 +945,82 @@ __global__ void k_nuss_cluster(NussArgs A, ClArgs C) {
     for (int q = threadIdx.x; q < n; q += blockDim.x) xs[q] = A.x_cat[A.x_off[p] + q];
     __syncthreads();
     for (int D = 0; D < nt; ++D) {
+      if (A.round_ns && cid == 0 && rank == 0 && threadIdx.x == 0) {  // DP_NUSS_ROUNDS (diagnostic)
+        unsigned long long tm;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tm));
+        A.round_ns[2 * D] = tm;
+      }
       // this CTA's tiles of diagonal D: J = I + D with J mod kcl == rank, one warp each
       const int I0 = ((rank - D) % kcl + kcl) % kcl;
-      for (int I = I0 + kcl * warp; I + D < nt; I += kcl * W) {
-        const int J = I + D;
-        const bool diag = D == 0;
-        const int below = diag ? 0 : tab.U16(I + 1, J)[lane * T + 0];           // X[32][c], c = lane
-        const int left = diag ? 0 : tab.U16(I, J - 1)[(T - 1) * T + lane];      // gamma(32I + r, 32J - 1)
-        const int corner = (!diag && I + 1 <= J - 1) ? tab.U16(I + 1, J - 1)[(T - 1) * T] : 0;
+      const int TD = nt - D, NW = kcl * W;
+      if (TD * 2 > NW) {
+        // many tiles: each tile on one warp of its owner CTA (at most W per owner)
+        for (int I = I0 + kcl * warp; I < TD; I += kcl * W) {
+          const int J = I + D;
+          const bool diag = D == 0;
+          const int below = diag ? 0 : tab.U16(I + 1, J)[lane * T + 0];           // X[32][c], c = lane
+          const int left = diag ? 0 : tab.U16(I, J - 1)[(T - 1) * T + lane];      // gamma(32I + r, 32J - 1)
+          const int corner = (!diag && I + 1 <= J - 1) ? tab.U16(I + 1, J - 1)[(T - 1) * T] : 0;
+          uint32_t acc[16];
+#pragma unroll
+          for (int q = 0; q < 16; ++q) acc[q] = 0;
+          cl_products(tab, I, J, I + 1, J, wbuf, acc, lane, clk);
+          cl_tile_finish(tab, I, J, acc, below, left, corner, IB, xs, pm, n, A.hairpin, lane, clk);
+        }
+      } else {
+        // few tiles: split-K over the whole cluster. Tile t's leader is warp t / kcl of its owner
+        // CTA (part 0 of its K range); the other warps are helpers, helper h taking part
+        // 1 + h / TD of tile h mod TD. Partial products stay in the computing warp's buffer; after
+        // a cluster barrier each leader merges its helpers' partials through DSMEM and finishes the
+        // tile (a leader's buffer only ever holds its own tile's part: no leader reads another's).
+        int H = 0, h = -1;  // helpers in total, this warp's helper index
+        for (int r2 = 0; r2 < kcl; ++r2) {
+          const int i0 = ((r2 - D) % kcl + kcl) % kcl;
+          const int lead = i0 < TD ? (TD - i0 + kcl - 1) / kcl : 0;  // leaders in CTA r2 (<= W / 2)
+          if (r2 == rank && warp >= lead) h = H + (warp - lead);
+          H += W - lead;
+        }
+        const bool leader = h < 0;
+        const int t = leader ? I0 + kcl * warp : h % TD;  // my tile
+        const int part = leader ? 0 : 1 + h / TD;
+        const int parts = 1 + (H > t ? (H - 1 - t) / TD + 1 : 0);
+        const int I = t, J = t + D, nk = J - I - 1;
         uint32_t acc[16];
 #pragma unroll
         for (int q = 0; q < 16; ++q) acc[q] = 0;
-        cl_products(tab, I, J, I + 1, J, wbuf, acc, lane);
-        cl_tile_finish(tab, I, J, acc, below, left, corner, IB, xs, pm, n, A.hairpin, lane);
+        cl_products(tab, I, J, I + 1 + nk * part / parts, I + 1 + nk * (part + 1) / parts, wbuf, acc, lane, clk);
+        __syncwarp();
+        uint32_t* pw = reinterpret_cast<uint32_t*>(wbuf);  // the partial: word q * 32 + lane
+        if (!leader) {
+#pragma unroll
+          for (int q = 0; q < 16; ++q) pw[q * 32 + lane] = acc[q];
+        }
+        cluster_sync_all();  // every partial of the diagonal written
+        if (A.round_ns && cid == 0 && rank == 0 && threadIdx.x == 0) {
+          unsigned long long tm;
+          asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tm));
+          A.round_ns[2 * D + 1] = tm;
+        }
+        if (leader) {
+          for (int pp = 1; pp < parts; ++pp) {
+            const int hh = t + TD * (pp - 1);  // helper index of part pp
+            int rq = 0, wq = 0, acc_h = 0;     // its CTA and warp
+            for (int r2 = 0; r2 < kcl; ++r2) {
+              const int i0 = ((r2 - D) % kcl + kcl) % kcl;
+              const int lead = i0 < TD ? (TD - i0 + kcl - 1) / kcl : 0;
+              if (hh < acc_h + (W - lead)) { rq = r2; wq = lead + (hh - acc_h); break; }
+              acc_h += W - lead;
+            }
+            const uint32_t* rp = cluster.map_shared_rank(reinterpret_cast<uint32_t*>(pm + 16 + wq * kBatchBuf), rq);
+#pragma unroll
+            for (int q = 0; q < 16; ++q) acc[q] = __vmaxs2(acc[q], rp[q * 32 + lane]);
+          }
+          const bool diag = D == 0;
+          const int below = diag ? 0 : tab.U16(I + 1, J)[lane * T + 0];
+          const int left = diag ? 0 : tab.U16(I, J - 1)[(T - 1) * T + lane];
+          const int corner = (!diag && I + 1 <= J - 1) ? tab.U16(I + 1, J - 1)[(T - 1) * T] : 0;
+          cl_tile_finish(tab, I, J, acc, below, left, corner, IB, xs, pm, n, A.hairpin, lane, clk);
+        }
       }
       cluster_sync_all();  // diagonal D's records visible to every rank
     }
