@@ -73,15 +73,6 @@ def blosum62() -> np.ndarray:
     return m
 
 
-def edit_sigma(asz: int = 26) -> np.ndarray:
-    """Unit-cost table for the edit-distance mode, stated as a scoring input
-    (0 on the diagonal, -1 elsewhere). Only the GPU's max-plus alignment kernel
-    consumes it; the oracle evaluates Fig.7's comparison s[i-1]==t[j-1] itself."""
-    m = -np.ones((asz, asz), dtype=np.int8)
-    np.fill_diagonal(m, 0)
-    return m
-
-
 def rna_pair_mask(gu: bool = True) -> np.ndarray:
     """4x4 uint8 mask over ACGU: 1 where the two bases may pair (WC + optional GU wobble)."""
     m = np.zeros((4, 4), dtype=np.uint8)
