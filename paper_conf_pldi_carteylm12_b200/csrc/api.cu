@@ -594,7 +594,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       A.scratch = p->scratch.ptr;
       unsigned long long* rounds = nullptr;
       A.tbw = p->env.nuss_tbw;
-      if (p->env.nuss_rounds && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), A.round_ns = rounds;
+      if (p->env.nuss_rounds && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), cudaMemset(rounds, 0, 8 * 8192), A.round_ns = rounds;
       unsigned long long* dbg = nullptr;
       if (p->env.nuss_timing && tiled) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
       e = tiled ? dpk::nuss_tiled_solve(A, s, &p->launches) : dpk::nuss_solve(A, s, &p->launches);
@@ -616,6 +616,8 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         for (int d = 0; d + 1 < nt; ++d) fprintf(stderr, "round %d %.1f us\n", d, (h[d + 1] - h[d]) * 1e-3);
         fprintf(stderr, "last round + score %.1f us\n", (h[nt] - h[nt - 1]) * 1e-3);
         if (h[nt + 1] > h[nt]) fprintf(stderr, "traceback %.1f us\n", (h[nt + 1] - h[nt]) * 1e-3);
+        fprintf(stderr, "traceback warps: max %llu cycles, sum %llu cycles, %llu intervals, %llu steps\n", h[nt + 2],
+                h[nt + 3], h[nt + 4], h[nt + 5]);
         cudaFree(rounds);
       }
       break;

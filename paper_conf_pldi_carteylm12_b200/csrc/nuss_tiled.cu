@@ -331,6 +331,10 @@ struct GridQueue {
   int cap;
 };
 __host__ __device__ __forceinline__ int grid_queue_cap(int64_t max_len) { return (int)max_len + 8192; }
+// head, tail and outstanding count each on a 128-byte line of their own: the idle warps poll the
+// count while the working warps push (tail, count) and pop (head)
+constexpr int kQH = 32;             // ints per header line
+constexpr int kQHdr = 3 * kQH;      // header ints before the flags
 
 // ------------------------------------------------------------------ batch driver (one warp per problem)
 // k_nuss_batch: every warp owns one problem at a time (no CTA barriers; 1-warp CTAs, as many
@@ -577,8 +581,11 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   __syncthreads();
   uint8_t* stg = smem + warp * kBatchBuf;
   InTileBuf& IB = *reinterpret_cast<InTileBuf*>(stg);
-  const uint8_t* x = A.x_cat + A.x_off[p];
   const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
+  // the sequence in shared memory (the pair tests of phase B and of the traceback's steps)
+  uint8_t* x = smem + kGridWarps * kBatchBuf;
+  for (int q = threadIdx.x; q < n; q += blockDim.x) x[q] = A.x_cat[A.x_off[p] + q];
+  __syncthreads();
   const int nt = (n + T - 1) / T;
   Tab2 tab;
   tab.base = reinterpret_cast<uint32_t*>(A.scratch);
@@ -587,12 +594,12 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   GridQueue Q;
   Q.hdr = Cg + 2 * (int64_t)nt * T * T;
   Q.cap = grid_queue_cap(A.max_len);
-  Q.flag = Q.hdr + 4;
+  Q.flag = Q.hdr + kQHdr;
   Q.item = reinterpret_cast<int2*>(Q.flag + Q.cap + (Q.cap & 1));
   PhaseClock clk;
   clk.dbg = A.dbg;  // DP_NUSS_TIMING: phase-B warps' per-tile phases (diagnostic)
   const int ty = lane >> 2, tx = lane & 3;
-  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T + 4 + Q.cap;
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < 2 * (int64_t)nt * T * T + kQHdr + Q.cap;
        q += (int64_t)gridDim.x * blockDim.x)
     Cg[q] = 0;  // C buffers, queue counters and flags
   grid.sync();
@@ -685,17 +692,19 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   if (gtid == 0 && n > 1) {
     Q.item[0] = make_int2(0, n - 1);
     Q.flag[0] = 1;
-    Q.hdr[1] = 1;  // tail
-    Q.hdr[2] = 1;  // outstanding
+    Q.hdr[kQH] = 1;      // tail
+    Q.hdr[2 * kQH] = 1;  // outstanding
   }
   grid.sync();
   const unsigned full = 0xffffffffu;
   int* win = reinterpret_cast<int*>(stg);
   int guard = 4 * n + 8;
+  long long tb_cyc = 0;  // DP_NUSS_ROUNDS: cycles this warp spends tracing, intervals traced
+  int tb_iv = 0;
   auto push = [&](int a, int b) {
     if (lane == 0) {
-      atomicAdd(&Q.hdr[2], 1);
-      const int t = atomicAdd(&Q.hdr[1], 1);
+      atomicAdd(&Q.hdr[2 * kQH], 1);
+      const int t = atomicAdd(&Q.hdr[kQH], 1);
       if (t < Q.cap) {
         Q.item[t] = make_int2(a, b);
         __threadfence();
@@ -709,29 +718,40 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
     if (lane == 0) idx = atomicAdd(&Q.hdr[0], 1);
     idx = __shfl_sync(full, idx, 0);
     int got = 0;
+    unsigned backoff = 64;  // polling back-off (ns), so idle warps do not crowd the queue's lines
     for (;;) {
       int f = 0, o = 0;
       if (lane == 0) {
         f = idx < Q.cap ? *reinterpret_cast<volatile int*>(&Q.flag[idx]) : 0;
-        o = *reinterpret_cast<volatile int*>(&Q.hdr[2]);
+        o = *reinterpret_cast<volatile int*>(&Q.hdr[2 * kQH]);
       }
       f = __shfl_sync(full, f, 0);
       o = __shfl_sync(full, o, 0);
       if (f) { got = 1; break; }
       if (o <= 0) break;
-      __nanosleep(128);
+      __nanosleep(backoff);
+      backoff = min(2 * backoff, 2048u);
     }
     if (!got) break;
     __threadfence();
     const int2 iv = __ldcg(&Q.item[idx]);
+    const long long c0 = clock64();
     trace_interval<NUSS_TBW_G, NUSS_TBK_G>(tab, x, pm, n, A.hairpin, db, iv.x, iv.y, win, guard, push, lane);
     __syncwarp();
+    tb_cyc += clock64() - c0;
+    ++tb_iv;
     if (lane == 0) {
       __threadfence();
-      atomicSub(&Q.hdr[2], 1);
+      atomicSub(&Q.hdr[2 * kQH], 1);
     }
   }
   if (A.round_ns) {
+    if (lane == 0) {  // [nt + 2]: max cycles of one warp, [nt + 3]: sum, [nt + 4]: intervals, [nt + 5]: steps
+      atomicMax(A.round_ns + nt + 2, (unsigned long long)tb_cyc);
+      atomicAdd(A.round_ns + nt + 3, (unsigned long long)tb_cyc);
+      atomicAdd(A.round_ns + nt + 4, (unsigned long long)tb_iv);
+      atomicAdd(A.round_ns + nt + 5, (unsigned long long)(4 * n + 8 - guard));
+    }
     grid.sync();
     if (gtid == 0) {
       unsigned long long t;
@@ -1164,7 +1184,7 @@ int64_t nuss_tiled_scratch_bytes(int64_t max_len, int64_t n, int device) {
   const int nt = (int)((max_len + T - 1) / T);
   if (n == 1 && max_len > kGridMin)
     return (tiles_of(nt) * kRecW + (int64_t)nt * kDiagW + 2 * (int64_t)nt * T * T) * 4 +
-           (4 + 3 * (int64_t)grid_queue_cap(max_len) + 2) * 4 + 256;
+           (kQHdr + 3 * (int64_t)grid_queue_cap(max_len) + 2) * 4 + 256;
   const int64_t grid = std::min<int64_t>(n, (int64_t)batch_ctas_per_sm(max_len) * num_sms_t(device));
   // + the work queue: counter, length histogram, permutation
   return grid * batch_slot_words(max_len) * 4 + 256 + 16 + (max_len + 1) * 4 + n * 4 + 256;
@@ -1176,7 +1196,7 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
   cudaGetDevice(&dev);
   const int sms = num_sms_t(dev);
   if (A.n == 1 && A.max_len > kGridMin) {
-    const size_t smem = kGridWarps * kBatchBuf;
+    const size_t smem = kGridWarps * kBatchBuf + ((A.max_len + 15) & ~int64_t(15));
     cudaError_t e = cudaFuncSetAttribute(k_nuss_grid2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int per_sm = 0;
@@ -1212,3 +1232,4 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
 }
 
 }  // namespace dpk
+
