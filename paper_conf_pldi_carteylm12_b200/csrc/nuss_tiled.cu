@@ -115,20 +115,21 @@ __device__ __forceinline__ bool pairable(const uint8_t* x, const uint8_t* pm, in
   return i < n && j < n && pm[x[i] * 4 + x[j]] && j - i - 1 >= h;
 }
 
-// Bit c of lane r: (i0 + r, j0 + c) may pair (pair set and hairpin). One coalesced load
-// per lane; the column bases are shuffled across the warp.
+// Bit c of lane r: (i0 + r, j0 + c) may pair (pair set and hairpin). Four ballots give, per base,
+// the columns holding it; lane r ORs the masks of the bases its own base pairs with, then clears
+// the columns closer than the hairpin (about 15 instructions instead of 32 shuffles and lookups).
 __device__ __forceinline__ uint32_t pair_bits(const uint8_t* x, const uint8_t* pm, int n, int i0, int j0, int h,
                                               int lane) {
-  const int i = i0 + lane;
-  const int xi = i < n ? x[i] : 0;
-  const int xjl = (j0 + lane < n) ? x[j0 + lane] : 0;
-  uint32_t bits = 0;
-#pragma unroll
-  for (int c = 0; c < T; ++c) {
-    const int xj = __shfl_sync(0xffffffffu, xjl, c);
-    const int j = j0 + c;
-    bits |= (uint32_t)(i < n && j < n && j - i - 1 >= h && pm[xi * 4 + xj]) << c;
-  }
+  const unsigned full = 0xffffffffu;
+  const int i = i0 + lane, jl = j0 + lane;
+  const int xj = jl < n ? x[jl] : 4;  // 4: no base (past the end)
+  const uint32_t m0 = __ballot_sync(full, xj == 0), m1 = __ballot_sync(full, xj == 1);
+  const uint32_t m2 = __ballot_sync(full, xj == 2), m3 = __ballot_sync(full, xj == 3);
+  if (i >= n) return 0u;
+  const uint8_t* row = pm + 4 * x[i];
+  uint32_t bits = (row[0] ? m0 : 0u) | (row[1] ? m1 : 0u) | (row[2] ? m2 : 0u) | (row[3] ? m3 : 0u);
+  const int cmin = h + 1 + i - j0;  // j - i - 1 >= h  <=>  c >= cmin
+  if (cmin > 0) bits = cmin >= 32 ? 0u : bits & ~((1u << cmin) - 1u);
   return bits;
 }
 
