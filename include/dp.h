@@ -166,7 +166,16 @@ int dp_abi_version(void);
 const char* dp_status_string(dp_status s);
 
 /* Validates d, derives (or verifies) the schedule via dp_schedule_derive, picks
- * the kernel variant, copies the scoring parameters to the current CUDA device. */
+ * the kernel variant, copies the scoring parameters to the current CUDA device.
+ * Variants: SW_LINEAR with max(max_len_a, max_len_b) <= 64 runs the
+ * inter-task kernel (one pair per thread; the short side of the §6.1 hybrid), longer
+ * plans the intra-task warp kernels (two problems per warp in s16x2 when the score
+ * range allows, else int32). NUSSINOV picks per batch at solve time: a few problems of
+ * <= 128 nt -> one small CTA each; a few (<= 64) of 129..1024 nt -> one thread-block
+ * cluster each, table in distributed shared memory; one problem > 1024 nt -> the whole
+ * grid (cooperative launch); otherwise one warp per problem. Results are identical
+ * whichever variant runs. DP_* environment variables, read here once per plan, force
+ * variants for tests and measurements only. */
 dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out);
 void dp_plan_destroy(dp_plan_t p);
 
