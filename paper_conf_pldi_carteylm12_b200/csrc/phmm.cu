@@ -17,8 +17,9 @@
 // works on column i = k - l at step k; the row above travels down the warp by __shfl_up_sync (the
 // new column) and the value shuffled one step earlier (the diagonal). Row 0 (I_0, begin) is a
 // register of lane 0; between strips the last row goes through shared memory, per column.
-// Transition coefficients live in registers (9 per row), the emission pair (eM_j(c), eI_j(c)) per
-// residue c and row in a shared table [c][j] (one LDS.128 per two rows), dead residue K -> 0.
+// Transition coefficients live in registers (9 per row), the emission pairs (eM_j(c), eI_j(c)) per
+// residue c in a shared table laid out per lane (one LDS.128 per two rows, conflict-free; see the
+// kernel), dead residue K -> 0.
 //
 // Range: probabilities underflow fp32 after ~100 columns, so values are kept in scaled linear
 // space (the paper lets the framework pick the probability representation, §3.2) with
@@ -54,16 +55,25 @@ __device__ __forceinline__ float exp2i(int d) {
 __global__ void __launch_bounds__(kPW * 32, 2) k_phmm_forward(PhmmArgs A) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int L = A.L, K = A.K;
-  const int rows_tab = A.rows_tab;  // row stride of the emission table (256 x strips + 8)
-  // [K + 1][rows_tab] (eM_j(c), eI_j(c)) with row j at index j + 7 (so every lane's first row,
-  // j0 = 1 + 8 l, starts a 64-byte group: LDS.128 stays aligned); c = K is the dead residue
-  float2* em = reinterpret_cast<float2*>(smem);
-  for (int q = threadIdx.x; q < (K + 1) * rows_tab; q += blockDim.x) {
-    const int c = q / rows_tab, j = q - c * rows_tab - 7;
-    float2 v = make_float2(0.f, 0.f);
-    if (c < K && j >= 0 && j <= L) v = make_float2(j >= 1 ? A.emit_m[j * K + c] : 0.f, A.emit_i[j * K + c]);
+  // Emission table, bank-conflict free: per residue c (c = K: the dead residue) S = 128 x strips
+  // 16-byte chunks; the chunk of lane l's rows j0 + 2k, j0 + 2k + 1 (j0 = 1 + 256 st + 8 l) sits at
+  // 128 st + 32 k + l and holds (eM, eI) of both rows. A step's four loads per lane (k = 0..3) then
+  // put the 8 lanes of a quarter-warp on 8 distinct bank quads whatever residues their columns
+  // hold (the row-major table had lanes 2 apart on the same quad: 73 % of the wavefronts were
+  // conflicts). Row 0 (I_0's emissions) is a separate [K + 1] table.
+  const int S = A.rows_tab;  // chunks per residue (128 x strips)
+  float4* em = reinterpret_cast<float4*>(smem);
+  float* ei0t = reinterpret_cast<float*>(em + (size_t)(K + 1) * S);
+  for (int q = threadIdx.x; q < (K + 1) * S; q += blockDim.x) {
+    const int c = q / S, h = q - c * S;
+    const int st = h >> 7, k = (h >> 5) & 3, l = h & 31;
+    const int r0 = 1 + 256 * st + 8 * l + 2 * k;
+    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (c < K && r0 <= L) { v.x = A.emit_m[r0 * K + c]; v.y = A.emit_i[r0 * K + c]; }
+    if (c < K && r0 + 1 <= L) { v.z = A.emit_m[(r0 + 1) * K + c]; v.w = A.emit_i[(r0 + 1) * K + c]; }
     em[q] = v;
   }
+  for (int c = threadIdx.x; c <= K; c += blockDim.x) ei0t[c] = c < K ? A.emit_i[c] : 0.f;
   __syncthreads();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t p = (int64_t)blockIdx.x * kPW + warp;
@@ -72,7 +82,7 @@ __global__ void __launch_bounds__(kPW * 32, 2) k_phmm_forward(PhmmArgs A) {
   const int T = (int)(A.x_off[p + 1] - A.x_off[p]);
   const int strips = (L + kStripRows - 1) / kStripRows;
   // strip boundary (last row of the strip above, per column): M, I, D and the lane exponent
-  float4* bnd = reinterpret_cast<float4*>(smem + (size_t)(K + 1) * rows_tab * sizeof(float2)) +
+  float4* bnd = reinterpret_cast<float4*>(smem + (size_t)(K + 1) * S * sizeof(float4) + 128 * sizeof(float)) +
                 (size_t)warp * (A.max_len + 1);
   const int jL = L;  // the last row: its owner lane captures P at column T
   float out_val = 0.f;
@@ -106,7 +116,7 @@ __global__ void __launch_bounds__(kPW * 32, 2) k_phmm_forward(PhmmArgs A) {
     const int steps = T + 1 + 31;
     const bool first_strip = st == 0;
     const bool last_strip_lane = lane == 31 && st + 1 < strips;
-    const uint32_t em32 = (uint32_t)__cvta_generic_to_shared(em) + (uint32_t)((j0 + 7) * 8);
+    const uint32_t em32 = (uint32_t)__cvta_generic_to_shared(em) + (uint32_t)((128 * st + lane) * 16);
     for (int k = 0; k < steps; ++k) {
       const int i = k - lane;
       const bool live = i >= 0 && i <= T;
@@ -119,7 +129,7 @@ __global__ void __launch_bounds__(kPW * 32, 2) k_phmm_forward(PhmmArgs A) {
       if (lane == 0) {
         if (first_strip) {
           // row 0 at column i: M_0(i) = [i == 0] (begin), I_0(i) = eI_0(x_i) (M_0(i-1) t0_MI + I_0(i-1) t0_II)
-          const float ei0 = em[c * rows_tab + 7].y;
+          const float ei0 = ei0t[c];
           const float ni0 = ei0 * fmaf(m0, t0_mi, i0 * t0_ii);
           const float nm0 = (i == 0) ? 1.0f : 0.f;   // e0 == 0 at i == 0
           m0 = nm0; i0 = ni0;
@@ -152,11 +162,11 @@ __global__ void __launch_bounds__(kPW * 32, 2) k_phmm_forward(PhmmArgs A) {
       // column i, rows j0 .. j0+7: the diagonal comes from (pM, pI, pD) then from my old row r-1
       float dM = pM, dI = pI, dD = pD;
       pM = uM; pI = uI; pD = uD;
-      const uint32_t ea = em32 + (uint32_t)(c * rows_tab * 8);
+      const uint32_t ea = em32 + (uint32_t)(c * S * 16);
 #pragma unroll
       for (int r = 0; r < kR; r += 2) {
-        float4 e;
-        asm("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(e.x), "=f"(e.y), "=f"(e.z), "=f"(e.w) : "r"(ea + 8 * r));
+        float4 e;  // rows j0 + r, j0 + r + 1: chunk k = r / 2 at 32 k chunks
+        asm("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(e.x), "=f"(e.y), "=f"(e.z), "=f"(e.w) : "r"(ea + 256 * r));
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           const int q = r + h;
@@ -202,13 +212,13 @@ __global__ void __launch_bounds__(kPW * 32, 2) k_phmm_forward(PhmmArgs A) {
 
 }  // namespace
 
-// every lane's 8 rows of every strip are in the table (rows past L read zeros)
-int rows_tab_of(int L) { return ((L + kStripRows - 1) / kStripRows) * kStripRows + 8; }
+// every lane's 8 rows of every strip are in the table (rows past L read zeros): 16-byte chunks
+// per residue
+int rows_tab_of(int L) { return ((L + kStripRows - 1) / kStripRows) * (kStripRows / 2); }
 
 size_t phmm_smem_bytes(int L, int K, int64_t max_len) {
-  const int rows_tab = rows_tab_of(L);
   const int strips = (L + kStripRows - 1) / kStripRows;
-  size_t b = (size_t)(K + 1) * rows_tab * sizeof(float2);
+  size_t b = (size_t)(K + 1) * rows_tab_of(L) * sizeof(float4) + 128 * sizeof(float);
   if (strips > 1) b += (size_t)kPW * (size_t)(max_len + 1) * sizeof(float4);
   return b;
 }
