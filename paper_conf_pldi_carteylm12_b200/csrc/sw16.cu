@@ -356,6 +356,8 @@ constexpr int kTbUnroll = TB5_UNROLL;   // re-run steps unrolled
 #ifndef TB5_MINB
 #define TB5_MINB 4                       // CTAs per SM (register cap; 4 / 5 / 6 with no unroll: 1.049 / 1.059 / 1.099 ms)
 #endif
+constexpr int kSigRow = 34;              // int16 per sigma row (17 words: see k_sw16_tb5)
+constexpr int kSigBytes = ((32 * kSigRow * 2 + 127) / 128) * 128;
 constexpr int kCW = kGL * kSlab;         // code words per group: [c - 1][m]
 constexpr int kCWp = kCW + 4;            // group stride: 4 banks apart, so the 8 groups' code stores hit 32 banks
 constexpr int kTS = 36;                  // top-row keys per group, c = 0..32
@@ -407,13 +409,16 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
                                                                        uint8_t* out, int64_t stride, int32_t* out_len,
                                                                        int32_t* coords) {
   extern __shared__ __align__(16) uint8_t tsm[];
-  int16_t* sig_s = reinterpret_cast<int16_t*>(tsm);  // [32][32] 4 sigma + 2, kDead4 outside the alphabet
-  for (int q = threadIdx.x; q < 32 * 32; q += blockDim.x) {
-    const int x = q >> 5, y = q & 31;
+  // [32][kSigRow] 4 sigma + 2, kDead4 outside the alphabet. Rows 17 words apart: a lookup's bank
+  // is (17 a + b / 2) mod 32, so the rows of a group's lanes (same b, different a) spread over
+  // the banks (with 16-word rows a only chose between two banks)
+  int16_t* sig_s = reinterpret_cast<int16_t*>(tsm);
+  for (int q = threadIdx.x; q < 32 * kSigRow; q += blockDim.x) {
+    const int x = q / kSigRow, y = q % kSigRow;
     sig_s[q] = (x < A.asz && y < A.asz) ? (int16_t)(4 * A.sigma[x * A.asz + y] + 2) : (int16_t)kDead4;
   }
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, gq = lane / kGL, m = lane % kGL;
-  uint8_t* wb = tsm + 2048 + warp * kTbWarpBytes;
+  uint8_t* wb = tsm + kSigBytes + warp * kTbWarpBytes;
   uint32_t* Cs = reinterpret_cast<uint32_t*>(wb) + gq * kCWp;
   uint32_t* Ts = reinterpret_cast<uint32_t*>(wb + kGroups * 4 * kCWp) + gq * kTS;
   uint8_t* bS = wb + kGroups * 4 * (kCWp + kTS) + gq * 2 * kBS;                  // [2][kBS] staged b residues
@@ -616,7 +621,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         // this half's residues and top-row keys to shared memory
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
-          sa[hf][r] = sig32 + 64 * av[r];
+          sa[hf][r] = sig32 + 2 * kSigRow * av[r];
           aS[hf * kBlk + kRows * m + r] = (uint8_t)av[r];
         }
 #pragma unroll
@@ -785,7 +790,7 @@ __global__ void __launch_bounds__(256) k_sw16_rev(int64_t count, uint8_t* out, i
   }
 }
 
-size_t tb5_smem_bytes() { return 2048 + (size_t)kTbWarps * kTbWarpBytes; }
+size_t tb5_smem_bytes() { return kSigBytes + (size_t)kTbWarps * kTbWarpBytes; }
 
 }  // namespace
 
