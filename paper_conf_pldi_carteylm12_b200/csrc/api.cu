@@ -99,6 +99,7 @@ struct dp_plan {
   static constexpr int kMaxChunks = 16;
   cudaEvent_t ev_start = nullptr, ev_in[kMaxChunks] = {}, ev_out[kMaxChunks] = {};
   int64_t launches = 0;
+  bool vit_walked = false;  // the last Viterbi solve walked its paths into tb_aux2
   // dp_solve: a ring of {0, len_a, 0, len_b} offset slots in device memory; a slot is reused only
   // after the event recorded behind the solve that read it has completed
   static constexpr int kSolveSlots = 16;
@@ -111,7 +112,7 @@ struct dp_plan {
     bool nuss_rounds = false, diag_generic = false, sw_intra = false;
     int64_t nuss_tiled_min = 32;
     int nuss_tbw = 0, diag_force = -1, host_chunks = 4;
-    bool hmm_simt = false, nuss_no_cluster = false;
+    bool hmm_simt = false, nuss_no_cluster = false, hmm_separate_walk = false;
     int hmm_ns = 0, hmm_tc_smem_kb = -1;
   } env;
 };
@@ -133,6 +134,7 @@ void read_env(dp_plan* p) {
   if (on("DP_DIAG_FORCE")) p->env.diag_force = atoi(getenv("DP_DIAG_FORCE"));
   p->env.hmm_simt = on("DP_HMM_SIMT");
   p->env.nuss_no_cluster = on("DP_NUSS_NO_CLUSTER");
+  p->env.hmm_separate_walk = on("DP_HMM_SEPARATE_WALK");
   if (on("DP_HMM_NS")) p->env.hmm_ns = atoi(getenv("DP_HMM_NS"));
   if (on("DP_HMM_TC_SMEM_KB")) p->env.hmm_tc_smem_kb = atoi(getenv("DP_HMM_TC_SMEM_KB"));
   if (on("DP_HOST_CHUNKS")) p->env.host_chunks = std::max(1, std::min(dp_plan::kMaxChunks, atoi(getenv("DP_HOST_CHUNKS"))));
@@ -669,6 +671,14 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
           if (e != cudaSuccess) break;
           H.bp = static_cast<uint8_t*>(p->tb_state.ptr);
           H.final_state = static_cast<int32_t*>(p->tb_aux.ptr);
+          // the paths, walked inside k_viterbi right behind the sweep (DP_HMM_SEPARATE_WALK: the
+          // walk as its own kernel at dp_traceback, for comparison)
+          if (!p->env.hmm_separate_walk) {
+            e = p->tb_aux2.ensure((size_t)(n * (max_len_a > 0 ? max_len_a : 1) + 16));
+            if (e != cudaSuccess) break;
+            H.path = static_cast<uint8_t*>(p->tb_aux2.ptr);
+          }
+          p->vit_walked = H.path != nullptr;
         }
         e = dpk::hmm_viterbi(H, s, &p->launches);
       }
@@ -796,6 +806,7 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
       dpk::HmmArgs H{};
       H.n = p->last_n; H.x_cat = p->last_a; H.x_off = p->last_aoff; H.max_len = p->last_max_la; H.S = p->S;
       H.K = p->K; H.bp = static_cast<uint8_t*>(p->tb_state.ptr); H.final_state = static_cast<int32_t*>(p->tb_aux.ptr);
+      if (p->vit_walked) H.path = static_cast<uint8_t*>(p->tb_aux2.ptr);
       e = dpk::hmm_viterbi_traceback(H, first, count, out, stride, out_len, s, &p->launches);
       break;
     }

@@ -157,6 +157,7 @@ struct HmmArgs {
   int32_t* vit_out;                 // Viterbi
   uint8_t* bp;                      // Viterbi back-pointers (n x max_len x 64) or nullptr
   int32_t* final_state;             // n
+  uint8_t* path = nullptr;          // Viterbi: the walked state path (n x max_len), written by k_viterbi
   unsigned long long* dbg = nullptr;  // diagnostic step timestamps (DP_HMM_TIMING), else nullptr
   int ns_override = 0;                // diagnostic: sequences per warp of the SIMT kernels (DP_HMM_NS)
   int tc_smem_kb = -1;                // shared memory the tcgen05 forward reserves per CTA (-1: default)

@@ -156,6 +156,53 @@ __global__ void __launch_bounds__(kHW * 32) k_forward(HmmArgs H) {
   }
 }
 
+// One warp walks sequence p's back-pointers from its final state s (T >= 1), the path into
+// o[0 .. T). The walk s_{i-1} = bp[i-1][s_i] is one dependent load per step; the warp stages the
+// back-pointer rows it will need 32 at a time (row i-1 by lane T - i - 32c, one coalesced 2 KB
+// read per chunk, the next chunk's loads in flight during the walk) in shared memory, lane 0
+// walks the 32 steps there, and the warp writes the 32 states out with one coalesced store.
+// fresh: the rows were just written by this kernel (L2 loads) rather than by an earlier one
+// (streaming loads).
+__device__ __forceinline__ void viterbi_walk(const HmmArgs& H, int64_t p, int T, int s, uint8_t* o,
+                                             uint8_t (*rows)[32][kMaxS], uint8_t* ob, int lane, bool fresh) {
+  const uint8_t* bp = H.bp + (p * H.max_len) * kMaxS;
+  const int nch = (T + 31) / 32;
+  // chunk c: lane t holds row r = T - 1 - 32 c - t (used at position i = r + 1), valid for r >= 1
+  auto load = [&](int c, uint4* v) {
+    const int r = T - 1 - 32 * c - lane;
+    const uint4* src = reinterpret_cast<const uint4*>(bp + (int64_t)(r >= 1 ? r : 1) * kMaxS);
+#pragma unroll
+    for (int w = 0; w < kMaxS / 16; ++w)
+      v[w] = r >= 1 ? (fresh ? __ldcg(src + w) : __ldcs(src + w)) : make_uint4(0, 0, 0, 0);
+  };
+  auto stash = [&](int buf, const uint4* v) {
+    uint4* dst = reinterpret_cast<uint4*>(rows[buf][lane]);
+#pragma unroll
+    for (int w = 0; w < kMaxS / 16; ++w) dst[w] = v[w];
+  };
+  uint4 v[kMaxS / 16];
+  load(0, v);
+  stash(0, v);
+  for (int c = 0; c < nch; ++c) {
+    if (c + 1 < nch) load(c + 1, v);   // in flight during the walk
+    __syncwarp();
+    if (lane == 0) {
+      const uint8_t* R = &rows[c & 1][0][0];
+      for (int t = 0; t < 32; ++t) {
+        const int i = T - 32 * c - t;   // position
+        if (i < 1) break;
+        ob[t] = (uint8_t)s;
+        if (i >= 2) s = R[t * kMaxS + s];
+      }
+    }
+    __syncwarp();
+    const int i = T - 32 * c - lane;
+    if (i >= 1) o[i - 1] = ob[lane];
+    if (c + 1 < nch) stash((c + 1) & 1, v);
+  }
+  __syncwarp();
+}
+
 constexpr int kNegKey = -(1 << 30);
 constexpr int kRenorm = 32;
 
@@ -164,6 +211,8 @@ __global__ void __launch_bounds__(kHW * 32) k_viterbi(HmmArgs H) {
   __shared__ __align__(16) int key[kHW][NS][kMaxS];
   __shared__ int Es[kMaxK][kMaxS];
   __shared__ uint8_t xs_all[kHW][NS][kChunk];
+  __shared__ __align__(16) uint8_t walk_rows[kHW][2][32][kMaxS];  // the fused walk's staged rows
+  __shared__ uint8_t walk_ob[kHW][32];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = H.S, K = H.K;
   for (int q = threadIdx.x; q < kMaxS * kMaxK; q += blockDim.x) {
@@ -267,15 +316,37 @@ __global__ void __launch_bounds__(kHW * 32) k_viterbi(HmmArgs H) {
         if (H.final_state) H.final_state[p0 + q] = 63 - (fk & 63);
       }
     }
+    // the walk right behind the sweep: this warp's back-pointers were just written (L2-resident),
+    // and other warps' sweeps keep the SM busy while it waits on them
+    if (H.path && p0 + q < H.n && T[q] > 0) {
+      __syncwarp();  // the final state and every back-pointer row of this warp are written
+      viterbi_walk(H, p0 + q, T[q], 63 - (fk & 63), H.path + (p0 + q) * H.max_len, walk_rows[warp], walk_ob[warp],
+                   lane, true);
+    }
   }
 }
 
-// Viterbi traceback: one warp per sequence. The walk s_{i-1} = bp[i-1][s_i] is one dependent load
-// per step; the warp stages the back-pointer rows it will need 32 at a time (row i-1 by lane
-// T - i - 32c, one coalesced 2 KB read per chunk, the next chunk's loads in flight during the
-// walk) in shared memory, lane 0 walks the 32 steps there, and the warp writes the 32 states out
-// with one coalesced store.
+// Viterbi traceback (dp_traceback): the paths were walked by k_viterbi right behind the sweep
+// (viterbi_walk); this copies rows [first, first + count) into the caller's layout, one warp per
+// row. k_viterbi_tb (the walk as a kernel of its own) serves plans whose solve did not walk.
 constexpr int kTbW = 4;  // warps per CTA
+
+__global__ void __launch_bounds__(kTbW * 32) k_viterbi_copy(HmmArgs H, int64_t first, int64_t count, uint8_t* out,
+                                                             int64_t stride, int32_t* out_len) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int64_t q = (int64_t)blockIdx.x * kTbW + warp; q < count; q += (int64_t)gridDim.x * kTbW) {
+    const int64_t p = first + q;
+    const int T = (int)(H.x_off[p + 1] - H.x_off[p]);
+    if (T > stride) {
+      if (lane == 0) out_len[q] = -1;
+      continue;
+    }
+    const uint8_t* src = H.path + p * H.max_len;
+    uint8_t* o = out + q * stride;
+    for (int i = lane; i < T; i += 32) o[i] = src[i];
+    if (lane == 0) out_len[q] = T;
+  }
+}
 
 __global__ void __launch_bounds__(kTbW * 32) k_viterbi_tb(HmmArgs H, int64_t first, int64_t count, uint8_t* out,
                                                            int64_t stride, int32_t* out_len) {
@@ -289,46 +360,7 @@ __global__ void __launch_bounds__(kTbW * 32) k_viterbi_tb(HmmArgs H, int64_t fir
       if (lane == 0) out_len[q] = -1;
       continue;
     }
-    if (T == 0) {
-      if (lane == 0) out_len[q] = 0;
-      continue;
-    }
-    const uint8_t* bp = H.bp + (p * H.max_len) * kMaxS;
-    uint8_t* o = out + q * stride;
-    int s = H.final_state[p];
-    const int nch = (T + 31) / 32;
-    // chunk c: lane t holds row r = T - 1 - 32 c - t (used at position i = r + 1), valid for r >= 1
-    auto load = [&](int c, uint4* v) {
-      const int r = T - 1 - 32 * c - lane;
-      const uint4* src = reinterpret_cast<const uint4*>(bp + (int64_t)(r >= 1 ? r : 1) * kMaxS);
-#pragma unroll
-      for (int w = 0; w < kMaxS / 16; ++w) v[w] = r >= 1 ? __ldcs(src + w) : make_uint4(0, 0, 0, 0);
-    };
-    auto stash = [&](int buf, const uint4* v) {
-      uint4* dst = reinterpret_cast<uint4*>(rows[warp][buf][lane]);
-#pragma unroll
-      for (int w = 0; w < kMaxS / 16; ++w) dst[w] = v[w];
-    };
-    uint4 v[kMaxS / 16];
-    load(0, v);
-    stash(0, v);
-    for (int c = 0; c < nch; ++c) {
-      if (c + 1 < nch) load(c + 1, v);   // in flight during the walk
-      __syncwarp();
-      if (lane == 0) {
-        const uint8_t* R = &rows[warp][c & 1][0][0];
-        for (int t = 0; t < 32; ++t) {
-          const int i = T - 32 * c - t;   // position
-          if (i < 1) break;
-          ob[warp][t] = (uint8_t)s;
-          if (i >= 2) s = R[t * kMaxS + s];
-        }
-      }
-      __syncwarp();
-      const int i = T - 32 * c - lane;
-      if (i >= 1) o[i - 1] = ob[warp][lane];
-      if (c + 1 < nch) stash((c + 1) & 1, v);
-    }
+    if (T > 0) viterbi_walk(H, p, T, H.final_state[p], out + q * stride, rows[warp], ob[warp], lane, false);
     if (lane == 0) out_len[q] = T;
   }
 }
@@ -397,7 +429,8 @@ cudaError_t hmm_viterbi_traceback(const HmmArgs& H, int64_t first, int64_t count
   if (count == 0) return cudaSuccess;
   const int64_t grid = std::min<int64_t>((count + kTbW - 1) / kTbW, (int64_t)sms_of_current() * 12);
   ++*launches;
-  k_viterbi_tb<<<(unsigned)grid, kTbW * 32, 0, s>>>(H, first, count, out, stride, out_len);
+  if (H.path) k_viterbi_copy<<<(unsigned)grid, kTbW * 32, 0, s>>>(H, first, count, out, stride, out_len);
+  else k_viterbi_tb<<<(unsigned)grid, kTbW * 32, 0, s>>>(H, first, count, out, stride, out_len);
   return cudaGetLastError();
 }
 
