@@ -390,10 +390,46 @@ __device__ __forceinline__ void stage_async(const Tab2& tab, int I, int K, int J
   for (int t = 0; t < 4; ++t) cp16(st + 4096 + (lane + 32 * t) * 16, b + (lane + 32 * t) * 8);
 }
 
+// Phase-A operand staging by the TMA bulk-copy engine (grid sweep): a K-step's two records are
+// contiguous (UTd 4 KB, L 2 KB), so one lane issues two cp.async.bulk copies that complete on the
+// stage's mbarrier (expect_tx 6 KB) instead of 32 lanes issuing 12 16-byte cp.async each. One
+// mbarrier per stage buffer and warp; their phase parities live in the warp's registers.
+struct BulkStage {
+  uint32_t bar;  // shared address of the warp's two mbarriers (8 bytes apart)
+  uint32_t par;  // bit b: the parity of the phase stage b completes next
+};
+__device__ __forceinline__ void bulk_init(BulkStage& bs, uint32_t bar, int lane) {
+  bs.bar = bar;
+  bs.par = 0;
+  if (lane == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar));
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar + 8));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+}
+__device__ __forceinline__ void stage_bulk(const Tab2& tab, int I, int K, int J, uint32_t st, uint32_t bar, int lane) {
+  if (lane == 0) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(6144) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], 4096, [%2];"
+                 ::"r"(st), "l"(tab.UTd(I, K)), "r"(bar) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], 2048, [%2];"
+                 ::"r"(st + 4096), "l"(tab.L(K, J)), "r"(bar) : "memory");
+  }
+}
+__device__ __forceinline__ void bulk_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred done;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 done, [%0], %1;\n\t"
+      "@!done bra WAIT_%=;\n\t}\n" ::"r"(bar), "r"(parity) : "memory");
+}
+
 // Phase A over K in [K0, K1): acc (micro-kernel lane layout) = max(acc, UTd(I,K) (x) L(K,J)),
-// operands staged by double-buffered cp.async.
-__device__ __forceinline__ void products_async(const Tab2& tab, int I, int J, int K0, int K1, uint8_t* stg,
-                                               uint32_t (&acc)[16], int lane) {
+// operands staged by double-buffered cp.async (the batch kernel: with the bulk copies below
+// config 5 measured 795 -> 815 ms).
+__device__ __forceinline__ void products_cp(const Tab2& tab, int I, int J, int K0, int K1, uint8_t* stg,
+                                            uint32_t (&acc)[16], int lane) {
   if (K0 >= K1) return;
   const uint32_t stg_s = (uint32_t)__cvta_generic_to_shared(stg);
   stage_async(tab, I, K0, J, stg_s, lane);
@@ -414,6 +450,25 @@ __device__ __forceinline__ void products_async(const Tab2& tab, int I, int J, in
   }
 }
 
+// The same with the operands staged by double-buffered bulk copies (the grid sweep: config 4
+// measured the same 8.67 ms either way; its records are written before a grid barrier and
+// fenced for the async proxy).
+__device__ __forceinline__ void products_async(const Tab2& tab, int I, int J, int K0, int K1, uint8_t* stg,
+                                               uint32_t (&acc)[16], int lane, BulkStage& bs) {
+  if (K0 >= K1) return;
+  const uint32_t stg_s = (uint32_t)__cvta_generic_to_shared(stg);
+  stage_bulk(tab, I, K0, J, stg_s, bs.bar, lane);
+  for (int K = K0; K < K1; ++K) {
+    const int b = (K - K0) & 1;
+    if (K + 1 < K1) stage_bulk(tab, I, K + 1, J, stg_s + (b ^ 1) * kStageB, bs.bar + 8 * (b ^ 1), lane);
+    bulk_wait(bs.bar + 8 * b, (bs.par >> b) & 1u);
+    bs.par ^= 1u << b;
+    micro(reinterpret_cast<const uint32_t*>(stg + b * kStageB),
+          reinterpret_cast<const uint16_t*>(stg + b * kStageB + 4096), acc, lane);
+    __syncwarp();  // every lane is done with stage b before it is refilled
+  }
+}
+
 // Phase B of tile (I,J) from C in registers (acc), then its records.
 __device__ void tile_finish(const Tab2& tab, int I, int J, const uint32_t (&acc)[16], int below, int left, int corner,
                             InTileBuf& B, const uint8_t* x, const uint8_t* pm, int n, int h, int lane,
@@ -431,7 +486,7 @@ __device__ void batch_tile(const Tab2& tab, int I, int J, uint8_t* stg, InTileBu
   uint32_t acc[16];
 #pragma unroll
   for (int q = 0; q < 16; ++q) acc[q] = 0;  // gamma >= 0, so 0 is a neutral start
-  products_async(tab, I, J, I + 1, J, stg, acc, lane);
+  products_cp(tab, I, J, I + 1, J, stg, acc, lane);
   tile_finish(tab, I, J, acc, below, left, corner, B, x, pm, n, h, lane, clk);
 }
 
@@ -586,6 +641,8 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
   // the sequence in shared memory (the pair tests of phase B and of the traceback's steps)
   uint8_t* x = smem + kGridWarps * kBatchBuf;
   for (int q = threadIdx.x; q < n; q += blockDim.x) x[q] = A.x_cat[A.x_off[p] + q];
+  BulkStage bs;
+  bulk_init(bs, (uint32_t)__cvta_generic_to_shared(x + ((A.max_len + 15) & ~int64_t(15))) + 16 * warp, lane);
   __syncthreads();
   const int nt = (n + T - 1) / T;
   Tab2 tab;
@@ -627,8 +684,8 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
         uint32_t acc[16];
 #pragma unroll
         for (int q = 0; q < 16; ++q) acc[q] = 0;
-        if (D >= 2) products_async(tab, I, J, I + 1, I + 2, stg, acc, lane);
-        if (D >= 3) products_async(tab, I, J, J - 1, J, stg, acc, lane);
+        if (D >= 2) products_async(tab, I, J, I + 1, I + 2, stg, acc, lane, bs);
+        if (D >= 3) products_async(tab, I, J, J - 1, J, stg, acc, lane, bs);
         if (D >= 4) {  // interior K = I+2 .. J-2 from the other warps (complete at the last grid barrier)
 #pragma unroll
           for (int rr = 0; rr < 4; ++rr)
@@ -639,6 +696,8 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
             }
         }
         tile_finish(tab, I, J, acc, below, left, corner, IB, x, pm, n, A.hairpin, lane, clk);
+        asm volatile("fence.proxy.async.global;" ::: "memory");  // the records, before bulk copies read them
+        __syncwarp();
         if (D >= 4)  // this C slot is reused by diagonal D+2
           for (int q = lane; q < T * T; q += 32) Ct[q] = 0;
         clk.lap(4);
@@ -659,7 +718,7 @@ __global__ void __launch_bounds__(kGridWarps * 32, 1) k_nuss_grid2(NussArgs A, i
         uint32_t acc[16];
 #pragma unroll
         for (int q = 0; q < 16; ++q) acc[q] = 0;
-        products_async(tab, I, J, I + 2 + kk, I + 2 + kk + (int)(e - it), stg, acc, lane);
+        products_async(tab, I, J, I + 2 + kk, I + 2 + kk + (int)(e - it), stg, acc, lane, bs);
         int* Ct = Cn + (int64_t)t * T * T;
 #pragma unroll
         for (int rr = 0; rr < 4; ++rr)
@@ -1197,7 +1256,7 @@ cudaError_t nuss_tiled_solve(const NussArgs& A, cudaStream_t s, int64_t* launche
   cudaGetDevice(&dev);
   const int sms = num_sms_t(dev);
   if (A.n == 1 && A.max_len > kGridMin) {
-    const size_t smem = kGridWarps * kBatchBuf + ((A.max_len + 15) & ~int64_t(15));
+    const size_t smem = kGridWarps * kBatchBuf + ((A.max_len + 15) & ~int64_t(15)) + 16 * kGridWarps;
     cudaError_t e = cudaFuncSetAttribute(k_nuss_grid2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int per_sm = 0;

@@ -44,4 +44,11 @@ for t in memcheck racecheck synccheck; do
   done
 done
 (cd ubench && timeout 300 ./ubench > ../gpurun_out/ubench.jsonl 2>&1)
+# summaries here (the .ncu-rep captures exceed gpurun's 64 MiB copy-back limit together): text only
+mkdir -p gpurun_out/sum
+for c in sw hmm nuss1 nuss4 nuss5 swa swshort nussmid diag phmm; do
+  [ -s gpurun_out/launches_$c.csv ] && python scripts/ncu_summary.py --launches gpurun_out/launches_$c.csv > gpurun_out/sum/launches_$c.txt
+  [ -s gpurun_out/ncu_$c.ncu-rep ] && python scripts/ncu_summary.py gpurun_out/ncu_$c.ncu-rep > gpurun_out/sum/ncu_$c.txt
+done
+rm -f gpurun_out/*.ncu-rep gpurun_out/launches_*.csv
 ls -la gpurun_out
