@@ -662,7 +662,7 @@ def roofline(W, name, phase_ms, alone, pk):
     # HMM: Viterbi (max-plus, SIMT, the step's critical path) and the tcgen05 forward on its own time
     vit_ms = alone.get("k_viterbi", phase_ms[1])
     vit = alu("k_viterbi", W["inner_local"], vit_ms, peak32,
-              "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (one add-max per (p, s, t))")
+              "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (one add-max per (p, s, t)); the kernel time includes the fused path walk")
     vit["kernel_ms_in_step"] = round(phase_ms[1], 4)
     fl = 2 * W["inner_local"]
     fw_ms = alone.get("k_forward_tc", phase_ms[0])
