@@ -386,6 +386,23 @@ def test_nussinov_cluster_path(dp, orc, lens, monkeypatch):
     assert list(r2["scores"]) == list(r["scores"]) and r2["db"] == r["db"]
 
 
+@pytest.mark.parametrize("lens", [[128, 127, 5], [129, 128, 5], [1024, 700], [1025]])
+def test_nussinov_dispatch_boundaries(dp, orc, lens):
+    """The plan's Nussinov variants meet at 128 / 129 nt (one small CTA per problem vs a cluster
+    per problem) and 1024 / 1025 nt (a cluster per problem vs the whole grid for one problem):
+    batches on either side of each boundary, with and without tracebacks, bit-exact."""
+    g = np.random.default_rng(190 + sum(lens))
+    seqs = [g.integers(0, 4, size=l).astype(np.uint8) for l in lens]
+    pm = dpgen.rna_pair_mask()
+    with concurrent.futures.ThreadPoolExecutor(THREADS) as ex:
+        want = list(ex.map(lambda x: orc.nussinov_traceback(x, pm, 3), seqs))
+    r = run_nuss(dp, seqs)
+    for q, x in enumerate(seqs):
+        assert (r["scores"][q], r["db"][q]) == want[q], (q, len(x))
+    r0 = run_nuss(dp, seqs, tb=False)
+    assert [int(v) for v in r0["scores"]] == [w[0] for w in want]
+
+
 def test_nussinov_cell_level_path(dp, orc, monkeypatch):
     """The cell-level CTA kernels (shared-memory table; L2 table above 340) on the same cases."""
     monkeypatch.setenv("DP_NUSS_CELL", "1")
