@@ -111,7 +111,7 @@ struct dp_plan {
     bool force_int32 = false, nuss_cell = false, hmm_timing = false, nuss_timing = false, sw_timing = false;
     bool nuss_rounds = false, diag_generic = false, sw_intra = false;
     int64_t nuss_tiled_min = 32;
-    int nuss_tbw = 0, diag_force = -1, host_chunks = 4;
+    int nuss_tbw = 0, diag_force = -1, host_chunks = 0;  // 0: per kind (see dp_solve_batch_host)
     bool hmm_simt = false, nuss_no_cluster = false, hmm_separate_walk = false;
     int hmm_ns = 0, hmm_tc_smem_kb = -1;
   } env;
@@ -866,9 +866,13 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   // byte q of a_cat lives at h_a + (q - a_off[0]), so the kernels take the
   // caller's (absolute) offsets with a rebased base pointer.
   // a chunk must still fill the GPU: ~3 waves of the sweep kernels
-  // (config 2, measured: 1 / 2 / 3 / 4 / 8 / 12 chunks -> 4.53 / 3.73 / 3.55 / 3.46 / 4.14 / 4.31 ms)
+  // (config 2, round 1: 1 / 2 / 3 / 4 / 8 / 12 chunks -> 4.53 / 3.73 / 3.55 / 3.46 / 4.14 / 4.31 ms)
   const int64_t min_chunk = align ? 16384 : (p->kind == DP_NUSSINOV ? 65536 : 32768);
-  const int max_ch = p->env.host_chunks;  // env DP_HOST_CHUNKS: diagnostic
+  // packed SW alternates two compute streams (a chunk's sweep under the previous chunk's
+  // traceback) and gains from finer chunks (config 2, 2 / 4 / 6 chunks: 3.90 / 3.22 / 3.00 ms);
+  // the one-stream kinds measured best at 4 (affine SW 9.57 vs 9.95 ms at 6, short pairs 5.25 vs
+  // 5.59); env DP_HOST_CHUNKS: diagnostic
+  const int max_ch = p->env.host_chunks > 0 ? p->env.host_chunks : (p->kind == DP_SW_LINEAR && p->packed16 ? 6 : 4);
   int nch = (int)std::min<int64_t>(max_ch, (n + min_chunk - 1) / min_chunk);
   if (nch < 1) nch = 1;
   const int64_t per = (n + nch - 1) / nch;
