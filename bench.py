@@ -350,7 +350,7 @@ PHASES = {
     "swa": ["k_align_affine (partition sweep)", "k_align_affine_tb (traceback)"],
     "nuss": ["k_nuss (fill + in-kernel traceback)", "dp_traceback (copy)"],
     "diag": ["k_diag (conditional schedule)"],
-    "hmm": ["k_forward_tc (tcgen05 forward)", "k_viterbi (max-plus + fused path walk)", "k_viterbi_copy (traceback: path copy)"],
+    "hmm": ["k_forward_tc (tcgen05 forward)", "k_viterbi16 (s16x2 max-plus, two sequences per register + fused path walk)", "k_viterbi_copy (traceback: path copy)"],
     "phmm": ["k_phmm_forward (anti-diagonal, three tables)"],
 }
 
@@ -502,6 +502,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
                 a1.record(stream)
             torch.cuda.synchronize(dev)
             alone[nm] = a0.elapsed_time(a1) / reps
+        alone["vit_kernel"] = plans[1].last_variant  # k_viterbi16 (s16x2) or k_viterbi (int32 keys)
         a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         with torch.cuda.stream(stream):
             a0.record(stream)
@@ -573,7 +574,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
                                               ("weak" if world > 1 else "strong"))),
         "dtype": {"sw": "s16x2 (int16 lanes; score range plan-checked, else int32)",
                   "swa": "int32", "swshort": "int32", "nuss": "int16 table, s16x2 max-plus (score <= n/2)",
-                  "diag": "uint16 table / int32", "hmm": "f32 (forward; bf16x3 tensor-core split) + int32 (Viterbi)",
+                  "diag": "uint16 table / int32", "hmm": "f32 (forward; bf16x3 tensor-core split) + s16x2 (Viterbi: int16 lanes relative to the row max, exactness plan-checked, else int32)",
                   "phmm": "f32 (scaled linear space, per-lane power-of-two exponents)"}[W["kind"]],
         "config": {"workload": W["workload"], "config": name, "problems": W["n_total"], "problems_per_gpu": n,
                    "cells": W["cells_total"],
@@ -660,9 +661,16 @@ def roofline(W, name, phase_ms, alone, pk):
         r["unit"] = "Tops/s (fp32 FMA pipe)"
         return r
     # HMM: Viterbi (max-plus, SIMT, the step's critical path) and the tcgen05 forward on its own time
+    vk = alone.get("vit_kernel", "k_viterbi")
     vit_ms = alone.get("k_viterbi", phase_ms[1])
-    vit = alu("k_viterbi", W["inner_local"], vit_ms, peak32,
-              "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (one add-max per (p, s, t)); the kernel time includes the fused path walk")
+    if vk == "k_viterbi16":
+        vit = alu(vk, W["inner_local"], vit_ms, peak16,
+                  "ubench_r01 VIADDMNMX.S16x2 128 lane-ops/clk/SM x 148 SMs x sm_max_mhz (one 16-bit add-max per "
+                  "(p, s, t)); the kernel time includes the fused path walk (argmax recovery)")
+    else:
+        vit = alu(vk, W["inner_local"], vit_ms, peak32,
+                  "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (one add-max per (p, s, t)); "
+                  "the kernel time includes the fused path walk")
     vit["kernel_ms_in_step"] = round(phase_ms[1], 4)
     fl = 2 * W["inner_local"]
     fw_ms = alone.get("k_forward_tc", phase_ms[0])

@@ -86,6 +86,8 @@ def lib():
                                            ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i32)]
         L.dp_plan_launch_count.restype = i64
         L.dp_plan_launch_count.argtypes = [vp]
+        L.dp_plan_last_variant.restype = ctypes.c_char_p
+        L.dp_plan_last_variant.argtypes = [vp]
         L.dp_solve_batch.restype = ctypes.c_int
         L.dp_solve_batch.argtypes = [vp, i64, vp, vp, vp, vp, i64, i64, vp, vp]
         L.dp_solve.restype = ctypes.c_int
@@ -101,7 +103,7 @@ def lib():
 EXPORTS = ["dp_abi_version", "dp_status_string", "dp_schedule_derive", "dp_schedule_conditional",
            "dp_schedule_select", "dp_plan_create", "dp_plan_destroy",
            "dp_plan_get_schedule", "dp_solve_batch", "dp_solve", "dp_solve_batch_host", "dp_traceback",
-           "dp_plan_launch_count"]
+           "dp_plan_launch_count", "dp_plan_last_variant"]
 
 
 def _check(code, where):
@@ -245,6 +247,11 @@ class Plan:
     @property
     def launches(self):
         return int(lib().dp_plan_launch_count(self._h))
+
+    @property
+    def last_variant(self):
+        """The kernel family the last solve ran (dp_plan_last_variant)."""
+        return lib().dp_plan_last_variant(self._h).decode()
 
     def schedule(self):
         co = (ctypes.c_int32 * MAX_DIM)()

@@ -80,6 +80,7 @@ struct dp_plan {
   uint8_t* d_pair = nullptr;
   float *d_pi = nullptr, *d_A = nullptr, *d_E = nullptr;
   int32_t *d_lpi = nullptr, *d_lA = nullptr, *d_lE = nullptr;
+  int v16_C = 0, v16_sat = 0;  // Viterbi on the s16x2 kernel when v16_C > 0 (hmm_vit16.cu guard)
   int L = 0;                                         // DP_PROFILE_FORWARD positions
   float *d_ptr = nullptr, *d_pem = nullptr, *d_pei = nullptr;
   // retained state of the most recent solve
@@ -99,6 +100,7 @@ struct dp_plan {
   static constexpr int kMaxChunks = 16;
   cudaEvent_t ev_start = nullptr, ev_in[kMaxChunks] = {}, ev_out[kMaxChunks] = {};
   int64_t launches = 0;
+  const char* variant = "";  // kernel family of the last solve (dp_plan_last_variant)
   bool vit_walked = false;  // the last Viterbi solve walked its paths into tb_aux2
   // dp_solve: a ring of {0, len_a, 0, len_b} offset slots in device memory; a slot is reused only
   // after the event recorded behind the solve that read it has completed
@@ -385,6 +387,8 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
         e = upload(&p->d_lpi, d->lpi, p->S);
         if (e == cudaSuccess) e = upload(&p->d_lA, d->lA, (size_t)p->S * p->S);
         if (e == cudaSuccess) e = upload(&p->d_lE, d->lE, (size_t)p->S * p->K);
+        // exact in 16 bits for these scores? (DP_FORCE_INT32: the int32 kernel regardless)
+        if (!p->env.force_int32) p->v16_C = dpk::vit16_clamp(d->lA, d->lE, p->S, p->K, &p->v16_sat);
       }
       break;
   }
@@ -437,6 +441,7 @@ dp_status dp_plan_get_schedule(dp_plan_t p, int32_t coeff[], int* ndim, int64_t*
 }
 
 int64_t dp_plan_launch_count(dp_plan_t p) { return p ? p->launches : -1; }
+const char* dp_plan_last_variant(dp_plan_t p) { return p ? p->variant : ""; }
 
 dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int64_t* a_off, const uint8_t* b_cat,
                          const int64_t* b_off, int64_t max_len_a, int64_t max_len_b, void* scores_out,
@@ -465,6 +470,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       for (int k = 0; k < p->ncand; ++k) { A.cand[k][0] = p->cand[k][0]; A.cand[k][1] = p->cand[k][1]; }
       A.force = p->env.diag_force >= 0 ? p->env.diag_force : p->force;  // env: diagnostic
       A.asz = p->env.diag_generic ? 0 : p->asz;  // env: diagnostic (the unpacked path)
+      p->variant = "k_diag";
       e = dpk::diag_solve(A, s, &p->launches);
       break;
     }
@@ -485,12 +491,14 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
           p->last_scores = A.scores;
         }
         e = p->scratch.ensure(dpk::sw_inter_work_bytes(n));
+        p->variant = "k_sw_inter";
         if (e == cudaSuccess) e = dpk::sw_inter_solve(A, p->scratch.ptr, s, &p->launches);
         break;
       }
       if (p->packed16) {
         dpk::Sw16Args A{};
         e = sw16_args(p, n, a_cat, a_off, b_cat, b_off, max_len_a, max_len_b, static_cast<int32_t*>(scores_out), &A);
+        p->variant = "k_sw16";
         if (e == cudaSuccess) e = dpk::sw16_solve(A, p->want_tb, s, &p->launches);
         break;
       }
@@ -510,6 +518,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
         p->last_scores = A.scores;
       }
+      p->variant = "k_align";
       e = dpk::align_solve(A, s, &p->launches);
       break;
     }
@@ -529,6 +538,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
         p->last_scores = A.scores;
       }
+      p->variant = "k_align_affine";
       e = dpk::align_affine_solve(A, s, &p->launches);
       break;
     }
@@ -552,6 +562,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       // traceback in shared memory, one barrier per partition (DP_NUSS_CELL / DP_NUSS_TILED_MIN: the
       // other paths, for comparison)
       if (dpk::nuss_small_supported(A.max_len, n, p->device) && !p->env.nuss_cell && p->env.nuss_tiled_min == 32) {
+        p->variant = "k_nuss_small";
         e = dpk::nuss_small_solve(A, s, &p->launches);
         break;
       }
@@ -567,6 +578,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         if (p->env.nuss_rounds) cudaMalloc(&rounds, 8 * 4096), cudaMemset(rounds, 0, 8 * 4096), A.round_ns = rounds;
         unsigned long long* dbg = nullptr;
         if (p->env.nuss_timing) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
+        p->variant = "k_nuss_cluster";
         e = dpk::nuss_cluster_solve(A, s, &p->launches);
         if (dbg) {  // diagnostic: cluster-kernel phase cycles summed over warps (stderr)
           unsigned long long h[8];
@@ -599,6 +611,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       if (p->env.nuss_rounds && tiled && n == 1) cudaMalloc(&rounds, 8 * 8192), cudaMemset(rounds, 0, 8 * 8192), A.round_ns = rounds;
       unsigned long long* dbg = nullptr;
       if (p->env.nuss_timing && tiled) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
+      p->variant = !tiled ? "k_nuss_cell" : (n == 1 && A.max_len > 1024) ? "k_nuss_grid2" : "k_nuss_batch";
       e = tiled ? dpk::nuss_tiled_solve(A, s, &p->launches) : dpk::nuss_solve(A, s, &p->launches);
       if (dbg) {  // diagnostic: batch-kernel phase cycles summed over warps (stderr)
         unsigned long long h[8];
@@ -629,6 +642,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       P.n = n; P.x_cat = a_cat; P.x_off = a_off; P.max_len = max_len_a; P.L = p->L; P.K = p->K;
       P.trans = p->d_ptr; P.emit_m = p->d_pem; P.emit_i = p->d_pei;
       P.ll_out = static_cast<float*>(scores_out);
+      p->variant = "k_phmm_forward";
       e = dpk::phmm_forward(P, s, &p->launches);
       break;
     }
@@ -644,8 +658,9 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
         unsigned long long* dbg = nullptr;
         if (p->env.hmm_timing) cudaMalloc(&dbg, 8 * 4 * 66), cudaMemset(dbg, 0, 8 * 4 * 66), H.dbg = dbg;
         H.tc_smem_kb = p->env.hmm_tc_smem_kb;
-        e = (dpk::hmm_forward_tc_supported(p->S) && !p->env.hmm_simt) ? dpk::hmm_forward_tc(H, s, &p->launches)
-                                                 : dpk::hmm_forward(H, s, &p->launches);
+        const bool tc = dpk::hmm_forward_tc_supported(p->S) && !p->env.hmm_simt;
+        p->variant = tc ? "k_forward_tc" : "k_forward";
+        e = tc ? dpk::hmm_forward_tc(H, s, &p->launches) : dpk::hmm_forward(H, s, &p->launches);
         if (dbg) {  // diagnostic: CTA 0 step phases (ns): MMA issue, wait for MMA, epilogue, barrier
           unsigned long long h[4 * 66];
           cudaStreamSynchronize(s);
@@ -665,6 +680,27 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       } else {
         H.lpi = p->d_lpi; H.lA = p->d_lA; H.lE = p->d_lE;
         H.vit_out = static_cast<int32_t*>(scores_out);
+        // the s16x2 kernel (two sequences per register, the argmax recovered by its fused walk);
+        // the int32 kernel when the scores do not fit or the walk is asked for as its own kernel
+        const bool v16 = p->v16_C > 0 && !(p->want_tb && p->env.hmm_separate_walk);
+        if (v16) {
+          H.v16_C = p->v16_C;
+          H.v16_sat = p->v16_sat;
+          if (p->want_tb) {
+            const int64_t ml = max_len_a > 0 ? max_len_a : 1;
+            e = p->tb_state.ensure((size_t)(((n + 1) / 2) * ml * 64 * 4 + 16));
+            if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 4 + 16));
+            if (e == cudaSuccess) e = p->tb_aux2.ensure((size_t)(n * ml + 16));
+            if (e != cudaSuccess) break;
+            H.rows16 = static_cast<uint32_t*>(p->tb_state.ptr);
+            H.final_state = static_cast<int32_t*>(p->tb_aux.ptr);
+            H.path = static_cast<uint8_t*>(p->tb_aux2.ptr);
+            p->vit_walked = true;
+          }
+          p->variant = "k_viterbi16";
+          e = dpk::hmm_viterbi16(H, s, &p->launches);
+          break;
+        }
         if (p->want_tb) {
           e = p->tb_state.ensure((size_t)(n * (max_len_a > 0 ? max_len_a : 1) * 64 + 16));
           if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 4 + 16));
@@ -680,6 +716,7 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
           }
           p->vit_walked = H.path != nullptr;
         }
+        p->variant = "k_viterbi";
         e = dpk::hmm_viterbi(H, s, &p->launches);
       }
       break;

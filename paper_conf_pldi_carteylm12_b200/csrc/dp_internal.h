@@ -161,11 +161,18 @@ struct HmmArgs {
   unsigned long long* dbg = nullptr;  // diagnostic step timestamps (DP_HMM_TIMING), else nullptr
   int ns_override = 0;                // diagnostic: sequences per warp of the SIMT kernels (DP_HMM_NS)
   int tc_smem_kb = -1;                // shared memory the tcgen05 forward reserves per CTA (-1: default)
+  // Viterbi in s16x2 (hmm_vit16.cu): clamp C (> 0: the 16-bit kernel runs), saturating emission add,
+  // and its per-position rows for the walk ((n+1)/2 pairs x max_len x 64 packed words) or nullptr
+  int v16_C = 0;
+  int v16_sat = 0;
+  uint32_t* rows16 = nullptr;
 };
 cudaError_t hmm_forward(const HmmArgs& a, cudaStream_t s, int64_t* launches);
 bool hmm_forward_tc_supported(int S);
 cudaError_t hmm_forward_tc(const HmmArgs& a, cudaStream_t s, int64_t* launches);  // tcgen05 path
 cudaError_t hmm_viterbi(const HmmArgs& a, cudaStream_t s, int64_t* launches);
+int vit16_clamp(const int32_t* lA, const int32_t* lE, int S, int K, int* sat);  // host: C, or 0 if not exact
+cudaError_t hmm_viterbi16(const HmmArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t hmm_viterbi_traceback(const HmmArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                                   int32_t* out_len, cudaStream_t s, int64_t* launches);
 

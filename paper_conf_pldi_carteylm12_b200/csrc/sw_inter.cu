@@ -101,7 +101,7 @@ __device__ __forceinline__ void inter_pair(const AlignArgs& A, const int8_t* sig
       bj = 64 - rk % 65;
     }
     if (TB) {  // column 16w + r sits at bits 2 (15 - r) of word w: left-align a partial last word
-      if (NC % 16) cw[NC / 16] <<= 2 * (16 - NC % 16);
+      if constexpr (NC % 16 != 0) cw[NC / 16] <<= 2 * (16 - NC % 16);
     }
     if (TB) reinterpret_cast<uint4*>(A.dirs)[(int64_t)(i - 1) * A.n + t] = make_uint4(cw[0], cw[1], cw[2], cw[3]);
   }

@@ -563,12 +563,64 @@ def test_viterbi_random(dp, orc, S):
     ml = max(len(s) for s in seqs)
     plan = dp.Plan(dp.HMM_VITERBI, ml, lpi=lpi, lA=lA, lE=lE, want_traceback=True)
     sc = host(plan.solve_batch(cuda(cat), cuda(off)))
+    assert plan.last_variant == "k_viterbi16"  # Dirichlet(1) scores fit the 16-bit guard
     out, ln, _ = plan.traceback(0, len(seqs), max(ml, 1), coords=False)
     out, ln = host(out), host(ln)
     for q, x in enumerate(seqs):
         v, path = orc.viterbi(x, lpi, lA, lE)
         assert sc[q] == v, q
         assert ln[q] == len(x) and (out[q, :len(x)] == path).all(), q
+
+
+def _viterbi_check(dp, orc, lpi, lA, lE, seqs, variant, tb=True):
+    cat, off = dpgen.pack(seqs)
+    ml = max(max(len(s) for s in seqs), 1)
+    plan = dp.Plan(dp.HMM_VITERBI, ml, lpi=lpi, lA=lA, lE=lE, want_traceback=tb)
+    sc = host(plan.solve_batch(cuda(cat), cuda(off)))
+    assert plan.last_variant == variant
+    if tb:
+        out, ln, _ = plan.traceback(0, len(seqs), ml, coords=False)
+        out, ln = host(out), host(ln)
+    for q, x in enumerate(seqs):
+        v, path = orc.viterbi(x, lpi, lA, lE)
+        assert sc[q] == v, q
+        if tb:
+            assert ln[q] == len(x) and (out[q, :len(x)] == path).all(), q
+
+
+@pytest.mark.parametrize("case", ["int32_forced", "guard_fails", "saturating", "ties", "odd_ragged", "score_only"])
+def test_viterbi_variants(dp, orc, case, monkeypatch):
+    """The s16x2 Viterbi's guard (hmm_vit16.cu: A' <= 16383 exact, saturating emission add when
+    A' + E'' > 32768) and the int32 kernel it falls back to, each bit-exact against the oracle."""
+    g = np.random.default_rng(150 + len(case))
+    S = 64 if case != "odd_ragged" else 23
+    pi, A, E = dpgen.hmm_params(g, S, 4)
+    lpi, lA, lE = dpgen.millibits(pi), dpgen.millibits(A), dpgen.millibits(E)
+    seqs = [dpgen.sample_hmm(g, pi, A, E, 1, int(g.integers(0, 200)))[0] for _ in range(21)]
+    variant = "k_viterbi16"
+    if case == "int32_forced":
+        monkeypatch.setenv("DP_FORCE_INT32", "1")
+        variant = "k_viterbi"
+    elif case == "guard_fails":      # one transition at the p = 0 floor: A' = 100000-ish > 16383
+        lA = lA.copy()
+        lA[3, 5] = dpgen.MILLIBIT_FLOOR
+        variant = "k_viterbi"
+    elif case == "saturating":       # A' within the guard, emissions down to 2^-24: A' + E'' > 32768
+        lA = np.maximum(lA, lA.max(axis=0, keepdims=True) - 12000).astype(np.int32)
+        lE = lE.copy()
+        lE[::3, 1] = -24000
+        cr = lA.max(axis=0)
+        ep = lE + cr[:, None]
+        assert (cr - lA.min(axis=0)).max() + (ep.max(axis=0) - ep.min(axis=0)).max() > 32768
+    elif case == "ties":             # uniform transitions and emissions: every predecessor ties
+        lpi = np.full(S, -6000, np.int32)
+        lA = np.full((S, S), -6000, np.int32)
+        lE = np.full((S, 4), -2000, np.int32)
+    elif case == "odd_ragged":       # S = 23 (inactive lanes), odd n, T = 0 and T = 1 rows
+        seqs[0] = seqs[0][:0]
+        seqs[7] = seqs[7][:1]
+        seqs.append(seqs[4][:1])
+    _viterbi_check(dp, orc, lpi, lA, lE, seqs, variant, tb=(case != "score_only"))
 
 
 def test_hmm_config3_sampled(dp, orc, capsys):
@@ -582,6 +634,7 @@ def test_hmm_config3_sampled(dp, orc, capsys):
     ll = host(pf.solve_batch(cuda(cat), cuda(off), max_len_a=T))
     pv = dp.Plan(dp.HMM_VITERBI, T, lpi=d["lpi"], lA=d["lA"], lE=d["lE"], want_traceback=True)
     vs = host(pv.solve_batch(cuda(cat), cuda(off), max_len_a=T))
+    assert pv.last_variant == "k_viterbi16"
     out, ln, _ = pv.traceback(0, n, T, coords=False)
     out = host(out)
     ids = np.random.default_rng(140).choice(n, size=24, replace=False)
