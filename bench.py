@@ -586,7 +586,7 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
         "roofline": roof,
         "gpu_launches": int(launches),
         "result_sha256": digest,
-        **({"alone_ms": {k: round(v, 4) for k, v in alone.items()}} if alone else {}),
+        **({"alone_ms": {k: (round(v, 4) if isinstance(v, float) else v) for k, v in alone.items()}} if alone else {}),
         **({"batch_kernel_ms": nocl, "cluster_kernel_ms": round(phase_ms[0], 4)} if nocl else {}),
         **({"intra_task_ms": intra, "inter_task_ms": round(ms_step, 4)} if intra else {}),
         **({"fixed_schedule_ms": fixed, "conditional_schedule_ms": round(ms_step, 4)} if fixed else {}),
