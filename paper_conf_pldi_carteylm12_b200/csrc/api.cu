@@ -150,6 +150,8 @@ int max_smem_optin(int dev) {
 
 dp_status cuda_status(cudaError_t e) {
   if (e == cudaSuccess) return DP_OK;
+  static const bool verbose = getenv("DP_VERBOSE_ERRORS") != nullptr;  // diagnostic: name the CUDA error
+  if (verbose) fprintf(stderr, "dp: CUDA error %s: %s\n", cudaGetErrorName(e), cudaGetErrorString(e));
   if (e == cudaErrorMemoryAllocation) return DP_E_NOMEM;
   return DP_E_CUDA;
 }
