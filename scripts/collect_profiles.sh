@@ -10,5 +10,7 @@ for c in sw hmm nuss1 nuss4 nuss5 swa swshort nussmid diag phmm; do  # summaries
   [ -s gpurun_out/sum/launches_$c.txt ] && cp gpurun_out/sum/launches_$c.txt profiles/launches_${c}_$R.txt
   [ -s gpurun_out/sum/ncu_$c.txt ] && cp gpurun_out/sum/ncu_$c.txt profiles/ncu_${c}_$R.txt
 done
-mkdir -p profiles/sanitizer_$R
-for f in gpurun_out/san/*.log; do tail -25 "$f" > profiles/sanitizer_$R/$(basename "$f"); done
+if ls gpurun_out/san/*.log > /dev/null 2>&1; then
+  mkdir -p profiles/sanitizer_$R
+  for f in gpurun_out/san/*.log; do tail -25 "$f" > profiles/sanitizer_$R/$(basename "$f"); done
+fi
