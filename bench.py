@@ -445,6 +445,9 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
     for _ in range(warmup):
         step(False)
     torch.cuda.synchronize(dev)
+    W["variant"] = plans[0].last_variant  # the kernel family the plan dispatched to
+    if W["kind"] == "swa" and W["variant"] == "k_affine16":
+        phase_names = ["k_affine16 (packed s16x2 partition sweep)", "k_affine16_tb (traceback)"]
     launches0 = sum(p.launches for p in plans)
     step_ms = []
     if world > 1:
@@ -573,7 +576,8 @@ def run_config(name, args, rank, world, local_rank, steps, warmup, headline):
         "scaling": ("strong" if sharded else ("replicas" if world > 1 and name in ("nuss1", "nuss4") else
                                               ("weak" if world > 1 else "strong"))),
         "dtype": {"sw": "s16x2 (int16 lanes; score range plan-checked, else int32)",
-                  "swa": "int32", "swshort": "int32", "nuss": "int16 table, s16x2 max-plus (score <= n/2)",
+                  "swa": ("s16x2 keys 4 v + code (int16 lanes; score range plan-checked, else int32)"
+                          if W.get("variant") == "k_affine16" else "int32"), "swshort": "int32", "nuss": "int16 table, s16x2 max-plus (score <= n/2)",
                   "diag": "uint16 table / int32", "hmm": "f32 (forward; bf16x3 tensor-core split) + s16x2 (Viterbi: int16 lanes relative to the row max, exactness plan-checked, else int32)",
                   "phmm": "f32 (scaled linear space, per-lane power-of-two exponents)"}[W["kind"]],
         "config": {"workload": W["workload"], "config": name, "problems": W["n_total"], "problems_per_gpu": n,
@@ -635,8 +639,15 @@ def roofline(W, name, phase_ms, alone, pk):
         r["traceback_ms"] = round(phase_ms[1], 4)
         return r
     if W["kind"] == "swa":
-        return alu("k_align_affine", W["ops_local"], phase_ms[0], peak32,
-                   "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (6 int32 ops per cell)")
+        if W.get("variant") == "k_affine16":
+            r = alu("k_affine16", W["ops_local"], phase_ms[0], peak16,
+                    "ubench_r01 VIADDMNMX.S16x2 128 lane-ops/clk/SM x 148 SMs x sm_max_mhz (6 max-plus ops per cell)")
+            r["frac_vs_int32_peak"] = round(W["ops_local"] / (phase_ms[0] * 1e-3) / peak32, 4)
+        else:
+            r = alu("k_align_affine", W["ops_local"], phase_ms[0], peak32,
+                    "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (6 int32 ops per cell)")
+        r["traceback_ms"] = round(phase_ms[1], 4)
+        return r
     if W["kind"] == "diag":
         return alu("k_diag", W["ops_local"], phase_ms[0], peak32,
                    "ubench_r01 VIADDMNMX s32 64 lane-ops/clk/SM x 148 SMs x sm_max_mhz (3 int ops per cell)")

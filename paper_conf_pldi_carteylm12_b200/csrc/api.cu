@@ -76,6 +76,7 @@ struct dp_plan {
   int8_t* d_sigma = nullptr;
   std::vector<int8_t> h_sigma;
   bool packed16 = false;  // SW on the s16x2 two-problems-per-warp kernels
+  bool affine16 = false;  // affine SW on the s16x2 two-problems-per-warp kernel
   bool inter = false;     // SW on the inter-task kernel (one pair per thread; short pairs)
   uint8_t* d_pair = nullptr;
   float *d_pi = nullptr, *d_A = nullptr, *d_E = nullptr;
@@ -336,7 +337,11 @@ dp_status dp_plan_create(const dp_desc* d, dp_plan_t* out) {
       if (p->asz > 32) { st = DP_E_UNSUPPORTED; break; }
       p->gap_open = d->gap_open; p->gap_ext = d->gap_extend;
       if (d->max_len_b > (1 << 20) || d->max_len_a > (1 << 20)) { st = DP_E_TOO_LARGE; break; }
-      if (smem_limit > 0 && dpk::align_affine_smem_bytes(p->asz, d->max_len_a, d->max_len_b) > (size_t)smem_limit) {
+      p->affine16 = dpk::affine16_eligible(d->max_len_a, d->max_len_b, d->sigma, p->asz, p->gap_open, p->gap_ext) &&
+                    !p->env.force_int32 &&
+                    (smem_limit <= 0 || dpk::affine16_smem_bytes(p->asz, d->max_len_a, d->max_len_b) <= (size_t)smem_limit);
+      if (!p->affine16 && smem_limit > 0 &&
+          dpk::align_affine_smem_bytes(p->asz, d->max_len_a, d->max_len_b) > (size_t)smem_limit) {
         st = DP_E_TOO_LARGE;
         break;
       }
@@ -532,16 +537,18 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       A.gap_open = p->gap_open; A.gap_ext = p->gap_ext;
       A.scores = static_cast<int32_t*>(scores_out);
       if (p->want_tb) {
-        A.dir_stride = dpk::align_affine_dir_words(A.max_la, A.max_lb);
-        e = p->tb_state.ensure((size_t)(n * A.dir_stride * 4 + 16));
+        // packed: codes per group of two problems; else per problem
+        A.dir_stride = p->affine16 ? dpk::affine16_dir_words(A.max_la, A.max_lb) : dpk::align_affine_dir_words(A.max_la, A.max_lb);
+        const int64_t units = p->affine16 ? (n + 1) / 2 : n;
+        e = p->tb_state.ensure((size_t)(units * A.dir_stride * 4 + 16));
         if (e == cudaSuccess) e = p->tb_aux.ensure((size_t)(n * 2 * 4 + 16));
         if (e != cudaSuccess) break;
         A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
         A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
         p->last_scores = A.scores;
       }
-      p->variant = "k_align_affine";
-      e = dpk::align_affine_solve(A, s, &p->launches);
+      p->variant = p->affine16 ? "k_affine16" : "k_align_affine";
+      e = p->affine16 ? dpk::affine16_solve(A, s, &p->launches) : dpk::align_affine_solve(A, s, &p->launches);
       break;
     }
     case DP_NUSSINOV: {
@@ -828,9 +835,14 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
       A.gap_open = p->gap_open; A.gap_ext = p->gap_ext;
       A.scores = p->last_scores;
       A.dirs = static_cast<uint32_t*>(p->tb_state.ptr);
-      A.dir_stride = dpk::align_affine_dir_words(A.max_la, A.max_lb);
       A.ends = static_cast<int32_t*>(p->tb_aux.ptr);
-      e = dpk::align_affine_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
+      if (p->affine16) {
+        A.dir_stride = dpk::affine16_dir_words(A.max_la, A.max_lb);
+        e = dpk::affine16_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
+      } else {
+        A.dir_stride = dpk::align_affine_dir_words(A.max_la, A.max_lb);
+        e = dpk::align_affine_traceback(A, first, count, out, stride, out_len, coords, s, &p->launches);
+      }
       break;
     }
     case DP_NUSSINOV: {

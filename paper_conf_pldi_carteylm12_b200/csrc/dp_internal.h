@@ -51,6 +51,13 @@ int64_t align_affine_dir_words(int64_t max_la, int64_t max_lb);  // affine: 4 bi
 cudaError_t align_affine_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t align_affine_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                                    int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
+// packed s16x2 affine SW (affine16.cu): two problems per warp, keyed codes; dirs strided per GROUP
+bool affine16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host, int asz, int go, int ge);
+size_t affine16_smem_bytes(int asz, int64_t max_la, int64_t max_lb);
+int64_t affine16_dir_words(int64_t max_la, int64_t max_lb);  // words per group of two problems
+cudaError_t affine16_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
+cudaError_t affine16_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
+                               int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);
 cudaError_t align_solve(const AlignArgs& a, cudaStream_t s, int64_t* launches);
 cudaError_t align_traceback(const AlignArgs& a, int64_t first, int64_t count, uint8_t* out, int64_t stride,
                             int32_t* out_len, int32_t* coords, cudaStream_t s, int64_t* launches);

@@ -250,6 +250,54 @@ def test_sw_affine_random_ragged(dp, orc, maxlen, go, ge):
             assert tuple(r["coords"][q]) == co, q
 
 
+def test_sw_affine_int32_kernel_path(dp, orc, monkeypatch):
+    """The int32 affine kernel (used when the s16x2 keys could overflow) on ragged cases."""
+    monkeypatch.setenv("DP_FORCE_INT32", "1")
+    g = np.random.default_rng(121)
+    sig = dpgen.blosum62()
+    a, _ = rand_batch(g, 60, 0, 300, 24)
+    b, _ = rand_batch(g, 60, 0, 300, 24)
+    r = run_align(dp, dp.SW_AFFINE, a, b, sigma=sig, asz=24, go=11, ge=1)
+    for q in range(60):
+        assert r["scores"][q] == orc.sw_affine(a[q], b[q], sig, 11, 1)[0], q
+        ops, co = orc.sw_affine_traceback(a[q], b[q], sig, 11, 1)
+        assert r["ops"][q] == ops and tuple(r["coords"][q]) == co, q
+
+
+def test_sw_affine_packed_variants(dp, orc):
+    """The packed s16x2 affine kernel: chosen for BLOSUM62-range scores (odd batch: the last warp
+    carries one problem), score-only equal to traceback mode, tie-heavy inputs (a 2-letter
+    alphabet, repeats, identical pairs); a sigma whose keys 4 sigma + 3 leave int8 falls back to
+    the int32 kernel, bit-exact as well."""
+    g = np.random.default_rng(122)
+    n = 81
+    a = [g.integers(0, 2, size=int(g.integers(0, 90))).astype(np.uint8) for _ in range(n)]
+    b = [g.integers(0, 2, size=int(g.integers(0, 90))).astype(np.uint8) for _ in range(n)]
+    a += [np.array([0, 1] * 20, np.uint8), np.zeros(30, np.uint8)]
+    b += [np.array([0, 1] * 20, np.uint8), np.zeros(25, np.uint8)]
+    a_cat, a_off = dpgen.pack(a)
+    b_cat, b_off = dpgen.pack(b)
+    A = (cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off))
+    m = len(a)
+    for sig, go, ge, want in ((np.array([[2, -1], [-1, 2]], np.int8), 2, 1, "k_affine16"),
+                              (np.array([[3, -3], [-3, 3]], np.int8), 0, 2, "k_affine16"),
+                              (np.array([[40, -9], [-9, 40]], np.int8), 5, 1, "k_align_affine")):
+        with dp.Plan(dp.SW_AFFINE, 90, 90, sigma=sig, alphabet_size=2, want_traceback=True, gap_open=go,
+                     gap_extend=ge) as p:
+            sc = host(p.solve_batch(*A, max_len_a=90, max_len_b=90))
+            assert p.last_variant == want
+            out, ln, co = p.traceback(0, m, 181)
+            out, ln, co = host(out), host(ln), host(co)
+        with dp.Plan(dp.SW_AFFINE, 90, 90, sigma=sig, alphabet_size=2, want_traceback=False, gap_open=go,
+                     gap_extend=ge) as p:
+            sc0 = host(p.solve_batch(*A, max_len_a=90, max_len_b=90))
+        assert (sc0 == sc).all()
+        for q in range(m):
+            assert sc[q] == orc.sw_affine(a[q], b[q], sig, go, ge)[0], (want, q)
+            ops, c = orc.sw_affine_traceback(a[q], b[q], sig, go, ge)
+            assert bytes(out[q, :ln[q]]).decode() == ops and tuple(co[q]) == c, (want, q)
+
+
 def test_sw_affine_config2_sampled(dp, orc):
     """BASELINE config 2's pairs with affine gaps (open 11, extend 1) at full size,
     in the bench's launch configuration; sampled pairs against the oracle."""
