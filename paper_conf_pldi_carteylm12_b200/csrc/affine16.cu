@@ -7,12 +7,13 @@
 //
 // Cells are KEYS 4 v + code (s16x2), so the maxima the recurrence takes anyway also pick the
 // traceback's tie-breaks (R-TB-SWA: in H diagonal > F > E; in E / F opening > extending):
-//   E4 = (max(H(i,j-1) - 4(go+ge) + 1, E4(i,j-1) - 4ge - 1) & ~3) | 1      (code 1 = open)
-//   F4 = (max(H(i-1,j) - 4(go+ge) + 1, F4(i-1,j) - 4ge - 2) & ~3) | 2
-//   H  = max(H(i-1,j-1) + 4 sigma + 3, F4, E4, 0) & ~3                      (H code: 3 diag, 2 F, 1 E)
-// (E4 / F4 carry their H-source code in the low bits, and the extension constants take it off
-// again.) Per packed cell: E 3 ops, F 3, the diagonal 1, H 2 — the critical path down a column
-// is 4 dependent ops per row. The traceback retains 4 bits per cell and problem: the H code,
+//   E4 = (max(Ho(i,j-1), E4(i,j-1) - 4ge - 1) & ~3) | 1      (code 1 = open)
+//   F4 = (max(Ho(i-1,j), F4(i-1,j) - 4ge - 2) & ~3) | 2
+//   Hk = max(Ho(i-1,j-1) + s(a_i,b_j), F4, E4, 0)             (H code: 3 diag, 2 F, 1 E, 0 zero)
+//   Ho = (Hk & ~3) + o,   o = -4(go+ge) + 1,   s = 4 sigma + 3 - o  (the profile holds s)
+// E4 / F4 carry their H-source code in the low bits, and the extension constants take it off
+// again; a cell is kept as Ho, the OPENING candidate of its right and lower neighbours, so one
+// add serves both. Per packed cell: E 2 ops, F 2, the diagonal 1, H 3. The traceback retains 4 bits per cell and problem: the H code,
 // F opened, E opened (one 32-bit word per lane, column and problem; one coalesced 64-bit store
 // per step), walked by one thread per problem (k_affine16_tb) with the score tracked exactly.
 // The end cell (first row-major maximum, R-TB-SW) comes from per-row running maxima and the
@@ -49,6 +50,13 @@ __device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c) {
   asm("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(d) : "r"(a), "r"(b), "r"(c), "n"(F));
   return d;
 }
+// a * b + c on the FMA pipe (the ALU pipe is the bound here): ~x as x * -1 - 1 (the 32-bit identity
+// holds for both halves at once), shifted merges of disjoint bit fields as multiply-adds
+__device__ __forceinline__ uint32_t mad(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm volatile("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
 __device__ __forceinline__ int lo16(uint32_t v) { return (int)(int16_t)(v & 0xffffu); }
 __device__ __forceinline__ int hi16(uint32_t v) { return (int)(int16_t)(v >> 16); }
 __device__ __forceinline__ uint32_t pk2(int v) { return (uint32_t)(uint16_t)(int16_t)v * 0x10001u; }
@@ -78,16 +86,17 @@ template <bool MULTI>
 __host__ __device__ constexpr int rec_bytes() { return MULTI ? 12 : 4; }  // u16 x 2 profile rows (+ H, F boundary)
 
 struct AffState {
-  uint32_t H[kRows];   // clean keys 4 H of my rows at my current column
+  uint32_t H[kRows];   // Ho = 4 H + o of my rows at my current column
   uint32_t E[kRows];   // E keys 4 E + 1
-  uint32_t rb[kRows];  // TB: per-row running maximum (clean keys); score-only: rb[0] is the lane maximum
+  uint32_t rb[kRows];  // TB: ~(per-row running maximum of Ho); score-only: rb[0] is the lane maximum of Ho
   uint32_t rc[kRows];  // TB: column where rb was first reached
   uint32_t prevH;      // H(row above my first row, j - 1)
   uint32_t F7;         // F key of my last row at my current column
 };
 
 struct AffK {          // packed constants
-  uint32_t open, exte, extf, negf;
+  uint32_t open, exte, extf, negf;  // o, -4ge - 1, -4ge - 2, F(0, j) = -inf
+  uint32_t m1;                      // 0xffffffff through an opaque move
 };
 
 // One step of one lane. CHECK: ramp steps (j may lie outside 1..lbm; dead profile values make
@@ -102,12 +111,12 @@ __device__ __forceinline__ uint2 aff_step(AffState& S, uint32_t rec, int j, uint
   const uint32_t fF = __shfl_up_sync(0xffffffffu, S.F7, 1);
   uint32_t Hup, Fup;
   if (MULTI) {  // only lane 0 reads the boundary words (lane 31 rewrites them a few steps later)
-    uint32_t bh = 0, bf = C.negf;
+    uint32_t bh = C.open, bf = C.negf;
     if (lane0 && from_bnd && live) { bh = lds_u32_v(rec + 4); bf = lds_u32_v(rec + 8); }
     Hup = lane0 ? bh : fH;
     Fup = lane0 ? bf : fF;
   } else {
-    Hup = lane0 ? 0u : fH;
+    Hup = lane0 ? C.open : fH;
     Fup = lane0 ? C.negf : fF;
   }
   const uint32_t Hd = S.prevH;
@@ -123,7 +132,7 @@ __device__ __forceinline__ uint2 aff_step(AffState& S, uint32_t rec, int j, uint
   uint32_t Ek[kRows], E4[kRows], Xp[kRows];
 #pragma unroll
   for (int r = 0; r < kRows; ++r) {
-    Ek[r] = __viaddmax_s16x2(S.H[r], C.open, __vadd2(S.E[r], C.exte));
+    Ek[r] = __viaddmax_s16x2(S.E[r], C.exte, S.H[r]);
     E4[r] = lop3<0xEA>(Ek[r], kClean, 0x00010001u);  // (Ek & ~3) | 1
     Xp[r] = __viaddmax_s16x2(r == 0 ? Hd : S.H[r - 1], sg[r], E4[r]);
   }
@@ -131,22 +140,23 @@ __device__ __forceinline__ uint2 aff_step(AffState& S, uint32_t rec, int j, uint
   uint32_t hu = Hup, fu = Fup, nib[kRows / 2], Hk0 = 0, Fk0 = 0;
 #pragma unroll
   for (int r = 0; r < kRows; ++r) {
-    const uint32_t Fk = __viaddmax_s16x2(hu, C.open, __vadd2(fu, C.extf));
+    const uint32_t Fk = __viaddmax_s16x2(fu, C.extf, hu);
     const uint32_t F4 = lop3<0xEA>(Fk, kClean, 0x00020002u);  // (Fk & ~3) | 2
     const uint32_t Hk = __vimax3_s16x2(Xp[r], F4, 0u);
-    const uint32_t Hc = Hk & kClean;
+    const uint32_t Hc = __vadd2(Hk & kClean, C.open);         // Ho
     if (TB) {
       // codes: bytes {r-1 lo, r-1 hi, r lo, r hi} of the three keys, one nibble per byte
       if (r & 1) {
         const uint32_t wH = prmt(Hk0, Hk, 0x6420u), wF = prmt(Fk0, Fk, 0x6420u), wE = prmt(Ek[r - 1], Ek[r], 0x6420u);
-        uint32_t n = (wH & 0x03030303u) + 4u * (wF & 0x01010101u);
-        nib[r >> 1] = n + 8u * (wE & 0x01010101u);
+        const uint32_t n = mad(wF & 0x01010101u, 4u, wH & 0x03030303u);
+        nib[r >> 1] = mad(wE & 0x01010101u, 8u, n);
       }
       Hk0 = Hk; Fk0 = Fk;
       // first row-major maximum: the column where each row's maximum is first reached
-      const uint32_t m = prmt(__vsub2(S.rb[r], Hc), 0u, 0xbb99u);  // 0xffff where Hc > rb
-      S.rc[r] = lop3<0xB8>(S.rc[r], m, j2);                        // (rc & ~m) | (j2 & m)
-      S.rb[r] = __vmaxs2(S.rb[r], Hc);
+      // rb holds ~max = -max - 1, so Hc + rb < 0 exactly when Hc <= max
+      const uint32_t m = prmt(__vadd2(Hc, S.rb[r]), 0u, 0xbb99u);  // 0xffff where Hc <= max
+      S.rc[r] = lop3<0xE2>(S.rc[r], m, j2);                        // (rc & m) | (j2 & ~m)
+      S.rb[r] = __vmins2(S.rb[r], mad(Hc, C.m1, C.m1));  // ~Hc (C.m1 = -1, opaque: kept an IMAD)
     }
     S.H[r] = Hc;
     S.E[r] = E4[r];
@@ -163,7 +173,7 @@ __device__ __forceinline__ uint2 aff_step(AffState& S, uint32_t rec, int j, uint
   if (MULTI && spill31 && live) { sts_u32_v(rec + 4, hu); sts_u32_v(rec + 8, fu); }
   if (!TB) return make_uint2(0, 0);
   // bytes [A0|A2<<4, B0|B2<<4, A1|A3<<4, B1|B3<<4] and the same for rows 4-7, then per problem
-  const uint32_t x = nib[0] + 16u * nib[1], y = nib[2] + 16u * nib[3];
+  const uint32_t x = mad(nib[1], 16u, nib[0]), y = mad(nib[3], 16u, nib[2]);
   return make_uint2(prmt(x, y, 0x6420u), prmt(x, y, 0x7531u));
 }
 
@@ -172,13 +182,14 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_affine16(AlignArgs A, int sm
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int asz = A.asz;
-  // keyed sigma transposed, sigT[c][a] = 4 sigma(a, c) + 3 (32 x 32 int8): kDead outside the
+  const int goe = A.gap_open + A.gap_ext, ge = A.gap_ext;
+  // keyed sigma transposed, sigT[c][a] = 4 sigma(a, c) + 3 - o (32 x 32 int8): kDead outside the
   // alphabet, so a = 31 is a dead residue and c = asz a dead column code
   int8_t* sigT = reinterpret_cast<int8_t*>(smem);
   constexpr int sig_bytes = 32 * 32;
   for (int q = threadIdx.x; q < 32 * 32; q += blockDim.x) {
     const int c = q >> 5, a = q & 31;
-    sigT[q] = (c < asz && a < asz) ? (int8_t)(4 * A.sigma[a * asz + c] + 3) : (int8_t)kDead;
+    sigT[q] = (c < asz && a < asz) ? (int8_t)(4 * A.sigma[a * asz + c] + 3 + 4 * goe - 1) : (int8_t)kDead;
   }
   __syncthreads();
   const int64_t grp = (int64_t)blockIdx.x * kWarps + warp;
@@ -219,12 +230,12 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_affine16(AlignArgs A, int sm
     const int cB = (jj >= 0 && jj < lbB && laB > 0) ? bB[jj] : asz;
     *reinterpret_cast<uint32_t*>(recg + q * kRec) = (uint32_t)(cA * kStrip) | ((uint32_t)(cB * kStrip) << 16);
   }
-  const int goe = A.gap_open + A.gap_ext, ge = A.gap_ext;
   AffK C;
   C.open = pk2(-4 * goe + 1);
   C.exte = pk2(-4 * ge - 1);
   C.extf = pk2(-4 * ge - 2);
   C.negf = pk2(-4 * (goe + 2) + 2);  // F(0, j) = -inf: below every opening (H = 0) after one extension
+  asm volatile("mov.b32 %0, %1;" : "=r"(C.m1) : "r"(0xffffffffu));
   const uint32_t nege = pk2(-4 * (goe + 2) + 1);  // E(i, 0) = -inf
   const int strips = (lam + kStrip - 1) / kStrip;
   const uint32_t laneA = (uint32_t)__cvta_generic_to_shared(profA) + lane * kRows;
@@ -232,7 +243,7 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_affine16(AlignArgs A, int sm
   const bool lane0 = lane == 0;
   // per half: best, its row and column (first row-major maximum)
   int bestv[2] = {0, 0}, besti[2] = {0, 0}, bestj[2] = {0, 0};
-  uint32_t lanemax = 0;
+  uint32_t lanemax = C.open;
   AffState S;
 
   for (int st = 0; st < strips; ++st) {
@@ -275,8 +286,8 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_affine16(AlignArgs A, int sm
     }
     __syncwarp();
 #pragma unroll
-    for (int r = 0; r < kRows; ++r) { S.H[r] = 0; S.E[r] = nege; S.rb[r] = 0; S.rc[r] = 0; }
-    S.prevH = 0; S.F7 = C.negf;
+    for (int r = 0; r < kRows; ++r) { S.H[r] = C.open; S.E[r] = nege; S.rb[r] = TB ? ~C.open : C.open; S.rc[r] = 0; }
+    S.prevH = C.open; S.F7 = C.negf;
     const bool from_bnd = st > 0;
     const bool spill31 = (st + 1 < strips) && lane == 31;
     uint2* cds = TB ? reinterpret_cast<uint2*>(A.dirs + grp * A.dir_stride) + (int64_t)st * A.max_lb * 32 + lane - 32
@@ -317,7 +328,8 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_affine16(AlignArgs A, int sm
       for (int r = 0; r < kRows; ++r) {
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
-          const int v = (h ? hi16(S.rb[r]) : lo16(S.rb[r])) >> 2;
+          const uint32_t mx = ~S.rb[r];
+          const int v = ((h ? hi16(mx) : lo16(mx)) + 4 * goe - 1) >> 2;
           if (v > bestv[h]) { bestv[h] = v; besti[h] = i0 + r + 1; bestj[h] = h ? hi16(S.rc[r]) : lo16(S.rc[r]); }
         }
       }
@@ -348,8 +360,8 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_affine16(AlignArgs A, int sm
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) lanemax = __vmaxs2(lanemax, __shfl_xor_sync(0xffffffffu, lanemax, o));
     if (lane == 0) {
-      A.scores[pA] = lo16(lanemax) >> 2;
-      if (hasB) A.scores[pB] = hi16(lanemax) >> 2;
+      A.scores[pA] = (lo16(lanemax) + 4 * goe - 1) >> 2;
+      if (hasB) A.scores[pB] = (hi16(lanemax) + 4 * goe - 1) >> 2;
     }
   }
 }
@@ -435,8 +447,9 @@ bool affine16_eligible(int64_t max_la, int64_t max_lb, const int8_t* sigma_host,
   const int64_t bound = (int64_t)smax * std::min(max_la, max_lb);  // H <= bound
   // keys 4 v + 3 in int16: 4 bound; E, F >= -(go + ge) after one opening; the -inf keys
   // -4 (go + ge + 2) minus one extension
-  return asz < 32 && 4 * smax + 3 <= 127 && 4 * smin + 3 >= -128 && 4 * bound + 3 <= 32000 && go >= 0 && ge >= 1 &&
-         4 * (go + 2 * ge + 3) <= 32000 && max_lb <= 32000;
+  // profile 4 sigma + 3 - o = 4 sigma + 4 (go + ge) + 2 in int8
+  return asz < 32 && 4 * smax + 4 * (go + ge) + 2 <= 127 && 4 * smin + 4 * (go + ge) + 2 >= -127 &&
+         4 * bound + 3 <= 32000 && go >= 0 && ge >= 1 && 4 * (go + 2 * ge + 3) <= 32000 && max_lb <= 32000;
 }
 
 size_t affine16_smem_bytes(int asz, int64_t max_la, int64_t max_lb) {
