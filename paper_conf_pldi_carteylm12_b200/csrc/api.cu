@@ -572,7 +572,16 @@ dp_status dp_solve_batch(dp_plan_t p, int64_t n, const uint8_t* a_cat, const int
       // other paths, for comparison)
       if (dpk::nuss_small_supported(A.max_len, n, p->device) && !p->env.nuss_cell && p->env.nuss_tiled_min == 32) {
         p->variant = "k_nuss_small";
+        unsigned long long* dbg = nullptr;
+        if (p->env.nuss_timing) cudaMalloc(&dbg, 64), cudaMemset(dbg, 0, 64), A.dbg = dbg;
         e = dpk::nuss_small_solve(A, s, &p->launches);
+        if (dbg) {  // diagnostic: CTA 0 thread 0 cycles (summed over problems): setup, fill, traceback
+          unsigned long long h[3];
+          cudaStreamSynchronize(s);
+          cudaMemcpy(h, dbg, sizeof(h), cudaMemcpyDeviceToHost);
+          fprintf(stderr, "nuss_small cycles: setup %llu fill %llu traceback %llu\n", h[0], h[1], h[2]);
+          cudaFree(dbg);
+        }
         break;
       }
       // a few mid-length problems: one thread-block cluster each, the table in distributed shared
