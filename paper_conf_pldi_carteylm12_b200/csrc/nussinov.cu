@@ -220,6 +220,14 @@ __global__ void __launch_bounds__(kSmallThreads) k_nuss_small(NussArgs A) {
   const int tid = threadIdx.x, lane = tid & 31;
   if (tid < 16) pm[tid] = A.pair_mask[tid];
   const uint32_t NEG2 = (uint32_t)(uint16_t)kSNeg * 0x10001u;
+  long long t0 = A.dbg ? clock64() : 0;  // DP_NUSS_TIMING: thread 0's cycles in setup / fill / traceback
+  auto lap = [&](int k) {
+    if (A.dbg && tid == 0) {
+      const long long t = clock64();
+      atomicAdd(A.dbg + k, (unsigned long long)(t - t0));
+      t0 = t;
+    }
+  };
   for (int64_t p = blockIdx.x; p < A.n; p += gridDim.x) {
     const int n = (int)(A.x_off[p + 1] - A.x_off[p]);
     __syncthreads();
@@ -239,6 +247,7 @@ __global__ void __launch_bounds__(kSmallThreads) k_nuss_small(NussArgs A) {
       prow[i] = (uint8_t)(pm[xi * 4] | pm[xi * 4 + 1] << 1 | pm[xi * 4 + 2] << 2 | pm[xi * 4 + 3] << 3);
     }
     __syncthreads();
+    lap(0);
     for (int d = 1; d < n; ++d) {
       // lane owns rows lane, lane + 32, ...: the cell (i, i + d) of each live row
 #pragma unroll 1
@@ -268,6 +277,7 @@ __global__ void __launch_bounds__(kSmallThreads) k_nuss_small(NussArgs A) {
       if (kSmallThreads == 32) __syncwarp();
       else __syncthreads();
     }
+    lap(1);
     if (tid == 0) A.scores[p] = n <= 1 ? 0 : (int)U[n - 1];
     if (A.db && tid < 32) {  // canonical traceback (R-TB-NUSS), one warp, stack in shared memory
       uint8_t* db = A.db + p * A.db_stride;
@@ -316,6 +326,7 @@ __global__ void __launch_bounds__(kSmallThreads) k_nuss_small(NussArgs A) {
       }
       if (lane == 0) A.db_len[p] = n;
     }
+    lap(2);
   }
 }
 
