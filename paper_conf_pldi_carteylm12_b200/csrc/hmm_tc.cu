@@ -141,6 +141,40 @@ __device__ __forceinline__ void split2(float a, float b, uint32_t& hi, uint32_t&
   lo = *reinterpret_cast<const uint32_t*>(&l);
 }
 
+// Packed fp32 pairs (Blackwell FMUL2 / FADD2: one instruction per two states)
+__device__ __forceinline__ uint64_t f2(float a, float b) {
+  uint64_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+  return r;
+}
+__device__ __forceinline__ uint64_t mul2(uint64_t a, uint64_t b) {
+  uint64_t r;
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+__device__ __forceinline__ uint64_t add2(uint64_t a, uint64_t b) {
+  uint64_t r;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+__device__ __forceinline__ uint64_t sub2(uint64_t a, uint64_t b) {
+  uint64_t r;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+// bf16x2 {lo: bf16(v.x), hi: bf16(v.y)}
+__device__ __forceinline__ uint32_t cvt_bf2(uint64_t v) {
+  uint32_t r;
+  asm("{\n\t.reg .f32 a, b;\n\tmov.b64 {a, b}, %1;\n\tcvt.rn.bf16x2.f32 %0, b, a;\n\t}" : "=r"(r) : "l"(v));
+  return r;
+}
+// (hi, lo) bf16x2 words with hi + lo = v to ~2^-16 (the two-term split, packed)
+__device__ __forceinline__ void split2p(uint64_t v, uint32_t& hi, uint32_t& lo) {
+  hi = cvt_bf2(v);
+  const uint64_t hf = f2(__uint_as_float(hi << 16), __uint_as_float(hi & 0xffff0000u));
+  lo = cvt_bf2(sub2(v, hf));
+}
+
 // Per step, with lagged scaling: alpha^_i = ((alpha^_{i-1} A) o e(x_i)) / R_{i-1},
 // R_i = sum_s alpha^_i(s); then P(x) = prod_{i<=T} R_i and log P = sum log R_i. Dividing by the
 // previous step's sum keeps R_i within the emission range because A is row-stochastic.
@@ -273,32 +307,41 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
       const float* er = &sm.E[(word >> (8 * (sh & 3))) & 0xff][0];
       mbar_wait(&sm.full[g], (uint32_t)(i - 2) & 1u);
       asm volatile("tcgen05.fence::after_thread_sync;");
-      float tot = 0.f;
+      uint64_t tot2 = 0;  // (+0.f, +0.f)
+      // a finished row keeps storing a zero operand (the .sync.aligned stores are warp-uniform
+      // calls): its scale is 0 (the accumulator and the emissions are finite)
+      const float sc = i > T ? 0.f : inv;
+      const uint64_t inv2 = f2(sc, sc);
       uint32_t r[kS];  // the row: 64 accumulators, four loads and one wait
       TMEM_LD16(taddr, r);
       TMEM_LD16(taddr + 16, (r + 16));
       TMEM_LD16(taddr + 32, (r + 32));
       TMEM_LD16(taddr + 48, (r + 48));
       asm volatile("tcgen05.wait::ld.sync.aligned;");
+      // per pair of states: (e * inv), times the accumulator, into the row sum, split to bf16
+      // hi / lo — 8 instructions per two states (FMUL2, FMUL2, FADD2, F2FP, 2 unpacks, FADD2, F2FP)
 #pragma unroll
       for (int k0 = 0; k0 < kS; k0 += 16) {
         const float4* e4 = reinterpret_cast<const float4*>(er + k0);
         const float4 e0 = e4[0], e1 = e4[1], e2 = e4[2], e3 = e4[3];
-        const float ev[16] = {e0.x, e0.y, e0.z, e0.w, e1.x, e1.y, e1.z, e1.w,
-                              e2.x, e2.y, e2.z, e2.w, e3.x, e3.y, e3.z, e3.w};
-        float v[16];
+        const uint64_t ev[8] = {f2(e0.x, e0.y), f2(e0.z, e0.w), f2(e1.x, e1.y), f2(e1.z, e1.w),
+                                f2(e2.x, e2.y), f2(e2.z, e2.w), f2(e3.x, e3.y), f2(e3.z, e3.w)};
+        uint32_t hw[8], lw[8];
 #pragma unroll
-        for (int u = 0; u < 16; ++u) {
-          v[u] = __uint_as_float(r[k0 + u]) * (ev[u] * inv);
-          tot += v[u];
+        for (int q = 0; q < 8; ++q) {
+          const uint64_t v = mul2(f2(__uint_as_float(r[k0 + 2 * q]), __uint_as_float(r[k0 + 2 * q + 1])),
+                                  mul2(ev[q], inv2));
+          tot2 = add2(tot2, v);
+          split2p(v, hw[q], lw[q]);
         }
-        if (i > T) {  // a finished row keeps its operand (.sync.aligned stores: warp-uniform calls)
-#pragma unroll
-          for (int u = 0; u < 16; ++u) v[u] = 0.f;
-        }
-        store16(k0, v);
+        TMEM_ST8(trow + kColsAHi + k0 / 2, hw);
+        TMEM_ST8(trow + kColsALo + k0 / 2, lw);
       }
-      if (i <= T) R = tot;
+      if (i <= T) {
+        float t0, t1;
+        asm("mov.b64 {%0, %1}, %2;" : "=f"(t0), "=f"(t1) : "l"(tot2));
+        R = t0 + t1;
+      }
       asm volatile("tcgen05.wait::st.sync.aligned;");
       asm volatile("tcgen05.fence::before_thread_sync;");
       mbar_arrive(&sm.empty[g]);
