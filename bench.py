@@ -692,7 +692,9 @@ def roofline(W, name, phase_ms, alone, pk):
         "peak": round(tc3 / 1e12, 1), "unit": "TFLOP/s", "frac": round(fl / (fw_ms * 1e-3) / tc3, 4),
         "traffic": (round(t["bytes_per_launch"]) if t else None), "kernel_ms": round(fw_ms, 4),
         "peak_source": "MEASURED_PEAKS.json bf16_tflops (burst) / 3: the fp32 product is computed as three bf16 "
-                       "MMAs (hi x hi, hi x lo, lo x hi); algorithmic flops 2 S^2 per cell; kernel timed alone"}
+                       "MMAs (hi x hi, hi x lo, lo x hi); algorithmic flops 2 S^2 per cell; kernel timed alone",
+        # SURVEY 8(d) D3's SIMT roofline: the same flops against the FFMA peak (2 flops per lane-op)
+        "frac_vs_ffma_peak": round(fl / (fw_ms * 1e-3) / (2 * MEASURED_UBENCH["ffma"] * SMS * pk["sm_max_mhz"] * 1e6), 4)}
     return vit
 
 
