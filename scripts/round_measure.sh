@@ -25,7 +25,7 @@ full hmm "k_forward_tc|k_viterbi" 3
 full nuss1 "k_nuss" 1
 full nuss4 "k_nuss" 1
 full nuss5 "k_nuss_batch" 1 DP_NUSS5_N=50000
-full swa "k_align_affine" 2
+full swa "k_affine16" 2
 full swshort "k_sw_inter" 2
 full nussmid "k_nuss_cluster" 1
 full diag "k_diag" 1
@@ -34,7 +34,7 @@ python scripts/ncu_traffic.py gpurun_out/traffic.json \
   k_sw16=gpurun_out/ncu_sw.ncu-rep k_sw16_tb5=gpurun_out/ncu_sw.ncu-rep \
   k_forward_tc=gpurun_out/ncu_hmm.ncu-rep k_viterbi16=gpurun_out/ncu_hmm.ncu-rep \
   k_nuss_batch=gpurun_out/ncu_nuss5.ncu-rep:20:"50k-problem capture of config 5 x 20" \
-  k_nuss_grid2=gpurun_out/ncu_nuss4.ncu-rep k_align_affine=gpurun_out/ncu_swa.ncu-rep \
+  k_nuss_grid2=gpurun_out/ncu_nuss4.ncu-rep k_affine16=gpurun_out/ncu_swa.ncu-rep \
   k_diag=gpurun_out/ncu_diag.ncu-rep k_phmm_forward=gpurun_out/ncu_phmm.ncu-rep \
   k_sw_inter=gpurun_out/ncu_swshort.ncu-rep k_sw_inter_tb=gpurun_out/ncu_swshort.ncu-rep \
   k_nuss_small=gpurun_out/ncu_nuss1.ncu-rep k_nuss_cluster=gpurun_out/ncu_nussmid.ncu-rep > gpurun_out/traffic.log 2>&1
