@@ -298,6 +298,31 @@ def test_sw_affine_packed_variants(dp, orc):
             assert bytes(out[q, :ln[q]]).decode() == ops and tuple(co[q]) == c, (want, q)
 
 
+def test_sw_affine_packed_guard_boundaries(dp, orc):
+    """SURVEY §8(c) C7 for the packed affine kernel: the plan checks 4 sigma_max min(|a|,|b|) + 3
+    <= 32000 (keys 4 v + code in int16) and 4 sigma + 4 (go + ge) + 2 in int8 (the profile holds the
+    opening-shifted diagonal term); one residue under / over each bound picks k_affine16 /
+    k_align_affine, both bit-exact on identical (high-scoring) and random pairs."""
+    sig = dpgen.blosum62()
+    g = np.random.default_rng(123)
+    for L, go, ge, want in ((727, 11, 1, "k_affine16"), (728, 11, 1, "k_align_affine"),
+                            (200, 19, 1, "k_affine16"), (200, 20, 1, "k_align_affine")):
+        x = g.integers(0, 20, size=L).astype(np.uint8)
+        y = g.integers(0, 20, size=L).astype(np.uint8)
+        a, b = [x, x, y], [x.copy(), y, x]
+        r = run_align(dp, dp.SW_AFFINE, a, b, sigma=sig, asz=24, go=go, ge=ge)
+        with dp.Plan(dp.SW_AFFINE, L, L, sigma=sig, alphabet_size=24, want_traceback=True, gap_open=go,
+                     gap_extend=ge) as p:
+            a_cat, a_off = dpgen.pack(a)
+            b_cat, b_off = dpgen.pack(b)
+            p.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=L, max_len_b=L)
+            assert p.last_variant == want, (L, go, want)
+        for q in range(3):
+            assert r["scores"][q] == orc.sw_affine(a[q], b[q], sig, go, ge)[0], (L, go, q)
+            ops, co = orc.sw_affine_traceback(a[q], b[q], sig, go, ge)
+            assert r["ops"][q] == ops and tuple(r["coords"][q]) == co, (L, go, q)
+
+
 def test_sw_affine_config2_sampled(dp, orc):
     """BASELINE config 2's pairs with affine gaps (open 11, extend 1) at full size,
     in the bench's launch configuration; sampled pairs against the oracle."""
