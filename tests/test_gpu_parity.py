@@ -836,6 +836,32 @@ def test_host_entry_point_chunked(dp, orc):
     plan.close()
 
 
+def test_host_entry_point_affine_chunked(dp, orc):
+    """The packed affine kernel through the host entry point in several chunks of odd size (a
+    chunk's last warp carries one problem): equal to the device path everywhere, the oracle on a
+    sample spread over the chunks."""
+    import torch
+    n = 40_001
+    a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(n)
+    sig = dpgen.blosum62()
+    plan = dp.Plan(dp.SW_AFFINE, 256, 256, sigma=sig, alphabet_size=24, want_traceback=True, gap_open=11,
+                   gap_extend=1)
+    sc, tb, tbl, tbc = plan.solve_batch_host(a_cat, a_off, b_cat, b_off, tb_stride=513)
+    dsc = host(plan.solve_batch(cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off), max_len_a=256, max_len_b=256))
+    assert plan.last_variant == "k_affine16"
+    out, ln, co = plan.traceback(0, n, 513)
+    torch.cuda.synchronize()
+    assert (sc == dsc).all()
+    assert (tbl == host(ln)).all() and (tbc == host(co)).all()
+    used = np.arange(513)[None, :] < tbl[:, None]
+    assert (tb[used] == host(out)[used]).all()
+    for q in list(range(0, n, 2500)) + [n - 1]:
+        x, y = a_cat[a_off[q]:a_off[q + 1]], b_cat[b_off[q]:b_off[q + 1]]
+        ops, c = orc.sw_affine_traceback(x, y, sig, 11, 1)
+        assert sc[q] == orc.sw_affine(x, y, sig, 11, 1)[0] and bytes(tb[q, :tbl[q]]).decode() == ops, q
+    plan.close()
+
+
 # ----------------------------------------------------------------------------- §4.7 diagonal-only
 def run_diag(dp, a_seqs, b_seqs, **kw):
     a_cat, a_off = dpgen.pack(a_seqs)
