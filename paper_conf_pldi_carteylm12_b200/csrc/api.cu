@@ -115,6 +115,7 @@ struct dp_plan {
     bool nuss_rounds = false, diag_generic = false, sw_intra = false;
     int64_t nuss_tiled_min = 32;
     int nuss_tbw = 0, diag_force = -1, host_chunks = 0;  // 0: per kind (see dp_solve_batch_host)
+    double host_edge = 0.5;  // first / last host chunk size relative to the others (config 2 e2e: 1.0 / 0.5 / 0.3: 2.97 / 2.91 / 2.92 ms)
     bool hmm_simt = false, nuss_no_cluster = false, hmm_separate_walk = false;
     int hmm_ns = 0, hmm_tc_smem_kb = -1;
   } env;
@@ -140,6 +141,7 @@ void read_env(dp_plan* p) {
   p->env.hmm_separate_walk = on("DP_HMM_SEPARATE_WALK");
   if (on("DP_HMM_NS")) p->env.hmm_ns = atoi(getenv("DP_HMM_NS"));
   if (on("DP_HMM_TC_SMEM_KB")) p->env.hmm_tc_smem_kb = atoi(getenv("DP_HMM_TC_SMEM_KB"));
+  if (on("DP_HOST_EDGE")) p->env.host_edge = std::max(0.05, std::min(1.0, atof(getenv("DP_HOST_EDGE"))));
   if (on("DP_HOST_CHUNKS")) p->env.host_chunks = std::max(1, std::min(dp_plan::kMaxChunks, atoi(getenv("DP_HOST_CHUNKS"))));
 }
 
@@ -935,7 +937,20 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   const int max_ch = p->env.host_chunks > 0 ? p->env.host_chunks : (p->kind == DP_SW_LINEAR && p->packed16 ? 6 : 4);
   int nch = (int)std::min<int64_t>(max_ch, (n + min_chunk - 1) / min_chunk);
   if (nch < 1) nch = 1;
-  const int64_t per = (n + nch - 1) / nch;
+  // chunk boundaries: the first chunk's H2D and the last chunk's D2H are exposed (nothing to
+  // overlap them with), so with 3+ chunks those two are `edge` times the size of the others
+  int64_t bound[dp_plan::kMaxChunks + 1];
+  {
+    const double edge = nch >= 3 ? p->env.host_edge : 1.0;
+    const double unit = (double)n / (nch >= 3 ? 2.0 * edge + (nch - 2) : (double)nch);
+    double acc = 0.0;
+    bound[0] = 0;
+    for (int c = 1; c < nch; ++c) {
+      acc += (nch >= 3 && c == 1) ? edge : 1.0;
+      bound[c] = std::min<int64_t>(n, ((int64_t)(acc * unit + 0.5) + 1) & ~int64_t(1));  // even: whole packed groups
+    }
+    bound[nch] = n;
+  }
   uint8_t* da = static_cast<uint8_t*>(p->h_a.ptr);
   uint8_t* db = align ? static_cast<uint8_t*>(p->h_b.ptr) : nullptr;
   int64_t* dao = static_cast<int64_t*>(p->h_aoff.ptr);
@@ -969,8 +984,8 @@ dp_status dp_solve_batch_host(dp_plan_t p, int64_t n, const uint8_t* a_cat, cons
   }
   int installed = 0;  // which state buffer is in p->tb_state
   for (int c = 0; c < nch; ++c) {
-    const int64_t k0 = c * per, k1 = std::min(n, k0 + per), nk = k1 - k0;
-    if (nk <= 0) break;
+    const int64_t k0 = bound[c], k1 = std::max(k0, bound[c + 1]), nk = k1 - k0;
+    if (nk <= 0) continue;
     const cudaStream_t sc = (two && (c & 1)) ? p->s_cmp : s;
     void* const scv = reinterpret_cast<void*>(sc);
     if (two && (c & 1) != installed) {
