@@ -21,6 +21,9 @@
 // The groups' chains are independent, so the tensor pipe works on one group while
 // the epilogue warps of the others run; no CTA-wide barrier inside the step loop
 // (the row sum needs no cross-warp reduction when a thread owns a whole row).
+// Within a group the steps overlap too: two accumulators alternate, and the epilogue signals
+// each 16 states of the next operand as soon as they are in TMEM (one `ready` mbarrier per K
+// chunk), so step i+1's MMAs for those K columns run while it still works on the rest.
 // Operands live in shared memory (alpha hi/lo 2 x 16 KB per group, transitions
 // hi/lo 16 KB); the accumulators in TMEM (4 x 64 columns).
 #include <algorithm>
@@ -113,7 +116,15 @@ constexpr int kEpiWarps = 4 * kNG;         // epilogue warps (4 per group: the T
 constexpr int kThreads = 32 * (kEpiWarps + 1);  // + the MMA warp
 // TMEM columns per group: the fp32 accumulator (64), then alpha_hi and alpha_lo as the next A
 // operand (64 bf16 = 32 columns each)
-constexpr int kColsAcc = 0, kColsAHi = kS, kColsALo = kS + kS / 2, kColsGroup = 2 * kS;
+// two fp32 accumulators (steps alternate: step i+1's MMAs run while the epilogue still works on
+// step i's row), then alpha_hi and alpha_lo as the next A operand (64 bf16 = 32 columns each)
+constexpr int kColsAcc = 0, kColsAHi = 2 * kS, kColsALo = 2 * kS + kS / 2, kColsGroup = 4 * kS;
+#ifndef HMM_TC_READY
+#define HMM_TC_READY 16  // states per operand-ready signal (16 / 32 / 64: forward alone 0.842 / 0.858 / 0.899 ms)
+#endif
+constexpr int kReadyS = HMM_TC_READY;
+constexpr int kChunks = kS / kReadyS;       // operand-ready signals per step
+static_assert(kNG * kColsGroup <= 512, "TMEM: 512 columns per SM");
 
 #define TMEM_ST8(taddr, w)                                                                      \
   asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr), \
@@ -123,7 +134,7 @@ struct TcSmem {
   alignas(128) uint8_t b_cat[kN2 * kS * 2];  // transitions (B operand): row n = s (A_hi) or 64 + s (A_lo), k = p
   alignas(16) float E[16][kS + 4];          // emission rows
   uint64_t full[kNG];                       // MMA -> epilogue: the group's accumulator is ready
-  uint64_t empty[kNG];                      // epilogue -> MMA: the group's next operand is stored
+  uint64_t ready[kNG][kChunks];             // epilogue -> MMA: states 16 kk .. 16 kk + 15 of the next operand stored
   uint32_t tmem_base;
   int tmax;
 };
@@ -200,7 +211,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
   if (tid == 0) {
     for (int g = 0; g < kNG; ++g) {
       mbar_init(&sm.full[g], 1);
-      mbar_init(&sm.empty[g], 128);
+      for (int kk = 0; kk < kChunks; ++kk) mbar_init(&sm.ready[g][kk], 128);
     }
     sm.tmax = 0;
     asm volatile("fence.mbarrier_init.release.cluster;");
@@ -236,13 +247,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
       // Descriptor address fields count 16-byte units: a K step of 16 is two core matrices.
       for (int i = 2; i <= Tmax; ++i) {
         for (int q = 0; q < kNG; ++q) {
-          mbar_wait(&sm.empty[q], (uint32_t)(i - 2) & 1u);
-          asm volatile("tcgen05.fence::after_thread_sync;");
-          const uint32_t td = tmem + (uint32_t)(q * kColsGroup + kColsAcc);
+          const uint32_t td = tmem + (uint32_t)(q * kColsGroup + kColsAcc + (i & 1) * kS);
           const uint32_t ta_hi = tmem + (uint32_t)(q * kColsGroup + kColsAHi);
           const uint32_t ta_lo = tmem + (uint32_t)(q * kColsGroup + kColsALo);
 #pragma unroll
-          for (int kk = 0; kk < kS / 16; ++kk) {  // a K step of 16 bf16: 8 TMEM columns of A
+          for (int kk = 0; kk < kS / 16; ++kk) {  // a K step of 16 bf16: 8 TMEM columns of A, issued as
+            if ((16 * kk) % kReadyS == 0) {       // soon as the epilogue stored them
+              mbar_wait(&sm.ready[q][16 * kk / kReadyS], (uint32_t)(i - 2) & 1u);
+              asm volatile("tcgen05.fence::after_thread_sync;");
+            }
             const uint64_t kb = (uint64_t)(2 * kk * (kN2 / 8) * kCore >> 4);
             mma_bf16_ts<kS>(td, ta_hi + 8 * kk, dB + kb, kk > 0);  // a_hi x A_hi
             mma_bf16_ts<kS>(td, ta_hi + 8 * kk, dB_lo + kb, 1);    // a_hi x A_lo
@@ -283,9 +296,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
     }
     asm volatile("tcgen05.wait::st.sync.aligned;");
     asm volatile("tcgen05.fence::before_thread_sync;");
-    mbar_arrive(&sm.empty[g]);
+#pragma unroll
+    for (int kk = 0; kk < kChunks; ++kk) mbar_arrive(&sm.ready[g][kk]);
     uint4 xs = make_uint4(0, 0, 0, 0);
-    const uint32_t taddr = trow + kColsAcc;
     for (int i = 2; i <= Tmax; ++i) {
       const float inv = R > 0.f ? 1.f / R : 0.f;
       if (i - 1 <= T) {
@@ -313,6 +326,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
       const float sc = i > T ? 0.f : inv;
       const uint64_t inv2 = f2(sc, sc);
       uint32_t r[kS];  // the row: 64 accumulators, four loads and one wait
+      const uint32_t taddr = trow + kColsAcc + (i & 1) * kS;
       TMEM_LD16(taddr, r);
       TMEM_LD16(taddr + 16, (r + 16));
       TMEM_LD16(taddr + 32, (r + 32));
@@ -336,15 +350,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_forward_tc(HmmArgs H) {
         }
         TMEM_ST8(trow + kColsAHi + k0 / 2, hw);
         TMEM_ST8(trow + kColsALo + k0 / 2, lw);
+        // these states of the next operand are in TMEM: the next step's K chunks may start
+        if ((k0 + 16) % kReadyS == 0) {
+          asm volatile("tcgen05.wait::st.sync.aligned;");
+          asm volatile("tcgen05.fence::before_thread_sync;");
+          mbar_arrive(&sm.ready[g][k0 / kReadyS]);
+        }
       }
       if (i <= T) {
         float t0, t1;
         asm("mov.b64 {%0, %1}, %2;" : "=f"(t0), "=f"(t1) : "l"(tot2));
         R = t0 + t1;
       }
-      asm volatile("tcgen05.wait::st.sync.aligned;");
-      asm volatile("tcgen05.fence::before_thread_sync;");
-      mbar_arrive(&sm.empty[g]);
     }
     if (Tmax >= 1 && Tmax <= T) prod *= (double)R;  // R_T of the sequences that run to the end
     if (live) H.ll_out[p] = T == 0 ? 0.f : (float)(log(prod) + (double)pexp * 0.69314718055994530942);
