@@ -7,7 +7,7 @@
 //
 // Warp-specialised CTA of kNG groups of 128 sequences (the MMA's M):
 //   * the MMA warp (one elected lane) issues, per step and group, 12
-//     tcgen05.mma.kind::f16 (M=128, N=64, K=16) into that group's fp32 TMEM
+//     tcgen05.mma.kind::f16 (M=128, N=64, K=16, A from TMEM) into that group's fp32 TMEM
 //     accumulator (64 columns): alpha_hi x A_hi + alpha_hi x A_lo + alpha_lo x A_hi,
 //     where x = x_hi + x_lo is a two-term bf16 split (the dropped lo x lo term is
 //     ~2^-16 of a 2^-8 term: ~1e-7 relative per step, DESIGN.md §2 "HMM precision");
@@ -15,17 +15,18 @@
 //   * four epilogue warps per group (warp w reads TMEM lane quarter w % 4), ONE
 //     SEQUENCE PER THREAD over all 64 states: tcgen05.ld of the row, times e_s(x_i),
 //     scaled by 1/R_{i-1} (the previous step's row sum, thread-local: lagged
-//     scaling, log P = sum_i log R_i), split into bf16 hi/lo and stored as the
-//     next A operand in the canonical K-major no-swizzle UMMA layout (8x16-byte
-//     core matrices); then all 128 threads arrive on the group's `empty` mbarrier.
+//     scaling, log P = sum_i log R_i; packed fp32 pairs, FMUL2 / FADD2), split into
+//     bf16 hi/lo and stored with tcgen05.st as the next A operand (TMEM, two bf16 per
+//     column, K-major); all 128 threads arrive on the group's `ready` mbarrier of each
+//     16-state K chunk as soon as it is stored.
 // The groups' chains are independent, so the tensor pipe works on one group while
 // the epilogue warps of the others run; no CTA-wide barrier inside the step loop
 // (the row sum needs no cross-warp reduction when a thread owns a whole row).
 // Within a group the steps overlap too: two accumulators alternate, and the epilogue signals
 // each 16 states of the next operand as soon as they are in TMEM (one `ready` mbarrier per K
 // chunk), so step i+1's MMAs for those K columns run while it still works on the rest.
-// Operands live in shared memory (alpha hi/lo 2 x 16 KB per group, transitions
-// hi/lo 16 KB); the accumulators in TMEM (4 x 64 columns).
+// The transitions (B operand, hi/lo, 16 KB) live in shared memory; per group TMEM holds two
+// fp32 accumulators (2 x 64 columns) and the next A operand alpha hi/lo (2 x 32 columns).
 #include <algorithm>
 #include <cstdint>
 #include <cstdlib>
