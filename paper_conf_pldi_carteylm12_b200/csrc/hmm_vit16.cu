@@ -101,14 +101,15 @@ __device__ __forceinline__ void walk16(const uint2* rws, int T, int sA, int sB, 
   flush(J);
 }
 
-template <bool SAT>
+// FULL: S == 64, every lane's two states exist (no per-step masking)
+template <bool SAT, bool FULL>
 __global__ void __launch_bounds__(32) k_viterbi16(HmmArgs H) {
   __shared__ __align__(16) V16Smem sm;
   const int lane = threadIdx.x;
-  const int S = H.S, K = H.K;
+  const int S = FULL ? kS : H.S, K = H.K;
   const int64_t pa = 2 * (int64_t)blockIdx.x, pb = pa + 1;
   const int s0 = lane, s1 = lane + 32;
-  const bool ok0 = s0 < S, ok1 = s1 < S;
+  const bool ok0 = FULL || s0 < S, ok1 = FULL || s1 < S;
   const int Ta = pa < H.n ? (int)(H.x_off[pa + 1] - H.x_off[pa]) : 0;
   const int Tb = pb < H.n ? (int)(H.x_off[pb + 1] - H.x_off[pb]) : 0;
   const int Tmax = max(Ta, Tb);
@@ -186,6 +187,7 @@ __global__ void __launch_bounds__(32) k_viterbi16(HmmArgs H) {
     if (Tb == 1) fb = final_state(r0, r1, true), vb = offb;
   }
   __syncwarp();
+  const int Tmin = min(Ta, Tb);
   for (int i = 2; i <= Tmax; ++i) {
     if (((i - 1) & (kCh - 1)) == 0) {
       __syncwarp();
@@ -215,9 +217,11 @@ __global__ void __launch_bounds__(32) k_viterbi16(HmmArgs H) {
     if (!ok0) n0 = 0x80008000u;
     if (!ok1) n1 = 0x80008000u;
     const uint32_t m = __vmaxs2(n0, n1);
-    const int Ma = __reduce_max_sync(0xffffffffu, (int)(m << 16)) >> 16;
-    const int Mb = __reduce_max_sync(0xffffffffu, (int)(m & 0xffff0000u)) >> 16;
-    const uint32_t negM = pk(-Ma, -Mb);
+    // the halves' maxima, shifted up 16: their negations' high halves are -M, packed by one PRMT
+    const int Ra = __reduce_max_sync(0xffffffffu, (int)(m << 16));
+    const int Rb = __reduce_max_sync(0xffffffffu, (int)(m & 0xffff0000u));
+    const int Ma = Ra >> 16, Mb = Rb >> 16;
+    const uint32_t negM = __byte_perm(0u - (uint32_t)Ra, 0u - (uint32_t)Rb, 0x7632);
     const uint32_t r0 = __viaddmax_s16x2(n0, negM, Cpk);
     const uint32_t r1 = __viaddmax_s16x2(n1, negM, Cpk);
     offa += sm.emax[ca] + Ma;
@@ -226,8 +230,10 @@ __global__ void __launch_bounds__(32) k_viterbi16(HmmArgs H) {
     sm.row[i & 1][s1] = r1;
     if (rows && i < Tmax)  // row of position i, read by the walk at position i + 1
       reinterpret_cast<uint2*>(rows + (int64_t)(i - 1) * kS)[lane] = make_uint2(r0, r1);
-    if (i == Ta) fa = final_state(r0, r1, false), va = offa;  // warp-uniform
-    if (i == Tb) fb = final_state(r0, r1, true), vb = offb;
+    if (i >= Tmin) {  // warp-uniform; only the last steps of the shorter sequence
+      if (i == Ta) fa = final_state(r0, r1, false), va = offa;
+      if (i == Tb) fb = final_state(r0, r1, true), vb = offb;
+    }
     __syncwarp();
   }
   if (lane == 0) {
@@ -291,7 +297,9 @@ cudaError_t hmm_viterbi16(const HmmArgs& H, cudaStream_t s, int64_t* launches) {
   void* args[1] = {&h2};
   ++*launches;
   const unsigned grid = (unsigned)((H.n + 1) / 2);
-  return cudaLaunchKernel(H.v16_sat ? (void*)k_viterbi16<true> : (void*)k_viterbi16<false>, dim3(grid), dim3(32),
+  void* kern = H.S == kS ? (H.v16_sat ? (void*)k_viterbi16<true, true> : (void*)k_viterbi16<false, true>)
+                         : (H.v16_sat ? (void*)k_viterbi16<true, false> : (void*)k_viterbi16<false, false>);
+  return cudaLaunchKernel(kern, dim3(grid), dim3(32),
                           args, 0, s);
 }
 
