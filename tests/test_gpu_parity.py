@@ -977,3 +977,60 @@ def test_nussinov_short_batches(dp, orc, count):
             if count > 120 and q % 7:
                 continue
             assert (r["scores"][q], r["db"][q]) == orc.nussinov_traceback(x, pm, h), (q, len(x))
+
+
+# ----------------------------------------------------------------------------- determinism
+def test_repeat_determinism(dp):
+    """Race detection by repetition (compute-sanitizer is closed on this GPU pool): the
+    warp-synchronous kernels with shared-memory hand-offs and the mbarrier-pipelined tcgen05
+    forward give bit-identical outputs when the same plan runs the same batch again, at sizes that
+    fill the GPU (several waves, both halves of every packed register, multi-strip columns)."""
+    import torch
+    sig = dpgen.blosum62()
+    a_cat, a_off, b_cat, b_off = dpgen.config2_protein_pairs(20_001)
+    A = (cuda(a_cat), cuda(a_off), cuda(b_cat), cuda(b_off))
+
+    def used(out, ln):  # bytes past a row's length are unspecified (dp.h): zero them
+        mask = torch.arange(out.shape[1], device=out.device)[None, :] < ln[:, None].long()
+        return torch.where(mask, out, torch.zeros_like(out))
+
+    def twice(plan, fn):
+        r1 = fn(plan)
+        torch.cuda.synchronize()
+        r2 = fn(plan)
+        torch.cuda.synchronize()
+        for k, (x, y) in enumerate(zip(r1, r2)):
+            assert torch.equal(x, y), k
+
+    def align(p):
+        sc = p.solve_batch(*A, max_len_a=256, max_len_b=256).clone()
+        out, ln, co = p.traceback(0, 20_001, 513)
+        return sc, used(out, ln), ln.clone(), co.clone()
+
+    with dp.Plan(dp.SW_LINEAR, 256, 256, sigma=sig, gap=dpgen.SW_GAP, want_traceback=True) as p:
+        twice(p, align)
+        assert p.last_variant == "k_sw16"
+    with dp.Plan(dp.SW_AFFINE, 256, 256, sigma=sig, alphabet_size=24, want_traceback=True, gap_open=11,
+                 gap_extend=1) as p:
+        twice(p, align)
+        assert p.last_variant == "k_affine16"
+    h = dpgen.config3_hmm(n_seqs=2_000, T=400)
+    cat, off = dpgen.pack(h["seqs"])
+    X = (cuda(cat), cuda(off))
+    with dp.Plan(dp.HMM_FORWARD, 400, pi=h["pi"], A=h["A"], E=h["E"]) as p:
+        twice(p, lambda q: (q.solve_batch(*X).clone(),))
+    with dp.Plan(dp.HMM_VITERBI, 400, lpi=h["lpi"], lA=h["lA"], lE=h["lE"], want_traceback=True) as p:
+        def vit(q):
+            sc = q.solve_batch(*X).clone()
+            out, ln, _ = q.traceback(0, 2_000, 400, coords=False)
+            return sc, used(out, ln), ln.clone()
+        twice(p, vit)
+        assert p.last_variant == "k_viterbi16"
+    rna = dpgen.config5_rna_batch(n_seqs=3_000)
+    R = (cuda(rna[0]), cuda(rna[1]))
+    with dp.Plan(dp.NUSSINOV, 512, pair_mask=dpgen.rna_pair_mask(), min_hairpin=3, want_traceback=True) as p:
+        def nuss(q):
+            sc = q.solve_batch(*R, max_len_a=512).clone()
+            out, ln, _ = q.traceback(0, 3_000, 512, coords=False)
+            return sc, used(out, ln), ln.clone()
+        twice(p, nuss)
