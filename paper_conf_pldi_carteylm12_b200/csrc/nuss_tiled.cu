@@ -240,7 +240,7 @@ __device__ __forceinline__ void wavefront(InTileBuf& B, bool diag, int left, int
 // j down by at most one, so a window serves up to 7 steps); split points cost one round
 // trip per 32 candidates. The interval stack lives in shared memory (kStk entries), deeper
 // entries in global memory.
-constexpr int kStk = 64;
+constexpr int kStk = 62;  // 62 (not 64): the batch kernel's 512-nt footprint then fits 16 CTAs per SM (228 KB)
 // Trace one interval [i, j] (canonical order); the right part of every split is handed to
 // push(k+1, j) and the walk continues on the left part. W x W window (rows i..i+W-1, columns
 // j-W+1..j; W*W/32 values per lane per round trip); KC split candidates per lane per round trip.
