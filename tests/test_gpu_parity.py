@@ -862,6 +862,28 @@ def test_host_entry_point_affine_chunked(dp, orc):
     plan.close()
 
 
+def test_host_entry_point_viterbi_chunked(dp, orc):
+    """The s16x2 Viterbi through the host entry point on a batch big enough for three chunks:
+    scores and paths equal to the device path, the oracle on a sample spread over the chunks; an
+    odd batch so a chunk's last warp carries one sequence."""
+    import torch
+    h = dpgen.config3_hmm(n_seqs=70_001, T=100)
+    cat, off = dpgen.pack(h["seqs"])
+    n = len(off) - 1
+    plan = dp.Plan(dp.HMM_VITERBI, 100, lpi=h["lpi"], lA=h["lA"], lE=h["lE"], want_traceback=True)
+    sc, tb, tbl, _ = plan.solve_batch_host(cat, off, tb_stride=100)
+    dsc = host(plan.solve_batch(cuda(cat), cuda(off)))
+    assert plan.last_variant == "k_viterbi16"
+    out, ln, _ = plan.traceback(0, n, 100, coords=False)
+    torch.cuda.synchronize()
+    out, ln = host(out), host(ln)
+    assert (sc == dsc).all() and (tbl == ln).all() and (tb == out).all()
+    for q in list(range(0, n, 5000)) + [n - 1]:
+        v, path = orc.viterbi(h["seqs"][q], h["lpi"], h["lA"], h["lE"])
+        assert sc[q] == v and (tb[q] == path).all(), q
+    plan.close()
+
+
 # ----------------------------------------------------------------------------- §4.7 diagonal-only
 def run_diag(dp, a_seqs, b_seqs, **kw):
     a_cat, a_off = dpgen.pack(a_seqs)
