@@ -17,10 +17,10 @@
 //
 // Traceback retention without per-cell direction codes: the forward pass
 // stores checkpoints of G — the bottom row of every 16-row band (odd lanes,
-// every column) and, after every block of 32 steps, every lane's 8 rows at the
-// column it is on (a staircase, column 32 s - lane: warp-uniform, coalesced,
+// every column) and, after every block of kSlab = 16 steps, every lane's 8 rows at the
+// column it is on (a staircase, column 16 s - lane: warp-uniform, coalesced,
 // no per-step branch), the G above it there and its best G over the block
-// (0.25 B/cell), plus every lane's maximum over the strip. k_sw16_tb5 recomputes
+// (0.25 + 0.5 B/cell), plus every lane's maximum over the strip. k_sw16_tb5 recomputes
 // only the 32x32 (sheared) blocks the canonical traceback needs, as 2-bit
 // direction codes that carry the oracle's tie-break (stop at H = 0, then
 // diag > up > left; end cell = first maximum in row-major order), and walks them.
@@ -42,7 +42,8 @@ constexpr int kStrip = 32 * kRows;    // rows per strip
 constexpr int kBand = 16;             // checkpoint band height (two lanes)
 constexpr int kLanesPerBand = kBand / kRows;
 constexpr int kBandsPerStrip = kStrip / kBand;
-constexpr int kSlab = 32;             // checkpoint column spacing
+constexpr int kSlab = 16;             // checkpoint column spacing (sweep steps)
+constexpr int kBW = 32;               // traceback block width (re-run steps): two checkpoint intervals
 constexpr int kDead = -100;           // profile value for rows/columns outside a problem
 constexpr int kPad = 32;              // dead columns on each side of the residue array
 
@@ -256,8 +257,8 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
       corner = A.corner + sb;
     }
     // step k works on column j = k - lane + 1, record address sh_rec + kRec (k - lane + kPad).
-    // Steps come in blocks of 32 (one slab); after block s every lane checkpoints
-    // at once (warp-uniform, coalesced): its 8 G values at column 32(s+1) - lane,
+    // Steps come in blocks of kSlab (one slab); after block s every lane checkpoints
+    // at once (warp-uniform, coalesced): its 8 G values at column kSlab (s+1) - lane,
     // the G above it there (corner), and its best G over the block.
     const uint32_t rec0 = sh_rec + kRec * (kPad - lane);
     const int K = lbm + 31;
@@ -325,8 +326,9 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
 // warps stay full until the queues drain.
 //
 // A traceback "block" is 32 rows (forward lanes L0..L0+3 of one strip,
-// L0 = 4 (blk mod 8)) x one slab: forward lane L0+m covered columns
-// j = D + c - m, c = 1..32, D = 32 slab - L0, at forward steps 32 slab + c - 1.
+// L0 = 4 (blk mod 8)) x two slabs from checkpoint sl (kBW = 32 steps): forward lane L0+m covered
+// columns j = D + c - m, c = 1..32, D = 16 sl - L0, at forward steps 16 sl + c - 1 (a walker's
+// block starts at the checkpoint that leaves it 17..32 columns of room).
 // So in the sheared column c all four lanes are at the SAME forward step and
 // group lane m re-runs forward lane L0+m (8 rows) for 32 steps exactly as the
 // sweep did (no ramp): the left column is its checkpoint, its first diagonal the
@@ -358,7 +360,7 @@ constexpr int kTbUnroll = TB5_UNROLL;   // re-run steps unrolled
 #endif
 constexpr int kSigRow = 34;              // int16 per sigma row (17 words: see k_sw16_tb5)
 constexpr int kSigBytes = ((32 * kSigRow * 2 + 127) / 128) * 128;
-constexpr int kCW = kGL * kSlab;         // code words per group: [c - 1][m]
+constexpr int kCW = kGL * kBW;           // code words per group: [c - 1][m]
 constexpr int kCWp = kCW + 4;            // group stride: 4 banks apart, so the 8 groups' code stores hit 32 banks
 constexpr int kTS = 36;                  // top-row keys per group, c = 0..32
 constexpr int kBS = 40;                  // staged b residues per half (columns D-3 .. D+36)
@@ -566,11 +568,13 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         } else if (mode == kWalk) {
           const int ln = ((S.i - 1) % kStrip) / kRows;
           r0 = (S.i - 1) / kStrip * kStrip + kRows * (kGL == 2 ? (ln & ~1) : (ln < 2 ? 0 : ((ln - 2) & ~1)));
-          sl = (S.j + ln - 1) / kSlab;
+          // the block starts at a checkpoint (every kSlab steps) that puts the walker at c in
+          // [kBW - kSlab + 1, kBW]: at least kSlab columns of room before leaving on the left
+          sl = max(0, (S.j + ln - 1) / kSlab - (kBW / kSlab - 1));
           // the next block is left (same rows or 16 up) or 32 rows up: pull their checkpoints into L2
 #pragma unroll
           for (int q = 0; q < 3; ++q) {
-            const int nr = r0 - (q == 0 ? 0 : (q == 1 ? 16 : 32)), ns = sl - (q < 2 ? 1 : 0);
+            const int nr = r0 - (q == 0 ? 0 : (q == 1 ? 16 : 32)), ns = sl - (q == 0 ? kBW / kSlab : (q == 1 ? 1 : 0));
             if (nr < 0 || ns < 1) continue;
             const int st = nr / kStrip, L0 = (nr % kStrip) / kRows;
             const int64_t base = (grp * SM + st) * NS + (ns - 1);
@@ -598,7 +602,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         const uint8_t* ap = S.a;
         const uint8_t* bp = S.b;
         const int la = S.la, lb = S.lb;
-        uint32_t av[kRows], bv[kBS / kGL], tv[(kSlab + kGL) / kGL];
+        uint32_t av[kRows], bv[kBS / kGL], tv[(kBW + kGL) / kGL];
 #pragma unroll
         for (int r = 0; r < kRows; ++r) {
           const int i = R0[hf] + kRows * m + r + 1;
@@ -614,9 +618,9 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         const uint32_t* rk = A.rowck + ((grp * SM + (bnd >= 0 ? bnd / kBandsPerStrip : 0)) * kBandsPerStrip +
                                         (bnd >= 0 ? bnd % kBandsPerStrip : 0)) * A.max_lb - 1;
 #pragma unroll
-        for (int k = 0; k < (kSlab + kGL) / kGL; ++k) {
+        for (int k = 0; k < (kBW + kGL) / kGL; ++k) {
           const int c = m + kGL * k, j = D[hf] + c;
-          tv[k] = (on && bnd >= 0 && c <= kSlab && j >= 1 && j <= lb) ? __ldcg(rk + j) : NEG_G2;
+          tv[k] = (on && bnd >= 0 && c <= kBW && j >= 1 && j <= lb) ? __ldcg(rk + j) : NEG_G2;
         }
         // this half's residues and top-row keys to shared memory
 #pragma unroll
@@ -628,8 +632,8 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         for (int k = 0; k < kBS / kGL; ++k) bS[hf * kBS + m + kGL * k] = (uint8_t)bv[k];
         int16_t* ts16 = reinterpret_cast<int16_t*>(Ts) + hf;
 #pragma unroll
-        for (int k = 0; k < (kSlab + kGL) / kGL; ++k)
-          if (m + kGL * k <= kSlab) ts16[2 * (m + kGL * k)] = (int16_t)(4 * half16(tv[k], hf));
+        for (int k = 0; k < (kBW + kGL) / kGL; ++k)
+          if (m + kGL * k <= kBW) ts16[2 * (m + kGL * k)] = (int16_t)(4 * half16(tv[k], hf));
       }
 #pragma unroll
       for (int r = 0; r < kRows; ++r) Kc[r] = key4(join(w[0][r], w[1][r]));
@@ -644,7 +648,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
       const uint32_t bA = bs32 + (3 - m), bB = bs32 + kBS + (3 - m);
       const uint32_t cw0 = cs32 + 4 * m;
 #pragma unroll kTbUnroll
-      for (int c = 1; c <= kSlab; ++c) {
+      for (int c = 1; c <= kBW; ++c) {
         const uint32_t topv = lds_u32(ts32 + 4 * c);
         const uint32_t fa = __shfl_up_sync(full, Kc[kRows - 1], 1, kGL);
         const uint32_t Ku = m == 0 ? topv : fa;
@@ -733,7 +737,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         int t = i - r0 - 1;
         int c = j - d0 + (t >> 3);
         bool stop = false;
-        if (t >= kBlk || c > kSlab) t = -1;  // a search just ended outside this block: walk next round
+        if (t >= kBlk || c > kBW) t = -1;  // a search just ended outside this block: walk next round
         while (t >= 0 && c >= 1) {
           const uint32_t wd = lds_u32(cw + 4 * kGL * c + 4 * (t >> 3));
           const uint32_t ra = lds_u8(as32 + i), rb = lds_u8(bsx + j);
@@ -815,7 +819,7 @@ size_t sw16_smem_bytes(int asz, int64_t max_la, int64_t max_lb) {
 void sw16_state_words(int64_t n, int64_t max_la, int64_t max_lb, int64_t* strips, int64_t* nslab, int64_t* rowck,
                       int64_t* colck, int64_t* slabbest) {
   *strips = (max_la + kStrip - 1) / kStrip;
-  *nslab = (max_lb + 31 + kSlab - 1) / kSlab;  // sweep steps lbm + 31 in blocks of 32
+  *nslab = (max_lb + 31 + kSlab - 1) / kSlab;  // sweep steps lbm + 31 in blocks of kSlab
   const int64_t groups = (n + 1) / 2;
   *rowck = groups * *strips * kBandsPerStrip * max_lb;
   *colck = groups * *strips * *nslab * kStrip;
