@@ -39,10 +39,16 @@ namespace {
 #endif
 constexpr int kRows = 8;              // rows per lane
 constexpr int kStrip = 32 * kRows;    // rows per strip
-constexpr int kBand = 16;             // checkpoint band height (two lanes)
+#ifndef SW16_BAND
+#define SW16_BAND 16
+#endif
+constexpr int kBand = SW16_BAND;      // checkpoint band height (16: two lanes, 8: every lane)
 constexpr int kLanesPerBand = kBand / kRows;
 constexpr int kBandsPerStrip = kStrip / kBand;
-constexpr int kSlab = 16;             // checkpoint column spacing (sweep steps)
+#ifndef SW16_SLAB
+#define SW16_SLAB 16
+#endif
+constexpr int kSlab = SW16_SLAB;      // checkpoint column spacing (sweep steps)
 constexpr int kBW = 32;               // traceback block width (re-run steps): two checkpoint intervals
 constexpr int kDead = -100;           // profile value for rows/columns outside a problem
 constexpr int kPad = 32;              // dead columns on each side of the residue array
@@ -198,7 +204,7 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
   const int strips = (lam + kStrip - 1) / kStrip;
   const uint32_t laneA = (uint32_t)__cvta_generic_to_shared(profA) + lane * kRows;
   const uint32_t laneB = (uint32_t)__cvta_generic_to_shared(profB) + lane * kRows;
-  const bool lane0 = lane == 0, odd = (lane & 1) != 0;
+  const bool lane0 = lane == 0, odd = (lane + 1) % kLanesPerBand == 0;  // "odd": the lane ends a band
   FwdState S;
   S.best2 = NEG_G2;  // max G = max h - g
 
@@ -567,7 +573,9 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
           }
         } else if (mode == kWalk) {
           const int ln = ((S.i - 1) % kStrip) / kRows;
-          r0 = (S.i - 1) / kStrip * kStrip + kRows * (kGL == 2 ? (ln & ~1) : (ln < 2 ? 0 : ((ln - 2) & ~1)));
+          r0 = (S.i - 1) / kStrip * kStrip +
+               kRows * (kBand == kRows ? (ln < kGL - 1 ? 0 : ln - (kGL - 1))  // walker in the block's last lane
+                                       : (kGL == 2 ? (ln & ~1) : (ln < 2 ? 0 : ((ln - 2) & ~1))));
           // the block starts at a checkpoint (every kSlab steps) that puts the walker at c in
           // [kBW - kSlab + 1, kBW]: at least kSlab columns of room before leaving on the left
           sl = max(0, (S.j + ln - 1) / kSlab - (kBW / kSlab - 1));
