@@ -233,7 +233,7 @@ dp_status dp_traceback(dp_plan_t p, int64_t first, int64_t count, uint8_t* out, 
 int64_t dp_plan_launch_count(dp_plan_t p);
 
 /* The kernel family the most recent dp_solve_batch / dp_solve / dp_solve_batch_host on this plan
- * ran (DESIGN.md §3 names: "k_sw16", "k_sw_inter", "k_align", "k_align_affine", "k_diag",
+ * ran (DESIGN.md §3 names: "k_sw16", "k_sw_inter", "k_align", "k_affine16", "k_align_affine", "k_diag",
  * "k_nuss_small", "k_nuss_cluster", "k_nuss_batch", "k_nuss_grid2", "k_nuss_cell",
  * "k_forward_tc", "k_forward", "k_viterbi16", "k_viterbi", "k_phmm_forward"); "" before the
  * first solve or for a NULL plan. Static storage; valid for the life of the library. Tests
