@@ -269,8 +269,18 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
     const uint32_t rec0 = sh_rec + kRec * (kPad - lane);
     const int K = lbm + 31;
     constexpr int U = SW16_UNROLL;
-    for (int kb = 0, sl = 0; kb < K; kb += kSlab, ++sl) {
-      const int ke = min(kb + kSlab, K);
+    constexpr int kB = TB ? kSlab : 2 * kSlab;  // steps per block (score only: no checkpoints)
+    for (int kb = 0, sl = 0; kb < K; kb += kB, ++sl) {
+      const int ke = min(kb + kB, K);
+      if (kB == U && kb >= 31 && ke <= lbm - 1) {  // a whole steady block: one unrolled run
+        const uint32_t rec = rec0 + kRec * kb;
+        uint32_t* rk = rowck + (kb - lane);
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+          sw_step<TB, false, MULTI>(S, rec + kRec * u, kb + u - lane + 1, lbm, lane0, odd, spill31, from_bnd, NEG_G2,
+                                    laneA, laneB, rk + u);
+        if (MULTI) __syncwarp();
+      } else {
       // steady range: lane 31 at j >= 1 and lane 0 at j <= lbm - 1
       const int s0 = min(max(kb, 31), ke), s1 = max(s0, min(ke, lbm - 1));
       int k = kb;
@@ -299,6 +309,7 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_sw16(Sw16Args A) {
         sw_step<TB, true, MULTI>(S, rec0 + kRec * k, k - lane + 1, lbm, lane0, odd, spill31, from_bnd, NEG_G2,
                                  laneA, laneB, rowck + (k - lane));
         if (MULTI) __syncwarp();
+      }
       }
       if (TB) {
         uint4* col = reinterpret_cast<uint4*>(colck + (int64_t)sl * kStrip);
