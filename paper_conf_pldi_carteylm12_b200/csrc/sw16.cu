@@ -401,6 +401,8 @@ struct TbState {      // one problem in one half of a group (shared memory; writ
 constexpr int kGroupBytes = 4 * kCWp + 4 * kTS + 2 * kBS + 2 * kBlk + 2 * (int)sizeof(TbState);
 constexpr int kTbWarpBytes = kGroups * kGroupBytes;
 
+// first forward lane of the search block of lane band ln (ln in the block's lane 2 or 3 when ln >= 2)
+__device__ __forceinline__ int search_l0(int ln) { return ln < 2 ? 0 : ((ln - 2) & ~1); }
 __device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
   uint32_t v;
   asm("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
@@ -576,9 +578,12 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
         // at least 16 rows before leaving upwards.
         int r0 = 0, sl = 0;
         if (srch) {
-          r0 = (S.band >> 5) * kStrip + kBlk * ((S.band & 31) / kGL);
-          sl = S.cand;
-          if (m == (S.band & 31) % kGL) {
+          // the search block puts the band in its lane 2 or 3 and the candidate slab in its second
+          // half, so a walk starting in this round from the end cell has room above and to the left
+          const int lnb = S.band & 31, L0b = search_l0(lnb);
+          r0 = (S.band >> 5) * kStrip + kRows * L0b;
+          sl = max(0, S.cand - (kBW / kSlab - 1));
+          if (m == lnb - L0b) {
             const uint32_t t = (uint32_t)(uint16_t)(int16_t)(4 * (S.best - g) - 1);
             T4m1 = hf ? ((T4m1 & 0xffffu) | (t << 16)) : ((T4m1 & 0xffff0000u) | t);
           }
@@ -719,7 +724,7 @@ __global__ void __launch_bounds__(kTbWarps * 32, TB5_MINB) k_sw16_tb5(Sw16Args A
       TbState& S = St[hf];
       if (m == 0 && S.mode == kSearch && S.cand >= 0) {
         if (key < (1 << 30)) {
-          const int m8 = (S.band & 31) % kGL, r = key >> 6, c = key & 63;
+          const int m8 = (S.band & 31) - search_l0(S.band & 31), r = key >> 6, c = key & 63;
           const long long k2 = ((long long)(R0[hf] + kRows * m8 + r + 1) << 32) | (long long)(D[hf] + c - m8);
           if (S.found < 0 || k2 < S.found) S.found = k2;
         }
